@@ -1,0 +1,26 @@
+"""Shared pytest configuration.
+
+Markers:
+  gpu -- needs a CUDA device (B200); run with ``-m gpu`` on the GPU box.
+Everything unmarked runs on the CPU-only dev box (``-m "not gpu"``).
+"""
+import os
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+
+def pytest_configure(config):
+    config.addinivalue_line("markers", "gpu: test needs a CUDA device (B200)")
+    config.addinivalue_line("markers", "slow: long-running test")
+
+
+@pytest.fixture(scope="session")
+def orc():
+    import oracle
+    oracle.build()
+    return oracle
