@@ -1,0 +1,670 @@
+// api.cu -- the C ABI (include/blsh.h): argument checks, memory, orchestration
+// of the build (b1-b4) and of the query hot path (a1-a6).
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <string>
+
+#include "internal.cuh"
+#include "query_kernels.cuh"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+blsh_status fail(blsh_status c, const std::string& m) {
+    g_last_error = m;
+    return c;
+}
+
+bool is_device_ptr(const void* p) {
+    if (!p) return false;
+    cudaPointerAttributes at{};
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+template <typename F>
+blsh_status guarded(F&& f) {
+    try {
+        f();
+        return BLSH_OK;
+    } catch (const blsh::Error& e) {
+        return fail(e.code, e.what());
+    } catch (const std::bad_alloc&) {
+        return fail(BLSH_ERR_OOM, "host allocation failed");
+    } catch (const std::exception& e) {
+        return fail(BLSH_ERR_CUDA, e.what());
+    }
+}
+
+__global__ void k_point_leaf(const uint32_t* __restrict__ order, const int64_t* __restrict__ seg, int G,
+                             int32_t* __restrict__ pt_leaf) {
+    const int g = blockIdx.y;
+    if (g >= G) return;
+    for (int64_t p = seg[g] + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < seg[g + 1];
+         p += (int64_t)gridDim.x * blockDim.x)
+        pt_leaf[order[p]] = g;
+}
+
+__global__ void k_point_key(const unsigned long long* __restrict__ hi, const unsigned long long* __restrict__ lo,
+                            const uint32_t* __restrict__ id, int64_t n, blsh::Key128* __restrict__ pt_key) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        pt_key[id[i]] = blsh::Key128{hi[i], lo[i]};
+}
+
+int64_t ipow3(int M) {
+    int64_t p = 1;
+    for (int i = 0; i < M; ++i) p *= 3;
+    return p;
+}
+
+}  // namespace
+
+extern "C" {
+
+void blsh_build_params_default(blsh_build_params* p) {
+    if (!p) return;
+    std::memset(p, 0, sizeof(*p));
+    p->n_leaves = 1;
+    p->rp_rule = 0;
+    p->rp_mean_c = 10.0;
+    p->rp_max_jitter = 0.0;
+    p->ek_iters = 40;
+    p->M = 8;
+    p->quantizer = 0;
+    p->W = 4.0f;
+    p->W_leaf = nullptr;
+    p->seed = 42;
+    p->rank = 0;
+    p->world = 1;
+    p->stream = nullptr;
+    p->keep_stages = 0;
+}
+
+void blsh_query_params_default(blsh_query_params* p) {
+    if (!p) return;
+    std::memset(p, 0, sizeof(*p));
+    p->probe = 0;
+    p->n_probes = 1;
+    p->hierarchy = 0;
+    p->hier_step_bits = 0;
+    p->min_cand = 0;
+    p->stream = nullptr;
+    p->keep_stages = 0;
+    p->timing = 0;
+}
+
+const char* blsh_last_error(void) { return g_last_error.c_str(); }
+
+void blsh_free(blsh_index* idx) {
+    if (!idx) return;
+    for (auto& e : idx->ev)
+        if (e) cudaEventDestroy(e);
+    delete idx;
+}
+
+blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_params* p, blsh_index** out) {
+    if (!out) return fail(BLSH_ERR_INVALID, "out is NULL");
+    *out = nullptr;
+    if (!p) return fail(BLSH_ERR_INVALID, "params is NULL");
+    if (n < 0 || n >= (int64_t(1) << 31)) return fail(BLSH_ERR_INVALID, "n must be in [0, 2^31)");
+    if (n > 0 && !X) return fail(BLSH_ERR_INVALID, "X is NULL");
+    if (d < 1 || d > 1024) return fail(BLSH_ERR_INVALID, "d must be in [1, 1024]");
+    const int G = p->n_leaves;
+    if (G < 1 || G > 4096 || (G & (G - 1))) return fail(BLSH_ERR_INVALID, "n_leaves must be a power of two in [1, 4096]");
+    if (p->M < 1 || p->M > 16) return fail(BLSH_ERR_INVALID, "M must be in [1, 16]");
+    if (p->quantizer != 0 && p->quantizer != 1) return fail(BLSH_ERR_INVALID, "quantizer must be 0 or 1");
+    if (p->quantizer == 1 && p->M != 8) return fail(BLSH_ERR_INVALID, "E8 quantizer needs M = 8");
+    if (!(p->W > 0.0f) || !std::isfinite(p->W)) return fail(BLSH_ERR_INVALID, "W must be > 0");
+    if (p->rp_rule != 0 && p->rp_rule != 1) return fail(BLSH_ERR_INVALID, "rp_rule must be 0 or 1");
+    if (p->ek_iters < 1) return fail(BLSH_ERR_INVALID, "ek_iters must be >= 1");
+    if (p->world < 1 || p->rank < 0 || p->rank >= p->world || G % p->world != 0)
+        return fail(BLSH_ERR_INVALID, "rank/world must satisfy 0 <= rank < world and world | n_leaves");
+    if (p->W_leaf)
+        for (int g = 0; g < G; ++g)
+            if (!(p->W_leaf[g] > 0.0f) || !std::isfinite(p->W_leaf[g])) return fail(BLSH_ERR_INVALID, "W_leaf must be > 0");
+    auto t0 = std::chrono::steady_clock::now();
+    blsh_index* ix = new (std::nothrow) blsh_index();
+    if (!ix) return fail(BLSH_ERR_OOM, "host allocation failed");
+    cudaStream_t s = (cudaStream_t)p->stream;
+    blsh_status st = guarded([&] {
+        blsh::upload_e8_roots();
+        ix->n = n;
+        ix->d = d;
+        ix->ds = (d + 3) & ~3;
+        ix->G = G;
+        ix->M = p->M;
+        ix->B = blsh::bits_per_coord(p->M);
+        ix->quantizer = p->quantizer;
+        ix->rp_rule = p->rp_rule;
+        ix->rp_mean_c = p->rp_mean_c;
+        ix->rp_max_jitter = p->rp_max_jitter;
+        ix->ek_iters = p->ek_iters;
+        ix->seed = p->seed;
+        ix->rank = p->rank;
+        ix->world = p->world;
+        ix->leaf_lo = p->rank * (G / p->world);
+        ix->leaf_hi = (p->rank + 1) * (G / p->world);
+        int depth = 0;
+        while ((1 << depth) < G) ++depth;
+        ix->depth = depth;
+        const int ds = ix->ds, M = ix->M, nn = std::max(G - 1, 1);
+        // b1: parameters (host, R2)
+        ix->W_h.resize(G);
+        for (int g = 0; g < G; ++g) ix->W_h[g] = p->W_leaf ? p->W_leaf[g] : p->W;
+        ix->A_h.assign((size_t)G * M * d, 0.0f);
+        ix->b_h.assign((size_t)G * M, 0.0f);
+        ix->dirs_h.assign((size_t)nn * d, 0.0f);
+        ix->jit_h.assign(nn, 0.0);
+        blsh::gen_params(p->seed, G, M, d, ix->W_h.data(), ix->A_h.data(), ix->b_h.data(), ix->dirs_h.data(),
+                         ix->jit_h.data());
+        ix->A.alloc(ix->A_h.size() * sizeof(float));
+        ix->b.alloc(ix->b_h.size() * sizeof(float));
+        ix->W.alloc(G * sizeof(float));
+        BLSH_CUDA(cudaMemcpyAsync(ix->A.p, ix->A_h.data(), ix->A_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+        BLSH_CUDA(cudaMemcpyAsync(ix->b.p, ix->b_h.data(), ix->b_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+        BLSH_CUDA(cudaMemcpyAsync(ix->W.p, ix->W_h.data(), G * sizeof(float), cudaMemcpyHostToDevice, s));
+        ix->dirs.alloc((size_t)nn * ds * sizeof(float));
+        BLSH_CUDA(cudaMemsetAsync(ix->dirs.p, 0, (size_t)nn * ds * sizeof(float), s));
+        if (G > 1)
+            BLSH_CUDA(cudaMemcpy2DAsync(ix->dirs.p, ds * sizeof(float), ix->dirs_h.data(), d * sizeof(float),
+                                        d * sizeof(float), G - 1, cudaMemcpyHostToDevice, s));
+        // data in the padded row layout
+        blsh::DevBuf Xs;
+        Xs.alloc((size_t)std::max<int64_t>(n, 1) * ds * sizeof(float));
+        if (ds != d) BLSH_CUDA(cudaMemsetAsync(Xs.p, 0, (size_t)std::max<int64_t>(n, 1) * ds * sizeof(float), s));
+        if (n > 0)
+            BLSH_CUDA(cudaMemcpy2DAsync(Xs.p, ds * sizeof(float), X, d * sizeof(float), d * sizeof(float), n,
+                                        cudaMemcpyDefault, s));
+        // b2: RP-tree
+        blsh::DevBuf order;
+        order.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(uint32_t));
+        std::vector<int64_t> seg;
+        blsh::build_rptree(*ix, Xs.as<float>(), order.as<uint32_t>(), seg, s);
+        const int64_t pos_lo = seg[ix->leaf_lo], pos_hi = seg[ix->leaf_hi];
+        const int64_t no = pos_hi - pos_lo;
+        ix->n_owned = no;
+        // b3: hash owned points
+        blsh::SortBufs sb;
+        for (int i = 0; i < 2; ++i) {
+            sb.hi[i].alloc((size_t)std::max<int64_t>(no, 1) * 8);
+            sb.lo[i].alloc((size_t)std::max<int64_t>(no, 1) * 8);
+            sb.leaf[i].alloc((size_t)std::max<int64_t>(no, 1) * 4);
+            sb.id[i].alloc((size_t)std::max<int64_t>(no, 1) * 4);
+        }
+        int32_t* code_out = nullptr;
+        if (p->keep_stages) {
+            ix->pt_code.alloc((size_t)std::max<int64_t>(n, 1) * M * sizeof(int32_t));
+            BLSH_CUDA(cudaMemsetAsync(ix->pt_code.p, 0, (size_t)std::max<int64_t>(n, 1) * M * sizeof(int32_t), s));
+            code_out = ix->pt_code.as<int32_t>();
+        }
+        const bool ok = blsh::hash_points(*ix, Xs.as<float>(), order.as<uint32_t>(), seg, pos_lo, pos_hi,
+                                          sb.hi[0].as<unsigned long long>(), sb.lo[0].as<unsigned long long>(),
+                                          sb.leaf[0].as<uint32_t>(), sb.id[0].as<uint32_t>(), code_out, s);
+        if (!ok) throw blsh::Error(BLSH_ERR_RANGE, "a data point's code leaves the Morton range (decrease M or increase W)");
+        if (p->keep_stages) {
+            ix->pt_leaf.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(int32_t));
+            ix->pt_key.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(blsh::Key128));
+            BLSH_CUDA(cudaMemsetAsync(ix->pt_key.p, 0, (size_t)std::max<int64_t>(n, 1) * sizeof(blsh::Key128), s));
+            blsh::DevBuf seg_d;
+            seg_d.alloc(seg.size() * sizeof(int64_t));
+            BLSH_CUDA(cudaMemcpyAsync(seg_d.p, seg.data(), seg.size() * sizeof(int64_t), cudaMemcpyHostToDevice, s));
+            dim3 g(64, G);
+            k_point_leaf<<<g, 256, 0, s>>>(order.as<uint32_t>(), seg_d.as<int64_t>(), G, ix->pt_leaf.as<int32_t>());
+            BLSH_LAUNCH_CHECK();
+            if (no > 0) {
+                k_point_key<<<592, 256, 0, s>>>(sb.hi[0].as<unsigned long long>(), sb.lo[0].as<unsigned long long>(),
+                                                sb.id[0].as<uint32_t>(), no, ix->pt_key.as<blsh::Key128>());
+                BLSH_LAUNCH_CHECK();
+            }
+            BLSH_CUDA(cudaStreamSynchronize(s));
+            ix->has_pt = true;
+        }
+        // b4: sort + table
+        int passes = 0;
+        const int cur = blsh::radix_sort_entries(sb, no, s, &passes);
+        blsh::build_table(*ix, Xs.as<float>(), sb.hi[cur].as<unsigned long long>(), sb.lo[cur].as<unsigned long long>(),
+                          sb.leaf[cur].as<uint32_t>(), sb.id[cur].as<uint32_t>(), no, sb.scan, s);
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        for (auto& e : ix->ev) BLSH_CUDA(cudaEventCreate(&e));
+    });
+    if (st != BLSH_OK) {
+        delete ix;
+        return st;
+    }
+    ix->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    *out = ix;
+    return BLSH_OK;
+}
+
+}  // extern "C"
+
+namespace blsh {
+
+void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k, const blsh_query_params& p,
+               int64_t* out_ids, float* out_d2, unsigned long long* out_packed, int64_t* out_ncand, bool out_host) {
+    cudaStream_t s = (cudaStream_t)p.stream;
+    QueryWork& w = ix.qw;
+    const int T = p.n_probes, M = ix.M, ds = ix.ds;
+    const bool keep = p.keep_stages != 0;
+    const bool tm = p.timing != 0;
+    blsh_stats& stt = ix.stats;
+    stt = blsh_stats{};
+    stt.nq = nq;
+    int launches = 0;
+    // ---- workspace ----
+    size_t need = 0;
+    auto add = [&](size_t cnt, size_t el) { need += Arena::need(cnt, el); };
+    add((size_t)nq * ds, 4);            // Qd
+    add(nq, 4); add((size_t)nq * M, 4); add((size_t)nq * M, 4); add(nq, 4); add(nq, 16);
+    add((size_t)nq * (T + 1), 8);       // ivl
+    add(nq, 8); add(nq, 8); add(nq, 4); // base cnt level
+    add(nq + 1, 8); add(nq + 1, 8);     // items, item_off
+    add(nq + 1, 8);                     // cand_off
+    add(4, 8);                          // tau + misc
+    if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
+    if (out_host) { add((size_t)nq * k, 8); add((size_t)nq * k, 4); add(nq, 8); add((size_t)nq * k, 8); }
+    w.arena.ensure(need);
+    Arena ar{w.arena.as<char>(), 0, w.arena.bytes};
+    w.Qd = ar.take<float>((size_t)nq * ds);
+    w.qleaf = ar.take<int32_t>(nq);
+    w.qt = ar.take<float>((size_t)nq * M);
+    w.qcode = ar.take<int32_t>((size_t)nq * M);
+    w.qoor = ar.take<int32_t>(nq);
+    w.qkey = ar.take<Key128>(nq);
+    w.ivl = ar.take<uint2>((size_t)nq * (T + 1));
+    w.base = ar.take<int64_t>(nq);
+    w.cnt = ar.take<int64_t>(nq);
+    w.level = ar.take<int32_t>(nq);
+    int64_t* items = ar.take<int64_t>(nq + 1);
+    w.item_off = ar.take<int64_t>(nq + 1);
+    int64_t* cand_off = ar.take<int64_t>(nq + 1);
+    w.tau = ar.take<int64_t>(4);
+    w.pkey = keep ? ar.take<Key128>((size_t)nq * T) : nullptr;
+    w.pvalid = keep ? ar.take<int32_t>((size_t)nq * T) : nullptr;
+    int64_t* d_ids = out_ids;
+    float* d_d2 = out_d2;
+    int64_t* d_nc = out_ncand;
+    unsigned long long* d_pk = out_packed;
+    if (out_host) {
+        int64_t* si = ar.take<int64_t>((size_t)nq * k);
+        float* sd = ar.take<float>((size_t)nq * k);
+        int64_t* sn = ar.take<int64_t>(nq);
+        unsigned long long* sp = ar.take<unsigned long long>((size_t)nq * k);
+        d_ids = out_ids ? si : nullptr;
+        d_d2 = out_d2 ? sd : nullptr;
+        d_nc = out_ncand ? sn : nullptr;
+        d_pk = out_packed ? sp : nullptr;
+    }
+    w.nq = nq;
+    w.T = T;
+    w.k = k;
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[0], s));
+    // ---- queries into the padded layout ----
+    if (ds != ix.d) BLSH_CUDA(cudaMemsetAsync(w.Qd, 0, (size_t)nq * ds * sizeof(float), s));
+    BLSH_CUDA(cudaMemcpy2DAsync(w.Qd, ds * sizeof(float), Q, ix.d * sizeof(float), ix.d * sizeof(float), nq,
+                                q_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, s));
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[1], s));
+    QueryArgs a{};
+    a.nq = nq; a.d = ix.d; a.ds = ds; a.G = ix.G; a.M = M; a.B = ix.B; a.depth = ix.depth;
+    a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi;
+    a.probe = p.probe; a.T = T; a.hstep = p.hier_step_bits > 0 ? p.hier_step_bits : M;
+    a.Q = w.Qd; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
+    a.ntype = ix.ntype.as<int32_t>(); a.A = ix.A.as<float>(); a.bvec = ix.b.as<float>(); a.Wl = ix.W.as<float>();
+    a.ukey = ix.ukey.as<Key128>(); a.uoff = ix.uoff.as<uint32_t>(); a.leaf_u = ix.leaf_u.as<int64_t>();
+    a.qleaf = w.qleaf; a.qt = w.qt; a.qcode = w.qcode; a.qoor = w.qoor; a.qkey = w.qkey;
+    a.pkey = w.pkey; a.pvalid = w.pvalid; a.ivl = w.ivl; a.base = w.base; a.cnt = w.cnt; a.level = w.level;
+    // a1+a2
+    launch_route_hash(a, s); ++launches;
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
+    // a3+a4
+    launch_probe_lookup(a, s); ++launches;
+    if (p.hierarchy) {
+        if (p.min_cand == 0) { launch_median(w.base, nq, w.tau, s); ++launches; }
+        launch_widen(a, w.tau, p.min_cand, s); ++launches;
+    }
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[3], s));
+    // plan: chunking of the candidate lists
+    scan_exclusive_i64(w.cnt, cand_off, nq, w.scan, s); launches += 3;
+    int64_t total = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    const int64_t target = 148 * 8 * 4;
+    int64_t ch = (total + target - 1) / std::max<int64_t>(target, 1);
+    ch = std::min<int64_t>(4096, std::max<int64_t>(256, (ch + 31) / 32 * 32));
+    launch_items(w.cnt, nq, (int)ch, items, s); ++launches;
+    scan_exclusive_i64(items, w.item_off, nq, w.scan, s); launches += 3;
+    int64_t n_items = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[4], s));
+    // a5
+    ShortlistArgs sa{};
+    sa.nq = nq; sa.n_items = n_items; sa.d = ix.d; sa.ds = ds; sa.T = T; sa.k = k; sa.chunk = (int)ch;
+    sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
+    sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
+    launch_shortlist(sa, s); if (n_items) ++launches;
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
+    launch_merge(sa, w.qoor, d_ids, d_d2, d_pk, d_nc, s); ++launches;
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
+    if (out_host) {
+        if (out_ids) BLSH_CUDA(cudaMemcpyAsync(out_ids, d_ids, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
+        if (out_d2) BLSH_CUDA(cudaMemcpyAsync(out_d2, d_d2, (size_t)nq * k * 4, cudaMemcpyDeviceToHost, s));
+        if (out_ncand) BLSH_CUDA(cudaMemcpyAsync(out_ncand, d_nc, (size_t)nq * 8, cudaMemcpyDeviceToHost, s));
+        if (out_packed) BLSH_CUDA(cudaMemcpyAsync(out_packed, d_pk, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
+    }
+    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[7], s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    stt.total_cand = total;
+    stt.n_items = n_items;
+    stt.chunk = (int32_t)ch;
+    stt.launches = launches;
+    stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 + (double)n_items * k * 8.0;
+    if (p.hierarchy) {
+        int64_t tau = p.min_cand;
+        if (p.min_cand == 0) BLSH_CUDA(cudaMemcpy(&tau, w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        stt.tau = tau;
+    }
+    if (tm) {
+        cudaEventElapsedTime(&stt.ms_route_hash, ix.ev[1], ix.ev[2]);
+        cudaEventElapsedTime(&stt.ms_probe, ix.ev[2], ix.ev[3]);
+        cudaEventElapsedTime(&stt.ms_plan, ix.ev[3], ix.ev[4]);
+        cudaEventElapsedTime(&stt.ms_shortlist, ix.ev[4], ix.ev[5]);
+        cudaEventElapsedTime(&stt.ms_merge, ix.ev[5], ix.ev[6]);
+        cudaEventElapsedTime(&stt.ms_total, ix.ev[0], ix.ev[7]);
+    }
+    ix.has_stages = keep;
+}
+
+}  // namespace blsh
+
+namespace {
+
+blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32_t k, const blsh_query_params* p) {
+    if (!idx) return fail(BLSH_ERR_INVALID, "index is NULL");
+    if (!p) return fail(BLSH_ERR_INVALID, "params is NULL");
+    if (nq < 0 || nq >= (int64_t(1) << 31)) return fail(BLSH_ERR_INVALID, "nq must be in [0, 2^31)");
+    if (nq > 0 && !Q) return fail(BLSH_ERR_INVALID, "Q is NULL");
+    if (k < 1) return fail(BLSH_ERR_INVALID, "k must be >= 1");
+    if (k > 64) return fail(BLSH_ERR_UNSUPPORTED, "k > 64 is not implemented in this build (NEXT: large-k short-list)");
+    if (p->n_probes < 1) return fail(BLSH_ERR_INVALID, "n_probes must be >= 1");
+    if (p->probe == 0 && p->n_probes != 1) return fail(BLSH_ERR_INVALID, "standard probing uses n_probes = 1");
+    if (p->probe == 1) {
+        if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "multiprobe needs a Z^M index");
+        if (idx->M > 10) return fail(BLSH_ERR_UNSUPPORTED, "multiprobe needs M <= 10");
+        if (p->n_probes > ipow3(idx->M)) return fail(BLSH_ERR_INVALID, "n_probes > 3^M");
+    } else if (p->probe == 2) {
+        if (idx->quantizer != 1) return fail(BLSH_ERR_INVALID, "lattice probing needs an E8 index");
+        if (p->n_probes > 241) return fail(BLSH_ERR_INVALID, "n_probes > 241");
+    } else if (p->probe != 0) {
+        return fail(BLSH_ERR_INVALID, "probe must be 0, 1 or 2");
+    }
+    if (p->n_probes > 256) return fail(BLSH_ERR_UNSUPPORTED, "n_probes > 256");
+    if (p->hierarchy) {
+        if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "the Morton hierarchy needs a Z^M index");
+        if (p->hier_step_bits < 0 || p->hier_step_bits > idx->M) return fail(BLSH_ERR_INVALID, "hier_step_bits must be in [0, M]");
+        if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");
+        if (p->min_cand == 0 && idx->world > 1)
+            return fail(BLSH_ERR_UNSUPPORTED, "batch-median tau on a sharded index needs a global median (pass min_cand)");
+    }
+    return BLSH_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+blsh_status blsh_query(const blsh_index* idx, const float* Q, int64_t nq, int32_t k, const blsh_query_params* p,
+                       int64_t* out_ids, float* out_dist2, int64_t* out_ncand) {
+    blsh_status c = check_query(idx, Q, nq, k, p);
+    if (c != BLSH_OK) return c;
+    if (nq > 0 && (!out_ids || !out_dist2)) return fail(BLSH_ERR_INVALID, "outputs are NULL");
+    if (nq == 0) return BLSH_OK;
+    const bool q_host = !is_device_ptr(Q);
+    const bool o_host = !is_device_ptr(out_ids);
+    if (o_host != !is_device_ptr(out_dist2) || (out_ncand && o_host != !is_device_ptr(out_ncand)))
+        return fail(BLSH_ERR_INVALID, "outputs must all be host or all be device memory");
+    return guarded([&] { blsh::run_query(*idx, Q, q_host, nq, k, *p, out_ids, out_dist2, nullptr, out_ncand, o_host); });
+}
+
+blsh_status blsh_query_packed(const blsh_index* idx, const float* Q, int64_t nq, int32_t k, const blsh_query_params* p,
+                              uint64_t* out_packed, int64_t* out_ncand) {
+    blsh_status c = check_query(idx, Q, nq, k, p);
+    if (c != BLSH_OK) return c;
+    if (nq > 0 && !out_packed) return fail(BLSH_ERR_INVALID, "out_packed is NULL");
+    if (idx->n >= (int64_t(1) << 32)) return fail(BLSH_ERR_UNSUPPORTED, "packed lists need n < 2^32");
+    if (nq == 0) return BLSH_OK;
+    const bool q_host = !is_device_ptr(Q);
+    const bool o_host = !is_device_ptr(out_packed);
+    if (out_ncand && o_host != !is_device_ptr(out_ncand))
+        return fail(BLSH_ERR_INVALID, "outputs must all be host or all be device memory");
+    return guarded([&] {
+        blsh::run_query(*idx, Q, q_host, nq, k, *p, nullptr, nullptr, reinterpret_cast<unsigned long long*>(out_packed),
+                        out_ncand, o_host);
+    });
+}
+
+blsh_status blsh_merge_topk(const uint64_t* packed, int32_t n_lists, int64_t nq, int32_t k, int64_t* out_ids,
+                            float* out_dist2, void* stream) {
+    if (n_lists < 1 || nq < 0 || k < 1) return fail(BLSH_ERR_INVALID, "bad sizes");
+    if (k > 64) return fail(BLSH_ERR_UNSUPPORTED, "k > 64");
+    if (nq == 0) return BLSH_OK;
+    if (!packed || !out_ids || !out_dist2) return fail(BLSH_ERR_INVALID, "NULL pointer");
+    if (!is_device_ptr(packed)) return fail(BLSH_ERR_INVALID, "packed must be device memory");
+    const bool o_host = !is_device_ptr(out_ids);
+    cudaStream_t s = (cudaStream_t)stream;
+    return guarded([&] {
+        blsh::DevBuf si, sd;
+        int64_t* di = out_ids;
+        float* dd = out_dist2;
+        if (o_host) {
+            si.alloc((size_t)nq * k * 8);
+            sd.alloc((size_t)nq * k * 4);
+            di = si.as<int64_t>();
+            dd = sd.as<float>();
+        }
+        blsh::merge_lists(reinterpret_cast<const unsigned long long*>(packed), n_lists, nq, k, di, dd, s);
+        if (o_host) {
+            BLSH_CUDA(cudaMemcpyAsync(out_ids, di, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
+            BLSH_CUDA(cudaMemcpyAsync(out_dist2, dd, (size_t)nq * k * 4, cudaMemcpyDeviceToHost, s));
+        }
+        BLSH_CUDA(cudaStreamSynchronize(s));
+    });
+}
+
+blsh_status blsh_index_info(const blsh_index* idx, blsh_info* out) {
+    if (!idx || !out) return fail(BLSH_ERR_INVALID, "NULL pointer");
+    out->n = idx->n;
+    out->n_owned = idx->n_owned;
+    out->nu = idx->nu;
+    out->d = idx->d;
+    out->d_stride = idx->ds;
+    out->G = idx->G;
+    out->M = idx->M;
+    out->B = idx->B;
+    out->quantizer = idx->quantizer;
+    out->leaf_lo = idx->leaf_lo;
+    out->leaf_hi = idx->leaf_hi;
+    out->device_bytes = (int64_t)(idx->A.bytes + idx->b.bytes + idx->W.bytes + idx->dirs.bytes + idx->mu.bytes +
+                                  idx->theta.bytes + idx->ntype.bytes + idx->Xp.bytes + idx->perm.bytes +
+                                  idx->ukey.bytes + idx->uleaf.bytes + idx->uoff.bytes + idx->leaf_u.bytes +
+                                  idx->pt_leaf.bytes + idx->pt_code.bytes + idx->pt_key.bytes);
+    out->build_ms = idx->build_ms;
+    return BLSH_OK;
+}
+
+blsh_status blsh_last_stats(const blsh_index* idx, blsh_stats* out) {
+    if (!idx || !out) return fail(BLSH_ERR_INVALID, "NULL pointer");
+    *out = idx->stats;
+    return BLSH_OK;
+}
+
+blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t cap, size_t* needed) {
+    if (!idx) return fail(BLSH_ERR_INVALID, "index is NULL");
+    const int64_t G = idx->G, M = idx->M, d = idx->d, nn = G > 1 ? G - 1 : 0;
+    const blsh::QueryWork& w = idx->qw;
+    const int64_t nq = w.nq;
+    const int T = w.T;
+    const void* host_src = nullptr;
+    const void* dev_src = nullptr;
+    size_t bytes = 0;
+    std::vector<char> tmp;
+    auto need_q = [&]() -> bool { return idx->has_stages; };
+    auto need_pt = [&]() -> bool { return idx->has_pt; };
+    switch (what) {
+        case BLSH_EX_A: host_src = idx->A_h.data(); bytes = idx->A_h.size() * 4; break;
+        case BLSH_EX_B: host_src = idx->b_h.data(); bytes = idx->b_h.size() * 4; break;
+        case BLSH_EX_W: host_src = idx->W_h.data(); bytes = idx->W_h.size() * 4; break;
+        case BLSH_EX_DIRS: host_src = idx->dirs_h.data(); bytes = (size_t)nn * d * 4; break;
+        case BLSH_EX_MU: host_src = idx->mu_h.data(); bytes = (size_t)nn * d * 4; break;
+        case BLSH_EX_THETA: host_src = idx->theta_h.data(); bytes = (size_t)nn * 4; break;
+        case BLSH_EX_NTYPE: host_src = idx->ntype_h.data(); bytes = (size_t)nn * 4; break;
+        case BLSH_EX_DIAM2: host_src = idx->diam2_h.data(); bytes = (size_t)nn * 8; break;
+        case BLSH_EX_DA2: host_src = idx->da2_h.data(); bytes = (size_t)nn * 8; break;
+        case BLSH_EX_PERM: {
+            bytes = (size_t)idx->n_owned * 8;
+            if (dst && cap >= bytes && bytes) {
+                std::vector<uint32_t> p32(idx->n_owned);
+                if (cudaMemcpy(p32.data(), idx->perm.p, p32.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    return fail(BLSH_ERR_CUDA, "export copy failed");
+                int64_t* o = (int64_t*)dst;
+                for (size_t i = 0; i < p32.size(); ++i) o[i] = p32[i];
+            }
+            if (needed) *needed = bytes;
+            return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+        }
+        case BLSH_EX_UKEY: {
+            bytes = (size_t)idx->nu * 16;
+            if (dst && cap >= bytes && bytes) {
+                std::vector<blsh::Key128> k(idx->nu);
+                if (cudaMemcpy(k.data(), idx->ukey.p, k.size() * 16, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    return fail(BLSH_ERR_CUDA, "export copy failed");
+                uint64_t* o = (uint64_t*)dst;
+                for (size_t i = 0; i < k.size(); ++i) { o[2 * i] = k[i].hi; o[2 * i + 1] = k[i].lo; }
+            }
+            if (needed) *needed = bytes;
+            return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+        }
+        case BLSH_EX_ULEAF: dev_src = idx->uleaf.p; bytes = (size_t)idx->nu * 4; break;
+        case BLSH_EX_UOFF: {
+            bytes = (size_t)(idx->nu + 1) * 8;
+            if (dst && cap >= bytes) {
+                std::vector<uint32_t> u(idx->nu + 1);
+                if (cudaMemcpy(u.data(), idx->uoff.p, u.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    return fail(BLSH_ERR_CUDA, "export copy failed");
+                int64_t* o = (int64_t*)dst;
+                for (size_t i = 0; i < u.size(); ++i) o[i] = u[i];
+            }
+            if (needed) *needed = bytes;
+            return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+        }
+        case BLSH_EX_LEAF_U: host_src = idx->leaf_u_h.data(); bytes = (size_t)(G + 1) * 8; break;
+        case BLSH_EX_POINT_LEAF:
+            if (!need_pt()) return fail(BLSH_ERR_INVALID, "build without keep_stages");
+            dev_src = idx->pt_leaf.p; bytes = (size_t)idx->n * 4; break;
+        case BLSH_EX_POINT_CODE:
+            if (!need_pt()) return fail(BLSH_ERR_INVALID, "build without keep_stages");
+            dev_src = idx->pt_code.p; bytes = (size_t)idx->n * M * 4; break;
+        case BLSH_EX_POINT_KEY: {
+            if (!need_pt()) return fail(BLSH_ERR_INVALID, "build without keep_stages");
+            bytes = (size_t)idx->n * 16;
+            if (dst && cap >= bytes && bytes) {
+                std::vector<blsh::Key128> k(idx->n);
+                if (cudaMemcpy(k.data(), idx->pt_key.p, k.size() * 16, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    return fail(BLSH_ERR_CUDA, "export copy failed");
+                uint64_t* o = (uint64_t*)dst;
+                for (size_t i = 0; i < k.size(); ++i) { o[2 * i] = k[i].hi; o[2 * i + 1] = k[i].lo; }
+            }
+            if (needed) *needed = bytes;
+            return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+        }
+        default: break;
+    }
+    if (what >= BLSH_EX_Q_LEAF && what <= BLSH_EX_Q_INTERVALS) {
+        if (!need_q()) return fail(BLSH_ERR_INVALID, "last query without keep_stages");
+        switch (what) {
+            case BLSH_EX_Q_LEAF: dev_src = w.qleaf; bytes = (size_t)nq * 4; break;
+            case BLSH_EX_Q_T: dev_src = w.qt; bytes = (size_t)nq * M * 4; break;
+            case BLSH_EX_Q_CODE: dev_src = w.qcode; bytes = (size_t)nq * M * 4; break;
+            case BLSH_EX_Q_OOR: {
+                bytes = (size_t)nq * 4;
+                if (dst && cap >= bytes) {
+                    if (cudaMemcpy(dst, w.qoor, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+                        return fail(BLSH_ERR_CUDA, "export copy failed");
+                    int32_t* o = (int32_t*)dst;
+                    for (int64_t i = 0; i < nq; ++i) o[i] &= 1;
+                }
+                if (needed) *needed = bytes;
+                return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+            }
+            case BLSH_EX_Q_KEY:
+            case BLSH_EX_Q_PKEY: {
+                const int64_t cnt = what == BLSH_EX_Q_KEY ? nq : nq * T;
+                bytes = (size_t)cnt * 16;
+                if (dst && cap >= bytes && bytes) {
+                    std::vector<blsh::Key128> k(cnt);
+                    std::vector<int32_t> oor(nq);
+                    if (cudaMemcpy(k.data(), what == BLSH_EX_Q_KEY ? (void*)w.qkey : (void*)w.pkey, bytes,
+                                   cudaMemcpyDeviceToHost) != cudaSuccess ||
+                        cudaMemcpy(oor.data(), w.qoor, nq * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                        return fail(BLSH_ERR_CUDA, "export copy failed");
+                    uint64_t* o = (uint64_t*)dst;
+                    for (int64_t i = 0; i < cnt; ++i) {
+                        const bool zero = what == BLSH_EX_Q_KEY && (oor[i] & 1);
+                        o[2 * i] = zero ? 0 : k[i].hi;
+                        o[2 * i + 1] = zero ? 0 : k[i].lo;
+                    }
+                }
+                if (needed) *needed = bytes;
+                return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+            }
+            case BLSH_EX_Q_PVALID: dev_src = w.pvalid; bytes = (size_t)nq * T * 4; break;
+            case BLSH_EX_Q_BASE: dev_src = w.base; bytes = (size_t)nq * 8; break;
+            case BLSH_EX_Q_LEVEL: dev_src = w.level; bytes = (size_t)nq * 4; break;
+            case BLSH_EX_Q_TAU: host_src = &idx->stats.tau; bytes = 8; break;
+            case BLSH_EX_Q_INTERVALS: {
+                bytes = (size_t)nq * (T + 1) * 16;
+                if (dst && cap >= bytes && bytes) {
+                    std::vector<uint2> iv((size_t)nq * (T + 1));
+                    if (cudaMemcpy(iv.data(), w.ivl, iv.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+                        return fail(BLSH_ERR_CUDA, "export copy failed");
+                    int64_t* o = (int64_t*)dst;
+                    for (size_t i = 0; i < iv.size(); ++i) { o[2 * i] = iv[i].x; o[2 * i + 1] = iv[i].y; }
+                }
+                if (needed) *needed = bytes;
+                return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
+            }
+            default: break;
+        }
+    }
+    if (!host_src && !dev_src && bytes == 0 && what != BLSH_EX_Q_TAU) {
+        if (needed) *needed = 0;
+        switch (what) {
+            case BLSH_EX_A: case BLSH_EX_B: case BLSH_EX_W: case BLSH_EX_DIRS: case BLSH_EX_MU: case BLSH_EX_THETA:
+            case BLSH_EX_NTYPE: case BLSH_EX_DIAM2: case BLSH_EX_DA2: case BLSH_EX_ULEAF: case BLSH_EX_LEAF_U:
+            case BLSH_EX_Q_LEAF: case BLSH_EX_Q_T: case BLSH_EX_Q_CODE: case BLSH_EX_Q_PVALID: case BLSH_EX_Q_BASE:
+            case BLSH_EX_Q_LEVEL: case BLSH_EX_POINT_LEAF: case BLSH_EX_POINT_CODE:
+                return BLSH_OK;
+            default:
+                return fail(BLSH_ERR_INVALID, "unknown export item");
+        }
+    }
+    if (needed) *needed = bytes;
+    if (!dst || cap < bytes) return fail(BLSH_ERR_INVALID, "dst too small");
+    if (bytes == 0) return BLSH_OK;
+    if (host_src) {
+        std::memcpy(dst, host_src, bytes);
+        return BLSH_OK;
+    }
+    if (cudaMemcpy(dst, dev_src, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+        return fail(BLSH_ERR_CUDA, "export copy failed");
+    return BLSH_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,185 @@
+// internal.cuh -- library-internal declarations (index layout, launchers).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/blsh.h"
+#include "common.cuh"
+
+namespace blsh {
+
+// Error carrying a blsh_status; converted at the ABI boundary.
+struct Error : std::runtime_error {
+    blsh_status code;
+    Error(blsh_status c, const std::string& m) : std::runtime_error(m), code(c) {}
+};
+
+#define BLSH_CUDA(expr)                                                                      \
+    do {                                                                                     \
+        cudaError_t e__ = (expr);                                                            \
+        if (e__ != cudaSuccess)                                                              \
+            throw ::blsh::Error(e__ == cudaErrorMemoryAllocation ? BLSH_ERR_OOM : BLSH_ERR_CUDA, \
+                                std::string(#expr) + ": " + cudaGetErrorString(e__) + " @" + \
+                                __FILE__ + ":" + std::to_string(__LINE__));                  \
+    } while (0)
+
+#define BLSH_LAUNCH_CHECK() BLSH_CUDA(cudaGetLastError())
+
+// Device buffer owned by RAII.
+struct DevBuf {
+    void* p = nullptr;
+    size_t bytes = 0;
+    DevBuf() = default;
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+    ~DevBuf() { release(); }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+    }
+    void alloc(size_t b) {
+        release();
+        if (b == 0) b = 16;
+        BLSH_CUDA(cudaMalloc(&p, b));
+        bytes = b;
+    }
+    void ensure(size_t b) {   // grow-only, contents not preserved
+        if (b > bytes) alloc(b + b / 4);
+    }
+    template <typename T> T* as() const { return reinterpret_cast<T*>(p); }
+};
+
+// Bump allocator over a DevBuf (alignment 256 B).
+struct Arena {
+    char* base = nullptr;
+    size_t off = 0, cap = 0;
+    template <typename T> T* take(size_t count) {
+        size_t b = (count * sizeof(T) + 255) & ~size_t(255);
+        if (off + b > cap) throw Error(BLSH_ERR_INVALID, "internal arena overflow");
+        T* r = reinterpret_cast<T*>(base + off);
+        off += b;
+        return r;
+    }
+    static size_t need(size_t count, size_t elem) { return (count * elem + 255) & ~size_t(255); }
+};
+
+// Temp storage of the device scan.
+struct ScanTemp {
+    DevBuf blocks;
+};
+
+// ---- primitives (scan.cu, sort.cu) ------------------------------------------
+// out[i] = sum_{j<i} in[j] for i in [0, n]; out has n+1 entries.
+void scan_exclusive_i64(const int64_t* in, int64_t* out, int64_t n, ScanTemp& t, cudaStream_t s);
+void scan_exclusive_u8(const uint8_t* in, int64_t* out, int64_t n, ScanTemp& t, cudaStream_t s);
+
+struct SortBufs {
+    DevBuf hi[2], lo[2], leaf[2], id[2], hist, off, stats;
+    ScanTemp scan;
+};
+// Stable LSD radix sort of (leaf, hi, lo) with payload id; result in buffer index returned.
+int radix_sort_entries(SortBufs& b, int64_t n, cudaStream_t s, int* passes_done);
+
+// ---- index -----------------------------------------------------------------
+struct QueryWork {
+    DevBuf arena;      // per-call carve-outs
+    DevBuf partials;   // per-item partial top-k lists
+    DevBuf host_stage; // device staging for host outputs
+    ScanTemp scan;
+    int64_t nq = 0;
+    int T = 0, k = 0;
+    // carved pointers of the last call
+    float* Qd = nullptr;
+    int32_t* qleaf = nullptr;
+    float* qt = nullptr;
+    int32_t* qcode = nullptr;
+    int32_t* qoor = nullptr;
+    Key128* qkey = nullptr;
+    Key128* pkey = nullptr;
+    int32_t* pvalid = nullptr;
+    uint2* ivl = nullptr;      // [nq][T+1] (start, end)
+    int64_t* base = nullptr;
+    int64_t* cnt = nullptr;
+    int32_t* level = nullptr;
+    int64_t* item_off = nullptr;  // [nq+1]
+    int64_t* tau = nullptr;
+    int64_t* ncand_dev = nullptr;
+    int64_t* misc = nullptr;      // small scalars
+};
+
+}  // namespace blsh
+
+struct blsh_index {
+    // metadata
+    int64_t n = 0, n_owned = 0, nu = 0;
+    int d = 0, ds = 0, G = 1, M = 8, B = 16, quantizer = 0, depth = 0;
+    int leaf_lo = 0, leaf_hi = 1, rank = 0, world = 1;
+    int rp_rule = 0, ek_iters = 40;
+    double rp_mean_c = 10.0, rp_max_jitter = 0.0;
+    uint64_t seed = 0;
+    double build_ms = 0.0;
+    // host copies (export)
+    std::vector<float> A_h, b_h, W_h, dirs_h, mu_h, theta_h;
+    std::vector<int32_t> ntype_h;
+    std::vector<double> diam2_h, da2_h, jit_h;
+    std::vector<int64_t> leaf_u_h;     // [G+1]
+    // device: parameters and tree
+    blsh::DevBuf A, b, W, dirs, mu, theta, ntype;
+    // device: table
+    blsh::DevBuf Xp;      // [n_owned][ds] fp32 rows in table order
+    blsh::DevBuf perm;    // [n_owned] uint32 original ids
+    blsh::DevBuf ukey;    // [nu] Key128
+    blsh::DevBuf uleaf;   // [nu] int32
+    blsh::DevBuf uoff;    // [nu+1] uint32
+    blsh::DevBuf leaf_u;  // [G+1] int64
+    // kept build stages (keep_stages)
+    blsh::DevBuf pt_leaf, pt_code, pt_key;
+    bool has_pt = false;
+    // query state
+    mutable blsh::QueryWork qw;
+    mutable blsh_stats stats{};
+    mutable bool has_stages = false;
+    mutable cudaEvent_t ev[8] = {};
+};
+
+namespace blsh {
+
+// ---- build (rptree.cu, hash.cu, table.cu) --------------------------------------
+// Host-side generator (params.cpp), reading R2.
+void gen_params(uint64_t seed, int G, int M, int d, const float* Wleaf, float* A, float* b,
+                float* dirs, double* jit);
+
+// RP-tree over Xs [n][ds]; fills idx tree arrays; returns leaf segments of the
+// final order (order_out [n] uint32 ids grouped by leaf, ascending id) and
+// seg [G+1] (host).
+void build_rptree(blsh_index& ix, const float* Xs, uint32_t* order_dev,
+                  std::vector<int64_t>& seg, cudaStream_t s);
+
+// Hash the points order[lo..hi) (grouped by leaf) with their leaf's params;
+// writes sort entries; returns false when a code leaves the Morton range.
+bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order,
+                 const std::vector<int64_t>& seg, int64_t pos_lo, int64_t pos_hi,
+                 unsigned long long* key_hi, unsigned long long* key_lo, uint32_t* leaf,
+                 uint32_t* id, int32_t* code_out /* nullable [n][M] by id */,
+                 cudaStream_t s);
+
+// After sorting: buckets, offsets, permuted rows.
+void build_table(blsh_index& ix, const float* Xs, const unsigned long long* key_hi,
+                 const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
+                 int64_t n_owned, ScanTemp& scan, cudaStream_t s);
+
+// ---- query (query.cu, shortlist.cu) ----------------------------------------------
+void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
+               const blsh_query_params& p, int64_t* out_ids, float* out_d2,
+               unsigned long long* out_packed, int64_t* out_ncand, bool out_host);
+
+void merge_lists(const unsigned long long* packed, int n_lists, int64_t nq, int k,
+                 int64_t* out_ids, float* out_d2, cudaStream_t s);
+
+}  // namespace blsh

@@ -1,0 +1,478 @@
+// query.cu -- a1-a4 of the query hot path.
+//   k_route_hash   a1+a2: RP-tree routing + E2LSH projection (Eq. 2) /
+//                  E8 decode (Eq. 6) + Morton key; canonical fp32 (R1).
+//   k_probe_lookup a3+a4: probe sequence (standard, multiprobe P:247 / R11,
+//                  E8 lattice P:147 / R15) and binary search of every probe key
+//                  among the leaf's sorted bucket keys (R10); candidate
+//                  intervals of the position-sorted table + |A0|.
+//   k_median       tau = lower median of |A0| over the batch (R18).
+//   k_widen        Morton-prefix widening until |R| >= tau (Eq. 7-8, R17).
+#include "hashcore.cuh"
+#include "internal.cuh"
+#include "query_kernels.cuh"
+
+namespace blsh {
+
+__constant__ int8_t c_e8_roots[240][8];   // doubled coordinates, canonical order (R15)
+
+namespace {
+
+// ---------------------------------------------------------------------------
+// a1 + a2
+// ---------------------------------------------------------------------------
+template <int MM>
+__global__ void __launch_bounds__(128) k_route_hash(QueryArgs a) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= a.nq) return;
+    const float* x = a.Q + (size_t)q * a.ds;
+    const int d = a.d;
+    int v = 0;
+    for (int l = 0; l < a.depth; ++l) {
+        float s = 0.0f;
+        if (a.ntype[v] == 0) {
+            const float* dir = a.dirs + (size_t)v * a.ds;
+            for (int j = 0; j < d; ++j) s = __fmaf_rn(__ldg(dir + j), __ldg(x + j), s);
+        } else {
+            const float* mu = a.mu + (size_t)v * a.ds;
+            for (int j = 0; j < d; ++j) {
+                const float e = __fsub_rn(__ldg(x + j), __ldg(mu + j));
+                s = __fmaf_rn(e, e, s);
+            }
+        }
+        v = 2 * v + 1 + (s > a.theta[v] ? 1 : 0);
+    }
+    const int g = v - (a.G - 1);
+    a.qleaf[q] = g;
+    const bool active = g >= a.leaf_lo && g < a.leaf_hi;
+    float s[MM];
+#pragma unroll
+    for (int i = 0; i < MM; ++i) s[i] = 0.0f;
+    const float* Ag = a.A + (size_t)g * MM * d;
+    for (int j = 0; j < d; ++j) {
+        const float xj = __ldg(x + j);
+#pragma unroll
+        for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(__ldg(Ag + (size_t)i * d + j), xj, s[i]);
+    }
+    const float W = a.Wl[g];
+    float t[MM];
+#pragma unroll
+    for (int i = 0; i < MM; ++i) {
+        t[i] = __fdiv_rn(__fadd_rn(s[i], a.bvec[g * MM + i]), W);
+        a.qt[(size_t)q * MM + i] = t[i];
+    }
+    int32_t code[MM];
+    const bool ok = quantise(t, MM, a.B, a.quantizer, code);
+#pragma unroll
+    for (int i = 0; i < MM; ++i) a.qcode[(size_t)q * MM + i] = code[i];
+    a.qoor[q] = ok ? 0 : 1;
+    a.qkey[q] = morton_key(code, MM, a.B);   // clamped home key (hierarchy uses it)
+    if (!active) a.qoor[q] |= 2;
+}
+
+// ---------------------------------------------------------------------------
+// a3 + a4
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ int64_t find_bucket(const Key128* __restrict__ ukey, int64_t lo, int64_t hi,
+                                               const Key128& k) {
+    const int64_t end = hi;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        const Key128 m = ukey[mid];
+        if (key_lt(m, k)) lo = mid + 1;
+        else hi = mid;
+    }
+    if (lo < end && key_eq(ukey[lo], k)) return lo;
+    return -1;
+}
+
+constexpr int kPW = 4;          // warps per block in k_probe_lookup
+constexpr int kMaxSel = 256;    // max probes (T <= 256)
+
+struct ProbeSmem {
+    uint32_t hist[256];
+    unsigned long long sbits[kMaxSel];
+    uint32_t sx[kMaxSel];
+    uint32_t order[kMaxSel];
+};
+
+// Multiprobe pool (R11 + the pruning bound in DESIGN.md "Probe generation"):
+// per coordinate the admissible options among {-1, 0, +1}.
+struct MPPool {
+    int M;
+    uint32_t P;                 // pool size (mixed radix product)
+    uint32_t home;              // pool index of delta = 0
+    int nopt[10];
+    int8_t opt[10][3];
+    uint32_t stride[10];
+    double sq[10][2];           // [i][0] = x_i(-1)^2, [i][1] = x_i(+1)^2
+};
+
+__device__ __forceinline__ double mp_score(const MPPool& P, uint32_t x, int8_t* delta) {
+    double s = 0.0;
+    for (int i = 0; i < P.M; ++i) {
+        const uint32_t dg = (x / P.stride[i]) % (uint32_t)P.nopt[i];
+        const int8_t dv = P.opt[i][dg];
+        delta[i] = dv;
+        if (dv != 0) s = __dadd_rn(s, P.sq[i][dv > 0 ? 1 : 0]);
+    }
+    return s;
+}
+
+__device__ __forceinline__ double lat_score(const float* y, const int32_t* c2, uint32_t r) {
+    int32_t p[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) p[j] = c2[j] + (int32_t)c_e8_roots[r][j];
+    return e8_dist2(y, p);
+}
+
+// Select the R smallest (score, pool index) of a pool with an exact warp radix
+// select over the fp64 score bits (scores >= 0: bit order == value order).
+// Writes the selection sorted by (score, index) into sm.sx[0..R).
+template <typename ScoreFn>
+__device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, ScoreFn score) {
+    const int lane = threadIdx.x & 31;
+    unsigned long long prefix = 0ull, mask = 0ull;
+    int r = R - 1;
+    for (int sh = 56; sh >= 0; sh -= 8) {
+        for (int i = lane; i < 256; i += 32) sm.hist[i] = 0;
+        __syncwarp();
+        for (uint32_t x = lane; x < P; x += 32) {
+            if (x == skip) continue;
+            const unsigned long long b = (unsigned long long)__double_as_longlong(score(x));
+            if ((b & mask) == prefix) atomicAdd(&sm.hist[(b >> sh) & 255ull], 1u);
+        }
+        __syncwarp();
+        uint32_t loc[8], tot = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) { loc[i] = sm.hist[lane * 8 + i]; tot += loc[i]; }
+        uint32_t inc = tot;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+            if (lane >= o) inc += y;
+        }
+        const uint32_t ex = inc - tot;
+        const bool mine = (uint32_t)r >= ex && (uint32_t)r < inc;
+        const unsigned who = __ballot_sync(BLSH_FULL, mine);
+        const int src = __ffs(who) - 1;
+        int dg = 0, nr = 0;
+        if (mine) {
+            uint32_t c = ex;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                if ((uint32_t)r < c + loc[i]) { dg = lane * 8 + i; nr = r - (int)c; break; }
+                c += loc[i];
+            }
+        }
+        dg = __shfl_sync(BLSH_FULL, dg, src);
+        r = __shfl_sync(BLSH_FULL, nr, src);
+        prefix |= (unsigned long long)dg << sh;
+        mask |= 255ull << sh;
+        __syncwarp();
+    }
+    // prefix = score bits of the R-th smallest; take all smaller plus the first r+1 ties (ascending index)
+    int cnt = 0, ties = 0;
+    for (uint32_t base = 0; base < P; base += 32) {
+        const uint32_t x = base + lane;
+        unsigned long long b = ~0ull;
+        if (x < P && x != skip) b = (unsigned long long)__double_as_longlong(score(x));
+        const bool tie = b == prefix;
+        const unsigned tm = __ballot_sync(BLSH_FULL, tie);
+        const int my_tie = ties + __popc(tm & lanemask_lt());
+        ties += __popc(tm);
+        const bool sel = b < prefix || (tie && my_tie <= r);
+        const unsigned smk = __ballot_sync(BLSH_FULL, sel);
+        if (sel) {
+            const int at = cnt + __popc(smk & lanemask_lt());
+            sm.sbits[at] = b;
+            sm.sx[at] = x;
+        }
+        cnt += __popc(smk);
+    }
+    __syncwarp();
+    // sort the R selected entries by (score bits, index): rank by counting
+    for (int e = lane; e < R; e += 32) {
+        const unsigned long long b = sm.sbits[e];
+        const uint32_t x = sm.sx[e];
+        int rk = 0;
+        for (int f = 0; f < R; ++f) {
+            const unsigned long long bf = sm.sbits[f];
+            rk += (bf < b || (bf == b && sm.sx[f] < x)) ? 1 : 0;
+        }
+        sm.order[rk] = x;
+    }
+    __syncwarp();
+}
+
+__global__ void __launch_bounds__(kPW * 32) k_probe_lookup(QueryArgs a) {
+    __shared__ ProbeSmem smem[kPW];
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    const int64_t q = blockIdx.x * (int64_t)kPW + w;
+    if (q >= a.nq) return;
+    ProbeSmem& sm = smem[w];
+    const int T = a.T, M = a.M;
+    const int oor = a.qoor[q];
+    uint2* ivl = a.ivl + (size_t)q * (T + 1);
+    if (oor & 2) {   // leaf not owned by this shard
+        for (int p = lane; p <= T; p += 32) ivl[p] = make_uint2(0, 0);
+        if (a.pkey)
+            for (int p = lane; p < T; p += 32) { a.pkey[(size_t)q * T + p] = Key128{0, 0}; a.pvalid[(size_t)q * T + p] = 0; }
+        if (lane == 0) { a.base[q] = 0; a.cnt[q] = 0; if (a.level) a.level[q] = 0; }
+        return;
+    }
+    const int g = a.qleaf[q];
+    const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
+    const float* t = a.qt + (size_t)q * M;
+    const int32_t* code = a.qcode + (size_t)q * M;
+    const int B = a.B;
+    MPPool pool;
+    if (a.probe == 1 && T > 1) {
+        // pruned pool of perturbations
+        pool.M = M;
+        double v[20];
+        for (int i = 0; i < M; ++i) {
+            const float xm = __fsub_rn(t[i], floorf(t[i]));
+            const float xp = __fsub_rn(1.0f, xm);
+            pool.sq[i][0] = (double)xm * (double)xm;
+            pool.sq[i][1] = (double)xp * (double)xp;
+            v[2 * i] = pool.sq[i][0];
+            v[2 * i + 1] = pool.sq[i][1];
+        }
+        // smallest J terms (ascending value, ties by index) until the valid subsets number >= T-1
+        int used[10];
+        for (int i = 0; i < M; ++i) used[i] = 0;
+        unsigned long long taken = 0ull;
+        double Bsum = 0.0;
+        for (int J = 0; J < 2 * M; ++J) {
+            int jb = -1;
+            for (int j = 0; j < 2 * M; ++j)
+                if (!((taken >> j) & 1ull) && (jb < 0 || v[j] < v[jb])) jb = j;
+            taken |= 1ull << jb;
+            used[jb >> 1] += 1;
+            Bsum = __dadd_rn(Bsum, v[jb]);
+            double prod = 1.0;
+            for (int i = 0; i < M; ++i) prod *= (double)(1 + used[i]);
+            if (prod - 1.0 >= (double)(T - 1)) break;
+        }
+        const double Bp = __dmul_ru(Bsum, 1.0 + 0x1p-40);
+        uint32_t P = 1;
+        for (int i = M - 1; i >= 0; --i) {
+            int n = 0;
+            if (pool.sq[i][0] <= Bp) pool.opt[i][n++] = -1;
+            pool.opt[i][n++] = 0;
+            if (pool.sq[i][1] <= Bp) pool.opt[i][n++] = 1;
+            pool.nopt[i] = n;
+            pool.stride[i] = P;
+            P *= (uint32_t)n;
+        }
+        pool.P = P;
+        uint32_t home = 0;
+        for (int i = 0; i < M; ++i) {
+            const int zi = pool.opt[i][0] == 0 ? 0 : 1;
+            home += (uint32_t)zi * pool.stride[i];
+        }
+        pool.home = home;
+        warp_select(sm, P, home, T - 1, [&](uint32_t x) {
+            int8_t dl[10];
+            return mp_score(pool, x, dl);
+        });
+    } else if (a.probe == 2 && T > 1) {
+        if (!(oor & 1)) {
+            warp_select(sm, 240u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat_score(t, code, x); });
+        }
+    }
+    // keys + binary search, one probe per lane
+    int64_t mysum = 0;
+    for (int p = lane; p < T; p += 32) {
+        int32_t pc[16];
+        bool valid = true;
+        if (a.quantizer == 0) {
+            int8_t dl[10];
+            if (p > 0) mp_score(pool, sm.order[p - 1], dl);
+            const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
+            for (int i = 0; i < M; ++i) {
+                const float f = __fadd_rn(floorf(t[i]), p == 0 ? 0.0f : (float)dl[i]);
+                if (!(f >= lo && f <= hi)) valid = false;
+                else pc[i] = (int32_t)f;
+            }
+        } else {
+            valid = !(oor & 1);
+            const uint32_t r = (p > 0 && valid) ? sm.order[p - 1] : 0u;
+            for (int i = 0; i < 8; ++i) pc[i] = code[i] + (p > 0 ? (int32_t)c_e8_roots[r][i] : 0);
+            const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
+            if (valid)
+                for (int i = 0; i < 8; ++i)
+                    if (pc[i] < lo || pc[i] > hi) valid = false;
+        }
+        Key128 k{0, 0};
+        uint2 iv = make_uint2(0, 0);
+        if (valid) {
+            k = morton_key(pc, M, B);
+            const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
+            if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
+        }
+        ivl[p] = iv;
+        mysum += (int64_t)(iv.y - iv.x);
+        if (a.pkey) {
+            a.pkey[(size_t)q * T + p] = k;
+            a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
+        }
+    }
+    if (lane == 0) ivl[T] = make_uint2(0, 0);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mysum += __shfl_xor_sync(BLSH_FULL, mysum, o);
+    if (lane == 0) {
+        a.base[q] = mysum;
+        a.cnt[q] = mysum;
+        if (a.level) a.level[q] = 0;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// tau = lower median of |A0| over the batch (single block radix select).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) k_median(const int64_t* __restrict__ base, int64_t nq, int64_t* __restrict__ tau) {
+    __shared__ uint32_t h[256];
+    __shared__ unsigned long long s_prefix;
+    __shared__ int64_t s_rank;
+    if (threadIdx.x == 0) { s_prefix = 0; s_rank = (nq - 1) / 2; }
+    unsigned long long mask = 0ull;
+    for (int sh = 56; sh >= 0; sh -= 8) {
+        if (threadIdx.x < 256) h[threadIdx.x] = 0;
+        __syncthreads();
+        const unsigned long long pre = s_prefix;
+        for (int64_t i = threadIdx.x; i < nq; i += blockDim.x) {
+            const unsigned long long v = (unsigned long long)base[i];
+            if ((v & mask) == pre) atomicAdd(&h[(v >> sh) & 255ull], 1u);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int64_t r = s_rank, c = 0;
+            for (int dg = 0; dg < 256; ++dg) {
+                if (r < c + (int64_t)h[dg]) { s_prefix = pre | ((unsigned long long)dg << sh); s_rank = r - c; break; }
+                c += h[dg];
+            }
+        }
+        mask |= 255ull << sh;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *tau = nq > 0 ? (int64_t)s_prefix : 0;
+}
+
+__device__ __forceinline__ int64_t lower_key(const Key128* __restrict__ ukey, int64_t lo, int64_t hi, const Key128& k) {
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (key_lt(ukey[mid], k)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+__device__ __forceinline__ int64_t upper_key(const Key128* __restrict__ ukey, int64_t lo, int64_t hi, const Key128& k) {
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (key_le(ukey[mid], k)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+__global__ void k_widen(QueryArgs a, const int64_t* __restrict__ tau_p, int64_t min_cand) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= a.nq) return;
+    const int64_t tau = min_cand > 0 ? min_cand : *tau_p;
+    if ((a.qoor[q] & 2) || a.base[q] >= tau) return;
+    const int g = a.qleaf[q];
+    const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
+    const int BM = a.B * a.M;
+    const Key128 k0 = a.qkey[q];
+    int cb = 0;
+    int64_t s = 0, e = 0;
+    for (int l = 1;; ++l) {
+        cb = min(l * a.hstep, BM);
+        Key128 lo = k0, hi = k0;
+        if (cb >= 128) { lo = Key128{0, 0}; hi = Key128{~0ull, ~0ull}; }
+        else if (cb >= 64) {
+            const unsigned long long mh = cb == 64 ? 0ull : ((1ull << (cb - 64)) - 1ull);
+            lo = Key128{k0.hi & ~mh, 0ull};
+            hi = Key128{lo.hi | mh, ~0ull};
+        } else {
+            const unsigned long long ml = (1ull << cb) - 1ull;
+            lo = Key128{k0.hi, k0.lo & ~ml};
+            hi = Key128{k0.hi, lo.lo | ml};
+        }
+        const int64_t ua = lower_key(a.ukey, ulo, uhi, lo);
+        const int64_t ub = upper_key(a.ukey, ua, uhi, hi);
+        s = ua < ub ? (int64_t)a.uoff[ua] : 0;
+        e = ua < ub ? (int64_t)a.uoff[ub] : 0;
+        if (e - s >= tau || cb == BM) break;
+    }
+    uint2* ivl = a.ivl + (size_t)q * (a.T + 1);
+    int64_t c = a.base[q];
+    for (int p = 0; p < a.T; ++p) {
+        const uint2 iv = ivl[p];
+        if (iv.y > iv.x && (int64_t)iv.x >= s && (int64_t)iv.y <= e) {
+            c -= (int64_t)(iv.y - iv.x);
+            ivl[p] = make_uint2(0, 0);
+        }
+    }
+    ivl[a.T] = make_uint2((uint32_t)s, (uint32_t)e);
+    a.cnt[q] = c + (e - s);
+    if (a.level) a.level[q] = cb;
+}
+
+}  // namespace
+
+void upload_e8_roots() {
+    static bool done = false;   // per process; roots are a constant table of this library
+    if (done) return;
+    int8_t roots[240][8] = {};
+    int r = 0;
+    for (int i = 0; i < 8; ++i)
+        for (int j = i + 1; j < 8; ++j)
+            for (int si = 0; si < 2; ++si)
+                for (int sj = 0; sj < 2; ++sj) {
+                    roots[r][i] = si ? -2 : 2;
+                    roots[r][j] = sj ? -2 : 2;
+                    ++r;
+                }
+    for (int mask = 0; mask < 256; ++mask) {
+        if (__builtin_popcount(mask) & 1) continue;
+        for (int j = 0; j < 8; ++j) roots[r][j] = ((mask >> j) & 1) ? -1 : 1;
+        ++r;
+    }
+    BLSH_CUDA(cudaMemcpyToSymbol(c_e8_roots, roots, sizeof(roots)));
+    done = true;
+}
+
+void launch_route_hash(const QueryArgs& a, cudaStream_t s) {
+    const unsigned grid = (unsigned)((a.nq + 127) / 128);
+#define BLSH_RH_CASE(MMV) \
+    case MMV: k_route_hash<MMV><<<grid, 128, 0, s>>>(a); break;
+    switch (a.M) {
+        BLSH_RH_CASE(1) BLSH_RH_CASE(2) BLSH_RH_CASE(3) BLSH_RH_CASE(4)
+        BLSH_RH_CASE(5) BLSH_RH_CASE(6) BLSH_RH_CASE(7) BLSH_RH_CASE(8)
+        BLSH_RH_CASE(9) BLSH_RH_CASE(10) BLSH_RH_CASE(11) BLSH_RH_CASE(12)
+        BLSH_RH_CASE(13) BLSH_RH_CASE(14) BLSH_RH_CASE(15) BLSH_RH_CASE(16)
+        default: throw Error(BLSH_ERR_INVALID, "M out of range");
+    }
+#undef BLSH_RH_CASE
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_probe_lookup(const QueryArgs& a, cudaStream_t s) {
+    k_probe_lookup<<<(unsigned)((a.nq + kPW - 1) / kPW), kPW * 32, 0, s>>>(a);
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_median(const int64_t* base, int64_t nq, int64_t* tau, cudaStream_t s) {
+    k_median<<<1, 1024, 0, s>>>(base, nq, tau);
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_widen(const QueryArgs& a, const int64_t* tau, int64_t min_cand, cudaStream_t s) {
+    k_widen<<<(unsigned)((a.nq + 127) / 128), 128, 0, s>>>(a, tau, min_cand);
+    BLSH_LAUNCH_CHECK();
+}
+
+}  // namespace blsh
