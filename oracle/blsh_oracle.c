@@ -383,19 +383,27 @@ typedef struct {
     int64_t *lq_cand;     /* sorted candidate ids */
 } orc_index;
 
-static void orc_chunked_sum_ids(const float *X, int d, const int64_t *ids, int64_t n, int j,
-                                double *out)
+static void orc_chunked_colsum(const float *X, int d, const int64_t *ids, int64_t n, double *tot)
 {
-    /* R7: ordered fp64 reduction; chunks of 4096 members (ascending id),
-     * each summed sequentially, chunk sums added in chunk order. */
-    double tot = 0.0;
-    for (int64_t c = 0; c < n; c += 4096) {
-        double p = 0.0;
-        int64_t e = c + 4096 < n ? c + 4096 : n;
-        for (int64_t i = c; i < e; i++) p += (double)X[ids[i] * (int64_t)d + j];
-        tot += p;
+    /* R7: ordered fp64 reduction per coordinate j; chunks of 4096 members
+     * (ascending id), each summed sequentially, chunk sums added in chunk
+     * order.  All coordinates are walked together row by row (the sequence
+     * of additions of every single coordinate is unchanged). */
+    int64_t nc = (n + 4095) / 4096;
+    double *part = (double *)calloc((size_t)(nc > 0 ? nc : 1) * d, sizeof(double));
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t c = 0; c < nc; c++) {
+        double *p = part + (size_t)c * d;
+        int64_t e = (c + 1) * 4096 < n ? (c + 1) * 4096 : n;
+        for (int64_t i = c * 4096; i < e; i++) {
+            const float *x = X + ids[i] * (int64_t)d;
+            for (int j = 0; j < d; j++) p[j] += (double)x[j];
+        }
     }
-    *out = tot;
+    for (int j = 0; j < d; j++) tot[j] = 0.0;
+    for (int64_t c = 0; c < nc; c++)
+        for (int j = 0; j < d; j++) tot[j] += part[(size_t)c * d + j];
+    free(part);
 }
 
 static double orc_chunked_sum_vals(const float *v, int64_t n)
@@ -474,11 +482,10 @@ static void orc_split_node(orc_index *ix, int v, const int64_t *S, int64_t nS, f
     if (ix->rp_rule == 0) {
         /* RP-tree mean: mean, average squared interpoint distance
          * Delta_A^2 = (2/|S|) sum |x - mu|^2, approximate diameter Delta. */
-        for (int j = 0; j < d; j++) {
-            double tot;
-            orc_chunked_sum_ids(X, d, S, nS, j, &tot);
-            mu[j] = (float)(tot / (double)nS);
-        }
+        double *tot = (double *)malloc(sizeof(double) * (size_t)d);
+        orc_chunked_colsum(X, d, S, nS, tot);
+        for (int j = 0; j < d; j++) mu[j] = (float)(tot[j] / (double)nS);
+        free(tot);
         float *e = (float *)malloc(sizeof(float) * (size_t)nS);
         #pragma omp parallel for schedule(static)
         for (int64_t i = 0; i < nS; i++) e[i] = orc_dist2c(X + S[i] * (int64_t)d, mu, d);

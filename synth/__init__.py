@@ -78,7 +78,7 @@ CONFIGS = {
                  between=0.05, backend="torch", seed_data=1003, seed_query=2003,
                  notes="BASELINE configs[2]: Tiny-Images-shaped, multiprobe + Morton hierarchy"),
     "c4": Config("c4", n=10_000_000, d=384, n_clusters=1024, spread=0.02, rank=16,
-                 nq=100_000, k=10, G=64, M=8, W=1.2, probe=1, T=16, backend="torch",
+                 nq=100_000, k=10, G=64, M=8, W=1.65, probe=1, T=32, backend="torch",
                  seed_data=1004, seed_query=2004,
                  notes="BASELINE configs[3]: 10M x 384 sharded by subgroup, NCCL top-k merge"),
     "c5": Config("c5", n=1_000_000, d=384, n_clusters=256, spread=0.02, rank=16, nq=100_000,

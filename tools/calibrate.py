@@ -1,0 +1,116 @@
+"""Calibration sweep.
+
+For a configuration: r10 = median exact 10-NN distance over a query sample,
+then for W in r10 * {2, 2.83, 4, 5.66, 8} and T in a probe list: recall@10,
+selectivity, leaf ceiling and full-batch QPS of the CUDA path.  Exact k-NN for
+*calibration only* is computed with plain torch on the GPU (fp32); reported
+recall in bench.py comes from the oracle's fp64 ground truth.
+
+    python tools/calibrate.py --config c4 [--sample 1000] [--probes 1,4,8,16,32,64]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+from paper_conf_icde_panm12_b200 import blsh  # noqa: E402
+
+
+def exact_knn_torch(X, Qs, k=10, chunk=4096):
+    """fp32 exact k-NN (calibration helper only): ||q||^2 + ||x||^2 - 2 q.x, re-ranked in fp64."""
+    xn = (X * X).sum(1)
+    best_d, best_i = None, None
+    for s in range(0, X.shape[0], 1 << 20):
+        Xc = X[s:s + (1 << 20)]
+        d = (Qs * Qs).sum(1, keepdim=True) + xn[s:s + (1 << 20)][None, :] - 2.0 * Qs @ Xc.T
+        v, i = torch.topk(d, min(4 * k, d.shape[1]), dim=1, largest=False)
+        i = i + s
+        if best_d is None:
+            best_d, best_i = v, i
+        else:
+            cd = torch.cat([best_d, v], 1)
+            ci = torch.cat([best_i, i], 1)
+            vv, o = torch.topk(cd, 4 * k, dim=1, largest=False)
+            best_d, best_i = vv, torch.gather(ci, 1, o)
+    # exact fp64 re-rank of the shortlist
+    cand = X[best_i].double()
+    dd = ((cand - Qs.double()[:, None, :]) ** 2).sum(-1)
+    o = torch.argsort(dd, dim=1)[:, :k]
+    return torch.gather(best_i, 1, o), torch.gather(dd, 1, o)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="c4")
+    ap.add_argument("--sample", type=int, default=1000)
+    ap.add_argument("--probes", default="1,4,8,16,32,64")
+    ap.add_argument("--wmult", default="2,2.83,4,5.66,8")
+    ap.add_argument("--lattice", action="store_true")
+    ap.add_argument("--hier", action="store_true", help="Morton hierarchy with tau = batch median")
+    ap.add_argument("--out", default=None)
+    a = ap.parse_args()
+    cfg = synth.CONFIGS[a.config]
+    t0 = time.time()
+    X, Q = synth.make_dataset(cfg, backend="torch", device="cuda:0")
+    torch.cuda.synchronize()
+    print(f"data {tuple(X.shape)} queries {tuple(Q.shape)} in {time.time() - t0:.1f}s", flush=True)
+    rng = np.random.default_rng(0)
+    sidx = torch.as_tensor(np.sort(rng.choice(Q.shape[0], min(a.sample, Q.shape[0]), replace=False)), device="cuda")
+    Qs = Q[sidx].contiguous()
+    gi, gd = exact_knn_torch(X, Qs, 10)
+    r10 = float(torch.median(gd[:, 9].sqrt()))
+    print(f"r10 = {r10:.4f}", flush=True)
+    rows = []
+    for wm in [float(w) for w in a.wmult.split(",")]:
+        W = wm * r10
+        t1 = time.time()
+        ix = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=W, seed=cfg.seed_index, keep_stages=True,
+                             quantizer=1 if a.lattice else 0)
+        torch.cuda.synchronize()
+        bt = time.time() - t1
+        pleaf = torch.as_tensor(ix.export("POINT_LEAF"), device="cuda").long()
+        for T in [int(t) for t in a.probes.split(",")]:
+            probe = (2 if a.lattice else 1) if T > 1 else 0
+            hk = dict(hierarchy=1) if a.hier else {}
+            ids, d2, nc = ix.query(Qs, 10, probe=probe, n_probes=T, keep_stages=True, **hk)
+            qleaf = torch.as_tensor(ix.export("Q_LEAF"), device="cuda").long()
+            ceiling = float((pleaf[gi] == qleaf[:, None]).float().mean())
+            hit = (ids[:, :, None] == gi[:, None, :]).any(-1).float().mean()
+            sel = float(nc.double().mean() / X.shape[0])
+            # full batch timing
+            for _ in range(2):
+                ix.query(Q, cfg.k, probe=probe, n_probes=T, **hk)
+            torch.cuda.synchronize()
+            t2 = time.time()
+            ix.query(Q, cfg.k, probe=probe, n_probes=T, timing=True, **hk)
+            torch.cuda.synchronize()
+            dt = time.time() - t2
+            st = ix.stats()
+            row = dict(W_mult=wm, W=W, T=T, recall10=float(hit), selectivity=sel, ceiling=ceiling,
+                       qps=Q.shape[0] / dt, ms=dt * 1e3, sl_ms=st.ms_shortlist, probe_ms=st.ms_probe,
+                       mean_cand=float(st.total_cand) / Q.shape[0], build_s=bt,
+                       sl_gbs=st.shortlist_bytes / (st.ms_shortlist * 1e-3) / 1e9 if st.ms_shortlist > 0 else 0)
+            rows.append(row)
+            print(json.dumps(row), flush=True)
+        ix.close()
+    ok = [r for r in rows if r["recall10"] >= 0.9]
+    if ok:
+        best = max(ok, key=lambda r: r["qps"])
+        print("BEST", json.dumps(best))
+    if a.out:
+        with open(a.out, "w") as f:
+            json.dump(dict(config=a.config, r10=r10, rows=rows), f, indent=1)
+
+
+if __name__ == "__main__":
+    main()
