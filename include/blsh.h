@@ -162,9 +162,14 @@ blsh_status blsh_index_info(const blsh_index* idx, blsh_info* out);
 /* Statistics of the last blsh_query / blsh_query_packed on this index. */
 typedef struct {
     int64_t nq, n_active, total_cand, n_items, tau;
-    int32_t chunk, launches;          /* candidates per work item; kernels launched by the call */
+    int32_t chunk, launches;          /* candidates (rows) per work item; kernels launched by the call */
     double  shortlist_bytes;          /* algorithmic bytes of the short-list: sum|A(q)|*d*4 + 4/candidate + outputs */
     float   ms_route_hash, ms_probe, ms_plan, ms_shortlist, ms_merge, ms_total;  /* timing = 1 */
+    int32_t tiled;                    /* 1 = query-tiled short-list (rows shared across a tile of 32 queries) */
+    int32_t pad_;
+    int64_t union_rows;               /* tiled: rows streamed from HBM (sum over tiles of the candidate union) */
+    int64_t pairs_scored;             /* (row, query) distance evaluations actually performed */
+    double  shortlist_flops;          /* algorithmic flops: 3*d per (query, candidate) pair */
 } blsh_stats;
 
 blsh_status blsh_last_stats(const blsh_index* idx, blsh_stats* out);

@@ -267,6 +267,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     add(nq + 1, 8); add(nq + 1, 8);     // items, item_off
     add(nq + 1, 8);                     // cand_off
     add(4, 8);                          // tau + misc
+    add(nq, 4);                         // qorder
     if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
     if (out_host) { add((size_t)nq * k, 8); add((size_t)nq * k, 4); add(nq, 8); add((size_t)nq * k, 8); }
     w.arena.ensure(need);
@@ -285,6 +286,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     w.item_off = ar.take<int64_t>(nq + 1);
     int64_t* cand_off = ar.take<int64_t>(nq + 1);
     w.tau = ar.take<int64_t>(4);
+    uint32_t* qorder = ar.take<uint32_t>(nq);
     w.pkey = keep ? ar.take<Key128>((size_t)nq * T) : nullptr;
     w.pvalid = keep ? ar.take<int32_t>((size_t)nq * T) : nullptr;
     int64_t* d_ids = out_ids;
@@ -334,25 +336,40 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t total = 0;
     BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    const int64_t target = 148 * 8 * 4;
-    int64_t ch = (total + target - 1) / std::max<int64_t>(target, 1);
-    ch = std::min<int64_t>(4096, std::max<int64_t>(256, (ch + 31) / 32 * 32));
-    launch_items(w.cnt, nq, (int)ch, items, s); ++launches;
-    scan_exclusive_i64(items, w.item_off, nq, w.scan, s); launches += 3;
-    int64_t n_items = 0;
-    BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    BLSH_CUDA(cudaStreamSynchronize(s));
-    w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
-    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[4], s));
-    // a5
-    ShortlistArgs sa{};
-    sa.nq = nq; sa.n_items = n_items; sa.d = ix.d; sa.ds = ds; sa.T = T; sa.k = k; sa.chunk = (int)ch;
-    sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
-    sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
-    launch_shortlist(sa, s); if (n_items) ++launches;
-    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
-    launch_merge(sa, w.qoor, d_ids, d_d2, d_pk, d_nc, s); ++launches;
-    if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
+    const char* mode = std::getenv("BLSH_SHORTLIST");
+    const bool tiled = tiled_supported(ds, T) && !(mode && std::strcmp(mode, "warp") == 0);
+    int64_t n_items = 0, union_rows = 0, pairs = total;
+    int64_t ch = 0;
+    if (tiled) {
+        // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
+        sort_queries(a, w.qsort, qorder, s, &launches);
+        int chr = 0;
+        run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
+                            ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
+                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs);
+        ch = chr;
+        if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
+    } else {
+        const int64_t target = 148 * 8 * 4;
+        ch = (total + target - 1) / std::max<int64_t>(target, 1);
+        ch = std::min<int64_t>(4096, std::max<int64_t>(256, (ch + 31) / 32 * 32));
+        launch_items(w.cnt, nq, (int)ch, items, s); ++launches;
+        scan_exclusive_i64(items, w.item_off, nq, w.scan, s); launches += 3;
+        BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
+        if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[4], s));
+        // a5, one warp per (query, chunk)
+        ShortlistArgs sa{};
+        sa.nq = nq; sa.n_items = n_items; sa.d = ix.d; sa.ds = ds; sa.T = T; sa.k = k; sa.chunk = (int)ch;
+        sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
+        sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
+        launch_shortlist(sa, s); if (n_items) ++launches;
+        if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
+        launch_merge(sa, w.qoor, d_ids, d_d2, d_pk, d_nc, s); ++launches;
+        if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
+        union_rows = total;
+    }
     if (out_host) {
         if (out_ids) BLSH_CUDA(cudaMemcpyAsync(out_ids, d_ids, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
         if (out_d2) BLSH_CUDA(cudaMemcpyAsync(out_d2, d_d2, (size_t)nq * k * 4, cudaMemcpyDeviceToHost, s));
@@ -366,6 +383,10 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     stt.chunk = (int32_t)ch;
     stt.launches = launches;
     stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 + (double)n_items * k * 8.0;
+    stt.tiled = tiled ? 1 : 0;
+    stt.union_rows = union_rows;
+    stt.pairs_scored = pairs;
+    stt.shortlist_flops = 3.0 * ix.d * (double)total;
     if (p.hierarchy) {
         int64_t tau = p.min_cand;
         if (p.min_cand == 0) BLSH_CUDA(cudaMemcpy(&tau, w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost));

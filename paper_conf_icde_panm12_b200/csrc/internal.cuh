@@ -91,6 +91,8 @@ struct QueryWork {
     DevBuf arena;      // per-call carve-outs
     DevBuf partials;   // per-item partial top-k lists
     DevBuf host_stage; // device staging for host outputs
+    DevBuf segbuf, tilebuf;   // tiled short-list: per-tile segments, tile arrays
+    SortBufs qsort;           // query sort by (leaf, key)
     ScanTemp scan;
     int64_t nq = 0;
     int T = 0, k = 0;

@@ -2,6 +2,7 @@
 #pragma once
 
 #include "common.cuh"
+#include "internal.cuh"
 
 namespace blsh {
 
@@ -55,6 +56,15 @@ struct ShortlistArgs {
     const int64_t* item_off; // [nq+1]
     unsigned long long* partials;   // [n_items][k]
 };
+
+// query-tiled short-list (shortlist_tiled.cu)
+bool tiled_supported(int ds, int T);
+void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
+void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
+                         DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
+                         unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
+                         cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out);
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s);
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s);

@@ -1,0 +1,540 @@
+// shortlist_tiled.cu -- a5 with cross-query reuse (the default short-list).
+//
+// Queries are sorted by their bi-level code (leaf, home Morton key), so
+// consecutive queries probe overlapping buckets.  A *tile* is QT = 32
+// consecutive queries.  k_tile_prep turns the tile's candidate intervals into
+// the sorted union of disjoint row segments, each with a 32-bit mask of the
+// tile queries whose A(q) contains it (interval boundaries -> sort -> XOR
+// toggles -> XOR prefix scan; a query's own intervals are disjoint).
+// k_shortlist_tiled streams that union once: rows are staged into shared
+// memory with 1-D TMA bulk copies (cp.async.bulk + mbarrier complete_tx,
+// double-buffered, 16-byte padded row pitch so one-row-per-lane reads are
+// bank-conflict free), and every warp scores the staged rows (one per lane)
+// against its 4 tile queries held in shared memory (broadcast reads).  A row
+// read from HBM once thus serves every query of the tile that needs it; the
+// per-(row, query) arithmetic is the same fp32 direct form as k_shortlist
+// (R22).  Each (work item, query) keeps a warp-register top-k; k_merge_tiled
+// merges the items of a tile per query.
+#include <algorithm>
+
+#include "internal.cuh"
+#include "query_kernels.cuh"
+
+namespace blsh {
+
+namespace {
+
+constexpr int QT = 32;            // queries per tile
+constexpr int kPrepThreads = 256;
+constexpr int kRows = 32;         // rows per stage (one per lane)
+constexpr int kTW = 8;            // warps per CTA (each owns 4 tile queries)
+
+struct Seg {
+    uint32_t start, len, mask, off;   // table rows [start, start+len), query mask, rows before it in the union
+};
+
+// ---------------------------------------------------------------------------
+// tile prep: union of the tile's candidate intervals, with query masks
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restrict__ ivl, int T,
+                                                            const uint32_t* __restrict__ qorder, int64_t nq,
+                                                            int segcap, Seg* __restrict__ segs,
+                                                            int32_t* __restrict__ nseg,
+                                                            int64_t* __restrict__ rows) {
+    extern __shared__ uint32_t sm[];
+    const int cap = 2 * QT * (T + 1);
+    int npow = 1;
+    while (npow < cap) npow <<= 1;
+    uint32_t* bnd = sm;             // [npow] boundaries (sorted, then unique)
+    uint32_t* tog = sm + npow;      // [npow] scratch -> toggles -> masks
+    uint32_t* pos = tog + npow;     // [npow] unique positions
+    __shared__ int s_cnt, s_nb;
+    const int t = blockIdx.x;
+    const int tid = threadIdx.x;
+    if (tid == 0) s_cnt = 0;
+    for (int i = tid; i < npow; i += kPrepThreads) bnd[i] = 0xFFFFFFFFu;
+    __syncthreads();
+    const int nint = QT * (T + 1);
+    for (int i = tid; i < nint; i += kPrepThreads) {
+        const int slot = i / (T + 1), p = i % (T + 1);
+        const int64_t qp = (int64_t)t * QT + slot;
+        if (qp >= nq) continue;
+        const uint2 iv = ivl[(size_t)qorder[qp] * (T + 1) + p];
+        if (iv.y > iv.x) {
+            const int at = atomicAdd(&s_cnt, 2);
+            bnd[at] = iv.x;
+            bnd[at + 1] = iv.y;
+        }
+    }
+    __syncthreads();
+    const int cnt = s_cnt;
+    if (cnt == 0) {
+        if (tid == 0) { nseg[t] = 0; rows[t] = 0; }
+        return;
+    }
+    int np2 = 1;
+    while (np2 < cnt) np2 <<= 1;
+    for (int k2 = 2; k2 <= np2; k2 <<= 1) {          // bitonic sort of bnd[0..np2)
+        for (int j = k2 >> 1; j > 0; j >>= 1) {
+            for (int i = tid; i < np2; i += kPrepThreads) {
+                const int ixj = i ^ j;
+                if (ixj > i) {
+                    const uint32_t a = bnd[i], b = bnd[ixj];
+                    if ((a > b) == ((i & k2) == 0)) { bnd[i] = b; bnd[ixj] = a; }
+                }
+            }
+            __syncthreads();
+        }
+    }
+    // unique boundaries (exclusive scan of first-occurrence flags by warp 0)
+    if (tid < 32) {
+        const int per = (cnt + 31) / 32;
+        const int lo = tid * per, hi = min(cnt, lo + per);
+        uint32_t c = 0;
+        for (int i = lo; i < hi; ++i) c += (i == 0 || bnd[i] != bnd[i - 1]) ? 1u : 0u;
+        uint32_t inc = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+            if (tid >= o) inc += y;
+        }
+        uint32_t run = inc - c;
+        for (int i = lo; i < hi; ++i) {
+            pos[i] = run;
+            run += (i == 0 || bnd[i] != bnd[i - 1]) ? 1u : 0u;
+        }
+        if (tid == 31) s_nb = (int)inc;
+    }
+    __syncthreads();
+    const int nb = s_nb;
+    for (int i = tid; i < cnt; i += kPrepThreads)
+        if (i == 0 || bnd[i] != bnd[i - 1]) tog[pos[i]] = bnd[i];
+    __syncthreads();
+    for (int i = tid; i < nb; i += kPrepThreads) bnd[i] = tog[i];
+    __syncthreads();
+    for (int i = tid; i < npow; i += kPrepThreads) tog[i] = 0u;
+    __syncthreads();
+    for (int i = tid; i < nint; i += kPrepThreads) {     // XOR toggles at both ends of every interval
+        const int slot = i / (T + 1), p = i % (T + 1);
+        const int64_t qp = (int64_t)t * QT + slot;
+        if (qp >= nq) continue;
+        const uint2 iv = ivl[(size_t)qorder[qp] * (T + 1) + p];
+        if (iv.y > iv.x) {
+            int lo = 0, hi = nb;
+            while (lo < hi) { const int m = (lo + hi) >> 1; if (bnd[m] < iv.x) lo = m + 1; else hi = m; }
+            const int is = lo;
+            hi = nb;
+            while (lo < hi) { const int m = (lo + hi) >> 1; if (bnd[m] < iv.y) lo = m + 1; else hi = m; }
+            atomicXor(&tog[is], 1u << slot);
+            atomicXor(&tog[lo], 1u << slot);
+        }
+    }
+    __syncthreads();
+    if (tid < 32) {                                        // inclusive XOR scan -> mask of [bnd[i], bnd[i+1])
+        const int per = (nb + 31) / 32;
+        const int lo = tid * per, hi = min(nb, lo + per);
+        uint32_t x = 0;
+        for (int i = lo; i < hi; ++i) x ^= tog[i];
+        uint32_t inc = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+            if (tid >= o) inc ^= y;
+        }
+        uint32_t run = inc ^ x;
+        for (int i = lo; i < hi; ++i) { run ^= tog[i]; tog[i] = run; }
+    }
+    __syncthreads();
+    if (tid < 32) {                                        // emit segments with a non-empty mask, in order
+        int out = 0;
+        uint32_t off = 0;
+        Seg* S = segs + (size_t)t * segcap;
+        for (int base = 0; base < nb - 1; base += 32) {
+            const int i = base + tid;
+            const bool v = i < nb - 1 && tog[i] != 0u;
+            const unsigned bm = __ballot_sync(BLSH_FULL, v);
+            const uint32_t len = v ? bnd[i + 1] - bnd[i] : 0u;
+            uint32_t inc = len;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+                if (tid >= o) inc += y;
+            }
+            if (v) S[out + __popc(bm & lanemask_lt())] = Seg{bnd[i], len, tog[i], off + inc - len};
+            off += __shfl_sync(BLSH_FULL, inc, 31);
+            out += __popc(bm);
+        }
+        if (tid == 0) { nseg[t] = out; rows[t] = off; }
+    }
+}
+
+__global__ void k_tile_items(const int64_t* __restrict__ rows, int64_t ntiles, int chr, int64_t* __restrict__ items) {
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t < ntiles) items[t] = (rows[t] + chr - 1) / chr;
+}
+
+// ---------------------------------------------------------------------------
+// TMA bulk copy + mbarrier
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+struct TiledArgs {
+    int64_t nq, ntiles, n_items;
+    int d, ds, k, chr, segcap;
+    const float* Q;
+    const float* Xp;
+    const uint32_t* perm;
+    const uint32_t* qorder;
+    const Seg* segs;
+    const int32_t* nseg;
+    const int64_t* rows;       // [ntiles] union rows per tile
+    const int64_t* item_off;   // [ntiles+1]
+    unsigned long long* partials;   // [n_items][QT][k]
+    unsigned long long* counters;   // [0] (row, query) pairs evaluated
+};
+
+struct TopK {
+    unsigned long long e0, e1;
+};
+
+__device__ __forceinline__ unsigned long long topk_thr(const TopK& t, int k) {
+    return __shfl_sync(BLSH_FULL, k <= 32 ? t.e0 : t.e1, (k - 1) & 31);
+}
+
+__device__ __forceinline__ void topk_insert(TopK& t, unsigned long long v, int lane) {
+    const int pos = __popc(__ballot_sync(BLSH_FULL, t.e0 < v)) + __popc(__ballot_sync(BLSH_FULL, t.e1 < v));
+    const unsigned long long up0 = __shfl_up_sync(BLSH_FULL, t.e0, 1);
+    unsigned long long up1 = __shfl_up_sync(BLSH_FULL, t.e1, 1);
+    const unsigned long long last0 = __shfl_sync(BLSH_FULL, t.e0, 31);
+    if (lane == 0) up1 = last0;
+    const int i1 = lane + 32;
+    t.e1 = i1 > pos ? up1 : (i1 == pos ? v : t.e1);
+    t.e0 = lane > pos ? up0 : (lane == pos ? v : t.e0);
+}
+
+// Offer one key per lane (kEmpty = none) to a warp top-k.
+__device__ __forceinline__ void topk_offer(TopK& tk, unsigned long long& thr, unsigned long long key, int k, int lane) {
+    unsigned m = __ballot_sync(BLSH_FULL, key < thr);
+    while (m) {
+        const int src = __ffs(m) - 1;
+        m &= m - 1;
+        const unsigned long long v = __shfl_sync(BLSH_FULL, key, src);
+        if (v < thr) {
+            topk_insert(tk, v, lane);
+            thr = topk_thr(tk, k);
+        }
+    }
+}
+
+#if 0   // superseded by tiled_kernel.cuh (kept until the next cleanup)
+__global__ void __launch_bounds__(kTW * 32, 1) k_shortlist_tiled_v1(TiledArgs a) {
+    extern __shared__ __align__(128) unsigned char smraw[];
+    const int nv4 = a.ds >> 2;
+    const int pitch = a.ds + 4;                              // floats per staged row
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smraw);      // [2]
+    uint32_t* rmask = reinterpret_cast<uint32_t*>(smraw + 16);   // [2][kRows]
+    uint32_t* rid = rmask + 2 * kRows;                            // [2][kRows]
+    int* nrows = reinterpret_cast<int*>(rid + 2 * kRows);         // [2]
+    float* qs = reinterpret_cast<float*>(smraw + 1024);           // [QT][ds]
+    float* rws = qs + (size_t)QT * a.ds;                          // [2][kRows][pitch]
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t item = blockIdx.x;
+    int64_t lo = 0, hi = a.ntiles;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (a.item_off[mid] <= item) lo = mid;
+        else hi = mid;
+    }
+    const int64_t tile = lo;
+    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
+    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    const Seg* S = a.segs + (size_t)tile * a.segcap;
+    const int ns = a.nseg[tile];
+    for (int i = threadIdx.x; i < QT * nv4; i += kTW * 32) {
+        const int slot = i / nv4, v = i % nv4;
+        const int64_t qp = tile * QT + slot;
+        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (qp < a.nq) x = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[qp] * a.ds)[v];
+        reinterpret_cast<float4*>(qs)[(size_t)slot * nv4 + v] = x;
+    }
+    if (threadIdx.x == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const uint32_t rowbytes = (uint32_t)a.ds * 4u;
+    // warp 0: stage rows [rs, rs + kRows) of the union into buffer st (one row per lane)
+    auto issue = [&](int st, int64_t rs) {
+        if (warp != 0) return;
+        const int64_t r = rs + lane;
+        const bool v = r < r1;
+        const int64_t left = r1 - rs;
+        const int n = left <= 0 ? 0 : (left < kRows ? (int)left : kRows);
+        uint32_t row = 0, msk = 0;
+        if (v) {
+            int l2 = 0, h2 = ns;                // last segment with off <= r
+            while (h2 - l2 > 1) {
+                const int m = (l2 + h2) >> 1;
+                if ((int64_t)S[m].off <= r) l2 = m;
+                else h2 = m;
+            }
+            const Seg sg = S[l2];
+            row = sg.start + (uint32_t)(r - sg.off);
+            msk = sg.mask;
+        }
+        rmask[st * kRows + lane] = msk;
+        rid[st * kRows + lane] = row;
+        if (lane == 0) nrows[st] = n;
+        if (n > 0) {
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&bar[st], (uint32_t)n * rowbytes);
+            }
+            __syncwarp();
+            if (v) bulk_g2s(rws + (size_t)(st * kRows + lane) * pitch, a.Xp + (size_t)row * a.ds, rowbytes, &bar[st]);
+        }
+        __syncwarp();
+    };
+    TopK tk[4];
+    unsigned long long thr[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { tk[j] = TopK{kEmpty, kEmpty}; thr[j] = kEmpty; }
+    const int k = a.k;
+    uint32_t phase0 = 0u, phase1 = 0u;
+    unsigned long long evaluated = 0ull;
+    int st = 0;
+    issue(0, r0);
+    __syncthreads();
+    int64_t rs = r0;
+    const float4* q4 = reinterpret_cast<const float4*>(qs) + (size_t)(warp * 4) * nv4;
+    while (true) {
+        const int n = nrows[st];
+        if (n == 0) break;
+        issue(st ^ 1, rs + n);                   // prefetch the next stage into the other buffer
+        mbar_wait(&bar[st], st ? phase1 : phase0);
+        if (st) phase1 ^= 1u; else phase0 ^= 1u;
+        const bool valid = lane < n;
+        const uint32_t msk = valid ? rmask[st * kRows + lane] : 0u;
+        const uint32_t prow = rid[st * kRows + lane];
+        const uint32_t myq = (msk >> (warp * 4)) & 15u;
+        const unsigned need = __ballot_sync(BLSH_FULL, myq != 0u);
+        if (need) {
+            evaluated += 4 * 32;
+            const uint32_t id = valid ? __ldg(a.perm + prow) : 0u;
+            const float4* xr = reinterpret_cast<const float4*>(rws + (size_t)(st * kRows + lane) * pitch);
+            // fp32 direct form in partial sums of <= 64 terms (16 float4), then summed (R22)
+            float tot[4] = {0.f, 0.f, 0.f, 0.f};
+            for (int vb = 0; vb < nv4; vb += 16) {
+                const int ve = min(nv4, vb + 16);
+                float acc[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll 4
+                for (int v = vb; v < ve; ++v) {
+                    const float4 x = xr[v];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const float4 q = q4[(size_t)j * nv4 + v];
+                        const float dx = q.x - x.x, dy = q.y - x.y, dz = q.z - x.z, dw = q.w - x.w;
+                        acc[j] = fmaf(dx, dx, acc[j]);
+                        acc[j] = fmaf(dy, dy, acc[j]);
+                        acc[j] = fmaf(dz, dz, acc[j]);
+                        acc[j] = fmaf(dw, dw, acc[j]);
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) tot[j] += acc[j];
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const bool mine = (myq >> j) & 1u;
+                const unsigned long long key = mine ? pack_entry(tot[j], id) : kEmpty;
+                topk_offer(tk[j], thr[j], key, k, lane);
+            }
+        }
+        __syncthreads();                          // buffer st fully consumed before it is refilled
+        rs += n;
+        st ^= 1;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        if (j == 0 && lane == 0 && a.counters) atomicAdd(a.counters, evaluated);
+        unsigned long long* out = a.partials + ((size_t)item * QT + warp * 4 + j) * k;
+        if (lane < k) out[lane] = tk[j].e0;
+        if (lane + 32 < k) out[lane + 32] = tk[j].e1;
+    }
+}
+
+#endif
+
+#include "tiled_kernel.cuh"
+
+__global__ void __launch_bounds__(256) k_merge_tiled(TiledArgs a, const int32_t* __restrict__ qoor,
+                                                     const int64_t* __restrict__ cnt, int64_t* out_ids, float* out_d2,
+                                                     unsigned long long* out_packed, int64_t* out_ncand) {
+    const int lane = threadIdx.x & 31;
+    const int64_t pos = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (pos >= a.nq) return;
+    const int64_t q = a.qorder[pos];
+    const int64_t tile = pos / QT;
+    const int slot = (int)(pos % QT);
+    const int k = a.k;
+    TopK tk{kEmpty, kEmpty};
+    unsigned long long thr = kEmpty;
+    for (int64_t it = a.item_off[tile]; it < a.item_off[tile + 1]; ++it) {
+        const unsigned long long* L = a.partials + ((size_t)it * QT + slot) * k;
+        const unsigned long long l0 = lane < k ? L[lane] : kEmpty;
+        const unsigned long long l1 = lane + 32 < k ? L[lane + 32] : kEmpty;
+        for (int j = 0; j < k; ++j) {
+            const unsigned long long v = __shfl_sync(BLSH_FULL, j < 32 ? l0 : l1, j & 31);
+            if (v >= thr) break;
+            topk_insert(tk, v, lane);
+            thr = topk_thr(tk, k);
+        }
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        const int i = lane + 32 * h;
+        if (i >= k) continue;
+        const unsigned long long e = h ? tk.e1 : tk.e0;
+        if (out_packed) out_packed[(size_t)q * k + i] = e == kEmpty ? kPadPacked : e;
+        if (out_ids) out_ids[(size_t)q * k + i] = e == kEmpty ? -1 : (int64_t)(uint32_t)(e & 0xFFFFFFFFull);
+        if (out_d2) out_d2[(size_t)q * k + i] = e == kEmpty ? __int_as_float(0x7F800000) : __uint_as_float((uint32_t)(e >> 32));
+    }
+    if (lane == 0 && out_ncand) out_ncand[q] = (qoor[q] & 2) ? 0 : cnt[q];
+}
+
+__global__ void k_qsort_keys(const Key128* __restrict__ qkey, const int32_t* __restrict__ qleaf,
+                             const int32_t* __restrict__ qoor, int64_t nq, unsigned long long* __restrict__ hi,
+                             unsigned long long* __restrict__ lo, uint32_t* __restrict__ leaf, uint32_t* __restrict__ id) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= nq) return;
+    const Key128 k = qkey[q];
+    hi[q] = k.hi;
+    lo[q] = k.lo;
+    leaf[q] = (qoor[q] & 2) ? 0xFFFFu : (uint32_t)qleaf[q];
+    id[q] = (uint32_t)q;
+}
+
+}  // namespace
+
+size_t tiled_smem_bytes(int ds) { return 1024 + (size_t)QT * ds * 4 + (size_t)kStages * 32 * (ds + 4) * 4; }
+
+bool tiled_supported(int ds, int T) {
+    int cap = 2 * QT * (T + 1), npow = 1;
+    while (npow < cap) npow <<= 1;
+    return tiled_smem_bytes(ds) <= 227 * 1024 && (size_t)3 * npow * 4 <= 227 * 1024;
+}
+
+// Sort the active queries by (leaf, home key): qorder[pos] = query.
+void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches) {
+    const int64_t nq = a.nq;
+    for (int i = 0; i < 2; ++i) {
+        sb.hi[i].ensure((size_t)nq * 8);
+        sb.lo[i].ensure((size_t)nq * 8);
+        sb.leaf[i].ensure((size_t)nq * 4);
+        sb.id[i].ensure((size_t)nq * 4);
+    }
+    k_qsort_keys<<<(unsigned)((nq + 255) / 256), 256, 0, s>>>(a.qkey, a.qleaf, a.qoor, nq,
+                                                               sb.hi[0].as<unsigned long long>(),
+                                                               sb.lo[0].as<unsigned long long>(),
+                                                               sb.leaf[0].as<uint32_t>(), sb.id[0].as<uint32_t>());
+    BLSH_LAUNCH_CHECK();
+    ++*launches;
+    int passes = 0;
+    const int cur = radix_sort_entries(sb, nq, s, &passes);
+    *launches += (nq > 1 ? 1 : 0) + passes * 5;
+    BLSH_CUDA(cudaMemcpyAsync(qorder, sb.id[cur].p, (size_t)nq * 4, cudaMemcpyDeviceToDevice, s));
+}
+
+void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
+                         DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
+                         unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
+                         cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out) {
+    const int64_t nq = a.nq;
+    const int64_t ntiles = (nq + QT - 1) / QT;
+    const int T = a.T;
+    const int segcap = 2 * QT * (T + 1);
+    segbuf.ensure((size_t)ntiles * segcap * sizeof(Seg));
+    const size_t slot = (((size_t)(ntiles + 1) * 8) + 255) & ~size_t(255);
+    tilebuf.ensure(slot * 5 + 256);
+    char* tb = tilebuf.as<char>();
+    unsigned long long* counters = reinterpret_cast<unsigned long long*>(tb + 5 * slot);
+    BLSH_CUDA(cudaMemsetAsync(counters, 0, 16, s));
+    int32_t* nseg = reinterpret_cast<int32_t*>(tb);
+    int64_t* rows = reinterpret_cast<int64_t*>(tb + slot);
+    int64_t* rows_off = reinterpret_cast<int64_t*>(tb + 2 * slot);
+    int64_t* items = reinterpret_cast<int64_t*>(tb + 3 * slot);
+    int64_t* item_off = reinterpret_cast<int64_t*>(tb + 4 * slot);
+    int npow = 1;
+    while (npow < segcap) npow <<= 1;
+    const size_t prep_smem = (size_t)3 * npow * 4;
+    BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
+    k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, nq, segcap, segbuf.as<Seg>(),
+                                                                  nseg, rows);
+    BLSH_LAUNCH_CHECK();
+    ++*launches;
+    scan_exclusive_i64(rows, rows_off, ntiles, scan, s);
+    *launches += 3;
+    int64_t total_rows = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&total_rows, rows_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    const int64_t target = 148 * 4;
+    int64_t chr = (total_rows + target - 1) / target;
+    chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 31) / 32 * 32));
+    k_tile_items<<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(rows, ntiles, (int)chr, items);
+    BLSH_LAUNCH_CHECK();
+    ++*launches;
+    scan_exclusive_i64(items, item_off, ntiles, scan, s);
+    *launches += 3;
+    int64_t n_items = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    partials.ensure((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8);
+    TiledArgs ta{};
+    ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
+    ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
+    ta.nseg = nseg; ta.rows = rows; ta.item_off = item_off; ta.partials = partials.as<unsigned long long>();
+    ta.counters = counters;
+    const size_t smem = tiled_smem_bytes(a.ds);
+    if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
+    if (n_items > 0) {
+        BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);
+        BLSH_LAUNCH_CHECK();
+        ++*launches;
+    }
+    if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
+    k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand);
+    BLSH_LAUNCH_CHECK();
+    ++*launches;
+    *n_items_out = n_items;
+    *chr_out = (int)chr;
+    *rows_out = total_rows;
+    unsigned long long ev = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&ev, counters, 8, cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    *pairs_out = (int64_t)ev;
+}
+
+}  // namespace blsh

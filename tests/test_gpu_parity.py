@@ -270,3 +270,26 @@ def test_c2_full(blsh, orc):
     ix, ox = build_pair(blsh, orc, X, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
     compare_build(ix, ox)
     run_query_pair(ix, ox, X, Q, cfg.k)
+
+
+def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
+    """The one-warp-per-(query, chunk) short-list (used when the tiled kernel's
+    shared memory does not fit, e.g. d > 512) against the oracle."""
+    X, Q = c1
+    monkeypatch.setenv("BLSH_SHORTLIST", "warp")
+    ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=4.0, seed=11)
+    run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
+    run_query_pair(ix, ox, X, Q, 50, probe=1, T=4, hierarchy=1)
+    assert ix.stats().tiled == 0
+    monkeypatch.delenv("BLSH_SHORTLIST")
+    run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
+    assert ix.stats().tiled == 1
+
+
+def test_large_d_uses_fallback(blsh, orc):
+    mix = synth.mixture(1000, 8, 8, 0.2, 5)
+    X = synth.sample_points(mix, 2500, 6)
+    Q = synth.sample_points(mix, 30, 7)
+    ix, ox = build_pair(blsh, orc, X, G=2, M=6, W=3.0)
+    run_query_pair(ix, ox, X, Q, 10, probe=1, T=8)
+    assert ix.stats().tiled == 0
