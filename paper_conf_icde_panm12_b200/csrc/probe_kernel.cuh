@@ -1,0 +1,205 @@
+// probe_kernel.cuh -- a3 + a4, one warp per query (included by query.cu inside
+// its anonymous namespace, after warp_select / find_bucket / lat_score).
+//
+// Z^M path templated on M so the perturbation pool lives in registers:
+// per coordinate the admissible options among {-1, 0, +1} (those whose term
+// x_i(delta)^2 is <= the bound B' of DESIGN.md §7), decoded from the pool
+// index with divisions by 1, 2 or 3 (multiply-high), least-significant
+// coordinate first; the score is then summed in ascending coordinate order
+// (R11), exactly as the oracle does.
+
+template <int MM>
+struct PoolT {
+    double sqm[MM], sqp[MM];   // x_i(-1)^2, x_i(+1)^2 (exact products of fp32 values)
+    uint32_t nopt[MM];         // 1..3 options per coordinate
+    uint32_t hasm[MM];         // 1 if -1 is an option
+    uint32_t P, home;
+};
+
+template <int MM>
+__device__ __forceinline__ double pool_score(const PoolT<MM>& pl, uint32_t x, int8_t* dl) {
+    int8_t d[MM];
+#pragma unroll
+    for (int i = MM - 1; i >= 0; --i) {
+        const uint32_t n = pl.nopt[i];
+        const uint32_t qv = n == 3u ? (__umulhi(x, 0xAAAAAAABu) >> 1) : (n == 2u ? (x >> 1) : x);
+        d[i] = (int8_t)((int)(x - qv * n) - (int)pl.hasm[i]);
+        x = qv;
+    }
+    double s = 0.0;
+#pragma unroll
+    for (int i = 0; i < MM; ++i) {
+        if (d[i] < 0) s = __dadd_rn(s, pl.sqm[i]);
+        else if (d[i] > 0) s = __dadd_rn(s, pl.sqp[i]);
+        dl[i] = d[i];
+    }
+    return s;
+}
+
+template <int MM>
+__device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int lane, int64_t ulo, int64_t uhi,
+                            uint2* ivl) {
+    const int T = a.T, B = a.B;
+    const float* tq = a.qt + (size_t)q * MM;
+    float t[MM], fl[MM];
+#pragma unroll
+    for (int i = 0; i < MM; ++i) {
+        t[i] = tq[i];
+        fl[i] = floorf(t[i]);
+    }
+    PoolT<MM> pl;
+    if (a.probe == 1 && T > 1) {
+        double v[2 * MM];
+#pragma unroll
+        for (int i = 0; i < MM; ++i) {
+            const float xm = __fsub_rn(t[i], fl[i]);
+            const float xp = __fsub_rn(1.0f, xm);
+            pl.sqm[i] = (double)xm * (double)xm;
+            pl.sqp[i] = (double)xp * (double)xp;
+            v[2 * i] = pl.sqm[i];
+            v[2 * i + 1] = pl.sqp[i];
+        }
+        // bound B': sum of the J smallest terms, J minimal with >= T-1 valid subsets
+        uint32_t used = 0;            // 2 bits per coordinate
+        unsigned long long taken = 0ull;
+        double Bsum = 0.0;
+        for (int J = 0; J < 2 * MM; ++J) {
+            int jb = -1;
+            double vb = 0.0;
+#pragma unroll
+            for (int j = 0; j < 2 * MM; ++j)
+                if (!((taken >> j) & 1ull) && (jb < 0 || v[j] < vb)) { jb = j; vb = v[j]; }
+            taken |= 1ull << jb;
+            used += 1u << (2 * (jb >> 1));
+            Bsum = __dadd_rn(Bsum, vb);
+            uint32_t prod = 1;
+#pragma unroll
+            for (int i = 0; i < MM; ++i) prod *= 1u + ((used >> (2 * i)) & 3u);
+            if (prod - 1u >= (uint32_t)(T - 1)) break;
+        }
+        const double Bp = __dmul_ru(Bsum, 1.0 + 0x1p-40);
+        uint32_t P = 1, home = 0;
+#pragma unroll
+        for (int i = MM - 1; i >= 0; --i) {
+            const uint32_t hm = pl.sqm[i] <= Bp ? 1u : 0u;
+            const uint32_t hp = pl.sqp[i] <= Bp ? 1u : 0u;
+            pl.hasm[i] = hm;
+            pl.nopt[i] = 1u + hm + hp;
+            home += hm * P;
+            P *= pl.nopt[i];
+        }
+        pl.P = P;
+        pl.home = home;
+        warp_select(sm, P, home, T - 1, [&](uint32_t x) {
+            int8_t dl[MM];
+            return pool_score<MM>(pl, x, dl);
+        });
+    }
+    int64_t mysum = 0;
+    const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
+    for (int p = lane; p < T; p += 32) {
+        int8_t dl[MM];
+#pragma unroll
+        for (int i = 0; i < MM; ++i) dl[i] = 0;
+        if (p > 0) pool_score<MM>(pl, sm.order[p - 1], dl);
+        int32_t pc[MM];
+        bool valid = true;
+#pragma unroll
+        for (int i = 0; i < MM; ++i) {
+            const float f = __fadd_rn(fl[i], (float)dl[i]);
+            if (!(f >= lo && f <= hi)) valid = false;
+            pc[i] = valid ? (int32_t)f : 0;
+        }
+        Key128 k{0, 0};
+        uint2 iv = make_uint2(0, 0);
+        if (valid) {
+            k = morton_key(pc, MM, B);
+            const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
+            if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
+        }
+        ivl[p] = iv;
+        mysum += (int64_t)(iv.y - iv.x);
+        if (a.pkey) {
+            a.pkey[(size_t)q * T + p] = k;
+            a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
+        }
+    }
+    return mysum;
+}
+
+__device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int lane, int oor, int64_t ulo,
+                            int64_t uhi, uint2* ivl) {
+    const int T = a.T, B = a.B;
+    const float* t = a.qt + (size_t)q * 8;
+    const int32_t* code = a.qcode + (size_t)q * 8;
+    if (a.probe == 2 && T > 1 && !(oor & 1))
+        warp_select(sm, 240u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat_score(t, code, x); });
+    int64_t mysum = 0;
+    for (int p = lane; p < T; p += 32) {
+        int32_t pc[8];
+        bool valid = !(oor & 1);
+        const uint32_t r = (p > 0 && valid) ? sm.order[p - 1] : 0u;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) pc[i] = code[i] + (p > 0 ? (int32_t)c_e8_roots[r][i] : 0);
+        const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
+        if (valid)
+            for (int i = 0; i < 8; ++i)
+                if (pc[i] < lo || pc[i] > hi) valid = false;
+        Key128 k{0, 0};
+        uint2 iv = make_uint2(0, 0);
+        if (valid) {
+            k = morton_key(pc, 8, B);
+            const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
+            if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
+        }
+        ivl[p] = iv;
+        mysum += (int64_t)(iv.y - iv.x);
+        if (a.pkey) {
+            a.pkey[(size_t)q * T + p] = k;
+            a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
+        }
+    }
+    return mysum;
+}
+
+__global__ void __launch_bounds__(kPW * 32, 4) k_probe_lookup(QueryArgs a) {
+    __shared__ ProbeSmem smem[kPW];
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    const int64_t q = blockIdx.x * (int64_t)kPW + w;
+    if (q >= a.nq) return;
+    ProbeSmem& sm = smem[w];
+    const int T = a.T;
+    const int oor = a.qoor[q];
+    uint2* ivl = a.ivl + (size_t)q * (T + 1);
+    if (oor & 2) {   // leaf not owned by this shard
+        for (int p = lane; p <= T; p += 32) ivl[p] = make_uint2(0, 0);
+        if (a.pkey)
+            for (int p = lane; p < T; p += 32) { a.pkey[(size_t)q * T + p] = Key128{0, 0}; a.pvalid[(size_t)q * T + p] = 0; }
+        if (lane == 0) { a.base[q] = 0; a.cnt[q] = 0; if (a.level) a.level[q] = 0; }
+        return;
+    }
+    const int g = a.qleaf[q];
+    const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
+    int64_t mysum = 0;
+    if (a.quantizer == 1) {
+        mysum = probe_e8(a, sm, q, lane, oor, ulo, uhi, ivl);
+    } else {
+        switch (a.M) {
+#define BLSH_ZM_CASE(MMV) case MMV: mysum = probe_zm<MMV>(a, sm, q, lane, ulo, uhi, ivl); break;
+            BLSH_ZM_CASE(1) BLSH_ZM_CASE(2) BLSH_ZM_CASE(3) BLSH_ZM_CASE(4) BLSH_ZM_CASE(5) BLSH_ZM_CASE(6)
+            BLSH_ZM_CASE(7) BLSH_ZM_CASE(8) BLSH_ZM_CASE(9) BLSH_ZM_CASE(10) BLSH_ZM_CASE(11) BLSH_ZM_CASE(12)
+            BLSH_ZM_CASE(13) BLSH_ZM_CASE(14) BLSH_ZM_CASE(15) BLSH_ZM_CASE(16)
+#undef BLSH_ZM_CASE
+            default: break;
+        }
+    }
+    if (lane == 0) ivl[T] = make_uint2(0, 0);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mysum += __shfl_xor_sync(BLSH_FULL, mysum, o);
+    if (lane == 0) {
+        a.base[q] = mysum;
+        a.cnt[q] = mysum;
+        if (a.level) a.level[q] = 0;
+    }
+}

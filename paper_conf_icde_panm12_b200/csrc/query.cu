@@ -133,7 +133,32 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
     const int lane = threadIdx.x & 31;
     unsigned long long prefix = 0ull, mask = 0ull;
     int r = R - 1;
-    for (int sh = 56; sh >= 0; sh -= 8) {
+    // bits common to every key are skipped: start at the byte of the highest differing bit
+    unsigned long long kmin = ~0ull, kmax = 0ull;
+    for (uint32_t x = lane; x < P; x += 32) {
+        if (x == skip) continue;
+        const unsigned long long b = (unsigned long long)__double_as_longlong(score(x));
+        kmin = b < kmin ? b : kmin;
+        kmax = b > kmax ? b : kmax;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long a0 = __shfl_xor_sync(BLSH_FULL, kmin, o);
+        const unsigned long long a1 = __shfl_xor_sync(BLSH_FULL, kmax, o);
+        kmin = a0 < kmin ? a0 : kmin;
+        kmax = a1 > kmax ? a1 : kmax;
+    }
+    int sh0 = -8;
+    if (kmin != kmax) {
+        const int hb = 63 - __clzll((long long)(kmin ^ kmax));
+        sh0 = (hb / 8) * 8;
+        mask = sh0 + 8 >= 64 ? 0ull : ~((1ull << (sh0 + 8)) - 1ull);
+        prefix = kmin & mask;
+    } else {
+        mask = ~0ull;
+        prefix = kmin;
+    }
+    for (int sh = sh0; sh >= 0; sh -= 8) {
         for (int i = lane; i < 256; i += 32) sm.hist[i] = 0;
         __syncwarp();
         for (uint32_t x = lane; x < P; x += 32) {
@@ -166,21 +191,27 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
         }
         dg = __shfl_sync(BLSH_FULL, dg, src);
         r = __shfl_sync(BLSH_FULL, nr, src);
+        const uint32_t binc = __shfl_sync(BLSH_FULL, sm.hist[dg], 0);
         prefix |= (unsigned long long)dg << sh;
         mask |= 255ull << sh;
         __syncwarp();
+        if ((uint32_t)r + 1u == binc) break;   // the whole bin is taken: no finer digit needed
     }
-    // prefix = score bits of the R-th smallest; take all smaller plus the first r+1 ties (ascending index)
+    // take every key whose masked bits are < prefix, plus the first r+1 (ascending index)
+    // of those equal to it (either all of them, or exact ties after the last digit)
     int cnt = 0, ties = 0;
     for (uint32_t base = 0; base < P; base += 32) {
         const uint32_t x = base + lane;
-        unsigned long long b = ~0ull;
-        if (x < P && x != skip) b = (unsigned long long)__double_as_longlong(score(x));
-        const bool tie = b == prefix;
+        unsigned long long b = ~0ull, bm = ~0ull;
+        if (x < P && x != skip) {
+            b = (unsigned long long)__double_as_longlong(score(x));
+            bm = b & mask;
+        }
+        const bool tie = bm == prefix;
         const unsigned tm = __ballot_sync(BLSH_FULL, tie);
         const int my_tie = ties + __popc(tm & lanemask_lt());
         ties += __popc(tm);
-        const bool sel = b < prefix || (tie && my_tie <= r);
+        const bool sel = bm < prefix || (tie && my_tie <= r);
         const unsigned smk = __ballot_sync(BLSH_FULL, sel);
         if (sel) {
             const int at = cnt + __popc(smk & lanemask_lt());
@@ -204,7 +235,8 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
     __syncwarp();
 }
 
-__global__ void __launch_bounds__(kPW * 32) k_probe_lookup(QueryArgs a) {
+#if 0   // superseded by probe_kernel.cuh (kept until the next cleanup)
+__global__ void __launch_bounds__(kPW * 32) k_probe_lookup_v1(QueryArgs a) {
     __shared__ ProbeSmem smem[kPW];
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
@@ -328,6 +360,10 @@ __global__ void __launch_bounds__(kPW * 32) k_probe_lookup(QueryArgs a) {
         if (a.level) a.level[q] = 0;
     }
 }
+
+#endif
+
+#include "probe_kernel.cuh"
 
 // ---------------------------------------------------------------------------
 // tau = lower median of |A0| over the batch (single block radix select).
