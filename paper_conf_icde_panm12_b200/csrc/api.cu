@@ -339,6 +339,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     const char* mode = std::getenv("BLSH_SHORTLIST");
     const bool tiled = tiled_supported(ds, T) && !(mode && std::strcmp(mode, "warp") == 0);
     int64_t n_items = 0, union_rows = 0, pairs = total;
+    int tcpath = 0;
     int64_t ch = 0;
     if (tiled) {
         // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
@@ -346,7 +347,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         int chr = 0;
         run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
-                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs);
+                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs, &tcpath);
         ch = chr;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {
@@ -383,7 +384,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     stt.chunk = (int32_t)ch;
     stt.launches = launches;
     stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 + (double)n_items * k * 8.0;
-    stt.tiled = tiled ? 1 : 0;
+    stt.tiled = tiled ? (tcpath ? 2 : 1) : 0;
     stt.union_rows = union_rows;
     stt.pairs_scored = pairs;
     stt.shortlist_flops = 3.0 * ix.d * (double)total;

@@ -16,6 +16,9 @@
 // (R22).  Each (work item, query) keeps a warp-register top-k; k_merge_tiled
 // merges the items of a tile per query.
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
 
 #include "internal.cuh"
 #include "query_kernels.cuh"
@@ -37,7 +40,8 @@ struct Seg {
 // tile prep: union of the tile's candidate intervals, with query masks
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restrict__ ivl, int T,
-                                                            const uint32_t* __restrict__ qorder, int64_t nq,
+                                                            const uint32_t* __restrict__ qorder,
+                                                            const int64_t* __restrict__ tile_off,
                                                             int segcap, Seg* __restrict__ segs,
                                                             int32_t* __restrict__ nseg,
                                                             int64_t* __restrict__ rows) {
@@ -57,8 +61,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
     const int nint = QT * (T + 1);
     for (int i = tid; i < nint; i += kPrepThreads) {
         const int slot = i / (T + 1), p = i % (T + 1);
-        const int64_t qp = (int64_t)t * QT + slot;
-        if (qp >= nq) continue;
+        const int64_t qp = tile_off[t] + slot;
+        if (qp >= tile_off[t + 1]) continue;
         const uint2 iv = ivl[(size_t)qorder[qp] * (T + 1) + p];
         if (iv.y > iv.x) {
             const int at = atomicAdd(&s_cnt, 2);
@@ -116,8 +120,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
     __syncthreads();
     for (int i = tid; i < nint; i += kPrepThreads) {     // XOR toggles at both ends of every interval
         const int slot = i / (T + 1), p = i % (T + 1);
-        const int64_t qp = (int64_t)t * QT + slot;
-        if (qp >= nq) continue;
+        const int64_t qp = tile_off[t] + slot;
+        if (qp >= tile_off[t + 1]) continue;
         const uint2 iv = ivl[(size_t)qorder[qp] * (T + 1) + p];
         if (iv.y > iv.x) {
             int lo = 0, hi = nb;
@@ -210,7 +214,12 @@ struct TiledArgs {
     const int64_t* rows;       // [ntiles] union rows per tile
     const int64_t* item_off;   // [ntiles+1]
     unsigned long long* partials;   // [n_items][QT][k]
-    unsigned long long* counters;   // [0] (row, query) pairs evaluated
+    const int64_t* tile_off;        // [ntiles+1] sorted-query positions of each tile
+    const int32_t* tile_of;         // [nq] tile of each sorted position
+    unsigned long long* counters;   // [0] (row, query) pairs evaluated, [1] screen survivors (TC)
+    float* dbg;                     // optional (BLSH_TC_DEBUG): item 0, block 0 dots / |x'|^2 / rows
+    unsigned long long* sbuf;       // TC: [n_items][QT][scap] buffered (lower bound, row) pairs
+    int scap;
 };
 
 struct TopK {
@@ -387,6 +396,7 @@ __global__ void __launch_bounds__(kTW * 32, 1) k_shortlist_tiled_v1(TiledArgs a)
 #endif
 
 #include "tiled_kernel.cuh"
+#include "tc_kernel.cuh"
 
 __global__ void __launch_bounds__(256) k_merge_tiled(TiledArgs a, const int32_t* __restrict__ qoor,
                                                      const int64_t* __restrict__ cnt, int64_t* out_ids, float* out_d2,
@@ -395,8 +405,8 @@ __global__ void __launch_bounds__(256) k_merge_tiled(TiledArgs a, const int32_t*
     const int64_t pos = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
     if (pos >= a.nq) return;
     const int64_t q = a.qorder[pos];
-    const int64_t tile = pos / QT;
-    const int slot = (int)(pos % QT);
+    const int64_t tile = a.tile_of[pos];
+    const int slot = (int)(pos - a.tile_off[tile]);
     const int k = a.k;
     TopK tk{kEmpty, kEmpty};
     unsigned long long thr = kEmpty;
@@ -435,6 +445,67 @@ __global__ void k_qsort_keys(const Key128* __restrict__ qkey, const int32_t* __r
     id[q] = (uint32_t)q;
 }
 
+// ---------------------------------------------------------------------------
+// tile formation: consecutive sorted queries, at most QT per tile, a new tile
+// at every leaf change and wherever two consecutive queries are far apart
+// (> 16 x the median consecutive squared distance), so a tile's queries sit
+// in one region of space (the TC screen's error bound grows with |q - c|).
+// ---------------------------------------------------------------------------
+__global__ void k_consec_d2(const float* __restrict__ Q, int ds, const uint32_t* __restrict__ qorder, int64_t nq,
+                            int64_t* __restrict__ d2bits) {
+    const int lane = threadIdx.x & 31;
+    const int64_t i = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5) + 1;
+    if (i >= nq) return;
+    const float4* a = reinterpret_cast<const float4*>(Q + (size_t)qorder[i] * ds);
+    const float4* b = reinterpret_cast<const float4*>(Q + (size_t)qorder[i - 1] * ds);
+    float s = 0.f;
+    for (int v = lane; v < (ds >> 2); v += 32) {
+        const float4 x = a[v], y = b[v];
+        const float dx = x.x - y.x, dy = x.y - y.y, dz = x.z - y.z, dw = x.w - y.w;
+        s += dx * dx + dy * dy + dz * dz + dw * dw;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(BLSH_FULL, s, o);
+    if (lane == 0) d2bits[i - 1] = (int64_t)__float_as_uint(s);
+}
+
+__global__ void k_tile_flags(const int64_t* __restrict__ d2bits, const int64_t* __restrict__ med,
+                             const int32_t* __restrict__ qleaf, const int32_t* __restrict__ qoor,
+                             const uint32_t* __restrict__ qorder, int64_t nq, uint8_t* __restrict__ brk) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= nq) return;
+    if (i == 0) { brk[0] = 1; return; }
+    const uint32_t a = qorder[i], b = qorder[i - 1];
+    const uint32_t la = (qoor[a] & 2) ? 0xFFFFu : (uint32_t)qleaf[a];
+    const uint32_t lb = (qoor[b] & 2) ? 0xFFFFu : (uint32_t)qleaf[b];
+    const float lim = 16.0f * __uint_as_float((uint32_t)*med);
+    brk[i] = (la != lb || __uint_as_float((uint32_t)d2bits[i - 1]) > lim) ? 1 : 0;
+}
+
+__global__ void k_run_start(const uint8_t* __restrict__ brk, const int64_t* __restrict__ excl, int64_t nq,
+                            int64_t* __restrict__ run_start) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < nq && brk[i]) run_start[excl[i]] = i;
+}
+
+__global__ void k_tile_start(const uint8_t* __restrict__ brk, const int64_t* __restrict__ excl,
+                             const int64_t* __restrict__ run_start, int64_t nq, uint8_t* __restrict__ ts) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= nq) return;
+    const int64_t rid = excl[i] + brk[i] - 1;
+    ts[i] = ((i - run_start[rid]) % QT == 0) ? 1 : 0;
+}
+
+__global__ void k_tile_scatter(const uint8_t* __restrict__ ts, const int64_t* __restrict__ excl, int64_t nq,
+                               int64_t* __restrict__ tile_off, int32_t* __restrict__ tile_of) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i >= nq) return;
+    const int64_t t = excl[i] + ts[i] - 1;
+    tile_of[i] = (int32_t)t;
+    if (ts[i]) tile_off[t] = i;
+    if (i == nq - 1) tile_off[t + 1] = nq;
+}
+
 }  // namespace
 
 size_t tiled_smem_bytes(int ds) { return 1024 + (size_t)QT * ds * 4 + (size_t)kStages * 32 * (ds + 4) * 4; }
@@ -470,17 +541,49 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
-                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out) {
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int* tc_out) {
     const int64_t nq = a.nq;
-    const int64_t ntiles = (nq + QT - 1) / QT;
     const int T = a.T;
     const int segcap = 2 * QT * (T + 1);
-    segbuf.ensure((size_t)ntiles * segcap * sizeof(Seg));
-    const size_t slot = (((size_t)(ntiles + 1) * 8) + 255) & ~size_t(255);
-    tilebuf.ensure(slot * 5 + 256);
+    // tile arrays are sized for the worst case (one query per tile)
+    const size_t slot = (((size_t)(nq + 1) * 8) + 255) & ~size_t(255);
+    tilebuf.ensure(slot * 13 + 256);
     char* tb = tilebuf.as<char>();
     unsigned long long* counters = reinterpret_cast<unsigned long long*>(tb + 5 * slot);
     BLSH_CUDA(cudaMemsetAsync(counters, 0, 16, s));
+    int64_t* tile_off = reinterpret_cast<int64_t*>(tb + 6 * slot);
+    int32_t* tile_of = reinterpret_cast<int32_t*>(tb + 7 * slot);
+    int64_t* d2bits = reinterpret_cast<int64_t*>(tb + 8 * slot);
+    int64_t* fexcl = reinterpret_cast<int64_t*>(tb + 9 * slot);
+    int64_t* run_start = reinterpret_cast<int64_t*>(tb + 10 * slot);
+    uint8_t* brk = reinterpret_cast<uint8_t*>(tb + 11 * slot);
+    uint8_t* tst = reinterpret_cast<uint8_t*>(tb + 11 * slot + (slot >> 1));
+    int64_t* med = reinterpret_cast<int64_t*>(tb + 12 * slot);
+    {
+        const unsigned g256 = (unsigned)((nq + 255) / 256);
+        BLSH_CUDA(cudaMemsetAsync(med, 0, 8, s));
+        if (nq > 1) {
+            k_consec_d2<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(a.Q, a.ds, qorder, nq, d2bits);
+            BLSH_LAUNCH_CHECK();
+            launch_median(d2bits, nq - 1, med, s);
+            *launches += 2;
+        }
+        k_tile_flags<<<g256, 256, 0, s>>>(d2bits, med, a.qleaf, a.qoor, qorder, nq, brk);
+        BLSH_LAUNCH_CHECK();
+        scan_exclusive_u8(brk, fexcl, nq, scan, s);
+        k_run_start<<<g256, 256, 0, s>>>(brk, fexcl, nq, run_start);
+        BLSH_LAUNCH_CHECK();
+        k_tile_start<<<g256, 256, 0, s>>>(brk, fexcl, run_start, nq, tst);
+        BLSH_LAUNCH_CHECK();
+        scan_exclusive_u8(tst, fexcl, nq, scan, s);
+        k_tile_scatter<<<g256, 256, 0, s>>>(tst, fexcl, nq, tile_off, tile_of);
+        BLSH_LAUNCH_CHECK();
+        *launches += 10;
+    }
+    int64_t ntiles = 0;
+    BLSH_CUDA(cudaMemcpyAsync(&ntiles, fexcl + nq, 8, cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    segbuf.ensure((size_t)std::max<int64_t>(ntiles, 1) * segcap * sizeof(Seg));
     int32_t* nseg = reinterpret_cast<int32_t*>(tb);
     int64_t* rows = reinterpret_cast<int64_t*>(tb + slot);
     int64_t* rows_off = reinterpret_cast<int64_t*>(tb + 2 * slot);
@@ -490,8 +593,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     while (npow < segcap) npow <<= 1;
     const size_t prep_smem = (size_t)3 * npow * 4;
     BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
-    k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, nq, segcap, segbuf.as<Seg>(),
-                                                                  nseg, rows);
+    k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, tile_off, segcap,
+                                                                  segbuf.as<Seg>(), nseg, rows);
     BLSH_LAUNCH_CHECK();
     ++*launches;
     scan_exclusive_i64(rows, rows_off, ntiles, scan, s);
@@ -510,20 +613,45 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int64_t n_items = 0;
     BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    partials.ensure((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8);
+    constexpr int kScap = 256;   // buffered (row, query) pairs per item and query before immediate rescoring
+    const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
+    partials.ensure(part_bytes + (size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
     ta.nseg = nseg; ta.rows = rows; ta.item_off = item_off; ta.partials = partials.as<unsigned long long>();
     ta.counters = counters;
+    ta.tile_off = tile_off;
+    ta.tile_of = tile_of;
+    ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
+    ta.scap = kScap;
     const size_t smem = tiled_smem_bytes(a.ds);
+    const size_t tc_smem = ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)2 * QT * a.ds * 4 +
+                           (size_t)kTcSlots * kTcChunkBytes;
+    const char* mode = std::getenv("BLSH_SHORTLIST");
+    // the tensor-core screen is opt-in (BLSH_SHORTLIST=tc) until it beats the SIMT tiled kernel
+    const bool use_tc = k <= kTcMaxK && a.ds % kTcChunk == 0 && a.ds <= 512 && tc_smem <= 227 * 1024 &&
+                        mode && std::strcmp(mode, "tc") == 0;
+    const char* dbg_path = std::getenv("BLSH_TC_DEBUG");
+    DevBuf dbgbuf;
+    if (use_tc && dbg_path) {
+        dbgbuf.alloc((4096 + 512) * sizeof(float));
+        BLSH_CUDA(cudaMemsetAsync(dbgbuf.p, 0, (4096 + 512) * sizeof(float), s));
+        ta.dbg = dbgbuf.as<float>();
+    }
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
-        BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);
+        if (use_tc) {
+            BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
+            k_shortlist_tc<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
+        } else {
+            BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);
+        }
         BLSH_LAUNCH_CHECK();
         ++*launches;
     }
+    *tc_out = use_tc ? 1 : 0;
     if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
     k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand);
     BLSH_LAUNCH_CHECK();
@@ -531,10 +659,21 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     *n_items_out = n_items;
     *chr_out = (int)chr;
     *rows_out = total_rows;
-    unsigned long long ev = 0;
-    BLSH_CUDA(cudaMemcpyAsync(&ev, counters, 8, cudaMemcpyDeviceToHost, s));
+    unsigned long long ev[2] = {0, 0};
+    BLSH_CUDA(cudaMemcpyAsync(ev, counters, 16, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    *pairs_out = (int64_t)ev;
+    *pairs_out = (int64_t)(use_tc ? ev[1] : ev[0]);   // TC: exact rescorings after the screen
+    if (ta.dbg) {
+        std::vector<float> h(4096 + 512);
+        BLSH_CUDA(cudaMemcpy(h.data(), ta.dbg, h.size() * sizeof(float), cudaMemcpyDeviceToHost));
+        std::vector<uint32_t> q0(QT);
+        BLSH_CUDA(cudaMemcpy(q0.data(), qorder, QT * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        if (FILE* f = std::fopen(dbg_path, "wb")) {
+            std::fwrite(h.data(), sizeof(float), h.size(), f);
+            std::fwrite(q0.data(), sizeof(uint32_t), q0.size(), f);
+            std::fclose(f);
+        }
+    }
 }
 
 }  // namespace blsh

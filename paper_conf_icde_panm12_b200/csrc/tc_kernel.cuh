@@ -1,0 +1,499 @@
+// tc_kernel.cuh -- query-tiled short-list with a tensor-core screen
+// (included by shortlist_tiled.cu inside its anonymous namespace).
+//
+// For a tile of QT = 32 queries and a 128-row block of the tile's candidate
+// union, the 128 x 32 dot products of the CENTRED vectors (x - c)(q - c),
+// c = the tile's first query, are one tcgen05.mma (kind::tf32, M = 128,
+// N = 32, K = 384 in 48 steps of K = 8) accumulated in TMEM.  The epilogue
+// turns them into approximate distances ~d^2 = |q'|^2 + |x'|^2 - 2 q'.x' and
+// keeps a (row, query) pair only if ~d^2 is within a rigorous margin of the
+// query's current k-th distance; every kept pair is rescored EXACTLY in the
+// fp32 direct form of k_shortlist (R22), so results are identical to the
+// SIMT kernels' -- the tensor cores only decide which pairs need exact work.
+//
+// Warp roles (13 warps):
+//   0-7  converters: gather the block's rows from HBM (16-byte loads),
+//        subtract c, write the TF32 A operand in the K-major no-swizzle UMMA
+//        layout (8-row x 16-byte core matrices), |x'|^2 per row;
+//   8    MMA issuer (one elected lane) + TMEM allocation;
+//   9-12 epilogue: tcgen05.ld of the 32 accumulators per row, screen, exact
+//        rescoring (warp-cooperative), per-(warp, query) top-k in smem.
+// Pipelines: 3-slot ring of 64-column A chunks (full / empty mbarriers, the
+// MMA frees a slot with tcgen05.commit), 2 TMEM accumulator slots
+// (tmem_full by commit / tmem_empty by the epilogue), 2 row-metadata slots.
+
+constexpr int kTcRows = 128;               // M
+constexpr int kTcChunk = 64;               // K columns per A chunk
+constexpr int kTcSlots = 3;                // A chunk ring
+constexpr int kTcConv = 8;                 // converter warps
+constexpr int kTcMmaWarp = 8;
+constexpr int kTcEpi0 = 9;                 // first epilogue warp
+constexpr int kTcThreads = 13 * 32;
+constexpr int kTcMaxK = 16;                // k supported by the TC path
+constexpr uint32_t kTcChunkBytes = kTcRows * kTcChunk * 4;   // 32 KB
+// instruction descriptor: D f32, A/B tf32, K-major both, N = 32, M = 128
+constexpr uint32_t kTcIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((32u >> 3) << 17) | ((128u >> 4) << 24);
+
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+    d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+    d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+    d |= 1ull << 46;   // descriptor version for sm_100
+    return d;          // base offset 0, SWIZZLE_NONE
+}
+__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(kTcIdesc), "r"(accum)
+        : "memory");
+}
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
+    uint32_t r[32];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+}
+
+struct TcSmem {
+    uint64_t full[kTcSlots], empty[kTcSlots];
+    uint64_t tfull[2], tempty[2], xready[2], mfree[2];
+    uint32_t tmem_base;
+    uint32_t thr[QT];                   // shared screen threshold (fp32 bits of the best k-th d^2)
+    float qn[QT];                       // |q'|^2
+    uint32_t rpos[2][kTcRows];          // table row of each block row
+    uint32_t rmask[2][kTcRows];         // query mask of each block row (0 = padding)
+    float xn[2][kTcRows];               // |x'|^2
+    unsigned long long tk[QT][kTcMaxK];      // per query sorted top-k (shared by the epilogue warps)
+    int lock[QT];                            // per query spinlock guarding tk[q] / ul[q]
+    float ul[QT][kTcMaxK];                   // per query k smallest upper bounds ~d2 + m (thr = ul[q][k-1])
+    int scnt[QT];                            // buffered pairs per query
+    alignas(16) float cen[512];              // centre of the tile (mean of its queries)
+};
+
+// exact fp32 direct-form d^2 (same partial-sum structure as k_shortlist: 12-term lanes + butterfly)
+__device__ __forceinline__ float exact_d2_warp(const float* __restrict__ x, const float* __restrict__ q, int nv4,
+                                               int lane) {
+    float p = 0.f;
+    for (int v = lane; v < nv4; v += 32) {
+        const float4 a = __ldg(reinterpret_cast<const float4*>(x) + v);
+        const float4 b = reinterpret_cast<const float4*>(q)[v];   // query row in shared memory
+        const float dx = b.x - a.x, dy = b.y - a.y, dz = b.z - a.z, dw = b.w - a.w;
+        p = fmaf(dx, dx, p);
+        p = fmaf(dy, dy, p);
+        p = fmaf(dz, dz, p);
+        p = fmaf(dw, dw, p);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(BLSH_FULL, p, o);
+    return p;
+}
+
+__global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
+    extern __shared__ __align__(1024) unsigned char smraw[];
+    TcSmem& S = *reinterpret_cast<TcSmem*>(smraw);
+    const int ds = a.ds, nv4 = ds >> 2, kp_total = ds >> 2;   // 16-byte K pieces
+    unsigned char* opbase = smraw + ((sizeof(TcSmem) + 1023) & ~size_t(1023));
+    unsigned char* Bop = opbase;                                    // [QT x ds] tf32, UMMA K-major
+    unsigned char* Aop = Bop + (size_t)QT * ds * 4;                 // [kTcSlots][128 x 64] tf32
+    float* Qf = reinterpret_cast<float*>(Aop + (size_t)kTcSlots * kTcChunkBytes);   // [QT][ds] original queries
+    const uint32_t sboB = (uint32_t)kp_total * 128u;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t item = blockIdx.x;
+    int64_t lo = 0, hi = a.ntiles;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (a.item_off[mid] <= item) lo = mid;
+        else hi = mid;
+    }
+    const int64_t tile = lo;
+    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
+    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    const int nblk = (int)((r1 - r0 + kTcRows - 1) / kTcRows);
+    const int nchunk = ds / kTcChunk;
+    const int k = a.k;
+    // ---- setup: queries, centre c = mean of the tile's queries, B operand (q - c), |q'|^2 ----
+    const int64_t q0 = a.tile_off[tile];
+    const int nqt = (int)(a.tile_off[tile + 1] - q0);
+    for (int i = threadIdx.x; i < QT * nv4; i += kTcThreads) {
+        const int n = i / nv4, v = i % nv4;
+        reinterpret_cast<float4*>(Qf)[i] = n < nqt ? reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + n] * ds)[v]
+                                                   : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    __syncthreads();
+    for (int j = threadIdx.x; j < ds; j += kTcThreads) {
+        float s = 0.f;
+        for (int n = 0; n < nqt; ++n) s += Qf[(size_t)n * ds + j];
+        S.cen[j] = s / (float)nqt;
+    }
+    __syncthreads();
+    const float* cen = S.cen;
+    for (int i = threadIdx.x; i < QT * kp_total; i += kTcThreads) {
+        const int n = i % QT, kp = i / QT;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (n < nqt) {
+            const float4 x = reinterpret_cast<const float4*>(Qf + (size_t)n * ds)[kp];
+            const float4 cc = reinterpret_cast<const float4*>(cen)[kp];
+            v = make_float4(x.x - cc.x, x.y - cc.y, x.z - cc.z, x.w - cc.w);
+        }
+        *reinterpret_cast<float4*>(Bop + (size_t)(n >> 3) * sboB + (size_t)kp * 128 + (n & 7) * 16) = v;
+    }
+    if (threadIdx.x < QT) {
+        const int n = threadIdx.x;
+        float s = 0.f;
+        if (n < nqt) {
+            const float* qq = Qf + (size_t)n * ds;
+            for (int j = 0; j < ds; ++j) {
+                const float e = qq[j] - cen[j];
+                s = fmaf(e, e, s);
+            }
+        }
+        S.qn[n] = s;
+        S.thr[n] = 0x7F800000u;   // +inf
+    }
+    for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) {
+        (&S.tk[0][0])[i] = kEmpty;
+        (&S.ul[0][0])[i] = __int_as_float(0x7F800000);
+    }
+    if (threadIdx.x < QT) { S.lock[threadIdx.x] = 0; S.scnt[threadIdx.x] = 0; }
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kTcSlots; ++s) {
+            mbar_init(&S.full[s], kTcConv);
+            mbar_init(&S.empty[s], 1);
+        }
+        for (int s = 0; s < 2; ++s) {
+            mbar_init(&S.tfull[s], 1);
+            mbar_init(&S.tempty[s], 4);
+            mbar_init(&S.xready[s], kTcConv);
+            mbar_init(&S.mfree[s], 4);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == kTcMmaWarp) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(smem_u32(&S.tmem_base)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B operand visible to the tensor core
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tbase = S.tmem_base;
+
+    if (warp < kTcConv) {
+        // ======================= converters =======================
+        const Seg* SG = a.segs + (size_t)tile * a.segcap;
+        const int ns = a.nseg[tile];
+        int cs = 0;
+        {
+            int l2 = 0, h2 = ns;
+            while (h2 - l2 > 1) {
+                const int m = (l2 + h2) >> 1;
+                if ((int64_t)SG[m].off <= r0) l2 = m;
+                else h2 = m;
+            }
+            cs = l2;
+        }
+        // Warp w converts block rows [16w, 16w + 16).  Lane -> (row rsub of an 8-row group,
+        // K piece offset ksub): one 16-byte load instruction covers 8 rows x 64 contiguous
+        // bytes (8 cache lines) and one 16-byte store covers 8 rows x one K piece (128
+        // contiguous bytes of a core matrix, bank-conflict free).
+        const int rsub = lane & 7, ksub = lane >> 3;
+        for (int b = 0; b < nblk; ++b) {
+            const int ms = b & 1;
+            if (b >= 2) mbar_wait(&S.mfree[ms], (uint32_t)(((b >> 1) - 1) & 1));
+            const int64_t bstart = r0 + (int64_t)b * kTcRows;
+            // the block's 128 rows lie in the 128 segments starting at cs (each has >= 1 row)
+            Seg sw[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int si = cs + lane + 32 * i;
+                sw[i] = si < ns ? SG[si] : Seg{0u, 0u, 0u, 0xFFFFFFFFu};
+            }
+            uint32_t my_pos = 0, my_mask = 0;   // lanes 0..15: row 16w + lane
+            for (int t2 = 0; t2 < 16; ++t2) {
+                const uint32_t r = (uint32_t)(bstart + 16 * warp + t2);
+                int cnt = 0;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) cnt += __popc(__ballot_sync(BLSH_FULL, sw[i].off <= r));
+                const int idx = cnt - 1, src = idx & 31, reg = idx >> 5;
+                uint32_t st = 0, of = 0, mk = 0;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const uint32_t a0 = __shfl_sync(BLSH_FULL, sw[i].start, src);
+                    const uint32_t a1 = __shfl_sync(BLSH_FULL, sw[i].off, src);
+                    const uint32_t a2 = __shfl_sync(BLSH_FULL, sw[i].mask, src);
+                    if (reg == i) { st = a0; of = a1; mk = a2; }
+                }
+                if (lane == t2) {
+                    const bool v = (int64_t)r < r1;
+                    my_pos = v ? st + (r - of) : 0u;
+                    my_mask = v ? mk : 0u;
+                }
+            }
+            {   // every converter warp advances cs identically (segment of the next block's first row)
+                const uint32_t rn = (uint32_t)(bstart + kTcRows);
+                int cnt = 0;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) cnt += __popc(__ballot_sync(BLSH_FULL, sw[i].off <= rn));
+                cs += cnt > 0 ? cnt - 1 : 0;
+            }
+            if (lane < 16) {
+                S.rpos[ms][16 * warp + lane] = my_pos;
+                S.rmask[ms][16 * warp + lane] = my_mask;
+            }
+            const uint32_t p0 = __shfl_sync(BLSH_FULL, my_pos, rsub), p1 = __shfl_sync(BLSH_FULL, my_pos, 8 + rsub);
+            const bool v0 = __shfl_sync(BLSH_FULL, my_mask, rsub) != 0u;
+            const bool v1 = __shfl_sync(BLSH_FULL, my_mask, 8 + rsub) != 0u;
+            const float4* x0 = reinterpret_cast<const float4*>(a.Xp + (size_t)p0 * ds);
+            const float4* x1 = reinterpret_cast<const float4*>(a.Xp + (size_t)p1 * ds);
+            float xs0 = 0.f, xs1 = 0.f;
+            auto load_chunk = [&](int c, float4* v) {
+#pragma unroll
+                for (int it = 0; it < 8; ++it) {
+                    const int kp = c * 16 + (it >> 1) * 4 + ksub;
+                    const bool vv = (it & 1) ? v1 : v0;
+                    v[it] = vv ? __ldg(((it & 1) ? x1 : x0) + kp) : make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+            };
+            auto convert_chunk = [&](int c, const float4* v) {
+                const int gch = b * nchunk + c;
+                const int slot = gch % kTcSlots;
+                if (gch >= kTcSlots) mbar_wait(&S.empty[slot], (uint32_t)((gch / kTcSlots - 1) & 1));
+                unsigned char* A = Aop + (size_t)slot * kTcChunkBytes;
+#pragma unroll
+                for (int it = 0; it < 8; ++it) {
+                    const int rg = it & 1;
+                    const int kpl = (it >> 1) * 4 + ksub;
+                    const float4 cc = reinterpret_cast<const float4*>(cen)[c * 16 + kpl];
+                    float4 x = v[it];
+                    if (rg ? v1 : v0) {
+                        x.x -= cc.x; x.y -= cc.y; x.z -= cc.z; x.w -= cc.w;
+                        float& xs = rg ? xs1 : xs0;
+                        xs = fmaf(x.x, x.x, xs);
+                        xs = fmaf(x.y, x.y, xs);
+                        xs = fmaf(x.z, x.z, xs);
+                        xs = fmaf(x.w, x.w, xs);
+                    }
+                    *reinterpret_cast<float4*>(A + (size_t)(2 * warp + rg) * 2048 + (size_t)kpl * 128 + rsub * 16) = x;
+                }
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&S.full[slot]);
+            };
+            // the next chunk's loads are in flight while the current chunk is converted
+            float4 va[8], vb[8];
+            load_chunk(0, va);
+            for (int c = 0; c < nchunk; c += 2) {
+                if (c + 1 < nchunk) load_chunk(c + 1, vb);
+                convert_chunk(c, va);
+                if (c + 1 < nchunk) {
+                    if (c + 2 < nchunk) load_chunk(c + 2, va);
+                    convert_chunk(c + 1, vb);
+                }
+            }
+            // |x'|^2 per row: reduce over the 4 lanes (ksub) sharing a row
+            xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 8);
+            xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 16);
+            xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 8);
+            xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 16);
+            if (lane < 8) S.xn[ms][16 * warp + lane] = xs0;
+            else if (lane < 16) S.xn[ms][16 * warp + lane] = xs1;
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.xready[ms]);
+        }
+    } else if (warp == kTcMmaWarp) {
+        // ======================= MMA issuer =======================
+        for (int b = 0; b < nblk; ++b) {
+            const int ts = b & 1;
+            if (b >= 2) mbar_wait(&S.tempty[ts], (uint32_t)(((b >> 1) - 1) & 1));
+            tc_fence_after();
+            const uint32_t dt = tbase + (uint32_t)ts * 32u;
+            for (int c = 0; c < nchunk; ++c) {
+                const int gch = b * nchunk + c;
+                const int slot = gch % kTcSlots;
+                mbar_wait(&S.full[slot], (uint32_t)((gch / kTcSlots) & 1));
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t abase = smem_u32(Aop + (size_t)slot * kTcChunkBytes);
+                    const uint32_t bbase = smem_u32(Bop) + (uint32_t)(c * 16) * 128u;
+#pragma unroll
+                    for (int s = 0; s < kTcChunk / 8; ++s) {
+                        const uint64_t ad = umma_desc(abase + (uint32_t)s * 256u, 128u, 2048u);
+                        const uint64_t bd = umma_desc(bbase + (uint32_t)s * 256u, 128u, sboB);
+                        tc_mma(dt, ad, bd, (c > 0 || s > 0) ? 1u : 0u);
+                    }
+                    tc_commit(&S.empty[slot]);
+                    if (c == nchunk - 1) tc_commit(&S.tfull[ts]);
+                }
+                __syncwarp();
+            }
+        }
+    } else {
+        // ======================= epilogue =======================
+        const int ew = warp - kTcEpi0;          // 0..3
+        const int quad = warp & 3;              // TMEM lane quadrant of this warp
+        const int brow = quad * 32 + lane;      // block row of this lane
+        for (int b = 0; b < nblk; ++b) {
+            const int ts = b & 1;
+            mbar_wait(&S.tfull[ts], (uint32_t)((b >> 1) & 1));
+            mbar_wait(&S.xready[ts], (uint32_t)((b >> 1) & 1));
+            tc_fence_after();
+            float dot[32];
+            tmem_ld32(tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 32u, dot);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.tempty[ts]);
+            const uint32_t msk = S.rmask[ts][brow];
+            const float xn = S.xn[ts][brow];
+            const uint32_t prow = S.rpos[ts][brow];
+            if (a.dbg && item == 0 && b == 0) {
+                for (int j = 0; j < 32; ++j) a.dbg[brow * 32 + j] = dot[j];
+                a.dbg[4096 + brow] = xn;
+                a.dbg[4096 + 128 + brow] = __uint_as_float(prow);
+                a.dbg[4096 + 256 + brow] = __uint_as_float(msk);
+                if (brow < 32) a.dbg[4096 + 384 + brow] = S.qn[brow];
+            }
+            // Screen with bounds: |~d2 - d2| <= m = 4e-3 (|q'|^2 + |x'|^2) + 1e-5 ~d2.  U_j = k-th
+            // smallest (~d2 + m) seen so far bounds the exact k-th from above; a pair with
+            // ~d2 - m > U_j can never enter the top-k.  Kept pairs are buffered per (item, query)
+            // and rescored exactly only at the end, against the final (tightest) U_j.
+            const uint32_t wmask = __reduce_or_sync(BLSH_FULL, msk);
+#pragma unroll
+            for (int j = 0; j < 32; ++j) {     // unrolled: dot[j] stays in registers
+                if (!((wmask >> j) & 1u)) continue;
+                const bool has = (msk >> j) & 1u;
+                const float qn = S.qn[j];
+                const float approx = qn + xn - 2.0f * dot[j];
+                const float m = 4e-3f * (qn + xn) + 1e-5f * fabsf(approx) + 1e-30f;
+                const float lo = approx - m, up = approx + m;
+                const float U = __uint_as_float(S.thr[j]);
+                const bool keep = has && lo <= U;
+                const unsigned km = __ballot_sync(BLSH_FULL, keep);
+                if (!km) continue;
+                // upper-bound list (k smallest ~d2 + m), updated by lane 0 under the query's lock
+                const unsigned um = __ballot_sync(BLSH_FULL, keep && up < U);
+                if (um) {
+                    // serial insertion of every lane's upper bound (lane order), lane 0 holds the lock
+                    if (lane == 0) {
+                        while (atomicCAS(&S.lock[j], 0, 1) != 0) {
+                        }
+                        __threadfence_block();
+                    }
+                    __syncwarp();
+                    unsigned mm = um;
+                    while (mm) {
+                        const int src = __ffs(mm) - 1;
+                        mm &= mm - 1;
+                        const float v = __shfl_sync(BLSH_FULL, up, src);
+                        if (lane == 0) {
+                            volatile float* UL = S.ul[j];
+                            if (v < UL[k - 1]) {
+                                int p = k - 1;
+                                while (p > 0 && UL[p - 1] > v) { UL[p] = UL[p - 1]; --p; }
+                                UL[p] = v;
+                                S.thr[j] = __float_as_uint(UL[k - 1]);
+                            }
+                        }
+                    }
+                    __syncwarp();
+                    if (lane == 0) {
+                        __threadfence_block();
+                        atomicExch(&S.lock[j], 0);
+                    }
+                }
+                // buffer the kept pairs: (lower bound bits << 32 | table row)
+                int base = 0;
+                if (lane == 0) base = atomicAdd(&S.scnt[j], __popc(km));
+                base = __shfl_sync(BLSH_FULL, base, 0);
+                const int at = base + __popc(km & lanemask_lt());
+                if (keep && at < a.scap)
+                    a.sbuf[((size_t)item * QT + j) * a.scap + at] =
+                        ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | prow;
+                // overflow: rescore those pairs now (warp-cooperative, same arithmetic)
+                unsigned om = __ballot_sync(BLSH_FULL, keep && at >= a.scap);
+                while (om) {
+                    const int src = __ffs(om) - 1;
+                    om &= om - 1;
+                    const uint32_t srow = __shfl_sync(BLSH_FULL, prow, src);
+                    const uint32_t sid = __ldg(a.perm + srow);
+                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, Qf + (size_t)j * ds, nv4, lane);
+                    const unsigned long long key = pack_entry(d2, sid);
+                    if (lane == 0) {
+                        while (atomicCAS(&S.lock[j], 0, 1) != 0) {
+                        }
+                        __threadfence_block();
+                        volatile unsigned long long* L = S.tk[j];
+                        if (key < L[k - 1]) {
+                            int p = k - 1;
+                            while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
+                            L[p] = key;
+                        }
+                        __threadfence_block();
+                        atomicExch(&S.lock[j], 0);
+                    }
+                    __syncwarp();
+                }
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.mfree[ts]);
+        }
+        // final: rescore the buffered pairs whose lower bound is <= the final U_j
+        named_bar(2, 4 * 32);
+        unsigned long long rescored = 0;
+        for (int j = ew * 8; j < ew * 8 + 8; ++j) {
+            const float U = __uint_as_float(S.thr[j]);
+            const int cnt = min(S.scnt[j], a.scap);
+            const unsigned long long* B = a.sbuf + ((size_t)item * QT + j) * a.scap;
+            for (int base = 0; base < cnt; base += 32) {
+                const int i = base + lane;
+                const unsigned long long e = i < cnt ? B[i] : ~0ull;
+                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+                unsigned nm = __ballot_sync(BLSH_FULL, need);
+                rescored += __popc(nm);
+                while (nm) {
+                    const int src = __ffs(nm) - 1;
+                    nm &= nm - 1;
+                    const uint32_t srow = (uint32_t)(__shfl_sync(BLSH_FULL, e, src) & 0xFFFFFFFFull);
+                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, Qf + (size_t)j * ds, nv4, lane);
+                    const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
+                    if (lane == 0) {
+                        unsigned long long* L = S.tk[j];
+                        if (key < L[k - 1]) {
+                            int p = k - 1;
+                            while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
+                            L[p] = key;
+                        }
+                    }
+                    __syncwarp();
+                }
+            }
+            unsigned long long* out = a.partials + ((size_t)item * QT + j) * k;
+            __syncwarp();
+            if (lane < k) out[lane] = S.tk[j][lane];
+        }
+        if (lane == 0 && a.counters) atomicAdd(a.counters + 1, rescored);
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == kTcMmaWarp) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tbase));
+    }
+}

@@ -75,9 +75,9 @@ __global__ void __launch_bounds__(kTiledThreads, 1) k_shortlist_tiled(TiledArgs 
     const int nst = (int)((r1 - r0 + 31) / 32);
     for (int i = threadIdx.x; i < QT * nv4; i += kTiledThreads) {
         const int slot = i / nv4, v = i % nv4;
-        const int64_t qp = tile * QT + slot;
+        const int64_t qp = a.tile_off[tile] + slot;
         float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (qp < a.nq) x = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[qp] * ds)[v];
+        if (qp < a.tile_off[tile + 1]) x = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[qp] * ds)[v];
         reinterpret_cast<float4*>(qs)[(size_t)slot * nv4 + v] = x;
     }
     if (threadIdx.x == 0) {

@@ -283,7 +283,7 @@ def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
     assert ix.stats().tiled == 0
     monkeypatch.delenv("BLSH_SHORTLIST")
     run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
-    assert ix.stats().tiled == 1
+    assert ix.stats().tiled >= 1
 
 
 def test_large_d_uses_fallback(blsh, orc):
@@ -293,3 +293,18 @@ def test_large_d_uses_fallback(blsh, orc):
     ix, ox = build_pair(blsh, orc, X, G=2, M=6, W=3.0)
     run_query_pair(ix, ox, X, Q, 10, probe=1, T=8)
     assert ix.stats().tiled == 0
+
+
+@pytest.mark.parametrize("mode", ["simt", "tc"])
+def test_tiled_shortlist_variants(blsh, orc, c1, monkeypatch, mode):
+    """Both query-tiled short-list kernels (SIMT and the tensor-core screen with
+    exact rescoring) against the oracle, k <= 16 so both are eligible."""
+    X, Q = c1
+    if mode == "simt":
+        monkeypatch.setenv("BLSH_SHORTLIST", "simt")
+    else:
+        monkeypatch.setenv("BLSH_SHORTLIST", "tc")
+    ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=4.0, seed=21)
+    for k, T in [(1, 1), (10, 16), (16, 64)]:
+        run_query_pair(ix, ox, X, Q, k, probe=1 if T > 1 else 0, T=T)
+        assert ix.stats().tiled == (1 if mode == "simt" else 2)
