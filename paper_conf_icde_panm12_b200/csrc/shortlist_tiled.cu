@@ -220,6 +220,7 @@ struct TiledArgs {
     float* dbg;                     // optional (BLSH_TC_DEBUG): item 0, block 0 dots / |x'|^2 / rows
     unsigned long long* sbuf;       // TC: [n_items][QT][scap] buffered (lower bound, row) pairs
     int scap;
+    int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA
 };
 
 struct TopK {
@@ -613,7 +614,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int64_t n_items = 0;
     BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    constexpr int kScap = 256;   // buffered (row, query) pairs per item and query before immediate rescoring
+    constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     partials.ensure(part_bytes + (size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8);
     TiledArgs ta{};
@@ -625,8 +626,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.tile_of = tile_of;
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
+    if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
-    const size_t tc_smem = ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)2 * QT * a.ds * 4 +
+    const size_t tc_smem = ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)QT * a.ds * 4 +
                            (size_t)kTcSlots * kTcChunkBytes;
     const char* mode = std::getenv("BLSH_SHORTLIST");
     // the tensor-core screen is opt-in (BLSH_SHORTLIST=tc) until it beats the SIMT tiled kernel
@@ -663,6 +665,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     BLSH_CUDA(cudaMemcpyAsync(ev, counters, 16, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     *pairs_out = (int64_t)(use_tc ? ev[1] : ev[0]);   // TC: exact rescorings after the screen
+    if (use_tc && std::getenv("BLSH_TC_MODE"))
+        std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld\n", (long long)n_items, ev[0], ev[1],
+                     (long long)total_rows);
     if (ta.dbg) {
         std::vector<float> h(4096 + 512);
         BLSH_CUDA(cudaMemcpy(h.data(), ta.dbg, h.size() * sizeof(float), cudaMemcpyDeviceToHost));

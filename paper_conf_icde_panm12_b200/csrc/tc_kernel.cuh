@@ -1,35 +1,48 @@
 // tc_kernel.cuh -- query-tiled short-list with a tensor-core screen
 // (included by shortlist_tiled.cu inside its anonymous namespace).
 //
-// For a tile of QT = 32 queries and a 128-row block of the tile's candidate
+// For a tile of <= QT = 32 queries and a 128-row block of the tile's candidate
 // union, the 128 x 32 dot products of the CENTRED vectors (x - c)(q - c),
-// c = the tile's first query, are one tcgen05.mma (kind::tf32, M = 128,
-// N = 32, K = 384 in 48 steps of K = 8) accumulated in TMEM.  The epilogue
-// turns them into approximate distances ~d^2 = |q'|^2 + |x'|^2 - 2 q'.x' and
-// keeps a (row, query) pair only if ~d^2 is within a rigorous margin of the
-// query's current k-th distance; every kept pair is rescored EXACTLY in the
-// fp32 direct form of k_shortlist (R22), so results are identical to the
-// SIMT kernels' -- the tensor cores only decide which pairs need exact work.
+// c = mean of the tile's queries, are one tcgen05.mma chain (kind::tf32,
+// M = 128, N = 32, K = d in steps of 8) accumulated in TMEM.  The epilogue
+// turns them into approximate distances ~d2 = |q'|^2 + |x'|^2 - 2 q'.x' with
+// the bound |~d2 - d2| <= m = 4e-3 (|q'|^2 + |x'|^2) + 1e-5 ~d2 (TF32 operand
+// truncation + fp32 accumulation, with margin).  U_j, the k-th smallest
+// ~d2 + m seen for query j, bounds its exact k-th distance from above, so a
+// pair with ~d2 - m > U_j can never enter the top-k.  Pairs that pass are
+// buffered (lower bound, row) and, after the whole union has been streamed,
+// only those with lower bound <= the final U_j are rescored EXACTLY in the
+// fp32 direct form of k_shortlist (R22).  The tensor cores only decide which
+// pairs need exact work; results equal the SIMT kernels' up to rounding of the
+// direct form (identical to k_shortlist's).
 //
 // Warp roles (13 warps):
-//   0-7  converters: gather the block's rows from HBM (16-byte loads),
-//        subtract c, write the TF32 A operand in the K-major no-swizzle UMMA
-//        layout (8-row x 16-byte core matrices), |x'|^2 per row;
+//   0-7  converters: per block, find each row's table position and query mask
+//        in the tile's segment list, gather the rows from HBM (coalesced
+//        16-byte loads: 8 rows x 64 bytes per instruction, the next chunk's
+//        loads in flight while the current one is converted), subtract c,
+//        write the TF32 A operand in the K-major no-swizzle UMMA layout
+//        (8-row x 16-byte core matrices), |x'|^2 per row;
 //   8    MMA issuer (one elected lane) + TMEM allocation;
-//   9-12 epilogue: tcgen05.ld of the 32 accumulators per row, screen, exact
-//        rescoring (warp-cooperative), per-(warp, query) top-k in smem.
-// Pipelines: 3-slot ring of 64-column A chunks (full / empty mbarriers, the
-// MMA frees a slot with tcgen05.commit), 2 TMEM accumulator slots
-// (tmem_full by commit / tmem_empty by the epilogue), 2 row-metadata slots.
+//   9-12 epilogue: tcgen05.ld of the 32 accumulators of its 32 rows, screen,
+//        per-warp upper-bound lists and per-warp pair buffers (registers and
+//        warp-private memory: no atomics or locks on the hot path), final
+//        exact rescoring.
+// Pipelines: 4-slot ring of 64-column A chunks (full / empty mbarriers; the
+// MMA frees a slot with tcgen05.commit), 4 TMEM accumulator slots and 4
+// row-metadata slots (tmem_full by commit, tmem_empty / meta_free by the
+// epilogue).
 
 constexpr int kTcRows = 128;               // M
 constexpr int kTcChunk = 64;               // K columns per A chunk
-constexpr int kTcSlots = 3;                // A chunk ring
+constexpr int kTcSlots = 4;                // A chunk ring
+constexpr int kTcBlk = 4;                  // TMEM / metadata slots
 constexpr int kTcConv = 8;                 // converter warps
 constexpr int kTcMmaWarp = 8;
 constexpr int kTcEpi0 = 9;                 // first epilogue warp
 constexpr int kTcThreads = 13 * 32;
 constexpr int kTcMaxK = 16;                // k supported by the TC path
+constexpr int kTcScap = 96;                // buffered pairs per (item, query, epilogue warp)
 constexpr uint32_t kTcChunkBytes = kTcRows * kTcChunk * 4;   // 32 KB
 // instruction descriptor: D f32, A/B tf32, K-major both, N = 32, M = 128
 constexpr uint32_t kTcIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((32u >> 3) << 17) | ((128u >> 4) << 24);
@@ -74,17 +87,16 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 struct TcSmem {
     uint64_t full[kTcSlots], empty[kTcSlots];
-    uint64_t tfull[2], tempty[2], xready[2], mfree[2];
+    uint64_t tfull[kTcBlk], tempty[kTcBlk], xready[kTcBlk], mfree[kTcBlk];
     uint32_t tmem_base;
-    uint32_t thr[QT];                   // shared screen threshold (fp32 bits of the best k-th d^2)
-    float qn[QT];                       // |q'|^2
-    uint32_t rpos[2][kTcRows];          // table row of each block row
-    uint32_t rmask[2][kTcRows];         // query mask of each block row (0 = padding)
-    float xn[2][kTcRows];               // |x'|^2
-    unsigned long long tk[QT][kTcMaxK];      // per query sorted top-k (shared by the epilogue warps)
-    int lock[QT];                            // per query spinlock guarding tk[q] / ul[q]
-    float ul[QT][kTcMaxK];                   // per query k smallest upper bounds ~d2 + m (thr = ul[q][k-1])
-    int scnt[QT];                            // buffered pairs per query
+    alignas(16) float qn[QT];                // |q'|^2
+    uint32_t rpos[kTcBlk][kTcRows];          // table row of each block row
+    uint32_t rmask[kTcBlk][kTcRows];         // query mask of each block row (0 = padding)
+    float xn[kTcBlk][kTcRows];               // |x'|^2
+    alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
+    int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
+    unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
+    int lock[QT];                            // guards tk[q] during overflow rescoring
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
 };
 
@@ -94,7 +106,7 @@ __device__ __forceinline__ float exact_d2_warp(const float* __restrict__ x, cons
     float p = 0.f;
     for (int v = lane; v < nv4; v += 32) {
         const float4 a = __ldg(reinterpret_cast<const float4*>(x) + v);
-        const float4 b = reinterpret_cast<const float4*>(q)[v];   // query row in shared memory
+        const float4 b = __ldg(reinterpret_cast<const float4*>(q) + v);
         const float dx = b.x - a.x, dy = b.y - a.y, dz = b.z - a.z, dw = b.w - a.w;
         p = fmaf(dx, dx, p);
         p = fmaf(dy, dy, p);
@@ -106,6 +118,14 @@ __device__ __forceinline__ float exact_d2_warp(const float* __restrict__ x, cons
     return p;
 }
 
+__device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned long long key) {
+    if (key < L[k - 1]) {
+        int p = k - 1;
+        while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
+        L[p] = key;
+    }
+}
+
 __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     extern __shared__ __align__(1024) unsigned char smraw[];
     TcSmem& S = *reinterpret_cast<TcSmem*>(smraw);
@@ -113,7 +133,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     unsigned char* opbase = smraw + ((sizeof(TcSmem) + 1023) & ~size_t(1023));
     unsigned char* Bop = opbase;                                    // [QT x ds] tf32, UMMA K-major
     unsigned char* Aop = Bop + (size_t)QT * ds * 4;                 // [kTcSlots][128 x 64] tf32
-    float* Qf = reinterpret_cast<float*>(Aop + (size_t)kTcSlots * kTcChunkBytes);   // [QT][ds] original queries
+    float* Qf = reinterpret_cast<float*>(Aop);                      // setup only: original queries (aliases A)
     const uint32_t sboB = (uint32_t)kp_total * 128u;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t item = blockIdx.x;
@@ -166,19 +186,16 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             }
         }
         S.qn[n] = s;
-        S.thr[n] = 0x7F800000u;   // +inf
+        S.lock[n] = 0;
     }
-    for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) {
-        (&S.tk[0][0])[i] = kEmpty;
-        (&S.ul[0][0])[i] = __int_as_float(0x7F800000);
-    }
-    if (threadIdx.x < QT) { S.lock[threadIdx.x] = 0; S.scnt[threadIdx.x] = 0; }
+    for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) (&S.tk[0][0])[i] = kEmpty;
+    if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kTcSlots; ++s) {
             mbar_init(&S.full[s], kTcConv);
             mbar_init(&S.empty[s], 1);
         }
-        for (int s = 0; s < 2; ++s) {
+        for (int s = 0; s < kTcBlk; ++s) {
             mbar_init(&S.tfull[s], 1);
             mbar_init(&S.tempty[s], 4);
             mbar_init(&S.xready[s], kTcConv);
@@ -187,12 +204,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == kTcMmaWarp) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 64;" ::"r"(smem_u32(&S.tmem_base)));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(smem_u32(&S.tmem_base)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B operand visible to the tensor core
     tc_fence_before();
-    __syncthreads();
+    __syncthreads();                                                // Qf (aliasing the A ring) is dead from here
     tc_fence_after();
     const uint32_t tbase = S.tmem_base;
 
@@ -216,8 +233,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         // contiguous bytes of a core matrix, bank-conflict free).
         const int rsub = lane & 7, ksub = lane >> 3;
         for (int b = 0; b < nblk; ++b) {
-            const int ms = b & 1;
-            if (b >= 2) mbar_wait(&S.mfree[ms], (uint32_t)(((b >> 1) - 1) & 1));
+            const int ms = b & (kTcBlk - 1);
+            if (b >= kTcBlk) mbar_wait(&S.mfree[ms], (uint32_t)(((b / kTcBlk) - 1) & 1));
             const int64_t bstart = r0 + (int64_t)b * kTcRows;
             // the block's 128 rows lie in the 128 segments starting at cs (each has >= 1 row)
             Seg sw[4];
@@ -269,7 +286,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 for (int it = 0; it < 8; ++it) {
                     const int kp = c * 16 + (it >> 1) * 4 + ksub;
                     const bool vv = (it & 1) ? v1 : v0;
-                    v[it] = vv ? __ldg(((it & 1) ? x1 : x0) + kp) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    v[it] = (vv && !(a.dbgmode & 2)) ? __ldg(((it & 1) ? x1 : x0) + kp) : make_float4(0.f, 0.f, 0.f, 0.f);
                 }
             };
             auto convert_chunk = [&](int c, const float4* v) {
@@ -321,8 +338,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     } else if (warp == kTcMmaWarp) {
         // ======================= MMA issuer =======================
         for (int b = 0; b < nblk; ++b) {
-            const int ts = b & 1;
-            if (b >= 2) mbar_wait(&S.tempty[ts], (uint32_t)(((b >> 1) - 1) & 1));
+            const int ts = b & (kTcBlk - 1);
+            if (b >= kTcBlk) mbar_wait(&S.tempty[ts], (uint32_t)(((b / kTcBlk) - 1) & 1));
             tc_fence_after();
             const uint32_t dt = tbase + (uint32_t)ts * 32u;
             for (int c = 0; c < nchunk; ++c) {
@@ -337,7 +354,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                     for (int s = 0; s < kTcChunk / 8; ++s) {
                         const uint64_t ad = umma_desc(abase + (uint32_t)s * 256u, 128u, 2048u);
                         const uint64_t bd = umma_desc(bbase + (uint32_t)s * 256u, 128u, sboB);
-                        tc_mma(dt, ad, bd, (c > 0 || s > 0) ? 1u : 0u);
+                        if (!(a.dbgmode & 4)) tc_mma(dt, ad, bd, (c > 0 || s > 0) ? 1u : 0u);
                     }
                     tc_commit(&S.empty[slot]);
                     if (c == nchunk - 1) tc_commit(&S.tfull[ts]);
@@ -350,19 +367,29 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         const int ew = warp - kTcEpi0;          // 0..3
         const int quad = warp & 3;              // TMEM lane quadrant of this warp
         const int brow = quad * 32 + lane;      // block row of this lane
+        float my_qn = lane < QT ? S.qn[lane] : 0.f;     // lane j holds query j's values
+        float my_U = __int_as_float(0x7F800000);        // this warp's k-th smallest upper bound for query j
+        float ulr[kTcMaxK];                             // lane j: this warp's sorted upper bounds of query j
+#pragma unroll
+        for (int p = 0; p < kTcMaxK; ++p) ulr[p] = __int_as_float(0x7F800000);
+        int my_cnt = 0;                                 // this warp's buffered pairs for query j
+        unsigned long long* SB = a.sbuf + ((size_t)item * QT * 4 + ew) * kTcScap;   // + j * 4 * kTcScap
         for (int b = 0; b < nblk; ++b) {
-            const int ts = b & 1;
-            mbar_wait(&S.tfull[ts], (uint32_t)((b >> 1) & 1));
-            mbar_wait(&S.xready[ts], (uint32_t)((b >> 1) & 1));
+            const int ts = b & (kTcBlk - 1);
+            mbar_wait(&S.tfull[ts], (uint32_t)((b / kTcBlk) & 1));
+            mbar_wait(&S.xready[ts], (uint32_t)((b / kTcBlk) & 1));
             tc_fence_after();
             float dot[32];
             tmem_ld32(tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 32u, dot);
             tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&S.tempty[ts]);
             const uint32_t msk = S.rmask[ts][brow];
             const float xn = S.xn[ts][brow];
             const uint32_t prow = S.rpos[ts][brow];
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&S.tempty[ts]);
+                mbar_arrive(&S.mfree[ts]);
+            }
             if (a.dbg && item == 0 && b == 0) {
                 for (int j = 0; j < 32; ++j) a.dbg[brow * 32 + j] = dot[j];
                 a.dbg[4096 + brow] = xn;
@@ -370,130 +397,129 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 a.dbg[4096 + 256 + brow] = __uint_as_float(msk);
                 if (brow < 32) a.dbg[4096 + 384 + brow] = S.qn[brow];
             }
-            // Screen with bounds: |~d2 - d2| <= m = 4e-3 (|q'|^2 + |x'|^2) + 1e-5 ~d2.  U_j = k-th
-            // smallest (~d2 + m) seen so far bounds the exact k-th from above; a pair with
-            // ~d2 - m > U_j can never enter the top-k.  Kept pairs are buffered per (item, query)
-            // and rescored exactly only at the end, against the final (tightest) U_j.
-            const uint32_t wmask = __reduce_or_sync(BLSH_FULL, msk);
+            // pass 1 (branch-free, all 32 queries): which (row, query) pairs pass the screen
+            uint32_t kmask = 0;
+            if (!(a.dbgmode & 1)) {
+#pragma unroll
+                for (int j4 = 0; j4 < 8; ++j4) {
+                    const float4 qn4 = reinterpret_cast<const float4*>(S.qn)[j4];
+                    const uint4 um4 = reinterpret_cast<const uint4*>(S.umin)[j4];
+                    const float qv[4] = {qn4.x, qn4.y, qn4.z, qn4.w};
+                    const uint32_t uv[4] = {um4.x, um4.y, um4.z, um4.w};
+#pragma unroll
+                    for (int t = 0; t < 4; ++t) {
+                        const int j = 4 * j4 + t;
+                        const float approx = qv[t] + xn - 2.0f * dot[j];
+                        const float m = 4e-3f * (qv[t] + xn) + 1e-5f * fabsf(approx) + 1e-30f;
+                        if (approx - m <= __uint_as_float(uv[t])) kmask |= 1u << j;
+                    }
+                }
+                kmask &= msk;
+            }
+            const uint32_t wmask = __reduce_or_sync(BLSH_FULL, kmask);
+            // pass 2 (only queries with a kept pair in this warp): bounds, buffers
 #pragma unroll
             for (int j = 0; j < 32; ++j) {     // unrolled: dot[j] stays in registers
                 if (!((wmask >> j) & 1u)) continue;
-                const bool has = (msk >> j) & 1u;
-                const float qn = S.qn[j];
+                const bool has = (kmask >> j) & 1u;
+                const float qn = __shfl_sync(BLSH_FULL, my_qn, j);
+                const float Uown = __shfl_sync(BLSH_FULL, my_U, j);
+                const float U = fminf(Uown, __uint_as_float(S.umin[j]));   // any warp's bound is valid
                 const float approx = qn + xn - 2.0f * dot[j];
                 const float m = 4e-3f * (qn + xn) + 1e-5f * fabsf(approx) + 1e-30f;
                 const float lo = approx - m, up = approx + m;
-                const float U = __uint_as_float(S.thr[j]);
                 const bool keep = has && lo <= U;
                 const unsigned km = __ballot_sync(BLSH_FULL, keep);
                 if (!km) continue;
-                // upper-bound list (k smallest ~d2 + m), updated by lane 0 under the query's lock
-                const unsigned um = __ballot_sync(BLSH_FULL, keep && up < U);
+                // this warp's upper-bound list of query j lives in lane j's registers
+                unsigned um = __ballot_sync(BLSH_FULL, keep && up < Uown);
                 if (um) {
-                    // serial insertion of every lane's upper bound (lane order), lane 0 holds the lock
-                    if (lane == 0) {
-                        while (atomicCAS(&S.lock[j], 0, 1) != 0) {
-                        }
-                        __threadfence_block();
-                    }
-                    __syncwarp();
-                    unsigned mm = um;
-                    while (mm) {
-                        const int src = __ffs(mm) - 1;
-                        mm &= mm - 1;
+                    while (um) {
+                        const int src = __ffs(um) - 1;
+                        um &= um - 1;
                         const float v = __shfl_sync(BLSH_FULL, up, src);
-                        if (lane == 0) {
-                            volatile float* UL = S.ul[j];
-                            if (v < UL[k - 1]) {
-                                int p = k - 1;
-                                while (p > 0 && UL[p - 1] > v) { UL[p] = UL[p - 1]; --p; }
-                                UL[p] = v;
-                                S.thr[j] = __float_as_uint(UL[k - 1]);
-                            }
+                        if (lane == j) {
+#pragma unroll
+                            for (int p = kTcMaxK - 1; p > 0; --p)
+                                ulr[p] = ulr[p - 1] > v ? ulr[p - 1] : (ulr[p] > v ? v : ulr[p]);
+                            ulr[0] = ulr[0] > v ? v : ulr[0];
                         }
                     }
-                    __syncwarp();
-                    if (lane == 0) {
-                        __threadfence_block();
-                        atomicExch(&S.lock[j], 0);
+                    if (lane == j) {
+                        float kth = ulr[0];
+#pragma unroll
+                        for (int p = 1; p < kTcMaxK; ++p)
+                            if (p == k - 1) kth = ulr[p];
+                        if (kth < my_U) {
+                            my_U = kth;
+                            atomicMin(&S.umin[j], __float_as_uint(kth));
+                        }
                     }
                 }
                 // buffer the kept pairs: (lower bound bits << 32 | table row)
-                int base = 0;
-                if (lane == 0) base = atomicAdd(&S.scnt[j], __popc(km));
-                base = __shfl_sync(BLSH_FULL, base, 0);
+                const int base = __shfl_sync(BLSH_FULL, my_cnt, j);
                 const int at = base + __popc(km & lanemask_lt());
-                if (keep && at < a.scap)
-                    a.sbuf[((size_t)item * QT + j) * a.scap + at] =
-                        ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | prow;
+                if (keep && at < kTcScap)
+                    SB[(size_t)j * 4 * kTcScap + at] = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | prow;
+                if (lane == j) my_cnt = base + __popc(km);
                 // overflow: rescore those pairs now (warp-cooperative, same arithmetic)
-                unsigned om = __ballot_sync(BLSH_FULL, keep && at >= a.scap);
+                unsigned om = __ballot_sync(BLSH_FULL, keep && at >= kTcScap);
                 while (om) {
                     const int src = __ffs(om) - 1;
                     om &= om - 1;
                     const uint32_t srow = __shfl_sync(BLSH_FULL, prow, src);
-                    const uint32_t sid = __ldg(a.perm + srow);
-                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, Qf + (size_t)j * ds, nv4, lane);
-                    const unsigned long long key = pack_entry(d2, sid);
+                    const float* qq = a.Q + (size_t)a.qorder[q0 + j] * ds;
+                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, qq, nv4, lane);
+                    const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
                     if (lane == 0) {
                         while (atomicCAS(&S.lock[j], 0, 1) != 0) {
                         }
                         __threadfence_block();
-                        volatile unsigned long long* L = S.tk[j];
-                        if (key < L[k - 1]) {
-                            int p = k - 1;
-                            while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
-                            L[p] = key;
-                        }
+                        tk_insert(S.tk[j], k, key);
                         __threadfence_block();
                         atomicExch(&S.lock[j], 0);
                     }
                     __syncwarp();
                 }
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&S.mfree[ts]);
         }
-        // final: rescore the buffered pairs whose lower bound is <= the final U_j
+        if (lane < QT) S.scnt[ew][lane] = my_cnt;
+        if (a.counters && lane < QT && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
+        // ---- final: rescore the buffered pairs whose lower bound is <= U_j ----
         named_bar(2, 4 * 32);
         unsigned long long rescored = 0;
-        for (int j = ew * 8; j < ew * 8 + 8; ++j) {
-            const float U = __uint_as_float(S.thr[j]);
-            const int cnt = min(S.scnt[j], a.scap);
-            const unsigned long long* B = a.sbuf + ((size_t)item * QT + j) * a.scap;
-            for (int base = 0; base < cnt; base += 32) {
-                const int i = base + lane;
-                const unsigned long long e = i < cnt ? B[i] : ~0ull;
-                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
-                unsigned nm = __ballot_sync(BLSH_FULL, need);
-                rescored += __popc(nm);
-                while (nm) {
-                    const int src = __ffs(nm) - 1;
-                    nm &= nm - 1;
-                    const uint32_t srow = (uint32_t)(__shfl_sync(BLSH_FULL, e, src) & 0xFFFFFFFFull);
-                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, Qf + (size_t)j * ds, nv4, lane);
-                    const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
-                    if (lane == 0) {
-                        unsigned long long* L = S.tk[j];
-                        if (key < L[k - 1]) {
-                            int p = k - 1;
-                            while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
-                            L[p] = key;
-                        }
+        for (int j = ew; j < nqt; j += 4) {
+            const float U = __uint_as_float(S.umin[j]);
+            const float* qq = a.Q + (size_t)a.qorder[q0 + j] * ds;
+            for (int w = 0; w < 4; ++w) {
+                const int cnt = min(S.scnt[w][j], kTcScap);
+                const unsigned long long* Bf = a.sbuf + (((size_t)item * QT + j) * 4 + w) * kTcScap;
+                for (int base = 0; base < cnt; base += 32) {
+                    const int i = base + lane;
+                    const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
+                    const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+                    unsigned nm = __ballot_sync(BLSH_FULL, need);
+                    rescored += __popc(nm);
+                    while (nm) {
+                        const int src = __ffs(nm) - 1;
+                        nm &= nm - 1;
+                        const uint32_t srow = (uint32_t)(__shfl_sync(BLSH_FULL, e, src) & 0xFFFFFFFFull);
+                        const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, qq, nv4, lane);
+                        const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
+                        if (lane == 0) tk_insert(S.tk[j], k, key);
+                        __syncwarp();
                     }
-                    __syncwarp();
                 }
             }
             unsigned long long* out = a.partials + ((size_t)item * QT + j) * k;
-            __syncwarp();
             if (lane < k) out[lane] = S.tk[j][lane];
         }
-        if (lane == 0 && a.counters) atomicAdd(a.counters + 1, rescored);
+        if (lane == 0 && a.counters && rescored) atomicAdd(a.counters + 1, rescored);
     }
     tc_fence_before();
     __syncthreads();
     if (warp == kTcMmaWarp) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 64;" ::"r"(tbase));
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tbase));
     }
 }
