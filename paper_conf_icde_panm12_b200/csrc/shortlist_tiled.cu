@@ -187,6 +187,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+// Warp-wide wait (every caller is a whole warp).  Lanes may leave the try_wait
+// loop on different iterations; the __syncwarp reconverges them so that the
+// warp collectives that follow take the converged fast path.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n\t.reg .pred p;\n"
@@ -195,6 +198,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
         "r"(parity)
         : "memory");
+    __syncwarp();
 }
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
@@ -220,7 +224,8 @@ struct TiledArgs {
     float* dbg;                     // optional (BLSH_TC_DEBUG): item 0, block 0 dots / |x'|^2 / rows
     unsigned long long* sbuf;       // TC: [n_items][QT][scap] buffered (lower bound, row) pairs
     int scap;
-    int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA
+    int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA, 32 phase timers
+    unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
 };
 
 struct TopK {
@@ -641,6 +646,12 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         BLSH_CUDA(cudaMemsetAsync(dbgbuf.p, 0, (4096 + 512) * sizeof(float), s));
         ta.dbg = dbgbuf.as<float>();
     }
+    DevBuf tsbuf;
+    if (use_tc && (ta.dbgmode & 32) && n_items > 0) {
+        tsbuf.alloc((size_t)n_items * 8 * 8);
+        BLSH_CUDA(cudaMemsetAsync(tsbuf.p, 0, (size_t)n_items * 8 * 8, s));
+        ta.tstamp = tsbuf.as<unsigned long long>();
+    }
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_tc) {
@@ -668,6 +679,17 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (use_tc && std::getenv("BLSH_TC_MODE"))
         std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld\n", (long long)n_items, ev[0], ev[1],
                      (long long)total_rows);
+    if (ta.tstamp) {   // mean phase durations over items (us)
+        std::vector<unsigned long long> h((size_t)n_items * 8);
+        BLSH_CUDA(cudaMemcpy(h.data(), ta.tstamp, h.size() * 8, cudaMemcpyDeviceToHost));
+        double acc[8] = {0};
+        for (int64_t i = 0; i < n_items; ++i)
+            for (int p = 1; p < 8; ++p)
+                if (h[i * 8 + p]) acc[p] += (double)(h[i * 8 + p] - h[i * 8]) * 1e-3;
+        std::fprintf(stderr, "[tc] phase us after start: setup %.1f conv %.1f mma %.1f epi %.1f sync %.1f compact %.1f end %.1f\n",
+                     acc[1] / n_items, acc[2] / n_items, acc[3] / n_items, acc[4] / n_items, acc[5] / n_items,
+                     acc[6] / n_items, acc[7] / n_items);
+    }
     if (ta.dbg) {
         std::vector<float> h(4096 + 512);
         BLSH_CUDA(cudaMemcpy(h.data(), ta.dbg, h.size() * sizeof(float), cudaMemcpyDeviceToHost));

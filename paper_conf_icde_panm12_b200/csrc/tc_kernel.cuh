@@ -97,7 +97,10 @@ struct TcSmem {
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
     unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
     int lock[QT];                            // guards tk[q] during overflow rescoring
+    int rcnt[QT];                            // final: pairs to rescore per query
+    int roff[QT + 1];                        // final: their exclusive prefix
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
+    float sap[4][QT][32];                    // per epilogue warp: approximate d^2 [query][lane]
 };
 
 // exact fp32 direct-form d^2 (same partial-sum structure as k_shortlist: 12-term lanes + butterfly)
@@ -118,11 +121,71 @@ __device__ __forceinline__ float exact_d2_warp(const float* __restrict__ x, cons
     return p;
 }
 
+// exact fp32 direct-form d^2 by one thread, in the partial-sum structure of the
+// SIMT tiled kernel's score_rows (blocks of 16 float4, two 32-term chains each,
+// blocks summed in order): TC and SIMT tiled results are bit-identical.  The
+// block's 16 row loads are issued before any arithmetic (memory-level parallelism).
+__device__ __forceinline__ float exact_d2_thread(const float4* __restrict__ x, const float4* __restrict__ q, int nv4) {
+    float tot = 0.f;
+    for (int vb = 0; vb < nv4; vb += 16) {
+        const int ne = min(16, nv4 - vb);
+        float4 xv[16];
+#pragma unroll
+        for (int v = 0; v < 16; ++v)
+            if (v < ne) xv[v] = __ldg(x + vb + v);
+        float a0 = 0.f, a1 = 0.f;
+#pragma unroll
+        for (int v = 0; v < 16; ++v) {
+            if (v < ne) {
+                const float4 qq = __ldg(q + vb + v);
+                const float dx = qq.x - xv[v].x, dy = qq.y - xv[v].y, dz = qq.z - xv[v].z, dw = qq.w - xv[v].w;
+                a0 = fmaf(dx, dx, a0);
+                a1 = fmaf(dy, dy, a1);
+                a0 = fmaf(dz, dz, a0);
+                a1 = fmaf(dw, dw, a1);
+            }
+        }
+        tot += a0 + a1;
+    }
+    return tot;
+}
+
 __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned long long key) {
     if (key < L[k - 1]) {
         int p = k - 1;
         while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
         L[p] = key;
+    }
+}
+
+// Overflowing pairs of one query (lanes in om, table row in prow): exact d^2 now,
+// inserted into the query's shared top-k under its lock.  Rare; kept out of line.
+__device__ __noinline__ void tc_overflow(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
+                                         unsigned om, uint32_t prow, int lane) {
+    const int nv4 = a.ds >> 2;
+    while (om) {
+        const int src = __ffs(om) - 1;
+        om &= om - 1;
+        const uint32_t srow = __shfl_sync(BLSH_FULL, prow, src);
+        const float d2 = exact_d2_warp(a.Xp + (size_t)srow * a.ds, qq, nv4, lane);
+        const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
+        if (lane == 0) {
+            while (atomicCAS(lock, 0, 1) != 0) {
+            }
+            __threadfence_block();
+            tk_insert(tk, a.k, key);
+            __threadfence_block();
+            atomicExch(lock, 0);
+        }
+        __syncwarp();
+    }
+}
+
+__device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p) {
+    if (a.tstamp) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        a.tstamp[item * 8 + p] = t;
     }
 }
 
@@ -149,6 +212,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     const int nblk = (int)((r1 - r0 + kTcRows - 1) / kTcRows);
     const int nchunk = ds / kTcChunk;
     const int k = a.k;
+    if (threadIdx.x == 0) tc_stamp(a, item, 0);
     // ---- setup: queries, centre c = mean of the tile's queries, B operand (q - c), |q'|^2 ----
     const int64_t q0 = a.tile_off[tile];
     const int nqt = (int)(a.tile_off[tile + 1] - q0);
@@ -175,18 +239,21 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         }
         *reinterpret_cast<float4*>(Bop + (size_t)(n >> 3) * sboB + (size_t)kp * 128 + (n & 7) * 16) = v;
     }
-    if (threadIdx.x < QT) {
-        const int n = threadIdx.x;
+    for (int n = warp; n < QT; n += kTcThreads / 32) {   // |q'|^2: one warp per query
         float s = 0.f;
         if (n < nqt) {
             const float* qq = Qf + (size_t)n * ds;
-            for (int j = 0; j < ds; ++j) {
+            for (int j = lane; j < ds; j += 32) {
                 const float e = qq[j] - cen[j];
                 s = fmaf(e, e, s);
             }
         }
-        S.qn[n] = s;
-        S.lock[n] = 0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(BLSH_FULL, s, o);
+        if (lane == 0) {
+            S.qn[n] = s;
+            S.lock[n] = 0;
+        }
     }
     for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) (&S.tk[0][0])[i] = kEmpty;
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
@@ -212,6 +279,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     __syncthreads();                                                // Qf (aliasing the A ring) is dead from here
     tc_fence_after();
     const uint32_t tbase = S.tmem_base;
+    if (threadIdx.x == 0) tc_stamp(a, item, 1);
 
     if (warp < kTcConv) {
         // ======================= converters =======================
@@ -335,6 +403,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             __syncwarp();
             if (lane == 0) mbar_arrive(&S.xready[ms]);
         }
+        if (threadIdx.x == 0) tc_stamp(a, item, 2);
     } else if (warp == kTcMmaWarp) {
         // ======================= MMA issuer =======================
         for (int b = 0; b < nblk; ++b) {
@@ -362,6 +431,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 __syncwarp();
             }
         }
+        if (lane == 0) tc_stamp(a, item, 3);
     } else {
         // ======================= epilogue =======================
         const int ew = warp - kTcEpi0;          // 0..3
@@ -412,20 +482,23 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                         const float approx = qv[t] + xn - 2.0f * dot[j];
                         const float m = 4e-3f * (qv[t] + xn) + 1e-5f * fabsf(approx) + 1e-30f;
                         if (approx - m <= __uint_as_float(uv[t])) kmask |= 1u << j;
+                        S.sap[ew][j][lane] = approx;   // for pass 2 (dynamic j)
                     }
                 }
                 kmask &= msk;
             }
             const uint32_t wmask = __reduce_or_sync(BLSH_FULL, kmask);
-            // pass 2 (only queries with a kept pair in this warp): bounds, buffers
-#pragma unroll
-            for (int j = 0; j < 32; ++j) {     // unrolled: dot[j] stays in registers
-                if (!((wmask >> j) & 1u)) continue;
+            __syncwarp();
+            // pass 2 (only queries with a kept pair in this warp): bounds, buffers.  Not unrolled
+            // (a 32-fold copy of this body thrashes the instruction cache): the approximate
+            // distances come back from shared memory.
+            for (uint32_t wm = wmask; wm; wm &= wm - 1) {
+                const int j = __ffs(wm) - 1;
                 const bool has = (kmask >> j) & 1u;
                 const float qn = __shfl_sync(BLSH_FULL, my_qn, j);
                 const float Uown = __shfl_sync(BLSH_FULL, my_U, j);
                 const float U = fminf(Uown, __uint_as_float(S.umin[j]));   // any warp's bound is valid
-                const float approx = qn + xn - 2.0f * dot[j];
+                const float approx = S.sap[ew][j][lane];
                 const float m = 4e-3f * (qn + xn) + 1e-5f * fabsf(approx) + 1e-30f;
                 const float lo = approx - m, up = approx + m;
                 const bool keep = has && lo <= U;
@@ -462,35 +535,32 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 if (keep && at < kTcScap)
                     SB[(size_t)j * 4 * kTcScap + at] = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | prow;
                 if (lane == j) my_cnt = base + __popc(km);
-                // overflow: rescore those pairs now (warp-cooperative, same arithmetic)
-                unsigned om = __ballot_sync(BLSH_FULL, keep && at >= kTcScap);
-                while (om) {
-                    const int src = __ffs(om) - 1;
-                    om &= om - 1;
-                    const uint32_t srow = __shfl_sync(BLSH_FULL, prow, src);
-                    const float* qq = a.Q + (size_t)a.qorder[q0 + j] * ds;
-                    const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, qq, nv4, lane);
-                    const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
-                    if (lane == 0) {
-                        while (atomicCAS(&S.lock[j], 0, 1) != 0) {
-                        }
-                        __threadfence_block();
-                        tk_insert(S.tk[j], k, key);
-                        __threadfence_block();
-                        atomicExch(&S.lock[j], 0);
-                    }
-                    __syncwarp();
-                }
+                // overflow: rescore those pairs now (warp-cooperative)
+                const unsigned om = __ballot_sync(BLSH_FULL, keep && at >= kTcScap);
+                if (om) tc_overflow(a, S.tk[j], &S.lock[j], a.Q + (size_t)a.qorder[q0 + j] * ds, om, prow, lane);
             }
         }
         if (lane < QT) S.scnt[ew][lane] = my_cnt;
         if (a.counters && lane < QT && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
-        // ---- final: rescore the buffered pairs whose lower bound is <= U_j ----
-        named_bar(2, 4 * 32);
-        unsigned long long rescored = 0;
-        for (int j = ew; j < nqt; j += 4) {
+        if (warp == kTcEpi0 && lane == 0) tc_stamp(a, item, 4);
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == kTcMmaWarp) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tbase));
+    }
+    if (threadIdx.x == 0) tc_stamp(a, item, 5);
+    // ---- final (all warps): exact rescoring of the buffered pairs whose lower bound is <= U_j ----
+    // The B operand and the A ring are dead: L[j][0 .. 4 * kTcScap) holds query j's pairs,
+    // first as (j << 32 | table row), then, rescored in place, as packed (d2, id) keys.
+    constexpr int kNW = kTcThreads / 32;
+    constexpr int kPerQ = 4 * kTcScap;
+    unsigned long long* L = reinterpret_cast<unsigned long long*>(opbase);
+    for (int j = warp; j < QT; j += kNW) {              // (a) compact: one warp per query
+        int c = 0;
+        if (j < nqt) {
             const float U = __uint_as_float(S.umin[j]);
-            const float* qq = a.Q + (size_t)a.qorder[q0 + j] * ds;
             for (int w = 0; w < 4; ++w) {
                 const int cnt = min(S.scnt[w][j], kTcScap);
                 const unsigned long long* Bf = a.sbuf + (((size_t)item * QT + j) * 4 + w) * kTcScap;
@@ -498,28 +568,56 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                     const int i = base + lane;
                     const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
                     const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
-                    unsigned nm = __ballot_sync(BLSH_FULL, need);
-                    rescored += __popc(nm);
-                    while (nm) {
-                        const int src = __ffs(nm) - 1;
-                        nm &= nm - 1;
-                        const uint32_t srow = (uint32_t)(__shfl_sync(BLSH_FULL, e, src) & 0xFFFFFFFFull);
-                        const float d2 = exact_d2_warp(a.Xp + (size_t)srow * ds, qq, nv4, lane);
-                        const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
-                        if (lane == 0) tk_insert(S.tk[j], k, key);
-                        __syncwarp();
-                    }
+                    const unsigned nm = __ballot_sync(BLSH_FULL, need);
+                    if (need) L[(size_t)j * kPerQ + c + __popc(nm & lanemask_lt())] = ((unsigned long long)j << 32) | (e & 0xFFFFFFFFull);
+                    c += __popc(nm);
                 }
             }
-            unsigned long long* out = a.partials + ((size_t)item * QT + j) * k;
-            if (lane < k) out[lane] = S.tk[j][lane];
         }
-        if (lane == 0 && a.counters && rescored) atomicAdd(a.counters + 1, rescored);
+        if (lane == 0) S.rcnt[j] = c;
     }
-    tc_fence_before();
     __syncthreads();
-    if (warp == kTcMmaWarp) {
-        tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tbase));
+    if (warp == 0) {                                    // exclusive prefix of the per-query counts
+        const int c = S.rcnt[lane];
+        int inc = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(BLSH_FULL, inc, o);
+            if (lane >= o) inc += t;
+        }
+        S.roff[lane] = inc - c;
+        if (lane == 31) S.roff[32] = inc;
+    }
+    __syncthreads();
+    const int total = S.roff[32];
+    if (threadIdx.x == 0) tc_stamp(a, item, 6);
+    for (int idx = threadIdx.x; idx < total; idx += kTcThreads) {   // (b) one thread per pair
+        int lo2 = 0, hi2 = 32;                                      // query j: roff[j] <= idx < roff[j + 1]
+        while (hi2 - lo2 > 1) {
+            const int m = (lo2 + hi2) >> 1;
+            if (S.roff[m] <= idx) lo2 = m;
+            else hi2 = m;
+        }
+        unsigned long long& e = L[(size_t)lo2 * kPerQ + (idx - S.roff[lo2])];
+        const uint32_t srow = (uint32_t)(e & 0xFFFFFFFFull);
+        const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)srow * ds),
+                                         reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + lo2] * ds), nv4);
+        e = pack_entry(d2, __ldg(a.perm + srow));
+    }
+    __syncthreads();
+    for (int j = warp; j < nqt; j += kNW) {             // (c) per-query top-k of the rescored keys
+        TopK tk{kEmpty, kEmpty};
+        unsigned long long thr = kEmpty;
+        const int c = S.rcnt[j];
+        for (int base = 0; base < c; base += 32)
+            topk_offer(tk, thr, base + lane < c ? L[(size_t)j * kPerQ + base + lane] : kEmpty, k, lane);
+        topk_offer(tk, thr, lane < k ? S.tk[j][lane] : kEmpty, k, lane);   // overflow-path results
+        unsigned long long* out = a.partials + ((size_t)item * QT + j) * k;
+        if (lane < k) out[lane] = tk.e0;
+    }
+    if (threadIdx.x == 0 && a.counters && total) atomicAdd(a.counters + 1, (unsigned long long)total);
+    if (a.tstamp) {
+        __syncthreads();
+        if (threadIdx.x == 0) tc_stamp(a, item, 7);
     }
 }
