@@ -172,6 +172,23 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
     }
 }
 
+// Expand the tiles' segment lists to one (table row, query mask) entry per union row,
+// at rows_off[tile] + (row index within the tile's union): the TC short-list reads its
+// block metadata with one coalesced load instead of walking the segment list.
+__global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ segs, const int32_t* __restrict__ nseg,
+                                                     int segcap, const int64_t* __restrict__ rows_off,
+                                                     uint2* __restrict__ rowinfo) {
+    const int64_t t = blockIdx.x;
+    const Seg* S = segs + (size_t)t * segcap;
+    uint2* out = rowinfo + rows_off[t];
+    const int ns = nseg[t];
+    const int lane = threadIdx.x & 31;
+    for (int sI = threadIdx.x >> 5; sI < ns; sI += 8) {
+        const Seg sg = S[sI];
+        for (uint32_t i = lane; i < sg.len; i += 32) out[sg.off + i] = make_uint2(sg.start + i, sg.mask);
+    }
+}
+
 __global__ void k_tile_items(const int64_t* __restrict__ rows, int64_t ntiles, int chr, int64_t* __restrict__ items) {
     const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (t < ntiles) items[t] = (rows[t] + chr - 1) / chr;
@@ -226,6 +243,8 @@ struct TiledArgs {
     int scap;
     int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA, 32 phase timers
     unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
+    const int64_t* rows_off;        // [ntiles + 1] union rows before each tile
+    const uint2* rowinfo;           // TC: [total rows] (table row, query mask) per union row
 };
 
 struct TopK {
@@ -621,7 +640,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     BLSH_CUDA(cudaStreamSynchronize(s));
     constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
-    partials.ensure(part_bytes + (size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8);
+    const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
+    partials.ensure(part_bytes + sbuf_bytes + (size_t)std::max<int64_t>(total_rows, 1) * 8);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
@@ -631,6 +651,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.tile_of = tile_of;
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
+    ta.rows_off = rows_off;
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
     const size_t tc_smem = ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)QT * a.ds * 4 +
@@ -651,6 +672,13 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         tsbuf.alloc((size_t)n_items * 8 * 8);
         BLSH_CUDA(cudaMemsetAsync(tsbuf.p, 0, (size_t)n_items * 8 * 8, s));
         ta.tstamp = tsbuf.as<unsigned long long>();
+    }
+    if (use_tc && ntiles > 0) {
+        uint2* ri = reinterpret_cast<uint2*>(partials.as<char>() + part_bytes + sbuf_bytes);
+        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(ta.segs, nseg, segcap, rows_off, ri);
+        BLSH_LAUNCH_CHECK();
+        ++*launches;
+        ta.rowinfo = ri;
     }
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {

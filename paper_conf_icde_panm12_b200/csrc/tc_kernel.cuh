@@ -36,6 +36,8 @@
 constexpr int kTcRows = 128;               // M
 constexpr int kTcChunk = 64;               // K columns per A chunk
 constexpr int kTcSlots = 4;                // A chunk ring
+constexpr int kTcAhead = 2;                // chunks in flight ahead of the conversion (kTcSlots - kTcAhead
+                                           // chunks of slack for the MMA to release a slot)
 constexpr int kTcBlk = 4;                  // TMEM / metadata slots
 constexpr int kTcConv = 8;                 // converter warps
 constexpr int kTcMmaWarp = 8;
@@ -283,125 +285,97 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
 
     if (warp < kTcConv) {
         // ======================= converters =======================
-        const Seg* SG = a.segs + (size_t)tile * a.segcap;
-        const int ns = a.nseg[tile];
-        int cs = 0;
-        {
-            int l2 = 0, h2 = ns;
-            while (h2 - l2 > 1) {
-                const int m = (l2 + h2) >> 1;
-                if ((int64_t)SG[m].off <= r0) l2 = m;
-                else h2 = m;
-            }
-            cs = l2;
-        }
-        // Warp w converts block rows [16w, 16w + 16).  Lane -> (row rsub of an 8-row group,
-        // K piece offset ksub): one 16-byte load instruction covers 8 rows x 64 contiguous
-        // bytes (8 cache lines) and one 16-byte store covers 8 rows x one K piece (128
-        // contiguous bytes of a core matrix, bank-conflict free).
+        // Warp w owns block rows [16w, 16w + 16).  Lane -> (row rsub of an 8-row group, K piece
+        // offset ksub).  Rows are copied straight into the A operand's K-major core-matrix layout
+        // with 16-byte cp.async (zero-fill for padding rows), kTcAhead chunks ahead of the
+        // conversion, so the HBM latency is covered by the ring instead of registers; the
+        // conversion (subtract c, |x'|^2) then works in place on shared memory.  Each lane
+        // converts exactly the pieces it copied, so cp.async.wait_group orders the two.
         const int rsub = lane & 7, ksub = lane >> 3;
-        for (int b = 0; b < nblk; ++b) {
+        const int nch_total = nblk * nchunk;
+        uint32_t ip0 = 0, ip1 = 0, isz0 = 0, isz1 = 0;   // issue side: this lane's two rows of the block
+        const uint2* RI = a.rowinfo + a.rows_off[tile];
+        auto fetch = [&](int b) {                         // this lane's metadata entry of block b
+            const int64_t r = r0 + (int64_t)b * kTcRows + 16 * warp + (lane & 15);
+            return (b < nblk && r < r1) ? RI[r] : make_uint2(0u, 0u);
+        };
+        uint2 e_next = fetch(0);                          // prefetched one block ahead
+        auto lookup = [&](int b) {                        // rows of block b: precomputed metadata
             const int ms = b & (kTcBlk - 1);
+            const uint2 e = e_next;
+            e_next = fetch(b + 1);
             if (b >= kTcBlk) mbar_wait(&S.mfree[ms], (uint32_t)(((b / kTcBlk) - 1) & 1));
-            const int64_t bstart = r0 + (int64_t)b * kTcRows;
-            // the block's 128 rows lie in the 128 segments starting at cs (each has >= 1 row)
-            Seg sw[4];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int si = cs + lane + 32 * i;
-                sw[i] = si < ns ? SG[si] : Seg{0u, 0u, 0u, 0xFFFFFFFFu};
-            }
-            uint32_t my_pos = 0, my_mask = 0;   // lanes 0..15: row 16w + lane
-            for (int t2 = 0; t2 < 16; ++t2) {
-                const uint32_t r = (uint32_t)(bstart + 16 * warp + t2);
-                int cnt = 0;
-#pragma unroll
-                for (int i = 0; i < 4; ++i) cnt += __popc(__ballot_sync(BLSH_FULL, sw[i].off <= r));
-                const int idx = cnt - 1, src = idx & 31, reg = idx >> 5;
-                uint32_t st = 0, of = 0, mk = 0;
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                    const uint32_t a0 = __shfl_sync(BLSH_FULL, sw[i].start, src);
-                    const uint32_t a1 = __shfl_sync(BLSH_FULL, sw[i].off, src);
-                    const uint32_t a2 = __shfl_sync(BLSH_FULL, sw[i].mask, src);
-                    if (reg == i) { st = a0; of = a1; mk = a2; }
-                }
-                if (lane == t2) {
-                    const bool v = (int64_t)r < r1;
-                    my_pos = v ? st + (r - of) : 0u;
-                    my_mask = v ? mk : 0u;
-                }
-            }
-            {   // every converter warp advances cs identically (segment of the next block's first row)
-                const uint32_t rn = (uint32_t)(bstart + kTcRows);
-                int cnt = 0;
-#pragma unroll
-                for (int i = 0; i < 4; ++i) cnt += __popc(__ballot_sync(BLSH_FULL, sw[i].off <= rn));
-                cs += cnt > 0 ? cnt - 1 : 0;
-            }
             if (lane < 16) {
-                S.rpos[ms][16 * warp + lane] = my_pos;
-                S.rmask[ms][16 * warp + lane] = my_mask;
+                S.rpos[ms][16 * warp + lane] = e.x;
+                S.rmask[ms][16 * warp + lane] = e.y;
             }
-            const uint32_t p0 = __shfl_sync(BLSH_FULL, my_pos, rsub), p1 = __shfl_sync(BLSH_FULL, my_pos, 8 + rsub);
-            const bool v0 = __shfl_sync(BLSH_FULL, my_mask, rsub) != 0u;
-            const bool v1 = __shfl_sync(BLSH_FULL, my_mask, 8 + rsub) != 0u;
-            const float4* x0 = reinterpret_cast<const float4*>(a.Xp + (size_t)p0 * ds);
-            const float4* x1 = reinterpret_cast<const float4*>(a.Xp + (size_t)p1 * ds);
-            float xs0 = 0.f, xs1 = 0.f;
-            auto load_chunk = [&](int c, float4* v) {
-#pragma unroll
-                for (int it = 0; it < 8; ++it) {
-                    const int kp = c * 16 + (it >> 1) * 4 + ksub;
-                    const bool vv = (it & 1) ? v1 : v0;
-                    v[it] = (vv && !(a.dbgmode & 2)) ? __ldg(((it & 1) ? x1 : x0) + kp) : make_float4(0.f, 0.f, 0.f, 0.f);
-                }
-            };
-            auto convert_chunk = [&](int c, const float4* v) {
-                const int gch = b * nchunk + c;
-                const int slot = gch % kTcSlots;
-                if (gch >= kTcSlots) mbar_wait(&S.empty[slot], (uint32_t)((gch / kTcSlots - 1) & 1));
-                unsigned char* A = Aop + (size_t)slot * kTcChunkBytes;
+            ip0 = __shfl_sync(BLSH_FULL, e.x, rsub);
+            ip1 = __shfl_sync(BLSH_FULL, e.x, 8 + rsub);
+            const bool nol = (a.dbgmode & 2) != 0;
+            isz0 = (__shfl_sync(BLSH_FULL, e.y, rsub) != 0u && !nol) ? 16u : 0u;
+            isz1 = (__shfl_sync(BLSH_FULL, e.y, 8 + rsub) != 0u && !nol) ? 16u : 0u;
+        };
+        auto issue = [&](int g) {                         // cp.async of global chunk g into its slot
+            if (g < nch_total) {
+                const int b = g / nchunk, c = g - b * nchunk;
+                if (c == 0) lookup(b);
+                const int slot = g % kTcSlots;
+                if (g >= kTcSlots) mbar_wait(&S.empty[slot], (uint32_t)((g / kTcSlots - 1) & 1));
+                const uint32_t A = smem_u32(Aop + (size_t)slot * kTcChunkBytes);
+                const float* x0 = a.Xp + (size_t)ip0 * ds;
+                const float* x1 = a.Xp + (size_t)ip1 * ds;
 #pragma unroll
                 for (int it = 0; it < 8; ++it) {
                     const int rg = it & 1;
                     const int kpl = (it >> 1) * 4 + ksub;
-                    const float4 cc = reinterpret_cast<const float4*>(cen)[c * 16 + kpl];
-                    float4 x = v[it];
-                    if (rg ? v1 : v0) {
-                        x.x -= cc.x; x.y -= cc.y; x.z -= cc.z; x.w -= cc.w;
-                        float& xs = rg ? xs1 : xs0;
-                        xs = fmaf(x.x, x.x, xs);
-                        xs = fmaf(x.y, x.y, xs);
-                        xs = fmaf(x.z, x.z, xs);
-                        xs = fmaf(x.w, x.w, xs);
-                    }
-                    *reinterpret_cast<float4*>(A + (size_t)(2 * warp + rg) * 2048 + (size_t)kpl * 128 + rsub * 16) = x;
-                }
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&S.full[slot]);
-            };
-            // the next chunk's loads are in flight while the current chunk is converted
-            float4 va[8], vb[8];
-            load_chunk(0, va);
-            for (int c = 0; c < nchunk; c += 2) {
-                if (c + 1 < nchunk) load_chunk(c + 1, vb);
-                convert_chunk(c, va);
-                if (c + 1 < nchunk) {
-                    if (c + 2 < nchunk) load_chunk(c + 2, va);
-                    convert_chunk(c + 1, vb);
+                    const float* src = (rg ? x1 : x0) + (size_t)(c * 16 + kpl) * 4;
+                    const uint32_t dst = A + (uint32_t)((2 * warp + rg) * 2048 + kpl * 128 + rsub * 16);
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
+                                 "r"(rg ? isz1 : isz0)
+                                 : "memory");
                 }
             }
-            // |x'|^2 per row: reduce over the 4 lanes (ksub) sharing a row
-            xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 8);
-            xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 16);
-            xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 8);
-            xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 16);
-            if (lane < 8) S.xn[ms][16 * warp + lane] = xs0;
-            else if (lane < 16) S.xn[ms][16 * warp + lane] = xs1;
+            asm volatile("cp.async.commit_group;" ::: "memory");   // (possibly empty: uniform group count)
+        };
+        for (int g = 0; g < kTcAhead; ++g) issue(g);
+        float xs0 = 0.f, xs1 = 0.f;
+        for (int g = 0; g < nch_total; ++g) {
+            issue(g + kTcAhead);
+            asm volatile("cp.async.wait_group %0;" ::"n"(kTcAhead) : "memory");   // chunk g has landed
+            const int b = g / nchunk, c = g - b * nchunk;
+            const int slot = g % kTcSlots;
+            unsigned char* A = Aop + (size_t)slot * kTcChunkBytes;
+#pragma unroll
+            for (int it = 0; it < 8; ++it) {
+                const int rg = it & 1;
+                const int kpl = (it >> 1) * 4 + ksub;
+                const float4 cc = reinterpret_cast<const float4*>(cen)[c * 16 + kpl];
+                float4* px = reinterpret_cast<float4*>(A + (size_t)(2 * warp + rg) * 2048 + (size_t)kpl * 128 + rsub * 16);
+                float4 x = *px;
+                x.x -= cc.x; x.y -= cc.y; x.z -= cc.z; x.w -= cc.w;
+                float& xs = rg ? xs1 : xs0;
+                xs = fmaf(x.x, x.x, xs);
+                xs = fmaf(x.y, x.y, xs);
+                xs = fmaf(x.z, x.z, xs);
+                xs = fmaf(x.w, x.w, xs);
+                *px = x;
+            }
+            if (!(a.dbgmode & 64)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.xready[ms]);
+            if (lane == 0) mbar_arrive(&S.full[slot]);
+            if (c == nchunk - 1) {
+                // |x'|^2 per row: reduce over the 4 lanes (ksub) sharing a row
+                const int ms = b & (kTcBlk - 1);
+                xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 8);
+                xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 16);
+                xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 8);
+                xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 16);
+                if (lane < 8) S.xn[ms][16 * warp + lane] = xs0;
+                else if (lane < 16) S.xn[ms][16 * warp + lane] = xs1;
+                xs0 = xs1 = 0.f;
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&S.xready[ms]);
+            }
         }
         if (threadIdx.x == 0) tc_stamp(a, item, 2);
     } else if (warp == kTcMmaWarp) {
