@@ -336,10 +336,10 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t total = 0;
     BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    const char* mode = std::getenv("BLSH_SHORTLIST");
-    const bool tiled = tiled_supported(ds, T) && !(mode && std::strcmp(mode, "warp") == 0);
+    const int kind = shortlist_kind(ds, T, k);
+    const bool tiled = kind > 0;
     int64_t n_items = 0, union_rows = 0, pairs = total;
-    int tcpath = 0;
+    const int tcpath = kind == 2 ? 1 : 0;
     int64_t ch = 0;
     if (tiled) {
         // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
@@ -347,7 +347,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         int chr = 0;
         run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
-                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs, &tcpath);
+                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs, kind);
         ch = chr;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {

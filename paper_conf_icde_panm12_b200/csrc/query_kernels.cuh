@@ -58,13 +58,16 @@ struct ShortlistArgs {
 };
 
 // query-tiled short-list (shortlist_tiled.cu)
-bool tiled_supported(int ds, int T);
+// 0: warp short-list, 1: SIMT query-tiled, 2: tensor-core screened query-tiled.  The TC
+// kernel is the default where it applies (k <= 16, d_stride a multiple of 64 and <= 512);
+// BLSH_SHORTLIST=warp|simt forces the others.
+int shortlist_kind(int ds, int T, int k);
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
 void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
-                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int* tc_out);
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int kind);
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s);
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s);

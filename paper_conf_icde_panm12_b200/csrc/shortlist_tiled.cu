@@ -535,10 +535,21 @@ __global__ void k_tile_scatter(const uint8_t* __restrict__ ts, const int64_t* __
 
 size_t tiled_smem_bytes(int ds) { return 1024 + (size_t)QT * ds * 4 + (size_t)kStages * 32 * (ds + 4) * 4; }
 
-bool tiled_supported(int ds, int T) {
+size_t tc_smem_bytes(int ds) {
+    return ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)QT * ds * 4 + (size_t)kTcSlots * kTcChunkBytes;
+}
+
+int shortlist_kind(int ds, int T, int k) {
+    const char* mode = std::getenv("BLSH_SHORTLIST");
+    if (mode && std::strcmp(mode, "warp") == 0) return 0;
     int cap = 2 * QT * (T + 1), npow = 1;
     while (npow < cap) npow <<= 1;
-    return tiled_smem_bytes(ds) <= 227 * 1024 && (size_t)3 * npow * 4 <= 227 * 1024;
+    if ((size_t)3 * npow * 4 > 227 * 1024) return 0;   // tile prep does not fit
+    const bool simt_ok = tiled_smem_bytes(ds) <= 227 * 1024;
+    const bool tc_ok = k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024;
+    if (mode && std::strcmp(mode, "simt") == 0) return simt_ok ? 1 : 0;
+    if (tc_ok) return 2;
+    return simt_ok ? 1 : 0;
 }
 
 // Sort the active queries by (leaf, home key): qorder[pos] = query.
@@ -566,7 +577,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
-                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int* tc_out) {
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int kind) {
     const int64_t nq = a.nq;
     const int T = a.T;
     const int segcap = 2 * QT * (T + 1);
@@ -654,12 +665,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.rows_off = rows_off;
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
-    const size_t tc_smem = ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)QT * a.ds * 4 +
-                           (size_t)kTcSlots * kTcChunkBytes;
-    const char* mode = std::getenv("BLSH_SHORTLIST");
-    // the tensor-core screen is opt-in (BLSH_SHORTLIST=tc) until it beats the SIMT tiled kernel
-    const bool use_tc = k <= kTcMaxK && a.ds % kTcChunk == 0 && a.ds <= 512 && tc_smem <= 227 * 1024 &&
-                        mode && std::strcmp(mode, "tc") == 0;
+    const size_t tc_smem = tc_smem_bytes(a.ds);
+    const bool use_tc = kind == 2;   // chosen by shortlist_kind()
     const char* dbg_path = std::getenv("BLSH_TC_DEBUG");
     DevBuf dbgbuf;
     if (use_tc && dbg_path) {
@@ -692,7 +699,6 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         BLSH_LAUNCH_CHECK();
         ++*launches;
     }
-    *tc_out = use_tc ? 1 : 0;
     if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
     k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand);
     BLSH_LAUNCH_CHECK();

@@ -36,8 +36,7 @@
 constexpr int kTcRows = 128;               // M
 constexpr int kTcChunk = 64;               // K columns per A chunk
 constexpr int kTcSlots = 4;                // A chunk ring
-constexpr int kTcAhead = 2;                // chunks in flight ahead of the conversion (kTcSlots - kTcAhead
-                                           // chunks of slack for the MMA to release a slot)
+constexpr int kTcAhead = 3;                // staged chunks in flight ahead of the conversion (< kTcSlots)
 constexpr int kTcBlk = 4;                  // TMEM / metadata slots
 constexpr int kTcConv = 8;                 // converter warps
 constexpr int kTcMmaWarp = 8;
@@ -45,7 +44,10 @@ constexpr int kTcEpi0 = 9;                 // first epilogue warp
 constexpr int kTcThreads = 13 * 32;
 constexpr int kTcMaxK = 16;                // k supported by the TC path
 constexpr int kTcScap = 96;                // buffered pairs per (item, query, epilogue warp)
-constexpr uint32_t kTcChunkBytes = kTcRows * kTcChunk * 4;   // 32 KB
+constexpr uint32_t kTcStageBytes = kTcRows * kTcChunk * 4;   // 32 KB staging per chunk
+constexpr uint32_t kTcChunkBytes = kTcStageBytes;
+constexpr int kTcASlots = 4;               // A ring in tensor memory (64 columns each)
+constexpr uint32_t kTcACol0 = kTcBlk * 32; // first TMEM column of the A ring (after the accumulators)
 // instruction descriptor: D f32, A/B tf32, K-major both, N = 32, M = 128
 constexpr uint32_t kTcIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((32u >> 3) << 17) | ((128u >> 4) << 24);
 
@@ -64,6 +66,14 @@ __device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t
         "l"(adesc), "l"(bdesc), "r"(kTcIdesc), "r"(accum)
         : "memory");
 }
+// A from tensor memory (tf32, M = 128: row m in lane m, one K element per column)
+__device__ __forceinline__ void tc_mma_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t bdesc, uint32_t accum) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "r"(a_tmem), "l"(bdesc), "r"(kTcIdesc), "r"(accum)
+        : "memory");
+}
 __device__ __forceinline__ void tc_commit(uint64_t* bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
                  : "memory");
@@ -71,6 +81,18 @@ __device__ __forceinline__ void tc_commit(uint64_t* bar) {
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t* r) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+        "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+        "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]),
+        "r"(r[16]), "r"(r[17]), "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]),
+        "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+        : "memory");
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
     uint32_t r[32];
@@ -88,13 +110,13 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 }
 
 struct TcSmem {
-    uint64_t full[kTcSlots], empty[kTcSlots];
+    uint64_t afull[kTcASlots], aempty[kTcASlots];
     uint64_t tfull[kTcBlk], tempty[kTcBlk], xready[kTcBlk], mfree[kTcBlk];
     uint32_t tmem_base;
     alignas(16) float qn[QT];                // |q'|^2
     uint32_t rpos[kTcBlk][kTcRows];          // table row of each block row
     uint32_t rmask[kTcBlk][kTcRows];         // query mask of each block row (0 = padding)
-    float xn[kTcBlk][kTcRows];               // |x'|^2
+    float xn2[kTcBlk][2][kTcRows];           // |x'|^2, per column half
     alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
     unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
@@ -104,24 +126,6 @@ struct TcSmem {
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
     float sap[4][QT][32];                    // per epilogue warp: approximate d^2 [query][lane]
 };
-
-// exact fp32 direct-form d^2 (same partial-sum structure as k_shortlist: 12-term lanes + butterfly)
-__device__ __forceinline__ float exact_d2_warp(const float* __restrict__ x, const float* __restrict__ q, int nv4,
-                                               int lane) {
-    float p = 0.f;
-    for (int v = lane; v < nv4; v += 32) {
-        const float4 a = __ldg(reinterpret_cast<const float4*>(x) + v);
-        const float4 b = __ldg(reinterpret_cast<const float4*>(q) + v);
-        const float dx = b.x - a.x, dy = b.y - a.y, dz = b.z - a.z, dw = b.w - a.w;
-        p = fmaf(dx, dx, p);
-        p = fmaf(dy, dy, p);
-        p = fmaf(dz, dz, p);
-        p = fmaf(dw, dw, p);
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(BLSH_FULL, p, o);
-    return p;
-}
 
 // exact fp32 direct-form d^2 by one thread, in the partial-sum structure of the
 // SIMT tiled kernel's score_rows (blocks of 16 float4, two 32-term chains each,
@@ -139,7 +143,7 @@ __device__ __forceinline__ float exact_d2_thread(const float4* __restrict__ x, c
 #pragma unroll
         for (int v = 0; v < 16; ++v) {
             if (v < ne) {
-                const float4 qq = __ldg(q + vb + v);
+                const float4 qq = q[vb + v];
                 const float dx = qq.x - xv[v].x, dy = qq.y - xv[v].y, dz = qq.z - xv[v].z, dw = qq.w - xv[v].w;
                 a0 = fmaf(dx, dx, a0);
                 a1 = fmaf(dy, dy, a1);
@@ -160,27 +164,34 @@ __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned
     }
 }
 
-// Overflowing pairs of one query (lanes in om, table row in prow): exact d^2 now,
-// inserted into the query's shared top-k under its lock.  Rare; kept out of line.
+// Overflowing pairs of one query (lanes in om, table row in prow): each such lane
+// computes its pair's exact d^2 (same arithmetic as the final rescoring), then lane 0
+// inserts the keys into the query's shared top-k under its lock.  Rare; out of line.
 __device__ __noinline__ void tc_overflow(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
                                          unsigned om, uint32_t prow, int lane) {
-    const int nv4 = a.ds >> 2;
+    unsigned long long key = kEmpty;
+    if ((om >> lane) & 1u) {
+        const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
+                                         reinterpret_cast<const float4*>(qq), a.ds >> 2);
+        key = pack_entry(d2, __ldg(a.perm + prow));
+    }
+    if (lane == 0) {
+        while (atomicCAS(lock, 0, 1) != 0) {
+        }
+        __threadfence_block();
+    }
+    __syncwarp();
     while (om) {
         const int src = __ffs(om) - 1;
         om &= om - 1;
-        const uint32_t srow = __shfl_sync(BLSH_FULL, prow, src);
-        const float d2 = exact_d2_warp(a.Xp + (size_t)srow * a.ds, qq, nv4, lane);
-        const unsigned long long key = pack_entry(d2, __ldg(a.perm + srow));
-        if (lane == 0) {
-            while (atomicCAS(lock, 0, 1) != 0) {
-            }
-            __threadfence_block();
-            tk_insert(tk, a.k, key);
-            __threadfence_block();
-            atomicExch(lock, 0);
-        }
-        __syncwarp();
+        const unsigned long long kk = __shfl_sync(BLSH_FULL, key, src);
+        if (lane == 0) tk_insert(tk, a.k, kk);
     }
+    if (lane == 0) {
+        __threadfence_block();
+        atomicExch(lock, 0);
+    }
+    __syncwarp();
 }
 
 __device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p) {
@@ -197,7 +208,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     const int ds = a.ds, nv4 = ds >> 2, kp_total = ds >> 2;   // 16-byte K pieces
     unsigned char* opbase = smraw + ((sizeof(TcSmem) + 1023) & ~size_t(1023));
     unsigned char* Bop = opbase;                                    // [QT x ds] tf32, UMMA K-major
-    unsigned char* Aop = Bop + (size_t)QT * ds * 4;                 // [kTcSlots][128 x 64] tf32
+    unsigned char* Aop = Bop + (size_t)QT * ds * 4;                 // [kTcSlots] staging (8 warps x 32 rows x 128 B)
     float* Qf = reinterpret_cast<float*>(Aop);                      // setup only: original queries (aliases A)
     const uint32_t sboB = (uint32_t)kp_total * 128u;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -260,9 +271,9 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) (&S.tk[0][0])[i] = kEmpty;
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < kTcSlots; ++s) {
-            mbar_init(&S.full[s], kTcConv);
-            mbar_init(&S.empty[s], 1);
+        for (int s = 0; s < kTcASlots; ++s) {
+            mbar_init(&S.afull[s], kTcConv);
+            mbar_init(&S.aempty[s], 1);
         }
         for (int s = 0; s < kTcBlk; ++s) {
             mbar_init(&S.tfull[s], 1);
@@ -273,7 +284,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == kTcMmaWarp) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 128;" ::"r"(smem_u32(&S.tmem_base)));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&S.tmem_base)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B operand visible to the tensor core
@@ -285,94 +296,90 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
 
     if (warp < kTcConv) {
         // ======================= converters =======================
-        // Warp w owns block rows [16w, 16w + 16).  Lane -> (row rsub of an 8-row group, K piece
-        // offset ksub).  Rows are copied straight into the A operand's K-major core-matrix layout
-        // with 16-byte cp.async (zero-fill for padding rows), kTcAhead chunks ahead of the
-        // conversion, so the HBM latency is covered by the ring instead of registers; the
-        // conversion (subtract c, |x'|^2) then works in place on shared memory.  Each lane
-        // converts exactly the pieces it copied, so cp.async.wait_group orders the two.
-        const int rsub = lane & 7, ksub = lane >> 3;
+        // Converter warp w owns TMEM lane quadrant qd = w % 4 (block rows 32 qd + lane, one row
+        // per lane) and half hf = w / 4 of every 64-column chunk.  Its 32 rows x 32 columns are
+        // copied by 16-byte cp.async into a warp-private staging area (kTcAhead chunks ahead;
+        // 16-byte pieces XOR-swizzled by row so both the copy and the row-per-lane reads are
+        // bank-conflict free), then each lane subtracts c from its row, accumulates |x'|^2 and
+        // writes the 32 TF32 operands to the A ring in tensor memory (tcgen05.st).  Staging is
+        // warp-private (cp.async.wait_group orders it), so only the TMEM A slots and the block
+        // metadata need cross-warp barriers.
+        const int qd = warp & 3, hf = warp >> 2;
         const int nch_total = nblk * nchunk;
-        uint32_t ip0 = 0, ip1 = 0, isz0 = 0, isz1 = 0;   // issue side: this lane's two rows of the block
         const uint2* RI = a.rowinfo + a.rows_off[tile];
-        auto fetch = [&](int b) {                         // this lane's metadata entry of block b
-            const int64_t r = r0 + (int64_t)b * kTcRows + 16 * warp + (lane & 15);
+        unsigned char* stg = Aop + (size_t)warp * 4096;   // + slot * kTcStageBytes
+        auto fetch = [&](int b) {                          // this lane's row entry of block b
+            const int64_t r = r0 + (int64_t)b * kTcRows + 32 * qd + lane;
             return (b < nblk && r < r1) ? RI[r] : make_uint2(0u, 0u);
         };
-        uint2 e_next = fetch(0);                          // prefetched one block ahead
-        auto lookup = [&](int b) {                        // rows of block b: precomputed metadata
-            const int ms = b & (kTcBlk - 1);
-            const uint2 e = e_next;
-            e_next = fetch(b + 1);
-            if (b >= kTcBlk) mbar_wait(&S.mfree[ms], (uint32_t)(((b / kTcBlk) - 1) & 1));
-            if (lane < 16) {
-                S.rpos[ms][16 * warp + lane] = e.x;
-                S.rmask[ms][16 * warp + lane] = e.y;
-            }
-            ip0 = __shfl_sync(BLSH_FULL, e.x, rsub);
-            ip1 = __shfl_sync(BLSH_FULL, e.x, 8 + rsub);
-            const bool nol = (a.dbgmode & 2) != 0;
-            isz0 = (__shfl_sync(BLSH_FULL, e.y, rsub) != 0u && !nol) ? 16u : 0u;
-            isz1 = (__shfl_sync(BLSH_FULL, e.y, 8 + rsub) != 0u && !nol) ? 16u : 0u;
-        };
-        auto issue = [&](int g) {                         // cp.async of global chunk g into its slot
+        uint2 e_next = fetch(0), e_iss = make_uint2(0u, 0u);
+        auto issue = [&](int g) {                          // cp.async of chunk g (this warp's part)
             if (g < nch_total) {
                 const int b = g / nchunk, c = g - b * nchunk;
-                if (c == 0) lookup(b);
-                const int slot = g % kTcSlots;
-                if (g >= kTcSlots) mbar_wait(&S.empty[slot], (uint32_t)((g / kTcSlots - 1) & 1));
-                const uint32_t A = smem_u32(Aop + (size_t)slot * kTcChunkBytes);
-                const float* x0 = a.Xp + (size_t)ip0 * ds;
-                const float* x1 = a.Xp + (size_t)ip1 * ds;
+                if (c == 0) {                              // new block: its row metadata
+                    const int ms = b & (kTcBlk - 1);
+                    e_iss = e_next;
+                    e_next = fetch(b + 1);
+                    // every converter warp writes slot ms (metadata or |x'|^2): wait until the
+                    // epilogue has released it
+                    if (b >= kTcBlk) mbar_wait(&S.mfree[ms], (uint32_t)(((b / kTcBlk) - 1) & 1));
+                    if (hf == 0) {
+                        S.rpos[ms][32 * qd + lane] = e_iss.x;
+                        S.rmask[ms][32 * qd + lane] = e_iss.y;
+                    }
+                }
+                const uint32_t sb = smem_u32(stg + (size_t)(g % kTcSlots) * kTcStageBytes);
+                const bool nol = (a.dbgmode & 2) != 0;
+                const int p = lane & 7;
 #pragma unroll
                 for (int it = 0; it < 8; ++it) {
-                    const int rg = it & 1;
-                    const int kpl = (it >> 1) * 4 + ksub;
-                    const float* src = (rg ? x1 : x0) + (size_t)(c * 16 + kpl) * 4;
-                    const uint32_t dst = A + (uint32_t)((2 * warp + rg) * 2048 + kpl * 128 + rsub * 16);
+                    const int r = it * 4 + (lane >> 3);
+                    const uint32_t pos = __shfl_sync(BLSH_FULL, e_iss.x, r);
+                    const uint32_t msk = __shfl_sync(BLSH_FULL, e_iss.y, r);
+                    const float* src = a.Xp + (size_t)pos * ds + c * kTcChunk + hf * 32 + p * 4;
+                    const uint32_t dst = sb + (uint32_t)(r * 128 + ((p ^ (r & 7)) << 4));
                     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
-                                 "r"(rg ? isz1 : isz0)
+                                 "r"((msk != 0u && !nol) ? 16u : 0u)
                                  : "memory");
                 }
             }
             asm volatile("cp.async.commit_group;" ::: "memory");   // (possibly empty: uniform group count)
         };
         for (int g = 0; g < kTcAhead; ++g) issue(g);
-        float xs0 = 0.f, xs1 = 0.f;
+        float xs = 0.f;
+        const uint32_t tl = (uint32_t)(32 * qd) << 16;   // TMEM lane base of this warp
         for (int g = 0; g < nch_total; ++g) {
             issue(g + kTcAhead);
             asm volatile("cp.async.wait_group %0;" ::"n"(kTcAhead) : "memory");   // chunk g has landed
             const int b = g / nchunk, c = g - b * nchunk;
             const int slot = g % kTcSlots;
-            unsigned char* A = Aop + (size_t)slot * kTcChunkBytes;
+            const unsigned char* row = stg + (size_t)slot * kTcStageBytes + lane * 128;
+            uint32_t v[32];
 #pragma unroll
-            for (int it = 0; it < 8; ++it) {
-                const int rg = it & 1;
-                const int kpl = (it >> 1) * 4 + ksub;
-                const float4 cc = reinterpret_cast<const float4*>(cen)[c * 16 + kpl];
-                float4* px = reinterpret_cast<float4*>(A + (size_t)(2 * warp + rg) * 2048 + (size_t)kpl * 128 + rsub * 16);
-                float4 x = *px;
+            for (int p = 0; p < 8; ++p) {
+                float4 x = *reinterpret_cast<const float4*>(row + ((p ^ (lane & 7)) << 4));
+                const float4 cc = reinterpret_cast<const float4*>(cen)[(c * kTcChunk + hf * 32) / 4 + p];
                 x.x -= cc.x; x.y -= cc.y; x.z -= cc.z; x.w -= cc.w;
-                float& xs = rg ? xs1 : xs0;
                 xs = fmaf(x.x, x.x, xs);
                 xs = fmaf(x.y, x.y, xs);
                 xs = fmaf(x.z, x.z, xs);
                 xs = fmaf(x.w, x.w, xs);
-                *px = x;
+                v[4 * p] = __float_as_uint(x.x);
+                v[4 * p + 1] = __float_as_uint(x.y);
+                v[4 * p + 2] = __float_as_uint(x.z);
+                v[4 * p + 3] = __float_as_uint(x.w);
             }
-            if (!(a.dbgmode & 64)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            const int as = g % kTcASlots;
+            if (g >= kTcASlots) mbar_wait(&S.aempty[as], (uint32_t)((g / kTcASlots - 1) & 1));
+            tc_fence_after();
+            tmem_st32(tbase + tl + kTcACol0 + (uint32_t)(as * kTcChunk + hf * 32), v);
+            tc_fence_before();
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.full[slot]);
+            if (lane == 0) mbar_arrive(&S.afull[as]);
             if (c == nchunk - 1) {
-                // |x'|^2 per row: reduce over the 4 lanes (ksub) sharing a row
                 const int ms = b & (kTcBlk - 1);
-                xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 8);
-                xs0 += __shfl_xor_sync(BLSH_FULL, xs0, 16);
-                xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 8);
-                xs1 += __shfl_xor_sync(BLSH_FULL, xs1, 16);
-                if (lane < 8) S.xn[ms][16 * warp + lane] = xs0;
-                else if (lane < 16) S.xn[ms][16 * warp + lane] = xs1;
-                xs0 = xs1 = 0.f;
+                S.xn2[ms][hf][32 * qd + lane] = xs;
+                xs = 0.f;
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&S.xready[ms]);
             }
@@ -387,19 +394,18 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             const uint32_t dt = tbase + (uint32_t)ts * 32u;
             for (int c = 0; c < nchunk; ++c) {
                 const int gch = b * nchunk + c;
-                const int slot = gch % kTcSlots;
-                mbar_wait(&S.full[slot], (uint32_t)((gch / kTcSlots) & 1));
+                const int as = gch % kTcASlots;
+                mbar_wait(&S.afull[as], (uint32_t)((gch / kTcASlots) & 1));
                 tc_fence_after();
                 if (lane == 0) {
-                    const uint32_t abase = smem_u32(Aop + (size_t)slot * kTcChunkBytes);
+                    const uint32_t at = tbase + kTcACol0 + (uint32_t)(as * kTcChunk);
                     const uint32_t bbase = smem_u32(Bop) + (uint32_t)(c * 16) * 128u;
 #pragma unroll
                     for (int s = 0; s < kTcChunk / 8; ++s) {
-                        const uint64_t ad = umma_desc(abase + (uint32_t)s * 256u, 128u, 2048u);
                         const uint64_t bd = umma_desc(bbase + (uint32_t)s * 256u, 128u, sboB);
-                        if (!(a.dbgmode & 4)) tc_mma(dt, ad, bd, (c > 0 || s > 0) ? 1u : 0u);
+                        if (!(a.dbgmode & 4)) tc_mma_ts(dt, at + (uint32_t)s * 8u, bd, (c > 0 || s > 0) ? 1u : 0u);
                     }
-                    tc_commit(&S.empty[slot]);
+                    tc_commit(&S.aempty[as]);
                     if (c == nchunk - 1) tc_commit(&S.tfull[ts]);
                 }
                 __syncwarp();
@@ -427,7 +433,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             tmem_ld32(tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 32u, dot);
             tc_fence_before();
             const uint32_t msk = S.rmask[ts][brow];
-            const float xn = S.xn[ts][brow];
+            const float xn = S.xn2[ts][0][brow] + S.xn2[ts][1][brow];
             const uint32_t prow = S.rpos[ts][brow];
             __syncwarp();
             if (lane == 0) {
@@ -522,7 +528,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     __syncthreads();
     if (warp == kTcMmaWarp) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 128;" ::"r"(tbase));
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
     }
     if (threadIdx.x == 0) tc_stamp(a, item, 5);
     // ---- final (all warps): exact rescoring of the buffered pairs whose lower bound is <= U_j ----
@@ -564,6 +570,11 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     }
     __syncthreads();
     const int total = S.roff[32];
+    // the tile's queries, exact, into shared memory behind L (the rescoring reads them per pair)
+    float* Qx = reinterpret_cast<float*>(opbase + (size_t)QT * kPerQ * 8);
+    for (int i = threadIdx.x; i < nqt * nv4; i += kTcThreads)
+        reinterpret_cast<float4*>(Qx)[i] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + i / nv4] * ds) + i % nv4);
+    __syncthreads();
     if (threadIdx.x == 0) tc_stamp(a, item, 6);
     for (int idx = threadIdx.x; idx < total; idx += kTcThreads) {   // (b) one thread per pair
         int lo2 = 0, hi2 = 32;                                      // query j: roff[j] <= idx < roff[j + 1]
@@ -575,7 +586,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         unsigned long long& e = L[(size_t)lo2 * kPerQ + (idx - S.roff[lo2])];
         const uint32_t srow = (uint32_t)(e & 0xFFFFFFFFull);
         const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)srow * ds),
-                                         reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + lo2] * ds), nv4);
+                                         reinterpret_cast<const float4*>(Qx + (size_t)lo2 * ds), nv4);
         e = pack_entry(d2, __ldg(a.perm + srow));
     }
     __syncthreads();

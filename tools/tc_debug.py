@@ -32,8 +32,10 @@ qn = raw[4096 + 384:4096 + 416]
 qord = np.fromfile(path, dtype=np.uint32)[4096 + 512:4096 + 512 + 32]
 perm = ix.export("PERM")
 Xp = X[perm]
-c = Q[qord[0]].astype(np.float64)
+nqt = int((qn > 0).sum())                     # tile 0's queries (qn = 0 for empty slots)
+c = Q[qord[:nqt]].astype(np.float64).mean(0)  # tile centre = mean of its queries
 qs = Q[qord].astype(np.float64) - c
+qs[nqt:] = 0.0
 valid = msk != 0
 xs = Xp[rpos].astype(np.float64) - c
 ref = xs @ qs.T
@@ -41,3 +43,7 @@ err = np.abs(dots - ref)[valid]
 print("rows valid", valid.sum(), "max |dot err|", err.max(), "max |dot|", np.abs(ref[valid]).max())
 print("xn err", np.abs(xn - (xs ** 2).sum(1))[valid].max(), "qn err", np.abs(qn - (qs ** 2).sum(1)).max())
 print("sample dots", dots[0, :4], ref[0, :4])
+# which (row, column) of the reference best explains each measured dot row (layout probe)
+for r in range(3):
+    best = [(float(np.abs(dots[r] - ref[rr]).max()), rr) for rr in range(128) if valid[rr]]
+    print("row", r, "closest ref row", min(best))
