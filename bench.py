@@ -217,6 +217,7 @@ def run_ours(a):
     import torch.distributed as dist
     import synth
     from paper_conf_icde_panm12_b200 import blsh
+    from paper_conf_icde_panm12_b200.sharded import ShardedIndex
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -233,6 +234,7 @@ def run_ours(a):
     t0 = time.time()
     ix = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, quantizer=cfg.quantizer,
                          rank=rank, world=world)
+    sh = ShardedIndex(ix) if world > 1 else None
     torch.cuda.synchronize()
     build_s = time.time() - t0
     info = ix.info()
@@ -242,7 +244,6 @@ def run_ours(a):
     out_d2 = torch.empty((nq, k), dtype=torch.float32, device=dev)
     out_nc = torch.empty((nq,), dtype=torch.int64, device=dev)
     pk = torch.empty((nq, k), dtype=torch.int64, device=dev)
-    gathered = torch.empty((world, nq, k), dtype=torch.int64, device=dev) if world > 1 else None
     stats = []
 
     def step(timing):
@@ -250,11 +251,10 @@ def run_ours(a):
             ix.query(Q, k, timing=timing, out=(out_ids, out_d2, out_nc), **kw)
             stats.append(ix.stats())
             return 0
-        ix.query_packed(Q, k, timing=timing, out=(pk, out_nc), **kw)
+        # leaf-sharded: this rank's packed lists -> NCCL all-gather -> blsh_merge_topk (sharded.py)
+        sh.query(Q, k, timing=timing, out=(out_ids, out_d2), packed_out=(pk, out_nc), **kw)
         stats.append(ix.stats())
-        dist.all_gather_into_tensor(gathered, pk)
-        blsh.blsh_merge_topk(gathered, world, nq, k, out=(out_ids, out_d2))
-        return 1
+        return 1 + (1 if cfg.hierarchy and not cfg.min_cand else 0)
 
     for _ in range(a.warmup):
         step(False)
@@ -308,9 +308,7 @@ def run_ours(a):
             if world == 1:
                 ix.query(Qh, k, out=(hi, hd, hn), **kw)
             else:
-                ix.query_packed(Qh, k, out=(hpk, out_nc), **kw)
-                dist.all_gather_into_tensor(gathered, hpk)
-                blsh.blsh_merge_topk(gathered, world, nq, k, out=(hi, hd))
+                sh.query(Qh, k, out=(hi, hd), packed_out=(hpk, out_nc), **kw)
 
         for _ in range(max(1, a.warmup // 2)):
             e2e_step()

@@ -76,6 +76,12 @@ typedef struct {
     void*   stream;         /* cudaStream_t                                                                   */
     int32_t keep_stages;    /* 1 = keep per-query stages of this call for blsh_export                         */
     int32_t timing;         /* 1 = record per-stage CUDA-event times into blsh_last_stats                     */
+    const int64_t* global_base; /* optional DEVICE array [nq]: |A0(q)| of every query of the batch summed over
+                               the shards (blsh_query_base_counts on each rank + a sum all-reduce).  With
+                               hierarchy = 1 and min_cand = 0, tau = its lower median (R18: P:249's "median
+                               over a set of queries" taken over the whole sharded batch, so a sharded index
+                               widens exactly like one GPU).  NULL = this call's own counts; must be non-NULL
+                               for that case when world > 1.  Read on `stream`; owned by the caller.          */
 } blsh_query_params;
 
 void blsh_build_params_default(blsh_build_params* p);
@@ -105,6 +111,16 @@ blsh_status blsh_query(const blsh_index* idx, const float* Q, int64_t nq, int32_
 blsh_status blsh_query_packed(const blsh_index* idx, const float* Q, int64_t nq, int32_t k,
                               const blsh_query_params* p, uint64_t* out_packed,
                               int64_t* out_ncand);
+
+/* a1-a4 only (route, hash, probe, look up; no widening, no short-list): the
+ * base candidate count |A0(q)| of every query (the count the hierarchy's
+ * threshold is a median of), 0 for queries whose leaf another shard owns.
+ *   Q        [nq x d] fp32 (device or host)
+ *   out_base [nq] int64 (device or host)
+ * On a sharded index the sum over ranks of out_base is the single-GPU base
+ * count of every query; pass it as p->global_base to blsh_query(_packed). */
+blsh_status blsh_query_base_counts(const blsh_index* idx, const float* Q, int64_t nq,
+                                   const blsh_query_params* p, int64_t* out_base);
 
 /* a6: merge n_lists per-rank packed lists (e.g. the output of an NCCL
  * all-gather, layout [n_lists][nq][k]) into the k smallest per query.

@@ -36,7 +36,7 @@ class BuildParams(C.Structure):
 class QueryParams(C.Structure):
     _fields_ = [("probe", C.c_int32), ("n_probes", C.c_int32), ("hierarchy", C.c_int32),
                 ("hier_step_bits", C.c_int32), ("min_cand", C.c_int64), ("stream", C.c_void_p),
-                ("keep_stages", C.c_int32), ("timing", C.c_int32)]
+                ("keep_stages", C.c_int32), ("timing", C.c_int32), ("global_base", C.c_void_p)]
 
 
 class Info(C.Structure):
@@ -84,6 +84,8 @@ def lib():
         L.blsh_query.restype = i32
         L.blsh_query_packed.argtypes = [P, P, i64, i32, C.POINTER(QueryParams), P, P]
         L.blsh_query_packed.restype = i32
+        L.blsh_query_base_counts.argtypes = [P, P, i64, C.POINTER(QueryParams), P]
+        L.blsh_query_base_counts.restype = i32
         L.blsh_merge_topk.argtypes = [P, i32, i64, i32, P, P, P]
         L.blsh_merge_topk.restype = i32
         L.blsh_export.argtypes = [P, i32, P, C.c_size_t, C.POINTER(C.c_size_t)]
@@ -101,7 +103,7 @@ def lib():
 
 
 EXPORTED_SYMBOLS = ("blsh_build_params_default", "blsh_query_params_default", "blsh_build", "blsh_query",
-                    "blsh_query_packed", "blsh_merge_topk", "blsh_export", "blsh_index_info",
+                    "blsh_query_packed", "blsh_query_base_counts", "blsh_merge_topk", "blsh_export", "blsh_index_info",
                     "blsh_last_stats", "blsh_free", "blsh_last_error")
 
 
@@ -170,11 +172,13 @@ def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42,
     return Index(h, n, d, M)
 
 
-def _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, stream):
+def _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, stream, global_base=None):
     p = QueryParams()
     lib().blsh_query_params_default(C.byref(p))
     p.probe, p.n_probes, p.hierarchy, p.hier_step_bits = probe, n_probes, int(hierarchy), hier_step_bits
     p.min_cand, p.keep_stages, p.timing, p.stream = min_cand, int(bool(keep_stages)), int(bool(timing)), stream
+    if global_base is not None:
+        p.global_base = C.c_void_p(global_base.data_ptr())   # CUDA int64 tensor [nq]
     return p
 
 
@@ -189,14 +193,15 @@ def _alloc_like(Q, shape, kind):
 
 def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
                hier_step_bits: int = 0, min_cand: int = 0, keep_stages: bool = False, timing: bool = False,
-               out=None):
+               out=None, global_base=None):
     """-> (ids [nq,k] int64, dist2 [nq,k] fp32, ncand [nq] int64), on Q's device."""
     Q = _f32(Q)
     nq = int(Q.shape[0])
     if out is None:
         out = (_alloc_like(Q, (nq, k), "i64"), _alloc_like(Q, (nq, k), "f32"), _alloc_like(Q, (nq,), "i64"))
     ids, d2, nc = out
-    p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, _stream_for(Q, ids))
+    p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, _stream_for(Q, ids),
+                 global_base)
     qp, kq, _ = _ptr(Q)
     ip, ki, _ = _ptr(ids)
     dp, kd, _ = _ptr(d2)
@@ -206,19 +211,35 @@ def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hie
 
 
 def blsh_query_packed(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
-                      hier_step_bits: int = 0, min_cand: int = 0, timing: bool = False, out=None):
+                      hier_step_bits: int = 0, min_cand: int = 0, timing: bool = False, out=None,
+                      global_base=None):
     """-> (packed [nq,k] (uint64 bits; int64 for torch), ncand [nq])."""
     Q = _f32(Q)
     nq = int(Q.shape[0])
     if out is None:
         out = (_alloc_like(Q, (nq, k), "u64"), _alloc_like(Q, (nq,), "i64"))
     pk, nc = out
-    p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, False, timing, _stream_for(Q, pk))
+    p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, False, timing, _stream_for(Q, pk),
+                 global_base)
     qp, kq, _ = _ptr(Q)
     pp, kp, _ = _ptr(pk)
     np_, kn, _ = _ptr(nc)
     _check(lib().blsh_query_packed(index.handle, qp, nq, k, C.byref(p), pp, np_))
     return pk, nc
+
+
+def blsh_query_base_counts(index: "Index", Q, probe: int = 0, n_probes: int = 1, timing: bool = False,
+                           out=None, **_ignored):
+    """a1-a4 only: |A0(q)| [nq] int64 (0 for queries another shard owns), on Q's device."""
+    Q = _f32(Q)
+    nq = int(Q.shape[0])
+    if out is None:
+        out = _alloc_like(Q, (nq,), "i64")
+    p = _qparams(probe, n_probes, 0, 0, 0, False, timing, _stream_for(Q, out))
+    qp, kq, _ = _ptr(Q)
+    op, ko, _ = _ptr(out)
+    _check(lib().blsh_query_base_counts(index.handle, qp, nq, C.byref(p), op))
+    return out
 
 
 def blsh_merge_topk(packed, n_lists: int, nq: int, k: int, out=None):
@@ -283,6 +304,9 @@ class Index:
 
     def query_packed(self, Q, k, **kw):
         return blsh_query_packed(self, Q, k, **kw)
+
+    def base_counts(self, Q, **kw):
+        return blsh_query_base_counts(self, Q, **kw)
 
     def export(self, what: str) -> np.ndarray:
         return blsh_export(self, what)

@@ -97,6 +97,7 @@ void blsh_query_params_default(blsh_query_params* p) {
     p->stream = nullptr;
     p->keep_stages = 0;
     p->timing = 0;
+    p->global_base = nullptr;
 }
 
 const char* blsh_last_error(void) { return g_last_error.c_str(); }
@@ -247,7 +248,8 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
 namespace blsh {
 
 void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k, const blsh_query_params& p,
-               int64_t* out_ids, float* out_d2, unsigned long long* out_packed, int64_t* out_ncand, bool out_host) {
+               int64_t* out_ids, float* out_d2, unsigned long long* out_packed, int64_t* out_ncand, bool out_host,
+               int64_t* out_base) {
     cudaStream_t s = (cudaStream_t)p.stream;
     QueryWork& w = ix.qw;
     const int T = p.n_probes, M = ix.M, ds = ix.ds;
@@ -326,8 +328,25 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // a3+a4
     launch_probe_lookup(a, s); ++launches;
+    if (out_base) {   // blsh_query_base_counts: a1-a4 only
+        BLSH_CUDA(cudaMemcpyAsync(out_base, w.base, (size_t)nq * 8, out_host ? cudaMemcpyDeviceToHost
+                                                                              : cudaMemcpyDeviceToDevice, s));
+        if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[3], s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        stt.launches = launches;
+        if (tm) {
+            cudaEventElapsedTime(&stt.ms_route_hash, ix.ev[1], ix.ev[2]);
+            cudaEventElapsedTime(&stt.ms_probe, ix.ev[2], ix.ev[3]);
+            cudaEventElapsedTime(&stt.ms_total, ix.ev[0], ix.ev[3]);
+        }
+        ix.has_stages = keep;
+        return;
+    }
     if (p.hierarchy) {
-        if (p.min_cand == 0) { launch_median(w.base, nq, w.tau, s); ++launches; }
+        if (p.min_cand == 0) {
+            launch_median(p.global_base ? p.global_base : w.base, nq, w.tau, s);
+            ++launches;
+        }
         launch_widen(a, w.tau, p.min_cand, s); ++launches;
     }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[3], s));
@@ -432,9 +451,11 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
         if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "the Morton hierarchy needs a Z^M index");
         if (p->hier_step_bits < 0 || p->hier_step_bits > idx->M) return fail(BLSH_ERR_INVALID, "hier_step_bits must be in [0, M]");
         if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");
-        if (p->min_cand == 0 && idx->world > 1)
-            return fail(BLSH_ERR_UNSUPPORTED, "batch-median tau on a sharded index needs a global median (pass min_cand)");
+        if (p->min_cand == 0 && idx->world > 1 && !p->global_base)
+            return fail(BLSH_ERR_INVALID, "batch-median tau on a sharded index needs p->global_base "
+                                          "(blsh_query_base_counts summed over ranks) or an explicit min_cand");
     }
+    if (p->global_base && !is_device_ptr(p->global_base)) return fail(BLSH_ERR_INVALID, "global_base must be device memory");
     return BLSH_OK;
 }
 
@@ -452,7 +473,7 @@ blsh_status blsh_query(const blsh_index* idx, const float* Q, int64_t nq, int32_
     const bool o_host = !is_device_ptr(out_ids);
     if (o_host != !is_device_ptr(out_dist2) || (out_ncand && o_host != !is_device_ptr(out_ncand)))
         return fail(BLSH_ERR_INVALID, "outputs must all be host or all be device memory");
-    return guarded([&] { blsh::run_query(*idx, Q, q_host, nq, k, *p, out_ids, out_dist2, nullptr, out_ncand, o_host); });
+    return guarded([&] { blsh::run_query(*idx, Q, q_host, nq, k, *p, out_ids, out_dist2, nullptr, out_ncand, o_host, nullptr); });
 }
 
 blsh_status blsh_query_packed(const blsh_index* idx, const float* Q, int64_t nq, int32_t k, const blsh_query_params* p,
@@ -468,7 +489,24 @@ blsh_status blsh_query_packed(const blsh_index* idx, const float* Q, int64_t nq,
         return fail(BLSH_ERR_INVALID, "outputs must all be host or all be device memory");
     return guarded([&] {
         blsh::run_query(*idx, Q, q_host, nq, k, *p, nullptr, nullptr, reinterpret_cast<unsigned long long*>(out_packed),
-                        out_ncand, o_host);
+                        out_ncand, o_host, nullptr);
+    });
+}
+
+blsh_status blsh_query_base_counts(const blsh_index* idx, const float* Q, int64_t nq, const blsh_query_params* p,
+                                   int64_t* out_base) {
+    if (!p) return fail(BLSH_ERR_INVALID, "params is NULL");
+    blsh_query_params p2 = *p;
+    p2.hierarchy = 0;     // the base set only: widening is not part of A0
+    p2.global_base = nullptr;
+    blsh_status c = check_query(idx, Q, nq, 1, &p2);
+    if (c != BLSH_OK) return c;
+    if (nq > 0 && !out_base) return fail(BLSH_ERR_INVALID, "out_base is NULL");
+    if (nq == 0) return BLSH_OK;
+    const bool q_host = !is_device_ptr(Q);
+    const bool o_host = !is_device_ptr(out_base);
+    return guarded([&] {
+        blsh::run_query(*idx, Q, q_host, nq, 1, p2, nullptr, nullptr, nullptr, nullptr, o_host, out_base);
     });
 }
 

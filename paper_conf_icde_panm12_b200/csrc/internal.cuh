@@ -179,7 +179,8 @@ void build_table(blsh_index& ix, const float* Xs, const unsigned long long* key_
 // ---- query (query.cu, shortlist.cu) ----------------------------------------------
 void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
                const blsh_query_params& p, int64_t* out_ids, float* out_d2,
-               unsigned long long* out_packed, int64_t* out_ncand, bool out_host);
+               unsigned long long* out_packed, int64_t* out_ncand, bool out_host,
+               int64_t* out_base);   // non-NULL: stop after a4 and write |A0(q)| (blsh_query_base_counts)
 
 void merge_lists(const unsigned long long* packed, int n_lists, int64_t nq, int k,
                  int64_t* out_ids, float* out_d2, cudaStream_t s);

@@ -690,8 +690,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_tc) {
-            BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
-            k_shortlist_tc<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
+            auto kern = k <= 8 ? k_shortlist_tc<8> : (k <= 12 ? k_shortlist_tc<12> : k_shortlist_tc<16>);
+            BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
+            kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
         } else {
             BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);

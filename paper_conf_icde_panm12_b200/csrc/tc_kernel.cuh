@@ -24,10 +24,10 @@
 //        write the TF32 A operand in the K-major no-swizzle UMMA layout
 //        (8-row x 16-byte core matrices), |x'|^2 per row;
 //   8    MMA issuer (one elected lane) + TMEM allocation;
-//   9-12 epilogue: tcgen05.ld of the 32 accumulators of its 32 rows, screen,
-//        per-warp upper-bound lists and per-warp pair buffers (registers and
-//        warp-private memory: no atomics or locks on the hot path), final
-//        exact rescoring.
+//   9-12 epilogue: tcgen05.ld of the 32 accumulators of its 32 rows, transpose
+//        through shared memory so that lane j screens query j: per-lane sorted
+//        upper-bound lists and per-lane pair buffers (registers and lane-private
+//        memory: no atomics or locks on the hot path), final exact rescoring.
 // Pipelines: 4-slot ring of 64-column A chunks (full / empty mbarriers; the
 // MMA frees a slot with tcgen05.commit), 4 TMEM accumulator slots and 4
 // row-metadata slots (tmem_full by commit, tmem_empty / meta_free by the
@@ -124,7 +124,8 @@ struct TcSmem {
     int rcnt[QT];                            // final: pairs to rescore per query
     int roff[QT + 1];                        // final: their exclusive prefix
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
-    float sap[4][QT][32];                    // per epilogue warp: approximate d^2 [query][lane]
+    float tr[4][32 * 33];                    // per epilogue warp: transposed dots [query][row], padded
+    uint4 rinfo[4][32];                      // per epilogue warp: (|x'|^2 bits, query mask, table row) per row
 };
 
 // exact fp32 direct-form d^2 by one thread, in the partial-sum structure of the
@@ -164,34 +165,20 @@ __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned
     }
 }
 
-// Overflowing pairs of one query (lanes in om, table row in prow): each such lane
-// computes its pair's exact d^2 (same arithmetic as the final rescoring), then lane 0
-// inserts the keys into the query's shared top-k under its lock.  Rare; out of line.
-__device__ __noinline__ void tc_overflow(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
-                                         unsigned om, uint32_t prow, int lane) {
-    unsigned long long key = kEmpty;
-    if ((om >> lane) & 1u) {
-        const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
-                                         reinterpret_cast<const float4*>(qq), a.ds >> 2);
-        key = pack_entry(d2, __ldg(a.perm + prow));
+// Overflow (screen phase, lane = query): the pair's exact d^2 by this thread,
+// inserted into the query's shared top-k under its lock.  Only when a pair buffer is
+// still full after dropping what the current bound excludes.
+__device__ __noinline__ void tc_overflow_lane(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
+                                              uint32_t prow) {
+    const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
+                                     reinterpret_cast<const float4*>(qq), a.ds >> 2);
+    const unsigned long long key = pack_entry(d2, __ldg(a.perm + prow));
+    while (atomicCAS(lock, 0, 1) != 0) {
     }
-    if (lane == 0) {
-        while (atomicCAS(lock, 0, 1) != 0) {
-        }
-        __threadfence_block();
-    }
-    __syncwarp();
-    while (om) {
-        const int src = __ffs(om) - 1;
-        om &= om - 1;
-        const unsigned long long kk = __shfl_sync(BLSH_FULL, key, src);
-        if (lane == 0) tk_insert(tk, a.k, kk);
-    }
-    if (lane == 0) {
-        __threadfence_block();
-        atomicExch(lock, 0);
-    }
-    __syncwarp();
+    __threadfence_block();
+    tk_insert(tk, a.k, key);
+    __threadfence_block();
+    atomicExch(lock, 0);
 }
 
 __device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p) {
@@ -202,6 +189,9 @@ __device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p
     }
 }
 
+// KT: length of the per-lane upper-bound lists (>= k; the first KT - k entries are -inf
+// placeholders, so the k-th smallest real bound is always ulr[KT - 1]).
+template <int KT>
 __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     extern __shared__ __align__(1024) unsigned char smraw[];
     TcSmem& S = *reinterpret_cast<TcSmem*>(smraw);
@@ -414,16 +404,29 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         if (lane == 0) tc_stamp(a, item, 3);
     } else {
         // ======================= epilogue =======================
+        // Lane = row when the accumulators come out of TMEM (tcgen05.ld 32x32b), lane = query
+        // for the screen: the 32 x 32 block of dot products is transposed through a padded
+        // shared tile (conflict-free both ways), then lane j runs query j's screen over the
+        // warp's 32 rows with its own sorted upper-bound list and its own pair buffer.  The
+        // 32 lists are updated in parallel (no serial per-pair insertion, no ballots).
         const int ew = warp - kTcEpi0;          // 0..3
         const int quad = warp & 3;              // TMEM lane quadrant of this warp
-        const int brow = quad * 32 + lane;      // block row of this lane
-        float my_qn = lane < QT ? S.qn[lane] : 0.f;     // lane j holds query j's values
-        float my_U = __int_as_float(0x7F800000);        // this warp's k-th smallest upper bound for query j
-        float ulr[kTcMaxK];                             // lane j: this warp's sorted upper bounds of query j
+        const int brow = quad * 32 + lane;      // block row of this lane (row phase)
+        const int j = lane;                     // query of this lane (screen phase)
+        // Screen bounds.  With s = |q'|^2 + |x'|^2 and t the TF32 dot of the centred vectors,
+        // |(s - 2t) - d2| <= 2.03e-3 s (TF32 operands: 2^-10 relative each; fp32 sums), and
+        // |s - 2t| <= 2.004 s, so lo = s (1 - kScr) - 2t <= d2 <= s (1 + kScr) - 2t = up with
+        // kScr = 4.03e-3 (2x slack; the rounding of these few fp32 operations is ~1e-7 s).
+        constexpr float kScr = 4.03e-3f;
+        const float qn = S.qn[j];
+        const float qa = qn * (1.0f - kScr), qb = qn * (1.0f + kScr);
+        float ulr[KT];                          // sorted k smallest upper bounds of query j seen by this warp
 #pragma unroll
-        for (int p = 0; p < kTcMaxK; ++p) ulr[p] = __int_as_float(0x7F800000);
-        int my_cnt = 0;                                 // this warp's buffered pairs for query j
-        unsigned long long* SB = a.sbuf + ((size_t)item * QT * 4 + ew) * kTcScap;   // + j * 4 * kTcScap
+        for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
+        int my_cnt = 0;                         // buffered pairs of query j in this warp's buffer
+        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * 4 + ew) * kTcScap;
+        float* Tt = S.tr[ew];
+        const bool screen = !(a.dbgmode & 1);
         for (int b = 0; b < nblk; ++b) {
             const int ts = b & (kTcBlk - 1);
             mbar_wait(&S.tfull[ts], (uint32_t)((b / kTcBlk) & 1));
@@ -441,87 +444,52 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 mbar_arrive(&S.mfree[ts]);
             }
             if (a.dbg && item == 0 && b == 0) {
-                for (int j = 0; j < 32; ++j) a.dbg[brow * 32 + j] = dot[j];
+                for (int jj = 0; jj < 32; ++jj) a.dbg[brow * 32 + jj] = dot[jj];
                 a.dbg[4096 + brow] = xn;
                 a.dbg[4096 + 128 + brow] = __uint_as_float(prow);
                 a.dbg[4096 + 256 + brow] = __uint_as_float(msk);
                 if (brow < 32) a.dbg[4096 + 384 + brow] = S.qn[brow];
             }
-            // pass 1 (branch-free, all 32 queries): which (row, query) pairs pass the screen
-            uint32_t kmask = 0;
-            if (!(a.dbgmode & 1)) {
+            if (!screen) continue;
+            // transpose: row lane writes its 32 dots, column j -> Tt[j][lane]
 #pragma unroll
-                for (int j4 = 0; j4 < 8; ++j4) {
-                    const float4 qn4 = reinterpret_cast<const float4*>(S.qn)[j4];
-                    const uint4 um4 = reinterpret_cast<const uint4*>(S.umin)[j4];
-                    const float qv[4] = {qn4.x, qn4.y, qn4.z, qn4.w};
-                    const uint32_t uv[4] = {um4.x, um4.y, um4.z, um4.w};
-#pragma unroll
-                    for (int t = 0; t < 4; ++t) {
-                        const int j = 4 * j4 + t;
-                        const float approx = qv[t] + xn - 2.0f * dot[j];
-                        const float m = 4e-3f * (qv[t] + xn) + 1e-5f * fabsf(approx) + 1e-30f;
-                        if (approx - m <= __uint_as_float(uv[t])) kmask |= 1u << j;
-                        S.sap[ew][j][lane] = approx;   // for pass 2 (dynamic j)
-                    }
-                }
-                kmask &= msk;
-            }
-            const uint32_t wmask = __reduce_or_sync(BLSH_FULL, kmask);
+            for (int jj = 0; jj < 32; ++jj) Tt[jj * 33 + lane] = dot[jj];
+            S.rinfo[ew][lane] = make_uint4(__float_as_uint(xn * (1.0f - kScr)), __float_as_uint(xn * (1.0f + kScr)),
+                                           msk, prow);
             __syncwarp();
-            // pass 2 (only queries with a kept pair in this warp): bounds, buffers.  Not unrolled
-            // (a 32-fold copy of this body thrashes the instruction cache): the approximate
-            // distances come back from shared memory.
-            for (uint32_t wm = wmask; wm; wm &= wm - 1) {
-                const int j = __ffs(wm) - 1;
-                const bool has = (kmask >> j) & 1u;
-                const float qn = __shfl_sync(BLSH_FULL, my_qn, j);
-                const float Uown = __shfl_sync(BLSH_FULL, my_U, j);
-                const float U = fminf(Uown, __uint_as_float(S.umin[j]));   // any warp's bound is valid
-                const float approx = S.sap[ew][j][lane];
-                const float m = 4e-3f * (qn + xn) + 1e-5f * fabsf(approx) + 1e-30f;
-                const float lo = approx - m, up = approx + m;
-                const bool keep = has && lo <= U;
-                const unsigned km = __ballot_sync(BLSH_FULL, keep);
-                if (!km) continue;
-                // this warp's upper-bound list of query j lives in lane j's registers
-                unsigned um = __ballot_sync(BLSH_FULL, keep && up < Uown);
-                if (um) {
-                    while (um) {
-                        const int src = __ffs(um) - 1;
-                        um &= um - 1;
-                        const float v = __shfl_sync(BLSH_FULL, up, src);
-                        if (lane == j) {
+            const float kth0 = ulr[KT - 1];
+            float U = fminf(kth0, __uint_as_float(S.umin[j]));    // any warp's bound is valid
+#pragma unroll 8
+            for (int i = 0; i < 32; ++i) {
+                const uint4 ri = S.rinfo[ew][i];                   // broadcast
+                const float t2 = -2.0f * Tt[j * 33 + i];
+                const float lo = (qa + __uint_as_float(ri.x)) + t2;
+                if (((ri.z >> j) & 1u) && lo <= U) {               // rare: keep the pair
+                    const float up = (qb + __uint_as_float(ri.y)) + t2;
+                    if (up < U) {                                  // sorted insert; only bounds below U matter
 #pragma unroll
-                            for (int p = kTcMaxK - 1; p > 0; --p)
-                                ulr[p] = ulr[p - 1] > v ? ulr[p - 1] : (ulr[p] > v ? v : ulr[p]);
-                            ulr[0] = ulr[0] > v ? v : ulr[0];
-                        }
+                        for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
+                        ulr[0] = fminf(ulr[0], up);
+                        U = fminf(U, ulr[KT - 1]);
                     }
-                    if (lane == j) {
-                        float kth = ulr[0];
-#pragma unroll
-                        for (int p = 1; p < kTcMaxK; ++p)
-                            if (p == k - 1) kth = ulr[p];
-                        if (kth < my_U) {
-                            my_U = kth;
-                            atomicMin(&S.umin[j], __float_as_uint(kth));
+                    const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ri.w;
+                    if (my_cnt == kTcScap) {                       // full: drop what the tighter U excludes
+                        int c2 = 0;
+                        for (int t = 0; t < kTcScap; ++t) {
+                            const unsigned long long f = SBj[t];
+                            if (__uint_as_float((uint32_t)(f >> 32)) <= U) SBj[c2++] = f;
                         }
+                        my_cnt = c2;
                     }
+                    if (my_cnt < kTcScap) SBj[my_cnt++] = e;
+                    else tc_overflow_lane(a, S.tk[j], &S.lock[j], a.Q + (size_t)a.qorder[q0 + j] * ds, ri.w);
                 }
-                // buffer the kept pairs: (lower bound bits << 32 | table row)
-                const int base = __shfl_sync(BLSH_FULL, my_cnt, j);
-                const int at = base + __popc(km & lanemask_lt());
-                if (keep && at < kTcScap)
-                    SB[(size_t)j * 4 * kTcScap + at] = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | prow;
-                if (lane == j) my_cnt = base + __popc(km);
-                // overflow: rescore those pairs now (warp-cooperative)
-                const unsigned om = __ballot_sync(BLSH_FULL, keep && at >= kTcScap);
-                if (om) tc_overflow(a, S.tk[j], &S.lock[j], a.Q + (size_t)a.qorder[q0 + j] * ds, om, prow, lane);
             }
+            if (ulr[KT - 1] < kth0) atomicMin(&S.umin[j], __float_as_uint(ulr[KT - 1]));
+            __syncwarp();                                          // Tt / rinfo reused by the next block
         }
-        if (lane < QT) S.scnt[ew][lane] = my_cnt;
-        if (a.counters && lane < QT && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
+        S.scnt[ew][j] = my_cnt;
+        if (a.counters && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
         if (warp == kTcEpi0 && lane == 0) tc_stamp(a, item, 4);
     }
     tc_fence_before();

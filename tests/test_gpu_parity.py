@@ -245,6 +245,32 @@ def test_sharded_build_and_merge(blsh, orc, c1):
     assert torch.all((torch.stack(counts) > 0).sum(0) <= 1)
 
 
+@pytest.mark.parametrize("probe,T", [(0, 1), (1, 8)])
+def test_sharded_hierarchy_global_median(blsh, orc, c1, probe, T):
+    """Batch-median tau on a sharded index (R18): blsh_query_base_counts per
+    shard, summed (what the SUM all-reduce of sharded.py does), passed as
+    global_base -> merged result == the single-GPU result == the oracle's."""
+    X, Q = c1
+    Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
+    full = blsh.blsh_build(Xd, n_leaves=8, M=8, W=4.0, seed=5)
+    fi, fd, fn = full.query(Qd, 10, probe=probe, n_probes=T, hierarchy=1)
+    ox = orc.OracleIndex(X, G=8, M=8, W=4.0, seed=5)
+    oi, od, onc = ox.query(Q, 10, probe=probe, T=T, hierarchy=1)
+    assert np.array_equal(fn.cpu().numpy(), onc)
+    shards = [blsh.blsh_build(Xd, n_leaves=8, M=8, W=4.0, seed=5, rank=r, world=2) for r in range(2)]
+    with pytest.raises(blsh.BlshError):     # a sharded index cannot take the median of its own half
+        shards[0].query_packed(Qd, 10, probe=probe, n_probes=T, hierarchy=1)
+    gb = sum(s.base_counts(Qd, probe=probe, n_probes=T) for s in shards)
+    assert np.array_equal(gb.cpu().numpy(), ox.get("q_base"))
+    lists = [s.query_packed(Qd, 10, probe=probe, n_probes=T, hierarchy=1, global_base=gb)[0] for s in shards]
+    mi, md = blsh.blsh_merge_topk(torch.stack(lists).contiguous(), 2, len(Q), 10)
+    torch.cuda.synchronize()
+    assert torch.equal(mi, fi) and torch.equal(md, fd)
+    # host output of the base counts, and widening with an explicit tau ignores global_base
+    hb = shards[1].base_counts(Q, probe=probe, n_probes=T)
+    assert isinstance(hb, np.ndarray) and np.array_equal(hb, shards[1].base_counts(Qd, probe=probe, n_probes=T).cpu().numpy())
+
+
 def test_merge_topk_against_numpy(blsh):
     rng = np.random.default_rng(9)
     L, nq, k = 5, 37, 13
