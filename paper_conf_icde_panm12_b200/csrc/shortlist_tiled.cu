@@ -245,6 +245,8 @@ struct TiledArgs {
     unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
     const int64_t* rows_off;        // [ntiles + 1] union rows before each tile
     const uint2* rowinfo;           // TC: [total rows] (table row, query mask) per union row
+    uint32_t* ufin;                 // TC -> k_tc_rescore: [n_items][QT] final screen bound U_j (fp32 bits)
+    int32_t* scnt;                  // TC -> k_tc_rescore: [n_items][QT][4] buffered pairs per epilogue warp
 };
 
 struct TopK {
@@ -652,7 +654,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
-    partials.ensure(part_bytes + sbuf_bytes + (size_t)std::max<int64_t>(total_rows, 1) * 8);
+    const size_t rinfo_bytes = ((size_t)std::max<int64_t>(total_rows, 1) * 8 + 255) & ~size_t(255);
+    const size_t ufin_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 4 + 255) & ~size_t(255);
+    partials.ensure(part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes + (size_t)std::max<int64_t>(n_items, 1) * QT * 16);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
@@ -663,6 +667,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
     ta.rows_off = rows_off;
+    ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes);
+    ta.scnt = reinterpret_cast<int32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes);
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
     const size_t tc_smem = tc_smem_bytes(a.ds);
@@ -676,8 +682,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     }
     DevBuf tsbuf;
     if (use_tc && (ta.dbgmode & 32) && n_items > 0) {
-        tsbuf.alloc((size_t)n_items * 8 * 8);
-        BLSH_CUDA(cudaMemsetAsync(tsbuf.p, 0, (size_t)n_items * 8 * 8, s));
+        tsbuf.alloc((size_t)n_items * 16 * 8);
+        BLSH_CUDA(cudaMemsetAsync(tsbuf.p, 0, (size_t)n_items * 16 * 8, s));
         ta.tstamp = tsbuf.as<unsigned long long>();
     }
     if (use_tc && ntiles > 0) {
@@ -693,6 +699,14 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
             auto kern = k <= 8 ? k_shortlist_tc<8> : (k <= 12 ? k_shortlist_tc<12> : k_shortlist_tc<16>);
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
+            BLSH_LAUNCH_CHECK();
+            ++*launches;
+            const unsigned rg = (unsigned)((n_items * QT + 7) / 8);
+            const int nvq = (a.ds / 4 + 31) / 32;
+            if (nvq <= 1) k_tc_rescore<1><<<rg, 256, 0, s>>>(ta);
+            else if (nvq == 2) k_tc_rescore<2><<<rg, 256, 0, s>>>(ta);
+            else if (nvq == 3) k_tc_rescore<3><<<rg, 256, 0, s>>>(ta);
+            else k_tc_rescore<4><<<rg, 256, 0, s>>>(ta);
         } else {
             BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);
@@ -715,15 +729,20 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld\n", (long long)n_items, ev[0], ev[1],
                      (long long)total_rows);
     if (ta.tstamp) {   // mean phase durations over items (us)
-        std::vector<unsigned long long> h((size_t)n_items * 8);
+        std::vector<unsigned long long> h((size_t)n_items * 16);
         BLSH_CUDA(cudaMemcpy(h.data(), ta.tstamp, h.size() * 8, cudaMemcpyDeviceToHost));
-        double acc[8] = {0};
-        for (int64_t i = 0; i < n_items; ++i)
-            for (int p = 1; p < 8; ++p)
-                if (h[i * 8 + p]) acc[p] += (double)(h[i * 8 + p] - h[i * 8]) * 1e-3;
-        std::fprintf(stderr, "[tc] phase us after start: setup %.1f conv %.1f mma %.1f epi %.1f sync %.1f compact %.1f end %.1f\n",
+        double acc[9] = {0};
+        unsigned long long pmax = 0, psum = 0;
+        for (int64_t i = 0; i < n_items; ++i) {
+            for (int p = 1; p < 9; ++p)
+                if (h[i * 16 + p]) acc[p] += (double)(h[i * 16 + p] - h[i * 16]) * 1e-3;
+            pmax = std::max(pmax, h[i * 16 + 9]);
+            psum += h[i * 16 + 9];
+        }
+        std::fprintf(stderr, "[tc] phase us after start: setup %.1f conv %.1f mma %.1f epi %.1f sync %.1f compact %.1f "
+                     "rescore %.1f end %.1f; rescored pairs per item mean %.0f max %llu\n",
                      acc[1] / n_items, acc[2] / n_items, acc[3] / n_items, acc[4] / n_items, acc[5] / n_items,
-                     acc[6] / n_items, acc[7] / n_items);
+                     acc[6] / n_items, acc[8] / n_items, acc[7] / n_items, (double)psum / n_items, pmax);
     }
     if (ta.dbg) {
         std::vector<float> h(4096 + 512);

@@ -121,41 +121,10 @@ struct TcSmem {
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
     unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
     int lock[QT];                            // guards tk[q] during overflow rescoring
-    int rcnt[QT];                            // final: pairs to rescore per query
-    int roff[QT + 1];                        // final: their exclusive prefix
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
     float tr[4][32 * 33];                    // per epilogue warp: transposed dots [query][row], padded
     uint4 rinfo[4][32];                      // per epilogue warp: (|x'|^2 bits, query mask, table row) per row
 };
-
-// exact fp32 direct-form d^2 by one thread, in the partial-sum structure of the
-// SIMT tiled kernel's score_rows (blocks of 16 float4, two 32-term chains each,
-// blocks summed in order): TC and SIMT tiled results are bit-identical.  The
-// block's 16 row loads are issued before any arithmetic (memory-level parallelism).
-__device__ __forceinline__ float exact_d2_thread(const float4* __restrict__ x, const float4* __restrict__ q, int nv4) {
-    float tot = 0.f;
-    for (int vb = 0; vb < nv4; vb += 16) {
-        const int ne = min(16, nv4 - vb);
-        float4 xv[16];
-#pragma unroll
-        for (int v = 0; v < 16; ++v)
-            if (v < ne) xv[v] = __ldg(x + vb + v);
-        float a0 = 0.f, a1 = 0.f;
-#pragma unroll
-        for (int v = 0; v < 16; ++v) {
-            if (v < ne) {
-                const float4 qq = q[vb + v];
-                const float dx = qq.x - xv[v].x, dy = qq.y - xv[v].y, dz = qq.z - xv[v].z, dw = qq.w - xv[v].w;
-                a0 = fmaf(dx, dx, a0);
-                a1 = fmaf(dy, dy, a1);
-                a0 = fmaf(dz, dz, a0);
-                a1 = fmaf(dw, dw, a1);
-            }
-        }
-        tot += a0 + a1;
-    }
-    return tot;
-}
 
 __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned long long key) {
     if (key < L[k - 1]) {
@@ -165,13 +134,38 @@ __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned
     }
 }
 
+// The warp short-list's fp32 direct form (k_shortlist, k_tc_rescore: lane l sums the
+// float4 columns l, l+32, .. in one fmaf chain, then a 5-level xor butterfly) evaluated
+// by ONE thread, so every distance the TC path reports has the same bits.
+__device__ __noinline__ float warp_order_d2_thread(const float4* __restrict__ x, const float4* __restrict__ q, int nv4) {
+    float p[32];
+#pragma unroll
+    for (int l = 0; l < 32; ++l) {
+        float acc = 0.0f;
+        for (int v = l; v < nv4; v += 32) {
+            const float4 xv = __ldg(x + v), qq = q[v];
+            const float dx = qq.x - xv.x, dy = qq.y - xv.y, dz = qq.z - xv.z, dw = qq.w - xv.w;
+            acc = fmaf(dx, dx, acc);
+            acc = fmaf(dy, dy, acc);
+            acc = fmaf(dz, dz, acc);
+            acc = fmaf(dw, dw, acc);
+        }
+        p[l] = acc;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+        for (int l = 0; l < o; ++l) p[l] = p[l] + p[l + o];
+    return p[0];
+}
+
 // Overflow (screen phase, lane = query): the pair's exact d^2 by this thread,
 // inserted into the query's shared top-k under its lock.  Only when a pair buffer is
 // still full after dropping what the current bound excludes.
 __device__ __noinline__ void tc_overflow_lane(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
                                               uint32_t prow) {
-    const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
-                                     reinterpret_cast<const float4*>(qq), a.ds >> 2);
+    const float d2 = warp_order_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
+                                          reinterpret_cast<const float4*>(qq), a.ds >> 2);
     const unsigned long long key = pack_entry(d2, __ldg(a.perm + prow));
     while (atomicCAS(lock, 0, 1) != 0) {
     }
@@ -185,7 +179,7 @@ __device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p
     if (a.tstamp) {
         unsigned long long t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-        a.tstamp[item * 8 + p] = t;
+        a.tstamp[item * 16 + p] = t;
     }
 }
 
@@ -499,78 +493,113 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
     }
     if (threadIdx.x == 0) tc_stamp(a, item, 5);
-    // ---- final (all warps): exact rescoring of the buffered pairs whose lower bound is <= U_j ----
-    // The B operand and the A ring are dead: L[j][0 .. 4 * kTcScap) holds query j's pairs,
-    // first as (j << 32 | table row), then, rescored in place, as packed (d2, id) keys.
-    constexpr int kNW = kTcThreads / 32;
-    constexpr int kPerQ = 4 * kTcScap;
-    unsigned long long* L = reinterpret_cast<unsigned long long*>(opbase);
-    for (int j = warp; j < QT; j += kNW) {              // (a) compact: one warp per query
-        int c = 0;
-        if (j < nqt) {
-            const float U = __uint_as_float(S.umin[j]);
-            for (int w = 0; w < 4; ++w) {
-                const int cnt = min(S.scnt[w][j], kTcScap);
-                const unsigned long long* Bf = a.sbuf + (((size_t)item * QT + j) * 4 + w) * kTcScap;
-                for (int base = 0; base < cnt; base += 32) {
-                    const int i = base + lane;
-                    const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
-                    const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
-                    const unsigned nm = __ballot_sync(BLSH_FULL, need);
-                    if (need) L[(size_t)j * kPerQ + c + __popc(nm & lanemask_lt())] = ((unsigned long long)j << 32) | (e & 0xFFFFFFFFull);
-                    c += __popc(nm);
+    // ---- hand-off to k_tc_rescore: final bound U_j, buffered pair counts, overflow top-k ----
+    if (threadIdx.x < QT) {
+        const int j = threadIdx.x;
+        a.ufin[(size_t)item * QT + j] = j < nqt ? S.umin[j] : 0u;   // 0.0f: nothing to rescore for padding slots
+#pragma unroll
+        for (int w = 0; w < 4; ++w) a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
+    }
+    for (int i = threadIdx.x; i < nqt * k; i += kTcThreads)
+        a.partials[((size_t)item * QT + i / k) * k + i % k] = S.tk[i / k][i % k];   // overflow-path results
+}
+
+// Exact rescoring of the TC screen's survivors, at full occupancy (one warp per
+// (item, query)): the buffered pairs whose lower bound is <= the final U_j get the
+// fp32 direct-form distance of k_shortlist (lane l: float4 columns l, l+32, ..,
+// per-lane fmaf chain, butterfly; bit-identical to the warp short-list), four rows
+// at a time, and a warp top-k that starts from the TC kernel's overflow results.
+template <int NV>
+__global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
+    const int lane = threadIdx.x & 31;
+    const int64_t unit = blockIdx.x * (int64_t)8 + (threadIdx.x >> 5);
+    if (unit >= a.n_items * QT) return;
+    const int64_t item = unit / QT;
+    const int j = (int)(unit % QT);
+    int64_t lo = 0, hi = a.ntiles;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (a.item_off[mid] <= item) lo = mid;
+        else hi = mid;
+    }
+    const int64_t q0 = a.tile_off[lo];
+    if (j >= (int)(a.tile_off[lo + 1] - q0)) return;
+    const int k = a.k, nv = a.ds >> 2;
+    unsigned long long* out = a.partials + (size_t)unit * k;
+    TopK tk{lane < k ? out[lane] : kEmpty, kEmpty};
+    unsigned long long thr = topk_thr(tk, k);
+    const float U = __uint_as_float(a.ufin[unit]);
+    const float4* qrow = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + j] * a.ds);
+    float4 qv[NV];
+#pragma unroll
+    for (int u = 0; u < NV; ++u) {
+        const int v = lane + 32 * u;
+        qv[u] = v < nv ? __ldg(qrow + v) : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    int rescored = 0;
+    for (int w = 0; w < 4; ++w) {
+        const int cnt = a.scnt[unit * 4 + w];
+        const unsigned long long* Bf = a.sbuf + ((size_t)unit * 4 + w) * kTcScap;
+        for (int base = 0; base < cnt; base += 32) {
+            const int i = base + lane;
+            const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
+            const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+            unsigned nm = __ballot_sync(BLSH_FULL, need);
+            rescored += __popc(nm);
+            while (nm) {
+                uint32_t row[4];
+                int nr = 0;
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    row[r] = 0u;
+                    if (nm) {
+                        const int src = __ffs(nm) - 1;
+                        nm &= nm - 1;
+                        row[r] = (uint32_t)__shfl_sync(BLSH_FULL, (unsigned)(e & 0xFFFFFFFFull), src);
+                        nr = r + 1;
+                    }
+                }
+                float part[4];
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    part[r] = 0.0f;
+                    if (r < nr) {
+                        const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)row[r] * a.ds);
+#pragma unroll
+                        for (int u = 0; u < NV; ++u) {
+                            const int v = lane + 32 * u;
+                            if (v < nv) {
+                                const float4 x = __ldg(xr + v);
+                                const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                                part[r] = fmaf(dx, dx, part[r]);
+                                part[r] = fmaf(dy, dy, part[r]);
+                                part[r] = fmaf(dz, dz, part[r]);
+                                part[r] = fmaf(dw, dw, part[r]);
+                            }
+                        }
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+                    for (int r = 0; r < 4; ++r) part[r] += __shfl_xor_sync(BLSH_FULL, part[r], o);
+                }
+                const uint32_t rl = (lane & 3) == 0 ? row[0] : (lane & 3) == 1 ? row[1] : (lane & 3) == 2 ? row[2] : row[3];
+                const uint32_t idl = lane < nr ? __ldg(a.perm + rl) : 0u;
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    const uint32_t id = __shfl_sync(BLSH_FULL, idl, r);
+                    if (r < nr) {
+                        const unsigned long long key = pack_entry(part[r], id);
+                        if (key < thr) {
+                            topk_insert(tk, key, lane);
+                            thr = topk_thr(tk, k);
+                        }
+                    }
                 }
             }
         }
-        if (lane == 0) S.rcnt[j] = c;
     }
-    __syncthreads();
-    if (warp == 0) {                                    // exclusive prefix of the per-query counts
-        const int c = S.rcnt[lane];
-        int inc = c;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(BLSH_FULL, inc, o);
-            if (lane >= o) inc += t;
-        }
-        S.roff[lane] = inc - c;
-        if (lane == 31) S.roff[32] = inc;
-    }
-    __syncthreads();
-    const int total = S.roff[32];
-    // the tile's queries, exact, into shared memory behind L (the rescoring reads them per pair)
-    float* Qx = reinterpret_cast<float*>(opbase + (size_t)QT * kPerQ * 8);
-    for (int i = threadIdx.x; i < nqt * nv4; i += kTcThreads)
-        reinterpret_cast<float4*>(Qx)[i] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + i / nv4] * ds) + i % nv4);
-    __syncthreads();
-    if (threadIdx.x == 0) tc_stamp(a, item, 6);
-    for (int idx = threadIdx.x; idx < total; idx += kTcThreads) {   // (b) one thread per pair
-        int lo2 = 0, hi2 = 32;                                      // query j: roff[j] <= idx < roff[j + 1]
-        while (hi2 - lo2 > 1) {
-            const int m = (lo2 + hi2) >> 1;
-            if (S.roff[m] <= idx) lo2 = m;
-            else hi2 = m;
-        }
-        unsigned long long& e = L[(size_t)lo2 * kPerQ + (idx - S.roff[lo2])];
-        const uint32_t srow = (uint32_t)(e & 0xFFFFFFFFull);
-        const float d2 = exact_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)srow * ds),
-                                         reinterpret_cast<const float4*>(Qx + (size_t)lo2 * ds), nv4);
-        e = pack_entry(d2, __ldg(a.perm + srow));
-    }
-    __syncthreads();
-    for (int j = warp; j < nqt; j += kNW) {             // (c) per-query top-k of the rescored keys
-        TopK tk{kEmpty, kEmpty};
-        unsigned long long thr = kEmpty;
-        const int c = S.rcnt[j];
-        for (int base = 0; base < c; base += 32)
-            topk_offer(tk, thr, base + lane < c ? L[(size_t)j * kPerQ + base + lane] : kEmpty, k, lane);
-        topk_offer(tk, thr, lane < k ? S.tk[j][lane] : kEmpty, k, lane);   // overflow-path results
-        unsigned long long* out = a.partials + ((size_t)item * QT + j) * k;
-        if (lane < k) out[lane] = tk.e0;
-    }
-    if (threadIdx.x == 0 && a.counters && total) atomicAdd(a.counters + 1, (unsigned long long)total);
-    if (a.tstamp) {
-        __syncthreads();
-        if (threadIdx.x == 0) tc_stamp(a, item, 7);
-    }
+    if (lane < k) out[lane] = tk.e0;
+    if (lane == 0 && a.counters && rescored) atomicAdd(a.counters + 1, (unsigned long long)rescored);
 }

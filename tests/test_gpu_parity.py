@@ -346,14 +346,14 @@ def _query_mode(ix, Q, k, mode, monkeypatch, **kw):
 
 
 @pytest.mark.parametrize("shape", ["lowrank384", "d512", "dup_overflow"])
-def test_tc_screen_equals_simt(blsh, orc, monkeypatch, shape):
+def test_tc_screen_equals_warp(blsh, orc, monkeypatch, shape):
     """The tensor-core screen only decides which pairs get exact fp32 work, and its exact
-    rescoring uses the SIMT tiled kernel's partial-sum order, so the two short-lists must
-    agree bit for bit (ids and d^2 bits); d512 (beyond the SIMT tiled kernel) is checked
-    against the oracle.  lowrank384: the C3/C4 shape (tight low-rank
-    clusters far from the origin, where the screen's bound matters); d512: the largest
-    d_stride the TC kernel takes; dup_overflow: 10 points repeated 1000x, so hundreds of
-    pairs tie inside the screen margin and the per-warp pair buffers overflow."""
+    rescoring (k_tc_rescore, and the overflow path) uses the warp short-list's partial-sum
+    order, so the two short-lists must agree bit for bit (ids and d^2 bits).  lowrank384:
+    the C3/C4 shape (tight low-rank clusters far from the origin, where the screen's bound
+    matters); d512: the largest d_stride the TC kernel takes; dup_overflow: 10 points
+    repeated 1000x, so hundreds of pairs tie inside the screen margin and the per-warp
+    pair buffers overflow."""
     if shape == "lowrank384":
         mix = synth.mixture(384, 64, 16, 0.02, 31)
         X = synth.sample_points(mix, 20000, 32)
@@ -371,15 +371,10 @@ def test_tc_screen_equals_simt(blsh, orc, monkeypatch, shape):
         Q = synth.sample_points(mix, 100, 53)
         G, W, T = 2, 3.0, 4
     ix, ox = build_pair(blsh, orc, X, G=G, M=8, W=W, seed=5)
-    if shape == "d512":   # the SIMT tiled kernel's staging does not fit at d = 512: TC vs the oracle
-        for k in (1, 10, 16):
-            run_query_pair(ix, ox, X, Q[:80], k, probe=1, T=T)
-            assert ix.stats().tiled == 2
-        return
     for k in (1, 10, 16):
-        a = _query_mode(ix, Q, k, "simt", monkeypatch, probe=1, n_probes=T)
+        a = _query_mode(ix, Q, k, "warp", monkeypatch, probe=1, n_probes=T)
         b = _query_mode(ix, Q, k, "tc", monkeypatch, probe=1, n_probes=T)
-        assert a[3] == 1 and b[3] == 2
+        assert a[3] == 0 and b[3] == 2
         np.testing.assert_array_equal(a[2], b[2])
         np.testing.assert_array_equal(a[0], b[0])
         np.testing.assert_array_equal(a[1].view(np.uint32), b[1].view(np.uint32))
