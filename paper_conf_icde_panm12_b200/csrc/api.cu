@@ -270,6 +270,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     add(nq + 1, 8);                     // cand_off
     add(4, 8);                          // tau + misc
     add(nq, 4);                         // qorder
+    add(nq, 4); add((size_t)2 * ix.G, 4);   // lperm, leaf counts + cursors
     if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
     if (out_host) { add((size_t)nq * k, 8); add((size_t)nq * k, 4); add(nq, 8); add((size_t)nq * k, 8); }
     w.arena.ensure(need);
@@ -289,6 +290,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t* cand_off = ar.take<int64_t>(nq + 1);
     w.tau = ar.take<int64_t>(4);
     uint32_t* qorder = ar.take<uint32_t>(nq);
+    uint32_t* lperm = ar.take<uint32_t>(nq);
+    int32_t* lcnt = ar.take<int32_t>((size_t)2 * ix.G);
     w.pkey = keep ? ar.take<Key128>((size_t)nq * T) : nullptr;
     w.pvalid = keep ? ar.take<int32_t>((size_t)nq * T) : nullptr;
     int64_t* d_ids = out_ids;
@@ -323,8 +326,9 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.ukey = ix.ukey.as<Key128>(); a.uoff = ix.uoff.as<uint32_t>(); a.leaf_u = ix.leaf_u.as<int64_t>();
     a.qleaf = w.qleaf; a.qt = w.qt; a.qcode = w.qcode; a.qoor = w.qoor; a.qkey = w.qkey;
     a.pkey = w.pkey; a.pvalid = w.pvalid; a.ivl = w.ivl; a.base = w.base; a.cnt = w.cnt; a.level = w.level;
+    a.lperm = lperm; a.lcnt = lcnt;
     // a1+a2
-    launch_route_hash(a, s); ++launches;
+    launches += launch_route_hash(a, s);
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // a3+a4
     launch_probe_lookup(a, s); ++launches;

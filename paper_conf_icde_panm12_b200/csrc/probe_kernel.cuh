@@ -36,6 +36,61 @@ __device__ __forceinline__ double pool_score(const PoolT<MM>& pl, uint32_t x, in
     return s;
 }
 
+// Every perturbation delta != 0 with score(delta) <= Bp, in enc order, by a
+// breadth-first expansion over the coordinates (i ascending): a partial
+// assignment keeps its running sum, which is exactly the score's summation
+// order (R11), and is dropped as soon as the sum exceeds Bp (rounded sums of
+// non-negative terms never decrease, so no completion of it can come back under
+// Bp).  Children are written in digit order after a warp scan, so each level is
+// sorted by enc prefix.  Returns false when a level would exceed kFCap.
+template <int MM>
+__device__ bool frontier_enum(ProbeSmem& sm, const PoolT<MM>& pl, double Bp, int lane, int* K, int* buf) {
+    int F = 1, cur = 0;
+    uint32_t home = 0;                  // enc prefix of the all-zero partial
+    if (lane == 0) {
+        sm.fs[0][0] = 0.0;
+        sm.fe[0][0] = 0u;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int i = 0; i < MM; ++i) {
+        const bool last = i == MM - 1;
+        int out = 0;
+        for (int base = 0; base < F; base += 32) {
+            const int e = base + lane;
+            const bool v = e < F;
+            const double sp = v ? sm.fs[cur][e] : 0.0;
+            const uint32_t en = v ? sm.fe[cur][e] : 0u;
+            const double sm1 = __dadd_rn(sp, pl.sqm[i]), sp1 = __dadd_rn(sp, pl.sqp[i]);
+            const bool cm = v && sm1 <= Bp;
+            const bool c0 = v && !(last && en == home);
+            const bool cp = v && sp1 <= Bp;
+            const int c = (int)cm + (int)c0 + (int)cp;
+            int inc = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(BLSH_FULL, inc, o);
+                if (lane >= o) inc += y;
+            }
+            const int tot = __shfl_sync(BLSH_FULL, inc, 31);
+            if (out + tot > kFCap) return false;
+            int at = out + inc - c;
+            const int nx = cur ^ 1;
+            if (cm) { sm.fs[nx][at] = sm1; sm.fe[nx][at] = en * 3u; ++at; }
+            if (c0) { sm.fs[nx][at] = sp; sm.fe[nx][at] = en * 3u + 1u; ++at; }
+            if (cp) { sm.fs[nx][at] = sp1; sm.fe[nx][at] = en * 3u + 2u; }
+            out += tot;
+        }
+        home = home * 3u + 1u;
+        F = out;
+        cur ^= 1;
+        __syncwarp();
+    }
+    *K = F;
+    *buf = cur;
+    return true;
+}
+
 template <int MM>
 __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int lane, int64_t ulo, int64_t uhi,
                             uint2* ivl) {
@@ -48,6 +103,7 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
         fl[i] = floorf(t[i]);
     }
     PoolT<MM> pl;
+    int fbuf = -1;                // >= 0: the selection indexes the frontier sm.fe[fbuf]
     if (a.probe == 1 && T > 1) {
         double v[2 * MM];
 #pragma unroll
@@ -90,10 +146,16 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
         }
         pl.P = P;
         pl.home = home;
-        warp_select(sm, P, home, T - 1, [&](uint32_t x) {
-            int8_t dl[MM];
-            return pool_score<MM>(pl, x, dl);
-        });
+        int K = 0;
+        if (MM <= 10 && frontier_enum<MM>(sm, pl, Bp, lane, &K, &fbuf)) {
+            warp_select(sm, (uint32_t)K, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return sm.fs[fbuf][x]; });
+        } else {
+            fbuf = -1;
+            warp_select(sm, P, home, T - 1, [&](uint32_t x) {
+                int8_t dl[MM];
+                return pool_score<MM>(pl, x, dl);
+            });
+        }
     }
     int64_t mysum = 0;
     const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
@@ -101,7 +163,19 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
         int8_t dl[MM];
 #pragma unroll
         for (int i = 0; i < MM; ++i) dl[i] = 0;
-        if (p > 0) pool_score<MM>(pl, sm.order[p - 1], dl);
+        if (p > 0) {
+            if (fbuf >= 0) {
+                uint32_t en = sm.fe[fbuf][sm.order[p - 1]];
+#pragma unroll
+                for (int i = MM - 1; i >= 0; --i) {
+                    const uint32_t qv = __umulhi(en, 0xAAAAAAABu) >> 1;
+                    dl[i] = (int8_t)((int)(en - qv * 3u) - 1);
+                    en = qv;
+                }
+            } else {
+                pool_score<MM>(pl, sm.order[p - 1], dl);
+            }
+        }
         int32_t pc[MM];
         bool valid = true;
 #pragma unroll

@@ -20,38 +20,156 @@ namespace {
 // ---------------------------------------------------------------------------
 // a1 + a2
 // ---------------------------------------------------------------------------
-template <int MM>
-__global__ void __launch_bounds__(128) k_route_hash(QueryArgs a) {
-    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (q >= a.nq) return;
-    const float* x = a.Q + (size_t)q * a.ds;
+// a1 and a2 run as two passes so that the projection reads its leaf's M x d
+// matrix from shared memory:
+//   k_route       one warp per block, one query per lane: the 32 query rows are
+//                 staged into shared memory with coalesced 16-byte loads (row
+//                 pitch ds + 4 floats, so the lanes' 16-byte reads at the same
+//                 column fall into distinct bank groups); each lane descends the
+//                 tree with its query's canonical chains (R1: strictly ascending
+//                 j, explicit fmaf), node vectors through L1; leaf histogram.
+//   k_leaf_scan / k_leaf_scatter   group the queries by leaf (lperm).
+//   k_hash        32 leaf-grouped queries per block; the block's leaf matrix A_g
+//                 is staged in shared memory (broadcast reads), the rows again;
+//                 each lane runs its M projection chains, Eq. 2 / E8, Morton key.
+constexpr int kRHQ = 32;
+
+__device__ __forceinline__ void stage_rows(const QueryArgs& a, float4* rows4, const uint32_t* qids, int64_t q0,
+                                           int nrow, int lane) {
+    const int nv4 = a.ds >> 2, pitch4 = nv4 + 1;
+    for (int r = 0; r < nrow; ++r) {
+        const int64_t q = qids ? (int64_t)qids[q0 + r] : q0 + r;
+        for (int v = lane; v < nv4; v += 32)
+            rows4[r * pitch4 + v] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds) + v);
+    }
+}
+
+__global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict__ lcnt) {
+    extern __shared__ __align__(16) float rh_rows[];
+    const int lane = threadIdx.x;
+    const int64_t q0 = blockIdx.x * (int64_t)kRHQ;
+    const int nrow = (int)min((int64_t)kRHQ, a.nq - q0);
+    float4* rows4 = reinterpret_cast<float4*>(rh_rows);
+    stage_rows(a, rows4, nullptr, q0, nrow, lane);
+    __syncwarp();
+    if (lane >= nrow) return;
+    const int64_t q = q0 + lane;
+    const float4* x4 = rows4 + lane * ((a.ds >> 2) + 1);
     const int d = a.d;
+    const int nfull = d >> 2, rem = d & 3;
     int v = 0;
     for (int l = 0; l < a.depth; ++l) {
         float s = 0.0f;
         if (a.ntype[v] == 0) {
-            const float* dir = a.dirs + (size_t)v * a.ds;
-            for (int j = 0; j < d; ++j) s = __fmaf_rn(__ldg(dir + j), __ldg(x + j), s);
+            const float4* dir4 = reinterpret_cast<const float4*>(a.dirs + (size_t)v * a.ds);
+#pragma unroll 4
+            for (int j4 = 0; j4 < nfull; ++j4) {
+                const float4 xv = x4[j4], dv = __ldg(dir4 + j4);
+                s = __fmaf_rn(dv.x, xv.x, s);
+                s = __fmaf_rn(dv.y, xv.y, s);
+                s = __fmaf_rn(dv.z, xv.z, s);
+                s = __fmaf_rn(dv.w, xv.w, s);
+            }
+            if (rem) {
+                const float4 xv = x4[nfull], dv = __ldg(dir4 + nfull);
+                s = __fmaf_rn(dv.x, xv.x, s);
+                if (rem > 1) s = __fmaf_rn(dv.y, xv.y, s);
+                if (rem > 2) s = __fmaf_rn(dv.z, xv.z, s);
+            }
         } else {
-            const float* mu = a.mu + (size_t)v * a.ds;
-            for (int j = 0; j < d; ++j) {
-                const float e = __fsub_rn(__ldg(x + j), __ldg(mu + j));
-                s = __fmaf_rn(e, e, s);
+            const float4* mu4 = reinterpret_cast<const float4*>(a.mu + (size_t)v * a.ds);
+            for (int j4 = 0; j4 < (d + 3) >> 2; ++j4) {
+                const float4 xv = x4[j4], mv = __ldg(mu4 + j4);
+                const float xs[4] = {xv.x, xv.y, xv.z, xv.w}, ms[4] = {mv.x, mv.y, mv.z, mv.w};
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    if (4 * j4 + c < d) {
+                        const float e = __fsub_rn(xs[c], ms[c]);
+                        s = __fmaf_rn(e, e, s);
+                    }
+                }
             }
         }
         v = 2 * v + 1 + (s > a.theta[v] ? 1 : 0);
     }
     const int g = v - (a.G - 1);
     a.qleaf[q] = g;
+    atomicAdd(&lcnt[g], 1);
+}
+
+// exclusive scan of the G leaf counts into the scatter cursors (one block)
+__global__ void __launch_bounds__(1024) k_leaf_scan(const int32_t* __restrict__ lcnt, int G, int32_t* __restrict__ lcur) {
+    __shared__ int32_t wsum[32];
+    const int per = (G + 1023) / 1024;
+    const int lo = threadIdx.x * per, hi = min(G, lo + per);
+    int32_t c = 0;
+    for (int i = lo; i < hi; ++i) c += lcnt[i];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int32_t inc = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) wsum[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+        int32_t x = wsum[lane], xi = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int32_t y = __shfl_up_sync(BLSH_FULL, xi, o);
+            if (lane >= o) xi += y;
+        }
+        wsum[lane] = xi - x;
+    }
+    __syncthreads();
+    int32_t run = wsum[w] + inc - c;
+    for (int i = lo; i < hi; ++i) {
+        lcur[i] = run;
+        run += lcnt[i];
+    }
+}
+
+__global__ void k_leaf_scatter(const int32_t* __restrict__ qleaf, int64_t nq, int32_t* __restrict__ lcur,
+                               uint32_t* __restrict__ lperm) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q < nq) lperm[atomicAdd(&lcur[qleaf[q]], 1)] = (uint32_t)q;
+}
+
+template <int MM>
+__global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __restrict__ lperm) {
+    extern __shared__ __align__(16) float rh_rows[];
+    const int lane = threadIdx.x;
+    const int64_t p0 = blockIdx.x * (int64_t)kRHQ;
+    const int nrow = (int)min((int64_t)kRHQ, a.nq - p0);
+    const int d = a.d;
+    float4* rows4 = reinterpret_cast<float4*>(rh_rows);
+    float* As = rh_rows + (size_t)kRHQ * (a.ds + 4);     // [MM][d] of the block's first leaf
+    const int g0 = a.qleaf[lperm[p0]];
+    const float* Ag0 = a.A + (size_t)g0 * MM * d;
+    for (int i = lane; i < MM * d; i += 32) As[i] = __ldg(Ag0 + i);
+    stage_rows(a, rows4, lperm, p0, nrow, lane);
+    __syncwarp();
+    if (lane >= nrow) return;
+    const int64_t q = lperm[p0 + lane];
+    const float4* x4 = rows4 + lane * ((a.ds >> 2) + 1);
+    const int g = a.qleaf[q];
     const bool active = g >= a.leaf_lo && g < a.leaf_hi;
+    const float* Ag = g == g0 ? As : a.A + (size_t)g * MM * d;   // generic: shared (broadcast) or global
     float s[MM];
 #pragma unroll
     for (int i = 0; i < MM; ++i) s[i] = 0.0f;
-    const float* Ag = a.A + (size_t)g * MM * d;
-    for (int j = 0; j < d; ++j) {
-        const float xj = __ldg(x + j);
+    for (int j4 = 0; j4 < (d + 3) >> 2; ++j4) {
+        const float4 xv = x4[j4];
+        const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
-        for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(__ldg(Ag + (size_t)i * d + j), xj, s[i]);
+        for (int c = 0; c < 4; ++c) {
+            const int j = 4 * j4 + c;
+            if (j < d) {
+#pragma unroll
+                for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(Ag[(size_t)i * d + j], xs[c], s[i]);
+            }
+        }
     }
     const float W = a.Wl[g];
     float t[MM];
@@ -88,11 +206,15 @@ __device__ __forceinline__ int64_t find_bucket(const Key128* __restrict__ ukey, 
 constexpr int kPW = 4;          // warps per block in k_probe_lookup
 constexpr int kMaxSel = 256;    // max probes (T <= 256)
 
+constexpr int kFCap = 256;      // multiprobe frontier capacity (larger sets fall back to the pool)
+
 struct ProbeSmem {
     uint32_t hist[256];
     unsigned long long sbits[kMaxSel];
     uint32_t sx[kMaxSel];
     uint32_t order[kMaxSel];
+    double fs[2][kFCap];        // frontier: partial scores
+    uint32_t fe[2][kFCap];      // frontier: partial enc (base-3 digits delta_i + 1, i = 0 most significant)
 };
 
 // Multiprobe pool (R11 + the pruning bound in DESIGN.md "Probe generation"):
@@ -127,19 +249,44 @@ __device__ __forceinline__ double lat_score(const float* y, const int32_t* c2, u
 
 // Select the R smallest (score, pool index) of a pool with an exact warp radix
 // select over the fp64 score bits (scores >= 0: bit order == value order).
-// Writes the selection sorted by (score, index) into sm.sx[0..R).
-template <typename ScoreFn>
-__device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, ScoreFn score) {
+// Writes the selection sorted by (score, index) into sm.order[0..R).
+// Pools of up to 32 * kSelCache entries (the common case: the pruning bound keeps
+// a few dozen) score every entry once into registers (lane l, slot c holds pool
+// index l + 32 c); larger pools re-score in every pass.
+constexpr int kSelCache = 8;
+
+template <bool CACHED, typename ScoreFn>
+__device__ void warp_select_impl(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, ScoreFn score) {
     const int lane = threadIdx.x & 31;
+    unsigned long long sc[CACHED ? kSelCache : 1];
+    // key of pool entry x = lane + 32 c (~0 = not in the pool)
+    auto key = [&](int c, uint32_t x) -> unsigned long long {
+        if (CACHED) return sc[c];
+        return (x < P && x != skip) ? (unsigned long long)__double_as_longlong(score(x)) : ~0ull;
+    };
+    const int nslot = (int)((P + 31) / 32);
+    if (CACHED) {
+#pragma unroll
+        for (int c = 0; c < kSelCache; ++c) {
+            const uint32_t x = lane + 32u * c;
+            sc[c] = (x < P && x != skip) ? (unsigned long long)__double_as_longlong(score(x)) : ~0ull;
+        }
+    }
     unsigned long long prefix = 0ull, mask = 0ull;
     int r = R - 1;
     // bits common to every key are skipped: start at the byte of the highest differing bit
     unsigned long long kmin = ~0ull, kmax = 0ull;
-    for (uint32_t x = lane; x < P; x += 32) {
-        if (x == skip) continue;
-        const unsigned long long b = (unsigned long long)__double_as_longlong(score(x));
-        kmin = b < kmin ? b : kmin;
-        kmax = b > kmax ? b : kmax;
+#pragma unroll
+    for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
+        for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
+            const uint32_t x = lane + 32u * cc;
+            const unsigned long long b = key(c, x);
+            if (b != ~0ull) {
+                kmin = b < kmin ? b : kmin;
+                kmax = b > kmax ? b : kmax;
+            }
+            if (CACHED) break;
+        }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
@@ -161,10 +308,13 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
     for (int sh = sh0; sh >= 0; sh -= 8) {
         for (int i = lane; i < 256; i += 32) sm.hist[i] = 0;
         __syncwarp();
-        for (uint32_t x = lane; x < P; x += 32) {
-            if (x == skip) continue;
-            const unsigned long long b = (unsigned long long)__double_as_longlong(score(x));
-            if ((b & mask) == prefix) atomicAdd(&sm.hist[(b >> sh) & 255ull], 1u);
+#pragma unroll
+        for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
+            for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
+                const unsigned long long b = key(c, lane + 32u * cc);
+                if (b != ~0ull && (b & mask) == prefix) atomicAdd(&sm.hist[(b >> sh) & 255ull], 1u);
+                if (CACHED) break;
+            }
         }
         __syncwarp();
         uint32_t loc[8], tot = 0;
@@ -200,25 +350,26 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
     // take every key whose masked bits are < prefix, plus the first r+1 (ascending index)
     // of those equal to it (either all of them, or exact ties after the last digit)
     int cnt = 0, ties = 0;
-    for (uint32_t base = 0; base < P; base += 32) {
-        const uint32_t x = base + lane;
-        unsigned long long b = ~0ull, bm = ~0ull;
-        if (x < P && x != skip) {
-            b = (unsigned long long)__double_as_longlong(score(x));
-            bm = b & mask;
+#pragma unroll
+    for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
+        for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
+            const uint32_t x = lane + 32u * cc;
+            const unsigned long long b = key(c, x);
+            const unsigned long long bm = b == ~0ull ? ~0ull : (b & mask);
+            const bool tie = b != ~0ull && bm == prefix;
+            const unsigned tm = __ballot_sync(BLSH_FULL, tie);
+            const int my_tie = ties + __popc(tm & lanemask_lt());
+            ties += __popc(tm);
+            const bool sel = (b != ~0ull && bm < prefix) || (tie && my_tie <= r);
+            const unsigned smk = __ballot_sync(BLSH_FULL, sel);
+            if (sel) {
+                const int at = cnt + __popc(smk & lanemask_lt());
+                sm.sbits[at] = b;
+                sm.sx[at] = x;
+            }
+            cnt += __popc(smk);
+            if (CACHED) break;
         }
-        const bool tie = bm == prefix;
-        const unsigned tm = __ballot_sync(BLSH_FULL, tie);
-        const int my_tie = ties + __popc(tm & lanemask_lt());
-        ties += __popc(tm);
-        const bool sel = bm < prefix || (tie && my_tie <= r);
-        const unsigned smk = __ballot_sync(BLSH_FULL, sel);
-        if (sel) {
-            const int at = cnt + __popc(smk & lanemask_lt());
-            sm.sbits[at] = b;
-            sm.sx[at] = x;
-        }
-        cnt += __popc(smk);
     }
     __syncwarp();
     // sort the R selected entries by (score bits, index): rank by counting
@@ -233,6 +384,12 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
         sm.order[rk] = x;
     }
     __syncwarp();
+}
+
+template <typename ScoreFn>
+__device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, ScoreFn score) {
+    if (P <= 32u * kSelCache) warp_select_impl<true>(sm, P, skip, R, score);
+    else warp_select_impl<false>(sm, P, skip, R, score);
 }
 
 #if 0   // superseded by probe_kernel.cuh (kept until the next cleanup)
@@ -481,10 +638,26 @@ void upload_e8_roots() {
     done = true;
 }
 
-void launch_route_hash(const QueryArgs& a, cudaStream_t s) {
-    const unsigned grid = (unsigned)((a.nq + 127) / 128);
-#define BLSH_RH_CASE(MMV) \
-    case MMV: k_route_hash<MMV><<<grid, 128, 0, s>>>(a); break;
+int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
+    if (a.nq == 0) return 0;
+    const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
+    const size_t smem_r = (size_t)kRHQ * (a.ds + 4) * sizeof(float);
+    const size_t smem_h = smem_r + (size_t)a.M * a.d * sizeof(float);
+    int32_t* lcnt = a.lcnt;
+    int32_t* lcur = a.lcnt + a.G;
+    BLSH_CUDA(cudaMemsetAsync(lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
+    BLSH_CUDA(cudaFuncSetAttribute(k_route, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_r));
+    k_route<<<grid, kRHQ, smem_r, s>>>(a, lcnt);
+    BLSH_LAUNCH_CHECK();
+    k_leaf_scan<<<1, 1024, 0, s>>>(lcnt, a.G, lcur);
+    BLSH_LAUNCH_CHECK();
+    k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, lcur, a.lperm);
+    BLSH_LAUNCH_CHECK();
+#define BLSH_RH_CASE(MMV)                                                                                   \
+    case MMV:                                                                                              \
+        BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        k_hash<MMV><<<grid, kRHQ, smem_h, s>>>(a, a.lperm);                                                 \
+        break;
     switch (a.M) {
         BLSH_RH_CASE(1) BLSH_RH_CASE(2) BLSH_RH_CASE(3) BLSH_RH_CASE(4)
         BLSH_RH_CASE(5) BLSH_RH_CASE(6) BLSH_RH_CASE(7) BLSH_RH_CASE(8)
@@ -494,6 +667,7 @@ void launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     }
 #undef BLSH_RH_CASE
     BLSH_LAUNCH_CHECK();
+    return 4;
 }
 
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s) {

@@ -37,10 +37,12 @@ struct QueryArgs {
     int64_t* base;
     int64_t* cnt;
     int32_t* level;          // nullable
+    uint32_t* lperm;         // [nq] queries grouped by leaf (a1 -> a2)
+    int32_t* lcnt;           // [2G] leaf counts, scatter cursors
 };
 
 void upload_e8_roots();
-void launch_route_hash(const QueryArgs& a, cudaStream_t s);
+int launch_route_hash(const QueryArgs& a, cudaStream_t s);   // returns kernels launched
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s);
 void launch_median(const int64_t* base, int64_t nq, int64_t* tau, cudaStream_t s);
 void launch_widen(const QueryArgs& a, const int64_t* tau, int64_t min_cand, cudaStream_t s);

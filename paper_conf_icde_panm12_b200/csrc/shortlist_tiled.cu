@@ -465,8 +465,12 @@ __global__ void k_qsort_keys(const Key128* __restrict__ qkey, const int32_t* __r
                              unsigned long long* __restrict__ lo, uint32_t* __restrict__ leaf, uint32_t* __restrict__ id) {
     const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (q >= nq) return;
+    // Sorting only groups similar queries into tiles (results do not depend on the order):
+    // the low 64 key bits are the Morton interleave of the low bit-planes of the codes
+    // (R9), which is where the queries of one leaf differ; the high bit-planes are mostly
+    // the offset-binary sign pattern.  hi = 0 is a constant digit the radix sort skips.
     const Key128 k = qkey[q];
-    hi[q] = k.hi;
+    hi[q] = 0ull;
     lo[q] = k.lo;
     leaf[q] = (qoor[q] & 2) ? 0xFFFFu : (uint32_t)qleaf[q];
     id[q] = (uint32_t)q;
