@@ -186,6 +186,10 @@ typedef struct {
     int64_t union_rows;               /* tiled: rows streamed from HBM (sum over tiles of the candidate union) */
     int64_t pairs_scored;             /* (row, query) distance evaluations actually performed */
     double  shortlist_flops;          /* algorithmic flops: 3*d per (query, candidate) pair */
+    float   ms_screen, ms_rescore;    /* tiled: the streaming kernel alone; TC: the exact rescoring kernel (timing = 1) */
+    double  union_bytes;              /* tiled: algorithmic bytes of the streaming kernel: union rows x (4 d_stride + 8)
+                                         + the tile queries each work item loads (4 d_stride per query)              */
+    int64_t pairs_kept;               /* TC: (row, query) pairs that passed the running screen and were buffered   */
 } blsh_stats;
 
 blsh_status blsh_last_stats(const blsh_index* idx, blsh_stats* out);

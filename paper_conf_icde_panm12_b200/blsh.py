@@ -53,7 +53,9 @@ class Stats(C.Structure):
                 ("ms_route_hash", C.c_float), ("ms_probe", C.c_float), ("ms_plan", C.c_float),
                 ("ms_shortlist", C.c_float), ("ms_merge", C.c_float), ("ms_total", C.c_float),
                 ("tiled", C.c_int32), ("pad_", C.c_int32), ("union_rows", C.c_int64),
-                ("pairs_scored", C.c_int64), ("shortlist_flops", C.c_double)]
+                ("pairs_scored", C.c_int64), ("shortlist_flops", C.c_double),
+                ("ms_screen", C.c_float), ("ms_rescore", C.c_float), ("union_bytes", C.c_double),
+                ("pairs_kept", C.c_int64)]
 
 
 class BlshError(RuntimeError):

@@ -361,7 +361,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     BLSH_CUDA(cudaStreamSynchronize(s));
     const int kind = shortlist_kind(ds, T, k);
     const bool tiled = kind > 0;
-    int64_t n_items = 0, union_rows = 0, pairs = total;
+    int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0;
+    double qload_rows = 0.0;
     const int tcpath = kind == 2 ? 1 : 0;
     int64_t ch = 0;
     if (tiled) {
@@ -370,7 +371,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         int chr = 0;
         run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
-                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[5] : nullptr, &pairs, kind);
+                            tm ? ix.ev[4] : nullptr, tm ? ix.ev[8] : nullptr, tm ? ix.ev[5] : nullptr, &pairs,
+                            &kept, &qload_rows, kind);
         ch = chr;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {
@@ -409,6 +411,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 + (double)n_items * k * 8.0;
     stt.tiled = tiled ? (tcpath ? 2 : 1) : 0;
     stt.union_rows = union_rows;
+    stt.pairs_kept = kept;
+    stt.union_bytes = tiled ? (double)union_rows * (4.0 * ds + 8.0) + qload_rows * 4.0 * ds : stt.shortlist_bytes;
     stt.pairs_scored = pairs;
     stt.shortlist_flops = 3.0 * ix.d * (double)total;
     if (p.hierarchy) {
@@ -421,6 +425,12 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         cudaEventElapsedTime(&stt.ms_probe, ix.ev[2], ix.ev[3]);
         cudaEventElapsedTime(&stt.ms_plan, ix.ev[3], ix.ev[4]);
         cudaEventElapsedTime(&stt.ms_shortlist, ix.ev[4], ix.ev[5]);
+        if (tiled) {
+            cudaEventElapsedTime(&stt.ms_screen, ix.ev[4], ix.ev[8]);
+            cudaEventElapsedTime(&stt.ms_rescore, ix.ev[8], ix.ev[5]);
+        } else {
+            stt.ms_screen = stt.ms_shortlist;
+        }
         cudaEventElapsedTime(&stt.ms_merge, ix.ev[5], ix.ev[6]);
         cudaEventElapsedTime(&stt.ms_total, ix.ev[0], ix.ev[7]);
     }

@@ -147,7 +147,7 @@ struct blsh_index {
     mutable blsh::QueryWork qw;
     mutable blsh_stats stats{};
     mutable bool has_stages = false;
-    mutable cudaEvent_t ev[8] = {};
+    mutable cudaEvent_t ev[10] = {};
 };
 
 namespace blsh {

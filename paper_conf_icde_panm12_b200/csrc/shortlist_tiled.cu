@@ -583,7 +583,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
-                         cudaEvent_t ev_sl0, cudaEvent_t ev_sl1, int64_t* pairs_out, int kind) {
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
+                         int64_t* kept_out, double* qload_rows_out, int kind) {
     const int64_t nq = a.nq;
     const int T = a.T;
     const int segcap = 2 * QT * (T + 1);
@@ -705,6 +706,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
             kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
             BLSH_LAUNCH_CHECK();
             ++*launches;
+            if (ev_mid) BLSH_CUDA(cudaEventRecord(ev_mid, s));
             const unsigned rg = (unsigned)((n_items * QT + 7) / 8);
             const int nvq = (a.ds / 4 + 31) / 32;
             if (nvq <= 1) k_tc_rescore<1><<<rg, 256, 0, s>>>(ta);
@@ -718,6 +720,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         BLSH_LAUNCH_CHECK();
         ++*launches;
     }
+    if (ev_mid && !use_tc) BLSH_CUDA(cudaEventRecord(ev_mid, s));
     if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
     k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand);
     BLSH_LAUNCH_CHECK();
@@ -729,6 +732,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     BLSH_CUDA(cudaMemcpyAsync(ev, counters, 16, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     *pairs_out = (int64_t)(use_tc ? ev[1] : ev[0]);   // TC: exact rescorings after the screen
+    *kept_out = use_tc ? (int64_t)ev[0] : 0;
+    // every work item loads its tile's queries: sum over tiles of |tile| x items(tile) ~ n_items x nq / ntiles
+    *qload_rows_out = ntiles > 0 ? (double)n_items * (double)nq / (double)ntiles : 0.0;
     if (use_tc && std::getenv("BLSH_TC_MODE"))
         std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld\n", (long long)n_items, ev[0], ev[1],
                      (long long)total_rows);
