@@ -72,12 +72,16 @@ def lib():
         L.orc_diameter_estimate.restype = f32
         L.orc_diameter_estimate.argtypes = [P, i32, P, i64, i32, P, P]
         L.orc_build.restype = P
-        L.orc_build.argtypes = [P, i64, i32, i32, i32, i32, f32, P, i32, f64, f64, i32, u64,
+        L.orc_build.argtypes = [P, i64, i32, i32, i32, i32, f32, P, i32, f64, f64, i32, u64, i32,
                                 C.POINTER(C.c_int)]
         L.orc_free.restype = None
         L.orc_free.argtypes = [P]
         L.orc_query.restype = i32
         L.orc_query.argtypes = [P, P, i64, i32, i32, i32, i32, i32, i64, P, P, P]
+        L.orc_query_union.restype = i32
+        L.orc_query_union.argtypes = [P, i32, P, i64, i32, i32, i32, P, P, P]
+        L.orc_gen_table_params.restype = None
+        L.orc_gen_table_params.argtypes = [u64, i32, i32, i32, i32, P, P, P]
         L.orc_bruteforce.restype = None
         L.orc_bruteforce.argtypes = [P, i64, i32, P, i64, i32, P, P]
         L.orc_info.restype = None
@@ -125,6 +129,15 @@ def gen_params(seed: int, G: int, M: int, d: int, W):
     jit = np.zeros(max(G - 1, 1), np.float64)
     lib().orc_gen_params(seed, G, M, d, _p(Wl), _p(A), _p(b), _p(dirs), _p(jit))
     return A, b, dirs[:G - 1], jit[:G - 1]
+
+
+def gen_table_params(seed: int, table: int, G: int, M: int, d: int, W):
+    """(A [G,M,d], b [G,M]) of hash table ``table`` (P:43 L tables, R2/R24)."""
+    Wl = _f32(np.broadcast_to(np.asarray(W, dtype=np.float32), (G,)))
+    A = np.empty((G, M, d), np.float32)
+    b = np.empty((G, M), np.float32)
+    lib().orc_gen_table_params(seed, table, G, M, d, _p(Wl), _p(A), _p(b))
+    return A, b
 
 
 def dot_canonical(a, x) -> np.float32:
@@ -271,39 +284,49 @@ class OracleIndex:
 
     def __init__(self, X, G: int, M: int = 8, W: float = 4.0, seed: int = 42, quantizer: int = 0,
                  W_leaf=None, rp_rule: int = 0, rp_mean_c: float = 10.0,
-                 rp_max_jitter: float = 0.0, ek_iters: int = 40):
+                 rp_max_jitter: float = 0.0, ek_iters: int = 40, L: int = 1):
+        """L > 1: L independent hash tables over the same RP-tree; table l
+        is the single-table index built with table = l (its own (a, b))."""
         self.X = _f32(X)
         n, d = self.X.shape
         Wl = None if W_leaf is None else _f32(W_leaf)
-        err = C.c_int(0)
-        h = lib().orc_build(_p(self.X), n, d, G, M, quantizer, float(W),
-                            _p(Wl) if Wl is not None else None, rp_rule, float(rp_mean_c),
-                            float(rp_max_jitter), ek_iters, seed, C.byref(err))
-        if not h:
-            raise OracleError(f"orc_build failed (code {err.value})", err.value)
-        self._h = h
+        self._tabs = []
+        for l in range(L):
+            err = C.c_int(0)
+            h = lib().orc_build(_p(self.X), n, d, G, M, quantizer, float(W),
+                                _p(Wl) if Wl is not None else None, rp_rule, float(rp_mean_c),
+                                float(rp_max_jitter), ek_iters, seed, l, C.byref(err))
+            if not h:
+                self.close()
+                raise OracleError(f"orc_build failed (code {err.value})", err.value)
+            self._tabs.append(h)
+        self._h = self._tabs[0]
         self._Wl = Wl
+        self.L = L
         self.n, self.d, self.G, self.M = n, d, G, M
         self.quantizer = quantizer
-        self._refresh()
         self.lq_T = 1
+        self._refresh()
 
-    def _refresh(self):
+    def _refresh(self, table: int = 0):
         info = np.zeros(8, np.int64)
-        lib().orc_info(self._h, _p(info))
+        h = self._tabs[table]
+        lib().orc_info(h, _p(info))
         self.B = int(info[4])
         self.nu = int(info[5])
         self.lq_n = int(info[6])
         self.tau = int(info[7])
-        self.ncand_total = int(lib().orc_last_ncand_total(self._h))
+        self.ncand_total = int(lib().orc_last_ncand_total(h))
 
-    def get(self, what: str) -> np.ndarray:
+    def get(self, what: str, table: int = 0) -> np.ndarray:
         code, dt, shape = self._GET[what]
+        self._refresh(table)
         out = np.zeros(shape(self), dt)
         if out.size:
-            rc = lib().orc_get(self._h, code, _p(out))
+            rc = lib().orc_get(self._tabs[table], code, _p(out))
             if rc:
                 raise OracleError(f"orc_get({what}) failed")
+        self._refresh(0)
         return out
 
     def query(self, Q, k: int, probe: int = 0, T: int = 1, hierarchy: int = 0,
@@ -313,24 +336,39 @@ class OracleIndex:
         ids = np.empty((nq, k), np.int64)
         d2 = np.empty((nq, k), np.float32)
         nc = np.empty(nq, np.int64)
-        rc = lib().orc_query(self._h, _p(Q), nq, k, probe, T, hierarchy, hier_step_bits,
-                             min_cand, _p(ids), _p(d2), _p(nc))
+        if self.L == 1:
+            rc = lib().orc_query(self._h, _p(Q), nq, k, probe, T, hierarchy, hier_step_bits,
+                                 min_cand, _p(ids), _p(d2), _p(nc))
+        elif hierarchy:
+            raise OracleError("the Morton hierarchy is defined for L = 1 only (R24)")
+        else:
+            arr = (C.c_void_p * self.L)(*self._tabs)
+            rc = lib().orc_query_union(arr, self.L, _p(Q), nq, k, probe, T, _p(ids), _p(d2), _p(nc))
         if rc:
             raise OracleError("orc_query: invalid arguments")
         self.lq_T = T
         self._refresh()
         return ids, d2, nc
 
-    def candidates(self):
-        """Candidate id sets A(q) of the last query, as a list of sorted arrays."""
-        off = self.get("q_coff")
-        ids = self.get("q_cand")
-        return [ids[off[i]:off[i + 1]] for i in range(len(off) - 1)]
+    def candidates(self, table=None):
+        """Candidate id sets A(q) of the last query (sorted arrays): the union
+        over the L tables, or one table's set when ``table`` is given."""
+        tabs = range(self.L) if table is None else [table]
+        per = []
+        for l in tabs:
+            off = self.get("q_coff", l)
+            ids = self.get("q_cand", l)
+            per.append([ids[off[i]:off[i + 1]] for i in range(len(off) - 1)])
+        if len(per) == 1:
+            return per[0]
+        return [np.unique(np.concatenate([p[q] for p in per])) for q in range(len(per[0]))]
 
     def close(self):
-        if getattr(self, "_h", None):
-            lib().orc_free(self._h)
-            self._h = None
+        for h in getattr(self, "_tabs", []):
+            if h:
+                lib().orc_free(h)
+        self._tabs = []
+        self._h = None
 
     def __del__(self):
         try:

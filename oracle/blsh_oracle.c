@@ -78,22 +78,32 @@ static uint64_t orc_stream(uint64_t kind, uint64_t table, uint64_t idx)
  *   b[g][i]    = fp32(W_g * U[0,1))  stream (2, 0, g), element i; clamped < W_g
  *   dir[v][j]  = fp32(g_j / |g|)     stream (3, 0, v), fp64 normalisation
  *   jit[v]     = U[0,1)              stream (4, 0, v), element 0 (max rule)  */
-void orc_gen_params(uint64_t seed, int G, int M, int d, const float *Wleaf,
-                    float *A, float *b, float *dirs, double *jit)
+/* The L hash tables of P:43 ("L hash tables are used and each of them is
+ * constructed independently with different dim-M hash functions") get their
+ * own (a, b) per leaf: table l draws from streams (1, l, g) and (2, l, g)
+ * (R2, R24).  Table 0 is the single table of the L = 1 index. */
+void orc_gen_table_params(uint64_t seed, int table, int G, int M, int d, const float *Wleaf,
+                          float *A, float *b)
 {
     for (int g = 0; g < G; g++) {
         for (int i = 0; i < M; i++)
             for (int j = 0; j < d; j++)
                 A[((size_t)g * M + i) * d + j] =
-                    (float)orc_rng_gauss(seed, orc_stream(1, 0, g), (uint64_t)i * d + j);
+                    (float)orc_rng_gauss(seed, orc_stream(1, (uint64_t)table, g), (uint64_t)i * d + j);
         for (int i = 0; i < M; i++) {
             float W = Wleaf[g];
-            double u = orc_rng_uniform(seed, orc_stream(2, 0, g), i);
+            double u = orc_rng_uniform(seed, orc_stream(2, (uint64_t)table, g), i);
             float bf = (float)((double)W * u);
             if (bf >= W) bf = nextafterf(W, 0.0f);      /* R2: keep b in [0, W) */
             b[(size_t)g * M + i] = bf;
         }
     }
+}
+
+void orc_gen_params(uint64_t seed, int G, int M, int d, const float *Wleaf,
+                    float *A, float *b, float *dirs, double *jit)
+{
+    orc_gen_table_params(seed, 0, G, M, d, Wleaf, A, b);
     double *gv = (double *)malloc(sizeof(double) * (size_t)d);
     for (int v = 0; v < G - 1; v++) {
         double s = 0.0;
@@ -619,10 +629,11 @@ static int orc_entry_cmp(const void *pa, const void *pb)
  * *err: 1 invalid argument, 4 code outside the Morton range (R9). */
 orc_index *orc_build(const float *X, int64_t n, int d, int G, int M, int quantizer, float W,
                      const float *Wleaf, int rp_rule, double rp_mean_c, double rp_max_jitter,
-                     int ek_iters, uint64_t seed, int *err)
+                     int ek_iters, uint64_t seed, int table, int *err)
 {
     *err = 1;
     if (n < 0 || d < 1 || G < 1 || G > 4096 || (G & (G - 1)) || M < 1 || M > 16) return NULL;
+    if (table < 0 || table > 255) return NULL;
     if (quantizer == 1 && M != 8) return NULL;
     if (!(W > 0.0f)) return NULL;
     orc_index *ix = (orc_index *)calloc(1, sizeof(orc_index));
@@ -648,6 +659,8 @@ orc_index *orc_build(const float *X, int64_t n, int d, int G, int M, int quantiz
     ix->diam2 = (double *)calloc((size_t)nn, sizeof(double));
     ix->da2 = (double *)calloc((size_t)nn, sizeof(double));
     orc_gen_params(seed, G, M, d, ix->Wl, ix->A, ix->b, ix->dirs, ix->jit);
+    /* table l of an L-table index: same RP-tree (dirs, jit), its own (a, b) */
+    if (table > 0) orc_gen_table_params(seed, table, G, M, d, ix->Wl, ix->A, ix->b);
 
     /* b2: level-by-level RP-tree; members of each node kept in ascending id. */
     int64_t *order = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
@@ -781,8 +794,9 @@ static void orc_shortlist(const float *X, int d, const float *q, const int64_t *
  * hierarchy (Z^M only): Morton-prefix widening (Eq. 7-8)
  * with threshold tau = min_cand, or the lower median of the base counts of
  * this batch when min_cand == 0 (R18).  Returns 0, or 1 on invalid args. */
-int orc_query(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
-              int hier_step, int64_t min_cand, int64_t *out_ids, float *out_d2, int64_t *out_ncand)
+static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
+                          int hier_step, int64_t min_cand, int64_t *out_ids, float *out_d2, int64_t *out_ncand,
+                          int do_shortlist)
 {
     const int M = ix->M, d = ix->d, B = ix->B;
     if (k < 1 || T < 1) return 1;
@@ -924,8 +938,9 @@ int orc_query(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T
         ncand[q] = m;
         if (out_ncand) out_ncand[q] = m;
         /* a5: short-list search */
-        orc_shortlist(ix->X, d, Q + q * (int64_t)d, pos, m, k, out_ids + q * (int64_t)k,
-                      out_d2 + q * (int64_t)k);
+        if (do_shortlist)
+            orc_shortlist(ix->X, d, Q + q * (int64_t)d, pos, m, k, out_ids + q * (int64_t)k,
+                          out_d2 + q * (int64_t)k);
     }
     ix->lq_coff[0] = 0;
     for (int64_t q = 0; q < nq; q++) ix->lq_coff[q + 1] = ix->lq_coff[q] + ncand[q];
@@ -935,6 +950,46 @@ int orc_query(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T
         free(cand[q]);
     }
     free(cand); free(ncand); free(bs); free(be); free(hs); free(he); free(hkey);
+    return 0;
+}
+
+int orc_query(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
+              int hier_step, int64_t min_cand, int64_t *out_ids, float *out_d2, int64_t *out_ncand)
+{
+    return orc_query_impl(ix, Q, nq, k, probe, T, hierarchy, hier_step, min_cand, out_ids, out_d2,
+                          out_ncand, 1);
+}
+
+/* L > 1 tables: "each of them is constructed independently with
+ * different dim-M hash functions"; the candidate set of a query is the union
+ * of the points of its probed buckets over the L tables, deduplicated (R24:
+ * every table probes T buckets the same way; the Morton hierarchy is not
+ * combined with L > 1).  tabs[l] is the index built with table = l (same
+ * data, tree and seed).  Short-list as for one table.  Returns 0, or 1 on
+ * invalid arguments. */
+int orc_query_union(orc_index **tabs, int L, const float *Q, int64_t nq, int k, int probe, int T,
+                    int64_t *out_ids, float *out_d2, int64_t *out_ncand)
+{
+    if (L < 1) return 1;
+    for (int l = 0; l < L; l++)
+        if (orc_query_impl(tabs[l], Q, nq, k, probe, T, 0, 0, 0, out_ids, out_d2, NULL, 0)) return 1;
+    const int d = tabs[0]->d;
+    #pragma omp parallel for schedule(dynamic, 16)
+    for (int64_t q = 0; q < nq; q++) {
+        int64_t cap = 0;
+        for (int l = 0; l < L; l++) cap += tabs[l]->lq_coff[q + 1] - tabs[l]->lq_coff[q];
+        int64_t *ids = (int64_t *)malloc(sizeof(int64_t) * (size_t)(cap > 0 ? cap : 1));
+        int64_t m = 0;
+        for (int l = 0; l < L; l++)
+            for (int64_t i = tabs[l]->lq_coff[q]; i < tabs[l]->lq_coff[q + 1]; i++) ids[m++] = tabs[l]->lq_cand[i];
+        qsort(ids, (size_t)m, sizeof(int64_t), orc_cmp_i64);
+        int64_t u = 0;
+        for (int64_t i = 0; i < m; i++) if (u == 0 || ids[i] != ids[u - 1]) ids[u++] = ids[i];
+        if (out_ncand) out_ncand[q] = u;
+        orc_shortlist(tabs[0]->X, d, Q + q * (int64_t)d, ids, u, k, out_ids + q * (int64_t)k,
+                      out_d2 + q * (int64_t)k);
+        free(ids);
+    }
     return 0;
 }
 
