@@ -96,7 +96,11 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
 
 /* a1-a5: route, hash, probe, look up, (widen), short-list.
  *   Q         [nq x d] fp32 queries (device or host)
- *   k         neighbours, 1..64 (k > 64 -> BLSH_ERR_UNSUPPORTED)
+ *   k         neighbours, 1..1024 (k > 1024 -> BLSH_ERR_UNSUPPORTED).  k <= 64 keeps
+ *             per-warp register top-k lists; 64 < k <= 1024 (the paper evaluates
+ *             k = 500) emits every candidate's packed (d^2, id) key to a
+ *             workspace of 8 B per candidate and selects per query (radix select);
+ *             both give the k smallest by (d^2, id).
  *   out_ids   [nq x k] int64 original row ids of X, ascending (d^2, id); -1 = padding
  *   out_dist2 [nq x k] fp32 squared L2 distances (fp32, direct form, R22); +inf = padding
  *   out_ncand [nq] int64 |A(q)| (may be NULL)
@@ -124,7 +128,7 @@ blsh_status blsh_query_base_counts(const blsh_index* idx, const float* Q, int64_
 
 /* a6: merge n_lists per-rank packed lists (e.g. the output of an NCCL
  * all-gather, layout [n_lists][nq][k]) into the k smallest per query.
- * packed is a device pointer; outputs device or host. */
+ * packed is a device pointer; outputs device or host.  k in 1..1024. */
 blsh_status blsh_merge_topk(const uint64_t* packed, int32_t n_lists, int64_t nq, int32_t k,
                             int64_t* out_ids, float* out_dist2, void* stream);
 

@@ -383,16 +383,22 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         scan_exclusive_i64(items, w.item_off, nq, w.scan, s); launches += 3;
         BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         BLSH_CUDA(cudaStreamSynchronize(s));
-        w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
+        const bool large_k = k > 64;
+        if (large_k) w.partials.ensure((size_t)std::max<int64_t>(total, 1) * sizeof(unsigned long long));
+        else w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[4], s));
         // a5, one warp per (query, chunk)
         ShortlistArgs sa{};
         sa.nq = nq; sa.n_items = n_items; sa.d = ix.d; sa.ds = ds; sa.T = T; sa.k = k; sa.chunk = (int)ch;
         sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
         sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
+        sa.cand_off = cand_off;
+        sa.cand_keys = large_k ? w.partials.as<unsigned long long>() : nullptr;
         launch_shortlist(sa, s); if (n_items) ++launches;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
-        launch_merge(sa, w.qoor, d_ids, d_d2, d_pk, d_nc, s); ++launches;
+        if (large_k) launch_select(sa.cand_keys, cand_off, nq, k, w.qoor, w.cnt, d_ids, d_d2, d_pk, d_nc, s);
+        else launch_merge(sa, w.qoor, d_ids, d_d2, d_pk, d_nc, s);
+        ++launches;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
         union_rows = total;
     }
@@ -408,7 +414,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     stt.n_items = n_items;
     stt.chunk = (int32_t)ch;
     stt.launches = launches;
-    stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 + (double)n_items * k * 8.0;
+    stt.shortlist_bytes = (double)total * ix.d * 4.0 + (double)total * 4.0 +
+                          (k > 64 && !tiled ? (double)total * 8.0 : (double)n_items * k * 8.0);
     stt.tiled = tiled ? (tcpath ? 2 : 1) : 0;
     stt.union_rows = union_rows;
     stt.pairs_kept = kept;
@@ -447,7 +454,7 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
     if (nq < 0 || nq >= (int64_t(1) << 31)) return fail(BLSH_ERR_INVALID, "nq must be in [0, 2^31)");
     if (nq > 0 && !Q) return fail(BLSH_ERR_INVALID, "Q is NULL");
     if (k < 1) return fail(BLSH_ERR_INVALID, "k must be >= 1");
-    if (k > 64) return fail(BLSH_ERR_UNSUPPORTED, "k > 64 is not implemented in this build (NEXT: large-k short-list)");
+    if (k > 1024) return fail(BLSH_ERR_UNSUPPORTED, "k > 1024");
     if (p->n_probes < 1) return fail(BLSH_ERR_INVALID, "n_probes must be >= 1");
     if (p->probe == 0 && p->n_probes != 1) return fail(BLSH_ERR_INVALID, "standard probing uses n_probes = 1");
     if (p->probe == 1) {
@@ -527,7 +534,7 @@ blsh_status blsh_query_base_counts(const blsh_index* idx, const float* Q, int64_
 blsh_status blsh_merge_topk(const uint64_t* packed, int32_t n_lists, int64_t nq, int32_t k, int64_t* out_ids,
                             float* out_dist2, void* stream) {
     if (n_lists < 1 || nq < 0 || k < 1) return fail(BLSH_ERR_INVALID, "bad sizes");
-    if (k > 64) return fail(BLSH_ERR_UNSUPPORTED, "k > 64");
+    if (k > 1024) return fail(BLSH_ERR_UNSUPPORTED, "k > 1024");
     if (nq == 0) return BLSH_OK;
     if (!packed || !out_ids || !out_dist2) return fail(BLSH_ERR_INVALID, "NULL pointer");
     if (!is_device_ptr(packed)) return fail(BLSH_ERR_INVALID, "packed must be device memory");

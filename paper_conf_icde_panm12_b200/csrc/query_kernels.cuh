@@ -57,6 +57,8 @@ struct ShortlistArgs {
     const int64_t* cnt;
     const int64_t* item_off; // [nq+1]
     unsigned long long* partials;   // [n_items][k]
+    const int64_t* cand_off;        // [nq+1] (large k)
+    unsigned long long* cand_keys;  // [total] non-NULL: emit every candidate key (large k)
 };
 
 // query-tiled short-list (shortlist_tiled.cu)
@@ -74,6 +76,9 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s);
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s);
+void launch_select(const unsigned long long* cand_keys, const int64_t* cand_off, int64_t nq, int k,
+                   const int32_t* qoor, const int64_t* cnt, int64_t* out_ids, float* out_d2,
+                   unsigned long long* out_packed, int64_t* out_ncand, cudaStream_t s);
 void launch_merge(const ShortlistArgs& a, const int32_t* qoor, int64_t* out_ids, float* out_d2,
                   unsigned long long* out_packed, int64_t* out_ncand, cudaStream_t s);
 

@@ -40,7 +40,12 @@ __device__ __forceinline__ void topk_insert(TopK& t, unsigned long long v, int l
     t.e0 = lane > pos ? up0 : (lane == pos ? v : t.e0);
 }
 
-template <int NV>
+// EMIT = false: register top-k per item (k <= 64) into a.partials.
+// EMIT = true (large k, k > 64): the packed key of every candidate goes to
+// a.cand_keys[a.cand_off[q] + c] (c = rank of the candidate in the query's
+// interval order); k_select then takes the k smallest per query.  The distance
+// arithmetic is the same in both modes (R22), so results agree bit for bit.
+template <int NV, bool EMIT>
 __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5);
@@ -102,6 +107,15 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
                     for (int j = 0; j < 4; ++j) part[j] += __shfl_xor_sync(BLSH_FULL, part[j], o);
                 }
                 const uint32_t idl = (lane < 4 && r0 + lane < pb) ? __ldg(a.perm + r0 + lane) : 0u;
+                if (EMIT) {
+                    if (lane < 4 && r0 + lane < pb) {
+                        float pj = part[0];
+#pragma unroll
+                        for (int j = 1; j < 4; ++j) pj = lane == j ? part[j] : pj;
+                        a.cand_keys[a.cand_off[q] + acc + (r0 - (int64_t)iv.x) + lane] = pack_entry(pj, idl);
+                    }
+                    continue;
+                }
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     const uint32_t id = __shfl_sync(BLSH_FULL, idl, j);
@@ -117,6 +131,7 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
         }
         acc += len;
     }
+    if (EMIT) return;
     unsigned long long* out = a.partials + (size_t)item * k;
     if (lane < k) out[lane] = tk.e0;
     if (lane + 32 < k) out[lane + 32] = tk.e1;
@@ -187,6 +202,160 @@ __global__ void __launch_bounds__(256) k_merge_lists(const unsigned long long* _
     write_out(tk, q, k, lane, out_ids, out_d2, nullptr);
 }
 
+// ---- large k (64 < k <= 1024): block radix select -------------------------------
+// One CTA per query selects the k smallest packed keys of the query's segment
+// (the candidate keys k_shortlist<.., true> emitted, or for the a6 merge the
+// n_lists sorted lists of k entries) and writes them in ascending order.  Keys
+// of distinct candidates are distinct (ids are); only padding repeats, and
+// padding is larger than every real key.
+//   MSB-first radix select, 8 bits per pass: histogram of the current byte over
+//   the keys that match the prefix so far, pick the bin holding the need-th
+//   key; stop early when that bin is taken whole.  Then the selected keys
+//   (<= k) are collected into shared memory and bitonic-sorted.
+constexpr int kSelThreads = 512;
+constexpr int kSelCap = 1024;   // max k
+
+struct SelSrc {
+    const unsigned long long* base;
+    int64_t off, len;      // segment mode: keys base[off .. off+len)
+    int n_lists;           // list mode (n_lists > 0): list l entries at base[(l*nq + q)*k + j]
+    int64_t nq, q;
+    int k;
+    __device__ __forceinline__ unsigned long long get(int64_t i) const {
+        if (n_lists == 0) return base[off + i];
+        const int64_t l = i / k, j = i - l * k;
+        const unsigned long long v = base[((size_t)l * nq + q) * k + j];
+        return v == kPadPacked ? kEmpty : v;
+    }
+};
+
+__device__ void block_select_write(const SelSrc& src, int k, int64_t q, int64_t* out_ids, float* out_d2,
+                                   unsigned long long* out_packed) {
+    __shared__ unsigned int hist[256];
+    __shared__ unsigned long long buf[kSelCap];
+    __shared__ unsigned long long s_prefix, s_mask;
+    __shared__ int s_need, s_whole, s_cnt;
+    const int tid = threadIdx.x;
+    const int64_t len = src.len;
+    unsigned long long thr_le;   // keys <= thr_le are all taken
+    int fill_eq = 0;             // ... plus fill_eq copies of thr_eq
+    unsigned long long thr_eq = kEmpty;
+    if (len <= k) {
+        thr_le = kEmpty;
+    } else {
+        if (tid == 0) { s_prefix = 0; s_mask = 0; s_need = k; s_whole = 0; }
+        __syncthreads();
+        for (int byte = 7; byte >= 0; --byte) {
+            for (int i = tid; i < 256; i += kSelThreads) hist[i] = 0;
+            __syncthreads();
+            const unsigned long long pre = s_prefix, msk = s_mask;
+            const int sh = byte * 8;
+            for (int64_t i = tid; i < len; i += kSelThreads) {
+                const unsigned long long v = src.get(i);
+                if ((v & msk) == pre) atomicAdd(&hist[(v >> sh) & 255], 1u);
+            }
+            __syncthreads();
+            if (tid < 32) {   // warp 0: find the bin of the need-th key
+                const int need = s_need;
+                unsigned int c[8], tot = 0;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) { c[j] = hist[tid * 8 + j]; tot += c[j]; }
+                unsigned int incl = tot;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned int t = __shfl_up_sync(BLSH_FULL, incl, o);
+                    if (tid >= o) incl += t;
+                }
+                const unsigned int excl = incl - tot;
+                const bool mine = excl < (unsigned)need && (unsigned)need <= incl;
+                if (mine) {
+                    unsigned int run = excl;
+                    int bin = tid * 8;
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        if (run + c[j] >= (unsigned)need) { bin = tid * 8 + j; break; }
+                        run += c[j];
+                    }
+                    const unsigned int inbin = hist[bin];
+                    s_need = need - (int)run;
+                    s_prefix = pre | ((unsigned long long)bin << sh);
+                    s_mask = msk | (255ull << sh);
+                    s_whole = (run + inbin == (unsigned)need) ? 1 : 0;
+                }
+            }
+            __syncthreads();
+            if (s_whole) break;
+        }
+        if (s_whole) {
+            thr_le = s_prefix | ~s_mask;          // exactly k keys are <= this
+        } else {
+            thr_eq = s_prefix;                    // the k-th key, repeated s_need times at the cut
+            fill_eq = s_need;
+            thr_le = thr_eq - 1;                  // keys strictly below it
+            if (thr_eq == 0) { thr_le = 0; fill_eq = 0; }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) s_cnt = 0;
+    for (int i = tid; i < kSelCap; i += kSelThreads) buf[i] = kEmpty;
+    __syncthreads();
+    const bool take_all = len <= k;
+    for (int64_t i = tid; i < len; i += kSelThreads) {
+        const unsigned long long v = src.get(i);
+        if (take_all || v <= thr_le) {
+            const int slot = atomicAdd(&s_cnt, 1);
+            if (slot < kSelCap) buf[slot] = v;
+        }
+    }
+    __syncthreads();
+    if (fill_eq > 0) {
+        const int base = s_cnt;
+        for (int i = tid; i < fill_eq; i += kSelThreads)
+            if (base + i < kSelCap) buf[base + i] = thr_eq;
+        __syncthreads();
+    }
+    // bitonic sort of kSelCap keys (padding kEmpty sorts last)
+    for (int size = 2; size <= kSelCap; size <<= 1) {
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            for (int i = tid; i < kSelCap / 2; i += kSelThreads) {
+                const int lo = 2 * i - (i & (stride - 1));
+                const int hi = lo + stride;
+                const bool up = (lo & size) == 0;
+                const unsigned long long x = buf[lo], y = buf[hi];
+                if ((x > y) == up) { buf[lo] = y; buf[hi] = x; }
+            }
+            __syncthreads();
+        }
+    }
+    for (int i = tid; i < k; i += kSelThreads) {
+        const unsigned long long e = buf[i];
+        if (out_packed) out_packed[(size_t)q * k + i] = e == kEmpty ? kPadPacked : e;
+        if (out_ids) out_ids[(size_t)q * k + i] = e == kEmpty ? -1 : (int64_t)(uint32_t)(e & 0xFFFFFFFFull);
+        if (out_d2) out_d2[(size_t)q * k + i] = e == kEmpty ? __int_as_float(0x7F800000) : __uint_as_float((uint32_t)(e >> 32));
+    }
+}
+
+// a5, large k: per query, the k smallest of its emitted candidate keys.
+__global__ void __launch_bounds__(kSelThreads) k_select(const unsigned long long* __restrict__ cand_keys,
+                                                        const int64_t* __restrict__ cand_off, int64_t nq, int k,
+                                                        const int32_t* __restrict__ qoor, const int64_t* __restrict__ cnt,
+                                                        int64_t* out_ids, float* out_d2, unsigned long long* out_packed,
+                                                        int64_t* out_ncand) {
+    const int64_t q = blockIdx.x;
+    SelSrc src{cand_keys, cand_off[q], cand_off[q + 1] - cand_off[q], 0, nq, q, k};
+    block_select_write(src, k, q, out_ids, out_d2, out_packed);
+    if (threadIdx.x == 0 && out_ncand) out_ncand[q] = (qoor[q] & 2) ? 0 : cnt[q];
+}
+
+// a6, large k: per query, the k smallest over n_lists packed lists.
+__global__ void __launch_bounds__(kSelThreads) k_select_lists(const unsigned long long* __restrict__ packed,
+                                                              int n_lists, int64_t nq, int k, int64_t* out_ids,
+                                                              float* out_d2) {
+    const int64_t q = blockIdx.x;
+    SelSrc src{packed, 0, (int64_t)n_lists * k, n_lists, nq, q, k};
+    block_select_write(src, k, q, out_ids, out_d2, nullptr);
+}
+
 }  // namespace
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s) {
@@ -199,17 +368,18 @@ void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     if (a.n_items == 0) return;
     const unsigned grid = (unsigned)((a.n_items + kSLWarps - 1) / kSLWarps);
     const int nvl = ((a.ds >> 2) + 31) / 32;
+
+#define BLSH_SL_CASE(V)                                                                         \
+    case V:                                                                                     \
+        if (a.cand_keys) k_shortlist<V, true><<<grid, kSLWarps * 32, 0, s>>>(a);                \
+        else k_shortlist<V, false><<<grid, kSLWarps * 32, 0, s>>>(a);                           \
+        break;
     switch (nvl) {
-        case 1: k_shortlist<1><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 2: k_shortlist<2><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 3: k_shortlist<3><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 4: k_shortlist<4><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 5: k_shortlist<5><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 6: k_shortlist<6><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 7: k_shortlist<7><<<grid, kSLWarps * 32, 0, s>>>(a); break;
-        case 8: k_shortlist<8><<<grid, kSLWarps * 32, 0, s>>>(a); break;
+        BLSH_SL_CASE(1) BLSH_SL_CASE(2) BLSH_SL_CASE(3) BLSH_SL_CASE(4)
+        BLSH_SL_CASE(5) BLSH_SL_CASE(6) BLSH_SL_CASE(7) BLSH_SL_CASE(8)
         default: throw Error(BLSH_ERR_UNSUPPORTED, "d > 1024");
     }
+#undef BLSH_SL_CASE
     BLSH_LAUNCH_CHECK();
 }
 
@@ -223,7 +393,22 @@ void launch_merge(const ShortlistArgs& a, const int32_t* qoor, int64_t* out_ids,
 void merge_lists(const unsigned long long* packed, int n_lists, int64_t nq, int k, int64_t* out_ids,
                  float* out_d2, cudaStream_t s) {
     if (nq == 0) return;
+    if (k > 64) {
+        k_select_lists<<<(unsigned)nq, kSelThreads, 0, s>>>(packed, n_lists, nq, k, out_ids, out_d2);
+        BLSH_LAUNCH_CHECK();
+        return;
+    }
     k_merge_lists<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(packed, n_lists, nq, k, out_ids, out_d2);
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_select(const unsigned long long* cand_keys, const int64_t* cand_off, int64_t nq, int k,
+                   const int32_t* qoor, const int64_t* cnt, int64_t* out_ids, float* out_d2,
+                   unsigned long long* out_packed, int64_t* out_ncand, cudaStream_t s) {
+    if (nq == 0) return;
+    if (k > kSelCap) throw Error(BLSH_ERR_UNSUPPORTED, "k > 1024");
+    k_select<<<(unsigned)nq, kSelThreads, 0, s>>>(cand_keys, cand_off, nq, k, qoor, cnt, out_ids, out_d2, out_packed,
+                                                  out_ncand);
     BLSH_LAUNCH_CHECK();
 }
 

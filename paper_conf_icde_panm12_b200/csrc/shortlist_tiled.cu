@@ -548,6 +548,7 @@ size_t tc_smem_bytes(int ds) {
 int shortlist_kind(int ds, int T, int k) {
     const char* mode = std::getenv("BLSH_SHORTLIST");
     if (mode && std::strcmp(mode, "warp") == 0) return 0;
+    if (k > 64) return 0;   // large k: warp short-list emitting every key + k_select
     int cap = 2 * QT * (T + 1), npow = 1;
     while (npow < cap) npow <<= 1;
     if ((size_t)3 * npow * 4 > 227 * 1024) return 0;   // tile prep does not fit
