@@ -64,6 +64,13 @@ typedef struct {
     int32_t rank, world;    /* shard: this index keeps leaves [rank*G/world, (rank+1)*G/world) (default 0,1)*/
     void*   stream;         /* cudaStream_t                                                                 */
     int32_t keep_stages;    /* 1 = keep per-point leaf/code/key for blsh_export (parity tests)              */
+    int32_t n_tables;       /* L hash tables per leaf, 1..64 ("L hash tables ... each constructed
+                               independently with different dim-M hash functions"; default 1).  Table l
+                               draws its own (a, b) (R2 streams (1, l, g), (2, l, g)); the RP-tree, W and
+                               the stored rows are shared.  A query's candidate set is the union of its
+                               probed buckets over the L tables, deduplicated (R24).  L > 1 needs every
+                               owned leaf to hold <= 1,600,000 points (the per-query dedup bitmap lives
+                               in shared memory) and excludes the Morton hierarchy.                      */
 } blsh_build_params;
 
 /* Query parameters.  Defaults: blsh_query_params_default(). */
@@ -165,6 +172,12 @@ typedef enum {
     BLSH_EX_Q_TAU = 39,     /* int64 [1]        threshold used                                */
     BLSH_EX_Q_INTERVALS = 40/* int64 [nq][T+1][2] candidate intervals [start, end) in table positions */
 } blsh_export_what;
+/* Table l of an L-table index (n_tables > 1): what = BLSH_EX_TABLE(l, item) for
+ * the per-table items A, B, PERM (original ids in table-l order), UKEY, ULEAF,
+ * UOFF (table-l positions), LEAF_U and the per-table query stages Q_T .. Q_BASE
+ * (Q_BASE = |A0_l(q)| of table l) and Q_INTERVALS (table-l positions).  l = 0
+ * is the primary table (plain item codes). */
+#define BLSH_EX_TABLE(l, item) ((int32_t)(((l) << 8) | (item)))
 
 blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t cap,
                         size_t* needed);
@@ -175,6 +188,8 @@ typedef struct {
     int32_t leaf_lo, leaf_hi;   /* owned leaves [leaf_lo, leaf_hi) */
     int64_t device_bytes;       /* persistent device memory held by the index */
     double  build_ms;           /* wall time of blsh_build                      */
+    int32_t n_tables;           /* L */
+    int32_t pad_;
 } blsh_info;
 
 blsh_status blsh_index_info(const blsh_index* idx, blsh_info* out);

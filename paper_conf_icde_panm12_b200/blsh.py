@@ -30,7 +30,7 @@ class BuildParams(C.Structure):
                 ("rp_max_jitter", C.c_double), ("ek_iters", C.c_int32), ("M", C.c_int32),
                 ("quantizer", C.c_int32), ("W", C.c_float), ("W_leaf", C.c_void_p), ("seed", C.c_uint64),
                 ("rank", C.c_int32), ("world", C.c_int32), ("stream", C.c_void_p),
-                ("keep_stages", C.c_int32)]
+                ("keep_stages", C.c_int32), ("n_tables", C.c_int32)]
 
 
 class QueryParams(C.Structure):
@@ -43,7 +43,8 @@ class Info(C.Structure):
     _fields_ = [("n", C.c_int64), ("n_owned", C.c_int64), ("nu", C.c_int64), ("d", C.c_int32),
                 ("d_stride", C.c_int32), ("G", C.c_int32), ("M", C.c_int32), ("B", C.c_int32),
                 ("quantizer", C.c_int32), ("leaf_lo", C.c_int32), ("leaf_hi", C.c_int32),
-                ("device_bytes", C.c_int64), ("build_ms", C.c_double)]
+                ("device_bytes", C.c_int64), ("build_ms", C.c_double), ("n_tables", C.c_int32),
+                ("pad_", C.c_int32)]
 
 
 class Stats(C.Structure):
@@ -155,7 +156,8 @@ def _f32(a):
 
 def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42, quantizer: int = 0,
                rp_rule: int = 0, rp_mean_c: float = 10.0, rp_max_jitter: float = 0.0, ek_iters: int = 40,
-               W_leaf=None, rank: int = 0, world: int = 1, keep_stages: bool = False) -> "Index":
+               W_leaf=None, rank: int = 0, world: int = 1, keep_stages: bool = False,
+               n_tables: int = 1) -> "Index":
     X = _f32(X)
     n, d = int(X.shape[0]), int(X.shape[1])
     p = BuildParams()
@@ -163,6 +165,7 @@ def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42,
     p.n_leaves, p.M, p.W, p.seed, p.quantizer = n_leaves, M, W, seed, quantizer
     p.rp_rule, p.rp_mean_c, p.rp_max_jitter, p.ek_iters = rp_rule, rp_mean_c, rp_max_jitter, ek_iters
     p.rank, p.world, p.keep_stages = rank, world, int(bool(keep_stages))
+    p.n_tables = n_tables
     wl = None
     if W_leaf is not None:
         wl = np.ascontiguousarray(np.asarray(W_leaf, dtype=np.float32))
@@ -265,8 +268,10 @@ _EX_DT = {"A": np.float32, "B": np.float32, "W": np.float32, "DIRS": np.float32,
           "Q_INTERVALS": np.int64}
 
 
-def blsh_export(index: "Index", what: str) -> np.ndarray:
-    code = EX[what]
+def blsh_export(index: "Index", what: str, table: int = 0) -> np.ndarray:
+    """Host copy of a build artefact / last-query stage; ``table`` selects hash
+    table l of an L-table index for the per-table items (BLSH_EX_TABLE)."""
+    code = EX[what] | (int(table) << 8)
     need = C.c_size_t(0)
     lib().blsh_export(index.handle, code, None, 0, C.byref(need))
     dt = _EX_DT[what]
@@ -310,8 +315,8 @@ class Index:
     def base_counts(self, Q, **kw):
         return blsh_query_base_counts(self, Q, **kw)
 
-    def export(self, what: str) -> np.ndarray:
-        return blsh_export(self, what)
+    def export(self, what: str, table: int = 0) -> np.ndarray:
+        return blsh_export(self, what, table)
 
     def info(self) -> Info:
         return blsh_index_info(self)

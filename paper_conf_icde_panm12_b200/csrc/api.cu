@@ -84,6 +84,7 @@ void blsh_build_params_default(blsh_build_params* p) {
     p->world = 1;
     p->stream = nullptr;
     p->keep_stages = 0;
+    p->n_tables = 1;
 }
 
 void blsh_query_params_default(blsh_query_params* p) {
@@ -126,6 +127,7 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
     if (p->ek_iters < 1) return fail(BLSH_ERR_INVALID, "ek_iters must be >= 1");
     if (p->world < 1 || p->rank < 0 || p->rank >= p->world || G % p->world != 0)
         return fail(BLSH_ERR_INVALID, "rank/world must satisfy 0 <= rank < world and world | n_leaves");
+    if (p->n_tables < 1 || p->n_tables > 64) return fail(BLSH_ERR_INVALID, "n_tables must be in [1, 64]");
     if (p->W_leaf)
         for (int g = 0; g < G; ++g)
             if (!(p->W_leaf[g] > 0.0f) || !std::isfinite(p->W_leaf[g])) return fail(BLSH_ERR_INVALID, "W_leaf must be > 0");
@@ -232,6 +234,48 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         blsh::build_table(*ix, Xs.as<float>(), sb.hi[cur].as<unsigned long long>(), sb.lo[cur].as<unsigned long long>(),
                           sb.leaf[cur].as<uint32_t>(), sb.id[cur].as<uint32_t>(), no, sb.scan, s);
         BLSH_CUDA(cudaStreamSynchronize(s));
+        // leaves as table position ranges (the same in every table: entries sort by leaf first)
+        ix->leaf_pos_h.assign(G + 1, 0);
+        ix->max_leaf_rows = 0;
+        for (int g = 0; g <= G; ++g)
+            ix->leaf_pos_h[g] = std::min<int64_t>(no, std::max<int64_t>(0, seg[g] - pos_lo));
+        for (int g = ix->leaf_lo; g < ix->leaf_hi; ++g)
+            ix->max_leaf_rows = std::max<int64_t>(ix->max_leaf_rows, ix->leaf_pos_h[g + 1] - ix->leaf_pos_h[g]);
+        ix->leaf_pos.alloc((G + 1) * sizeof(int64_t));
+        BLSH_CUDA(cudaMemcpyAsync(ix->leaf_pos.p, ix->leaf_pos_h.data(), (G + 1) * sizeof(int64_t),
+                                  cudaMemcpyHostToDevice, s));
+        // tables 1..L-1: own (a, b), same tree and rows
+        ix->L = p->n_tables;
+        std::vector<const uint32_t*> tab_pos(ix->L, nullptr);
+        if (ix->L > 1) {
+            blsh::DevBuf inv0;
+            inv0.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(uint32_t));
+            blsh::invert_perm(ix->perm.as<uint32_t>(), no, inv0.as<uint32_t>(), s);
+            for (int l = 1; l < ix->L; ++l) {
+                auto t = std::make_unique<blsh::ExtraTable>();
+                t->A_h.assign((size_t)G * M * d, 0.0f);
+                t->b_h.assign((size_t)G * M, 0.0f);
+                blsh::gen_table_params(p->seed, l, G, M, d, ix->W_h.data(), t->A_h.data(), t->b_h.data());
+                t->A.alloc(t->A_h.size() * sizeof(float));
+                t->b.alloc(t->b_h.size() * sizeof(float));
+                BLSH_CUDA(cudaMemcpyAsync(t->A.p, t->A_h.data(), t->A_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+                BLSH_CUDA(cudaMemcpyAsync(t->b.p, t->b_h.data(), t->b_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+                const bool okl = blsh::hash_points(*ix, Xs.as<float>(), order.as<uint32_t>(), seg, pos_lo, pos_hi,
+                                                   sb.hi[0].as<unsigned long long>(), sb.lo[0].as<unsigned long long>(),
+                                                   sb.leaf[0].as<uint32_t>(), sb.id[0].as<uint32_t>(), nullptr, s,
+                                                   t->A.as<float>(), t->b.as<float>());
+                if (!okl) throw blsh::Error(BLSH_ERR_RANGE, "a data point's code leaves the Morton range (decrease M or increase W)");
+                const int cl = blsh::radix_sort_entries(sb, no, s, &passes);
+                blsh::build_extra_table(*ix, *t, sb.hi[cl].as<unsigned long long>(), sb.lo[cl].as<unsigned long long>(),
+                                        sb.leaf[cl].as<uint32_t>(), sb.id[cl].as<uint32_t>(), inv0.as<uint32_t>(), no,
+                                        sb.scan, s);
+                tab_pos[l] = t->pos.as<uint32_t>();
+                ix->xt.push_back(std::move(t));
+            }
+        }
+        ix->tab_pos.alloc(ix->L * sizeof(const uint32_t*));
+        BLSH_CUDA(cudaMemcpyAsync(ix->tab_pos.p, tab_pos.data(), ix->L * sizeof(const uint32_t*), cudaMemcpyHostToDevice, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
         for (auto& e : ix->ev) BLSH_CUDA(cudaEventCreate(&e));
     });
     if (st != BLSH_OK) {
@@ -272,6 +316,13 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     add(nq, 4);                         // qorder
     add(nq, 4); add((size_t)2 * ix.G, 4);   // lperm, leaf counts + cursors
     if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
+    const int L = ix.L;
+    for (int l = 1; l < L; ++l) {      // per-table a2-a4 stages
+        add((size_t)nq * M, 4); add((size_t)nq * M, 4); add(nq, 4); add(nq, 16);
+        add((size_t)nq * (T + 1), 8); add(nq, 8); add(nq, 8);
+        if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
+    }
+    if (L > 1) { add(nq + 1, 8); add(nq, 8); add(L, 8); add(L, 8); }
     if (out_host) { add((size_t)nq * k, 8); add((size_t)nq * k, 4); add(nq, 8); add((size_t)nq * k, 8); }
     w.arena.ensure(need);
     Arena ar{w.arena.as<char>(), 0, w.arena.bytes};
@@ -294,6 +345,29 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int32_t* lcnt = ar.take<int32_t>((size_t)2 * ix.G);
     w.pkey = keep ? ar.take<Key128>((size_t)nq * T) : nullptr;
     w.pvalid = keep ? ar.take<int32_t>((size_t)nq * T) : nullptr;
+    w.tq.assign(L, QueryWork::TableQuery{});
+    w.tq[0] = {w.qt, w.qcode, w.qoor, w.qkey, w.pkey, w.pvalid, w.ivl, w.base, w.cnt};
+    for (int l = 1; l < L; ++l) {
+        auto& t = w.tq[l];
+        t.qt = ar.take<float>((size_t)nq * M);
+        t.qcode = ar.take<int32_t>((size_t)nq * M);
+        t.qoor = ar.take<int32_t>(nq);
+        t.qkey = ar.take<Key128>(nq);
+        t.ivl = ar.take<uint2>((size_t)nq * (T + 1));
+        t.base = ar.take<int64_t>(nq);
+        t.cnt = ar.take<int64_t>(nq);
+        t.pkey = keep ? ar.take<Key128>((size_t)nq * T) : nullptr;
+        t.pvalid = keep ? ar.take<int32_t>((size_t)nq * T) : nullptr;
+    }
+    int64_t* raw = nullptr;
+    const uint2** ivl_ptrs = nullptr;
+    const int64_t** cnt_ptrs = nullptr;
+    if (L > 1) {
+        w.raw_off = ar.take<int64_t>(nq + 1);
+        raw = ar.take<int64_t>(nq);
+        ivl_ptrs = ar.take<const uint2*>(L);
+        cnt_ptrs = ar.take<const int64_t*>(L);
+    }
     int64_t* d_ids = out_ids;
     float* d_d2 = out_d2;
     int64_t* d_nc = out_ncand;
@@ -329,9 +403,40 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.lperm = lperm; a.lcnt = lcnt;
     // a1+a2
     launches += launch_route_hash(a, s);
+    auto table_args = [&](int l) {   // QueryArgs of hash table l
+        QueryArgs al = a;
+        const auto& t = w.tq[l];
+        const auto& x = *ix.xt[l - 1];
+        al.A = x.A.as<float>(); al.bvec = x.b.as<float>();
+        al.ukey = x.ukey.as<Key128>(); al.uoff = x.uoff.as<uint32_t>(); al.leaf_u = x.leaf_u.as<int64_t>();
+        al.qt = t.qt; al.qcode = t.qcode; al.qoor = t.qoor; al.qkey = t.qkey; al.pkey = t.pkey;
+        al.pvalid = t.pvalid; al.ivl = t.ivl; al.base = t.base; al.cnt = t.cnt; al.level = nullptr;
+        return al;
+    };
+    for (int l = 1; l < L; ++l) { launch_hash(table_args(l), s); ++launches; }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // a3+a4
     launch_probe_lookup(a, s); ++launches;
+    for (int l = 1; l < L; ++l) { launch_probe_lookup(table_args(l), s); ++launches; }
+    int64_t total_raw = 0;
+    if (L > 1) {   // a4 across tables: deduplicated union of the L tables' buckets (R24)
+        std::vector<const uint2*> iv(L);
+        std::vector<const int64_t*> cn(L);
+        for (int l = 0; l < L; ++l) { iv[l] = w.tq[l].ivl; cn[l] = w.tq[l].cnt; }
+        BLSH_CUDA(cudaMemcpyAsync(ivl_ptrs, iv.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
+        BLSH_CUDA(cudaMemcpyAsync(cnt_ptrs, cn.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
+        UnionArgs u{};
+        u.nq = nq; u.L = L; u.T = T; u.qleaf = w.qleaf; u.qoor = w.qoor; u.ivl = ivl_ptrs; u.cnt = cnt_ptrs;
+        u.pos = ix.tab_pos.as<const uint32_t*>(); u.leaf_pos = ix.leaf_pos.as<int64_t>();
+        u.raw_off = w.raw_off; u.raw = raw; u.out_cnt = w.cnt;
+        launch_raw_counts(u, s); ++launches;
+        scan_exclusive_i64(raw, w.raw_off, nq, w.scan, s); launches += 3;
+        BLSH_CUDA(cudaMemcpyAsync(&total_raw, w.raw_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        w.listbuf.ensure((size_t)std::max<int64_t>(total_raw, 1) * sizeof(uint32_t));
+        u.list = w.listbuf.as<uint32_t>();
+        launch_union_tables(u, ix.max_leaf_rows, s); ++launches;
+    }
     if (out_base) {   // blsh_query_base_counts: a1-a4 only
         BLSH_CUDA(cudaMemcpyAsync(out_base, w.base, (size_t)nq * 8, out_host ? cudaMemcpyDeviceToHost
                                                                               : cudaMemcpyDeviceToDevice, s));
@@ -359,7 +464,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t total = 0;
     BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    const int kind = shortlist_kind(ds, T, k);
+    const int kind = L > 1 ? 0 : shortlist_kind(ds, T, k);   // L > 1: warp short-list over the position lists
     const bool tiled = kind > 0;
     int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0;
     double qload_rows = 0.0;
@@ -393,6 +498,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
         sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
         sa.cand_off = cand_off;
+        sa.list = L > 1 ? w.listbuf.as<uint32_t>() : nullptr;
+        sa.list_off = L > 1 ? w.raw_off : nullptr;
         sa.cand_keys = large_k ? w.partials.as<unsigned long long>() : nullptr;
         launch_shortlist(sa, s); if (n_items) ++launches;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
@@ -469,6 +576,7 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
     }
     if (p->n_probes > 256) return fail(BLSH_ERR_UNSUPPORTED, "n_probes > 256");
     if (p->hierarchy) {
+        if (idx->L > 1) return fail(BLSH_ERR_UNSUPPORTED, "the Morton hierarchy is defined for one table (R24)");
         if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "the Morton hierarchy needs a Z^M index");
         if (p->hier_step_bits < 0 || p->hier_step_bits > idx->M) return fail(BLSH_ERR_INVALID, "hier_step_bits must be in [0, M]");
         if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");
@@ -522,6 +630,7 @@ blsh_status blsh_query_base_counts(const blsh_index* idx, const float* Q, int64_
     p2.global_base = nullptr;
     blsh_status c = check_query(idx, Q, nq, 1, &p2);
     if (c != BLSH_OK) return c;
+    if (idx->L > 1) return fail(BLSH_ERR_UNSUPPORTED, "base counts serve the hierarchy, which needs L = 1");
     if (nq > 0 && !out_base) return fail(BLSH_ERR_INVALID, "out_base is NULL");
     if (nq == 0) return BLSH_OK;
     const bool q_host = !is_device_ptr(Q);
@@ -577,6 +686,11 @@ blsh_status blsh_index_info(const blsh_index* idx, blsh_info* out) {
                                   idx->ukey.bytes + idx->uleaf.bytes + idx->uoff.bytes + idx->leaf_u.bytes +
                                   idx->pt_leaf.bytes + idx->pt_code.bytes + idx->pt_key.bytes);
     out->build_ms = idx->build_ms;
+    out->n_tables = idx->L;
+    out->pad_ = 0;
+    for (const auto& t : idx->xt)
+        out->device_bytes += (int64_t)(t->A.bytes + t->b.bytes + t->ukey.bytes + t->uleaf.bytes + t->uoff.bytes +
+                                       t->leaf_u.bytes + t->pos.bytes + t->perm.bytes);
     return BLSH_OK;
 }
 
@@ -588,8 +702,29 @@ blsh_status blsh_last_stats(const blsh_index* idx, blsh_stats* out) {
 
 blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t cap, size_t* needed) {
     if (!idx) return fail(BLSH_ERR_INVALID, "index is NULL");
+    const int table = what >> 8;   // BLSH_EX_TABLE(l, item): table l of an L-table index
+    what &= 0xFF;
+    if (table < 0 || table >= idx->L) return fail(BLSH_ERR_INVALID, "table out of range");
+    const blsh::ExtraTable* xt = table > 0 ? idx->xt[table - 1].get() : nullptr;
+    if (xt && !(what == BLSH_EX_A || what == BLSH_EX_B || what == BLSH_EX_PERM || what == BLSH_EX_UKEY ||
+                what == BLSH_EX_ULEAF || what == BLSH_EX_UOFF || what == BLSH_EX_LEAF_U ||
+                (what >= BLSH_EX_Q_T && what <= BLSH_EX_Q_INTERVALS && what != BLSH_EX_Q_LEVEL &&
+                 what != BLSH_EX_Q_TAU && what != BLSH_EX_Q_LEAF)))
+        return fail(BLSH_ERR_INVALID, "item is not per table");
+    const std::vector<float>& A_h = xt ? xt->A_h : idx->A_h;
+    const std::vector<float>& b_h = xt ? xt->b_h : idx->b_h;
+    const void* perm_p = xt ? xt->perm.p : idx->perm.p;
+    const void* ukey_p = xt ? xt->ukey.p : idx->ukey.p;
+    const void* uleaf_p = xt ? xt->uleaf.p : idx->uleaf.p;
+    const void* uoff_p = xt ? xt->uoff.p : idx->uoff.p;
+    const int64_t nu = xt ? xt->nu : idx->nu;
+    const std::vector<int64_t>& leaf_u_h = xt ? xt->leaf_u_h : idx->leaf_u_h;
     const int64_t G = idx->G, M = idx->M, d = idx->d, nn = G > 1 ? G - 1 : 0;
     const blsh::QueryWork& w = idx->qw;
+    blsh::QueryWork::TableQuery tq0{w.qt, w.qcode, w.qoor, w.qkey, w.pkey, w.pvalid, w.ivl, w.base, w.cnt};
+    const blsh::QueryWork::TableQuery tq = (table > 0 && (size_t)table < w.tq.size()) ? w.tq[table] : tq0;
+    if (table > 0 && (size_t)table >= w.tq.size() && what >= BLSH_EX_Q_T)
+        return fail(BLSH_ERR_INVALID, "last query without keep_stages");
     const int64_t nq = w.nq;
     const int T = w.T;
     const void* host_src = nullptr;
@@ -599,8 +734,8 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
     auto need_q = [&]() -> bool { return idx->has_stages; };
     auto need_pt = [&]() -> bool { return idx->has_pt; };
     switch (what) {
-        case BLSH_EX_A: host_src = idx->A_h.data(); bytes = idx->A_h.size() * 4; break;
-        case BLSH_EX_B: host_src = idx->b_h.data(); bytes = idx->b_h.size() * 4; break;
+        case BLSH_EX_A: host_src = A_h.data(); bytes = A_h.size() * 4; break;
+        case BLSH_EX_B: host_src = b_h.data(); bytes = b_h.size() * 4; break;
         case BLSH_EX_W: host_src = idx->W_h.data(); bytes = idx->W_h.size() * 4; break;
         case BLSH_EX_DIRS: host_src = idx->dirs_h.data(); bytes = (size_t)nn * d * 4; break;
         case BLSH_EX_MU: host_src = idx->mu_h.data(); bytes = (size_t)nn * d * 4; break;
@@ -612,7 +747,7 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             bytes = (size_t)idx->n_owned * 8;
             if (dst && cap >= bytes && bytes) {
                 std::vector<uint32_t> p32(idx->n_owned);
-                if (cudaMemcpy(p32.data(), idx->perm.p, p32.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                if (cudaMemcpy(p32.data(), perm_p, p32.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
                     return fail(BLSH_ERR_CUDA, "export copy failed");
                 int64_t* o = (int64_t*)dst;
                 for (size_t i = 0; i < p32.size(); ++i) o[i] = p32[i];
@@ -621,10 +756,10 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
         }
         case BLSH_EX_UKEY: {
-            bytes = (size_t)idx->nu * 16;
+            bytes = (size_t)nu * 16;
             if (dst && cap >= bytes && bytes) {
-                std::vector<blsh::Key128> k(idx->nu);
-                if (cudaMemcpy(k.data(), idx->ukey.p, k.size() * 16, cudaMemcpyDeviceToHost) != cudaSuccess)
+                std::vector<blsh::Key128> k(nu);
+                if (cudaMemcpy(k.data(), ukey_p, k.size() * 16, cudaMemcpyDeviceToHost) != cudaSuccess)
                     return fail(BLSH_ERR_CUDA, "export copy failed");
                 uint64_t* o = (uint64_t*)dst;
                 for (size_t i = 0; i < k.size(); ++i) { o[2 * i] = k[i].hi; o[2 * i + 1] = k[i].lo; }
@@ -632,12 +767,12 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             if (needed) *needed = bytes;
             return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
         }
-        case BLSH_EX_ULEAF: dev_src = idx->uleaf.p; bytes = (size_t)idx->nu * 4; break;
+        case BLSH_EX_ULEAF: dev_src = uleaf_p; bytes = (size_t)nu * 4; break;
         case BLSH_EX_UOFF: {
-            bytes = (size_t)(idx->nu + 1) * 8;
+            bytes = (size_t)(nu + 1) * 8;
             if (dst && cap >= bytes) {
-                std::vector<uint32_t> u(idx->nu + 1);
-                if (cudaMemcpy(u.data(), idx->uoff.p, u.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                std::vector<uint32_t> u(nu + 1);
+                if (cudaMemcpy(u.data(), uoff_p, u.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
                     return fail(BLSH_ERR_CUDA, "export copy failed");
                 int64_t* o = (int64_t*)dst;
                 for (size_t i = 0; i < u.size(); ++i) o[i] = u[i];
@@ -645,7 +780,7 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             if (needed) *needed = bytes;
             return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
         }
-        case BLSH_EX_LEAF_U: host_src = idx->leaf_u_h.data(); bytes = (size_t)(G + 1) * 8; break;
+        case BLSH_EX_LEAF_U: host_src = leaf_u_h.data(); bytes = (size_t)(G + 1) * 8; break;
         case BLSH_EX_POINT_LEAF:
             if (!need_pt()) return fail(BLSH_ERR_INVALID, "build without keep_stages");
             dev_src = idx->pt_leaf.p; bytes = (size_t)idx->n * 4; break;
@@ -671,12 +806,12 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
         if (!need_q()) return fail(BLSH_ERR_INVALID, "last query without keep_stages");
         switch (what) {
             case BLSH_EX_Q_LEAF: dev_src = w.qleaf; bytes = (size_t)nq * 4; break;
-            case BLSH_EX_Q_T: dev_src = w.qt; bytes = (size_t)nq * M * 4; break;
-            case BLSH_EX_Q_CODE: dev_src = w.qcode; bytes = (size_t)nq * M * 4; break;
+            case BLSH_EX_Q_T: dev_src = tq.qt; bytes = (size_t)nq * M * 4; break;
+            case BLSH_EX_Q_CODE: dev_src = tq.qcode; bytes = (size_t)nq * M * 4; break;
             case BLSH_EX_Q_OOR: {
                 bytes = (size_t)nq * 4;
                 if (dst && cap >= bytes) {
-                    if (cudaMemcpy(dst, w.qoor, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    if (cudaMemcpy(dst, tq.qoor, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
                         return fail(BLSH_ERR_CUDA, "export copy failed");
                     int32_t* o = (int32_t*)dst;
                     for (int64_t i = 0; i < nq; ++i) o[i] &= 1;
@@ -691,9 +826,9 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
                 if (dst && cap >= bytes && bytes) {
                     std::vector<blsh::Key128> k(cnt);
                     std::vector<int32_t> oor(nq);
-                    if (cudaMemcpy(k.data(), what == BLSH_EX_Q_KEY ? (void*)w.qkey : (void*)w.pkey, bytes,
+                    if (cudaMemcpy(k.data(), what == BLSH_EX_Q_KEY ? (void*)tq.qkey : (void*)tq.pkey, bytes,
                                    cudaMemcpyDeviceToHost) != cudaSuccess ||
-                        cudaMemcpy(oor.data(), w.qoor, nq * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+                        cudaMemcpy(oor.data(), tq.qoor, nq * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
                         return fail(BLSH_ERR_CUDA, "export copy failed");
                     uint64_t* o = (uint64_t*)dst;
                     for (int64_t i = 0; i < cnt; ++i) {
@@ -705,15 +840,15 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
                 if (needed) *needed = bytes;
                 return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
             }
-            case BLSH_EX_Q_PVALID: dev_src = w.pvalid; bytes = (size_t)nq * T * 4; break;
-            case BLSH_EX_Q_BASE: dev_src = w.base; bytes = (size_t)nq * 8; break;
+            case BLSH_EX_Q_PVALID: dev_src = tq.pvalid; bytes = (size_t)nq * T * 4; break;
+            case BLSH_EX_Q_BASE: dev_src = tq.base; bytes = (size_t)nq * 8; break;
             case BLSH_EX_Q_LEVEL: dev_src = w.level; bytes = (size_t)nq * 4; break;
             case BLSH_EX_Q_TAU: host_src = &idx->stats.tau; bytes = 8; break;
             case BLSH_EX_Q_INTERVALS: {
                 bytes = (size_t)nq * (T + 1) * 16;
                 if (dst && cap >= bytes && bytes) {
                     std::vector<uint2> iv((size_t)nq * (T + 1));
-                    if (cudaMemcpy(iv.data(), w.ivl, iv.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+                    if (cudaMemcpy(iv.data(), tq.ivl, iv.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
                         return fail(BLSH_ERR_CUDA, "export copy failed");
                     int64_t* o = (int64_t*)dst;
                     for (size_t i = 0; i < iv.size(); ++i) { o[2 * i] = iv[i].x; o[2 * i + 1] = iv[i].y; }

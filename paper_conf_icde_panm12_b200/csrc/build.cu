@@ -132,11 +132,69 @@ __global__ void k_permute_rows(const float* __restrict__ Xs, int ds, const uint3
     }
 }
 
+__global__ void k_invert(const uint32_t* __restrict__ perm, int64_t n, uint32_t* __restrict__ inv) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        inv[perm[i]] = (uint32_t)i;
+}
+
+__global__ void k_map_pos(const uint32_t* __restrict__ perm_l, const uint32_t* __restrict__ inv0, int64_t n,
+                          uint32_t* __restrict__ pos) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        pos[i] = inv0[perm_l[i]];
+}
+
 }  // namespace
+
+void invert_perm(const uint32_t* perm, int64_t n_owned, uint32_t* inv, cudaStream_t s) {
+    if (n_owned == 0) return;
+    k_invert<<<592, 256, 0, s>>>(perm, n_owned, inv);
+    BLSH_LAUNCH_CHECK();
+}
+
+void build_extra_table(const blsh_index& ix, ExtraTable& t, const unsigned long long* key_hi,
+                       const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
+                       const uint32_t* inv0, int64_t n_owned, ScanTemp& scan, cudaStream_t s) {
+    const int64_t n = n_owned;
+    DevBuf flags, U;
+    flags.alloc(std::max<int64_t>(n, 1));
+    U.alloc((std::max<int64_t>(n, 1) + 1) * sizeof(int64_t));
+    t.perm.alloc(std::max<int64_t>(n, 1) * sizeof(uint32_t));
+    t.pos.alloc(std::max<int64_t>(n, 1) * sizeof(uint32_t));
+    int64_t nu = 0;
+    if (n > 0) {
+        k_flags<<<592, 256, 0, s>>>(key_hi, key_lo, leaf, n, flags.as<uint8_t>());
+        BLSH_LAUNCH_CHECK();
+        scan_exclusive_u8(flags.as<uint8_t>(), U.as<int64_t>(), n, scan, s);
+        BLSH_CUDA(cudaMemcpyAsync(&nu, U.as<int64_t>() + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+    }
+    t.nu = nu;
+    t.ukey.alloc(std::max<int64_t>(nu, 1) * sizeof(Key128));
+    t.uleaf.alloc(std::max<int64_t>(nu, 1) * sizeof(int32_t));
+    t.uoff.alloc((std::max<int64_t>(nu, 1) + 1) * sizeof(uint32_t));
+    BLSH_CUDA(cudaMemsetAsync(t.uoff.p, 0, sizeof(uint32_t), s));
+    if (n > 0) {
+        k_unique<<<592, 256, 0, s>>>(key_hi, key_lo, leaf, id, flags.as<uint8_t>(), U.as<int64_t>(), n,
+                                     t.ukey.as<Key128>(), t.uleaf.as<int32_t>(), t.uoff.as<uint32_t>(),
+                                     t.perm.as<uint32_t>());
+        BLSH_LAUNCH_CHECK();
+        k_map_pos<<<592, 256, 0, s>>>(t.perm.as<uint32_t>(), inv0, n, t.pos.as<uint32_t>());
+        BLSH_LAUNCH_CHECK();
+    }
+    t.leaf_u.alloc((ix.G + 1) * sizeof(int64_t));
+    k_leaf_u<<<(ix.G + 1 + 127) / 128, 128, 0, s>>>(t.uleaf.as<int32_t>(), nu, ix.G, t.leaf_u.as<int64_t>());
+    BLSH_LAUNCH_CHECK();
+    t.leaf_u_h.assign(ix.G + 1, 0);
+    BLSH_CUDA(cudaMemcpyAsync(t.leaf_u_h.data(), t.leaf_u.p, (ix.G + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+}
 
 bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order, const std::vector<int64_t>& seg,
                  int64_t pos_lo, int64_t pos_hi, unsigned long long* key_hi, unsigned long long* key_lo,
-                 uint32_t* leaf, uint32_t* id, int32_t* code_out, cudaStream_t s) {
+                 uint32_t* leaf, uint32_t* id, int32_t* code_out, cudaStream_t s, const float* A,
+                 const float* b) {
+    if (!A) A = ix.A.as<float>();
+    if (!b) b = ix.b.as<float>();
     std::vector<HTile> tiles;
     for (int g = ix.leaf_lo; g < ix.leaf_hi; ++g)
         for (int64_t p = seg[g]; p < seg[g + 1]; p += kTR)
@@ -151,7 +209,7 @@ bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order, c
 #define BLSH_HASH_CASE(MMV)                                                                                    \
     case MMV:                                                                                                  \
         k_hash_rows<MMV><<<nt, kTR, 0, s>>>(Xs, ix.ds, ix.d, order, tiles_d.as<HTile>(), pos_lo,              \
-                                            ix.A.as<float>(), ix.b.as<float>(), ix.W.as<float>(), ix.B,       \
+                                            A, b, ix.W.as<float>(), ix.B,                                     \
                                             ix.quantizer, key_hi, key_lo, leaf, id, code_out, bad_d.as<int>()); \
         break;
     switch (ix.M) {

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <memory>
 #include <stdexcept>
 #include <string>
 #include <vector>
@@ -113,6 +114,30 @@ struct QueryWork {
     int64_t* tau = nullptr;
     int64_t* ncand_dev = nullptr;
     int64_t* misc = nullptr;      // small scalars
+    // L > 1 tables: per-table a2-a4 stages (tq[0] aliases the fields above)
+    struct TableQuery {
+        float* qt; int32_t* qcode; int32_t* qoor; Key128* qkey; Key128* pkey; int32_t* pvalid;
+        uint2* ivl; int64_t* base; int64_t* cnt;
+    };
+    std::vector<TableQuery> tq;
+    DevBuf listbuf;               // deduplicated candidate positions (u32), at raw_off[q]
+    int64_t* raw_off = nullptr;   // [nq+1] scan of the per-query sums of the table counts
+};
+
+// Hash table l >= 1 of an L-table index.  Table 0 is the primary
+// table (blsh_index fields); the rows of X are stored once, in table-0 order,
+// and table l refers to them through pos (table-l position -> table-0 position).
+struct ExtraTable {
+    DevBuf A, b;          // [G][M][d], [G][M] this table's (a, b) (R2 streams (1, l, g), (2, l, g))
+    DevBuf ukey;          // [nu] Key128
+    DevBuf uleaf;         // [nu] int32
+    DevBuf uoff;          // [nu+1] uint32 (table-l positions)
+    DevBuf leaf_u;        // [G+1] int64
+    DevBuf pos;           // [n_owned] uint32 table-0 position of the row at table-l position i
+    DevBuf perm;          // [n_owned] uint32 original ids in table-l order (export / parity)
+    int64_t nu = 0;
+    std::vector<float> A_h, b_h;
+    std::vector<int64_t> leaf_u_h;
 };
 
 }  // namespace blsh
@@ -140,6 +165,13 @@ struct blsh_index {
     blsh::DevBuf uleaf;   // [nu] int32
     blsh::DevBuf uoff;    // [nu+1] uint32
     blsh::DevBuf leaf_u;  // [G+1] int64
+    // L > 1 hash tables
+    int L = 1;
+    std::vector<std::unique_ptr<blsh::ExtraTable>> xt;   // tables 1..L-1
+    std::vector<int64_t> leaf_pos_h;   // [G+1] first owned table position of each leaf (clamped)
+    blsh::DevBuf leaf_pos;             // device copy
+    blsh::DevBuf tab_pos;              // [L] const uint32_t* (pos of table l; [0] = NULL)
+    int64_t max_leaf_rows = 0;         // largest owned leaf
     // kept build stages (keep_stages)
     blsh::DevBuf pt_leaf, pt_code, pt_key;
     bool has_pt = false;
@@ -156,6 +188,8 @@ namespace blsh {
 // Host-side generator (params.cpp), reading R2.
 void gen_params(uint64_t seed, int G, int M, int d, const float* Wleaf, float* A, float* b,
                 float* dirs, double* jit);
+// (a, b) of hash table `table` (table 0 = the ones gen_params draws).
+void gen_table_params(uint64_t seed, int table, int G, int M, int d, const float* Wleaf, float* A, float* b);
 
 // RP-tree over Xs [n][ds]; fills idx tree arrays; returns leaf segments of the
 // final order (order_out [n] uint32 ids grouped by leaf, ascending id) and
@@ -169,12 +203,19 @@ bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order,
                  const std::vector<int64_t>& seg, int64_t pos_lo, int64_t pos_hi,
                  unsigned long long* key_hi, unsigned long long* key_lo, uint32_t* leaf,
                  uint32_t* id, int32_t* code_out /* nullable [n][M] by id */,
-                 cudaStream_t s);
+                 cudaStream_t s, const float* A = nullptr, const float* b = nullptr /* NULL: table 0's */);
 
 // After sorting: buckets, offsets, permuted rows.
 void build_table(blsh_index& ix, const float* Xs, const unsigned long long* key_hi,
                  const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
                  int64_t n_owned, ScanTemp& scan, cudaStream_t s);
+
+// Table l >= 1 (sorted entries of that table): bucket directory + pos via the
+// inverse of table 0's permutation (inv0[id] = table-0 position).
+void build_extra_table(const blsh_index& ix, ExtraTable& t, const unsigned long long* key_hi,
+                       const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
+                       const uint32_t* inv0, int64_t n_owned, ScanTemp& scan, cudaStream_t s);
+void invert_perm(const uint32_t* perm, int64_t n_owned, uint32_t* inv, cudaStream_t s);
 
 // ---- query (query.cu, shortlist.cu) ----------------------------------------------
 void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,

@@ -38,10 +38,11 @@ inline uint64_t stream_id(uint64_t kind, uint64_t table, uint64_t idx) {
 }
 }  // namespace
 
-void gen_params(uint64_t seed, int G, int M, int d, const float* Wleaf, float* A, float* b,
-                float* dirs, double* jit) {
+// L tables "constructed independently with different dim-M hash
+// functions": table l draws (a, b) from streams (1, l, g) and (2, l, g).
+void gen_table_params(uint64_t seed, int table, int G, int M, int d, const float* Wleaf, float* A, float* b) {
     for (int g = 0; g < G; ++g) {
-        const uint64_t sa = stream_id(1, 0, (uint64_t)g), sb = stream_id(2, 0, (uint64_t)g);
+        const uint64_t sa = stream_id(1, (uint64_t)table, (uint64_t)g), sb = stream_id(2, (uint64_t)table, (uint64_t)g);
         for (int i = 0; i < M; ++i)
             for (int j = 0; j < d; ++j)
                 A[((size_t)g * M + i) * d + j] = (float)counter_normal(seed, sa, (uint64_t)i * d + j);
@@ -52,6 +53,11 @@ void gen_params(uint64_t seed, int G, int M, int d, const float* Wleaf, float* A
             b[(size_t)g * M + i] = v;
         }
     }
+}
+
+void gen_params(uint64_t seed, int G, int M, int d, const float* Wleaf, float* A, float* b,
+                float* dirs, double* jit) {
+    gen_table_params(seed, 0, G, M, d, Wleaf, A, b);
     std::vector<double> gv((size_t)d);
     for (int v = 0; v + 1 < G; ++v) {
         const uint64_t sd = stream_id(3, 0, (uint64_t)v);

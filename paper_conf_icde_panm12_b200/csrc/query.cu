@@ -670,6 +670,26 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     return 4;
 }
 
+void launch_hash(const QueryArgs& a, cudaStream_t s) {
+    if (a.nq == 0) return;
+    const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
+    const size_t smem_h = (size_t)kRHQ * (a.ds + 4) * sizeof(float) + (size_t)a.M * a.d * sizeof(float);
+#define BLSH_H_CASE(MMV)                                                                                    \
+    case MMV:                                                                                              \
+        BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        k_hash<MMV><<<grid, kRHQ, smem_h, s>>>(a, a.lperm);                                                 \
+        break;
+    switch (a.M) {
+        BLSH_H_CASE(1) BLSH_H_CASE(2) BLSH_H_CASE(3) BLSH_H_CASE(4)
+        BLSH_H_CASE(5) BLSH_H_CASE(6) BLSH_H_CASE(7) BLSH_H_CASE(8)
+        BLSH_H_CASE(9) BLSH_H_CASE(10) BLSH_H_CASE(11) BLSH_H_CASE(12)
+        BLSH_H_CASE(13) BLSH_H_CASE(14) BLSH_H_CASE(15) BLSH_H_CASE(16)
+        default: throw Error(BLSH_ERR_INVALID, "M out of range");
+    }
+#undef BLSH_H_CASE
+    BLSH_LAUNCH_CHECK();
+}
+
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s) {
     k_probe_lookup<<<(unsigned)((a.nq + kPW - 1) / kPW), kPW * 32, 0, s>>>(a);
     BLSH_LAUNCH_CHECK();

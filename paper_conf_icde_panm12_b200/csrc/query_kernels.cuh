@@ -44,6 +44,27 @@ struct QueryArgs {
 void upload_e8_roots();
 int launch_route_hash(const QueryArgs& a, cudaStream_t s);   // returns kernels launched
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s);
+// a2 only (queries already routed and grouped by leaf in a.lperm): hash with a.A / a.bvec
+void launch_hash(const QueryArgs& a, cudaStream_t s);
+
+// L > 1 tables (tables.cu): raw[q] = sum over tables of |A0_l(q)|, then the
+// deduplicated union of the L tables' intervals as ascending table-0 positions.
+struct UnionArgs {
+    int64_t nq;
+    int L, T;
+    const int32_t* qleaf;
+    const int32_t* qoor;          // table 0's flags (bit 1: leaf not owned)
+    const uint2* const* ivl;      // [L] device pointers to [nq][T+1]
+    const int64_t* const* cnt;    // [L] device pointers to [nq]
+    const uint32_t* const* pos;   // [L] table-l position -> table-0 position ([0] = identity)
+    const int64_t* leaf_pos;      // [G+1]
+    const int64_t* raw_off;       // [nq+1]
+    int64_t* raw;                 // [nq]
+    uint32_t* list;               // [raw_off[nq]]
+    int64_t* out_cnt;             // [nq] |A(q)|
+};
+void launch_raw_counts(const UnionArgs& u, cudaStream_t s);
+void launch_union_tables(const UnionArgs& u, int64_t max_leaf_rows, cudaStream_t s);
 void launch_median(const int64_t* base, int64_t nq, int64_t* tau, cudaStream_t s);
 void launch_widen(const QueryArgs& a, const int64_t* tau, int64_t min_cand, cudaStream_t s);
 
@@ -59,6 +80,8 @@ struct ShortlistArgs {
     unsigned long long* partials;   // [n_items][k]
     const int64_t* cand_off;        // [nq+1] (large k)
     unsigned long long* cand_keys;  // [total] non-NULL: emit every candidate key (large k)
+    const uint32_t* list;           // non-NULL (L > 1): deduplicated candidate positions per query
+    const int64_t* list_off;        // [nq+1] start of each query's list
 };
 
 // query-tiled short-list (shortlist_tiled.cu)

@@ -43,9 +43,13 @@ __device__ __forceinline__ void topk_insert(TopK& t, unsigned long long v, int l
 // EMIT = false: register top-k per item (k <= 64) into a.partials.
 // EMIT = true (large k, k > 64): the packed key of every candidate goes to
 // a.cand_keys[a.cand_off[q] + c] (c = rank of the candidate in the query's
-// interval order); k_select then takes the k smallest per query.  The distance
-// arithmetic is the same in both modes (R22), so results agree bit for bit.
-template <int NV, bool EMIT>
+// candidate order); k_select then takes the k smallest per query.
+// LIST = false: the candidates are the query's T+1 position intervals (L = 1).
+// LIST = true (L > 1 tables): the candidates are the deduplicated position list
+// a.list[a.list_off[q] ..] that k_union_tables wrote (ascending positions).
+// The distance arithmetic is the same in every mode (R22), so the modes agree
+// bit for bit.
+template <int NV, bool EMIT, bool LIST>
 __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int lane = threadIdx.x & 31;
     const int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5);
@@ -71,65 +75,85 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     TopK tk{kEmpty, kEmpty};
     const int k = a.k;
     unsigned long long thr = kEmpty;
-    const uint2* ivl = a.ivl + (size_t)q * (a.T + 1);
-    int64_t acc = 0;   // candidates before the current interval
-    for (int p = 0; p <= a.T && acc < c1; ++p) {
-        const uint2 iv = ivl[p];
-        const int64_t len = (int64_t)iv.y - (int64_t)iv.x;
-        if (len <= 0) continue;
-        const int64_t s = max(c0, acc), e = min(c1, acc + len);
-        if (s < e) {
-            const int64_t pa = (int64_t)iv.x + (s - acc), pb = (int64_t)iv.x + (e - acc);
-            for (int64_t r0 = pa; r0 < pb; r0 += 4) {
-                float part[4];
+    // Rows r[0..nr) (table positions) that are candidates c, c+1, .. of q.
+    auto group = [&](const int64_t (&r)[4], int nr, int64_t c) {
+        float part[4];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    part[j] = 0.0f;
-                    if (r0 + j < pb) {
-                        const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)(r0 + j) * a.ds);
+        for (int j = 0; j < 4; ++j) {
+            part[j] = 0.0f;
+            if (j < nr) {
+                const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
 #pragma unroll
-                        for (int u = 0; u < NV; ++u) {
-                            const int v = lane + 32 * u;
-                            if (v < nv) {
-                                const float4 x = __ldg(xr + v);
-                                float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
-                                part[j] = fmaf(dx, dx, part[j]);
-                                part[j] = fmaf(dy, dy, part[j]);
-                                part[j] = fmaf(dz, dz, part[j]);
-                                part[j] = fmaf(dw, dw, part[j]);
-                            }
-                        }
-                    }
-                }
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) part[j] += __shfl_xor_sync(BLSH_FULL, part[j], o);
-                }
-                const uint32_t idl = (lane < 4 && r0 + lane < pb) ? __ldg(a.perm + r0 + lane) : 0u;
-                if (EMIT) {
-                    if (lane < 4 && r0 + lane < pb) {
-                        float pj = part[0];
-#pragma unroll
-                        for (int j = 1; j < 4; ++j) pj = lane == j ? part[j] : pj;
-                        a.cand_keys[a.cand_off[q] + acc + (r0 - (int64_t)iv.x) + lane] = pack_entry(pj, idl);
-                    }
-                    continue;
-                }
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    const uint32_t id = __shfl_sync(BLSH_FULL, idl, j);
-                    if (r0 + j < pb) {
-                        const unsigned long long key = pack_entry(part[j], id);
-                        if (key < thr) {
-                            topk_insert(tk, key, lane);
-                            thr = topk_thr(tk, k);
-                        }
+                for (int u = 0; u < NV; ++u) {
+                    const int v = lane + 32 * u;
+                    if (v < nv) {
+                        const float4 x = __ldg(xr + v);
+                        float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                        part[j] = fmaf(dx, dx, part[j]);
+                        part[j] = fmaf(dy, dy, part[j]);
+                        part[j] = fmaf(dz, dz, part[j]);
+                        part[j] = fmaf(dw, dw, part[j]);
                     }
                 }
             }
         }
-        acc += len;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) part[j] += __shfl_xor_sync(BLSH_FULL, part[j], o);
+        }
+        int64_t rl = r[0];
+#pragma unroll
+        for (int j = 1; j < 4; ++j) rl = lane == j ? r[j] : rl;
+        const uint32_t idl = (lane < nr) ? __ldg(a.perm + rl) : 0u;
+        if (EMIT) {
+            if (lane < nr) {
+                float pj = part[0];
+#pragma unroll
+                for (int j = 1; j < 4; ++j) pj = lane == j ? part[j] : pj;
+                a.cand_keys[a.cand_off[q] + c + lane] = pack_entry(pj, idl);
+            }
+            return;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const uint32_t id = __shfl_sync(BLSH_FULL, idl, j);
+            if (j < nr) {
+                const unsigned long long key = pack_entry(part[j], id);
+                if (key < thr) {
+                    topk_insert(tk, key, lane);
+                    thr = topk_thr(tk, k);
+                }
+            }
+        }
+    };
+    if (LIST) {
+        const uint32_t* L = a.list + a.list_off[q];
+        for (int64_t c = c0; c < c1; c += 4) {
+            const int nr = (int)min((int64_t)4, c1 - c);
+            int64_t r[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) r[j] = j < nr ? (int64_t)__ldg(L + c + j) : 0;
+            group(r, nr, c);
+        }
+    } else {
+        const uint2* ivl = a.ivl + (size_t)q * (a.T + 1);
+        int64_t acc = 0;   // candidates before the current interval
+        for (int p = 0; p <= a.T && acc < c1; ++p) {
+            const uint2 iv = ivl[p];
+            const int64_t len = (int64_t)iv.y - (int64_t)iv.x;
+            if (len <= 0) continue;
+            const int64_t s = max(c0, acc), e = min(c1, acc + len);
+            if (s < e) {
+                const int64_t pa = (int64_t)iv.x + (s - acc), pb = (int64_t)iv.x + (e - acc);
+                for (int64_t r0 = pa; r0 < pb; r0 += 4) {
+                    const int nr = (int)min((int64_t)4, pb - r0);
+                    const int64_t r[4] = {r0, r0 + 1, r0 + 2, r0 + 3};
+                    group(r, nr, acc + (r0 - (int64_t)iv.x));
+                }
+            }
+            acc += len;
+        }
     }
     if (EMIT) return;
     unsigned long long* out = a.partials + (size_t)item * k;
@@ -369,10 +393,15 @@ void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     const unsigned grid = (unsigned)((a.n_items + kSLWarps - 1) / kSLWarps);
     const int nvl = ((a.ds >> 2) + 31) / 32;
 
-#define BLSH_SL_CASE(V)                                                                         \
-    case V:                                                                                     \
-        if (a.cand_keys) k_shortlist<V, true><<<grid, kSLWarps * 32, 0, s>>>(a);                \
-        else k_shortlist<V, false><<<grid, kSLWarps * 32, 0, s>>>(a);                           \
+#define BLSH_SL_CASE(V)                                                                             \
+    case V:                                                                                         \
+        if (a.list) {                                                                               \
+            if (a.cand_keys) k_shortlist<V, true, true><<<grid, kSLWarps * 32, 0, s>>>(a);          \
+            else k_shortlist<V, false, true><<<grid, kSLWarps * 32, 0, s>>>(a);                     \
+        } else {                                                                                    \
+            if (a.cand_keys) k_shortlist<V, true, false><<<grid, kSLWarps * 32, 0, s>>>(a);         \
+            else k_shortlist<V, false, false><<<grid, kSLWarps * 32, 0, s>>>(a);                    \
+        }                                                                                           \
         break;
     switch (nvl) {
         BLSH_SL_CASE(1) BLSH_SL_CASE(2) BLSH_SL_CASE(3) BLSH_SL_CASE(4)

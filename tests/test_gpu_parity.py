@@ -208,7 +208,7 @@ def test_invalid_args(blsh, c1):
     X, Q = c1
     ix = blsh.blsh_build(torch.from_numpy(X).cuda(), n_leaves=4)
     Qd = torch.from_numpy(Q).cuda()
-    for kw, st in [(dict(k=0), blsh.BLSH_ERR_INVALID), (dict(k=65), blsh.BLSH_ERR_UNSUPPORTED),
+    for kw, st in [(dict(k=0), blsh.BLSH_ERR_INVALID), (dict(k=1025), blsh.BLSH_ERR_UNSUPPORTED),
                    (dict(k=5, probe=2, n_probes=4), blsh.BLSH_ERR_INVALID),
                    (dict(k=5, probe=0, n_probes=4), blsh.BLSH_ERR_INVALID),
                    (dict(k=5, probe=1, n_probes=300), blsh.BLSH_ERR_UNSUPPORTED)]:
