@@ -803,6 +803,8 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     if (probe == 0 && T != 1) return 1;
     if (probe == 1 && (ix->quantizer != 0 || M > 10 || T > orc_pow3(M))) return 1;
     if (probe == 2 && (ix->quantizer != 1 || T > 241)) return 1;
+    if (probe == 3 && ix->quantizer != 0) return 1;
+    if (probe < 0 || probe > 3) return 1;
     if (hierarchy && ix->quantizer != 0) return 1;
     if (min_cand < 0) return 1;
     int step = hier_step <= 0 ? M : hier_step;
@@ -850,7 +852,27 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         if (probe == 2 && T > 1 && ok) orc_lattice_order(t, code, T, ridx);
         const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
         int64_t base = 0;
-        for (int p = 0; p < T; p++) {
+        if (probe == 3) {
+            /* P:132 Morton-curve neighbours (R25): insertion position of the
+             * (clamped) home key among the leaf's sorted bucket keys, then the
+             * buckets after / before it alternately: offsets 0, -1, +1, -2, ... */
+            int64_t p0 = ix->leaf_u[g];
+            for (int64_t u = ix->leaf_u[g]; u < ix->leaf_u[g + 1]; u++)
+                if (ix->ukey[u] < hkey[q]) p0 = u + 1;
+            for (int p = 0; p < T; p++) {
+                int64_t off = (p % 2 == 1) ? -(int64_t)((p + 1) / 2) : (int64_t)(p / 2);
+                int64_t b = p0 + off;
+                int valid = b >= ix->leaf_u[g] && b < ix->leaf_u[g + 1];
+                u128 pk = valid ? ix->ukey[b] : 0;
+                ix->lq_pkey[((size_t)q * T + p) * 2] = (uint64_t)(pk >> 64);
+                ix->lq_pkey[((size_t)q * T + p) * 2 + 1] = (uint64_t)pk;
+                ix->lq_pvalid[(size_t)q * T + p] = valid;
+                bs[(size_t)q * T + p] = valid ? ix->uoff[b] : 0;
+                be[(size_t)q * T + p] = valid ? ix->uoff[b + 1] : 0;
+                base += be[(size_t)q * T + p] - bs[(size_t)q * T + p];
+            }
+        }
+        for (int p = 0; p < T && probe != 3; p++) {
             int32_t pc[16];
             int valid = 1;
             if (ix->quantizer == 0) {
