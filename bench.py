@@ -45,6 +45,12 @@ def parse():
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nq", type=int, default=None)
     ap.add_argument("--n", type=int, default=None)
+    ap.add_argument("--k", type=int, default=None)
+    ap.add_argument("--L", type=int, default=None, help="hash tables per leaf (P:43)")
+    ap.add_argument("--G", type=int, default=None)
+    ap.add_argument("--probe", type=int, default=None, help="0 standard, 1 multiprobe, 2 E8 lattice")
+    ap.add_argument("--quantizer", type=int, default=None, help="0 Z^M, 1 E8")
+    ap.add_argument("--hierarchy", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-sample-s", type=float, default=15.0, help="target seconds of oracle query work")
@@ -66,12 +72,18 @@ def load_cfg(a):
         kw["nq"] = a.nq
     if a.n is not None:
         kw["n"] = a.n
+    for f in ("k", "L", "G", "probe", "quantizer", "hierarchy"):
+        if getattr(a, f) is not None:
+            kw[f] = getattr(a, f)
     return replace(cfg, **kw) if kw else cfg
 
 
 def workload_str(cfg):
-    probe = {0: "standard", 1: f"multiprobe T={cfg.T}", 2: f"E8 lattice T={cfg.T}"}[cfg.probe]
+    probe = {0: "standard", 1: f"multiprobe T={cfg.T}", 2: f"E8 lattice T={cfg.T}",
+             3: f"Morton-curve neighbours T={cfg.T}"}[cfg.probe]
     hier = " + Morton hierarchy (tau=median)" if cfg.hierarchy else ""
+    if cfg.L > 1:
+        hier += f", L={cfg.L} tables"
     return (f"{cfg.name}: n={cfg.n} d={cfg.d} Gaussian-mixture (C={cfg.n_clusters}, spread={cfg.spread}), "
             f"{cfg.nq} queries, k={cfg.k}, RP-tree G={cfg.G}, M={cfg.M}, W={cfg.W:g}, {probe}{hier}")
 
@@ -171,6 +183,20 @@ def recall_from_gt(cfg, X, Q, ids_dev):
     """recall@10 on the committed oracle ground-truth sample (tools/make_gt.py), tie-aware (C9)."""
     import torch
     path = os.path.join(ROOT, "bench_data", f"{cfg.name}_gt.npz")
+    if not os.path.exists(path) and X.shape[0] <= 2_000_000 and ids_dev.shape[1] >= 10:
+        # no committed ground truth: exact 10-NN of a fixed 200-query sample by the oracle's fp64 brute force
+        import oracle
+        qidx = np.arange(0, Q.shape[0], max(1, Q.shape[0] // 200))[:200]
+        gi, gd = oracle.bruteforce(X.cpu().numpy(), Q[torch.as_tensor(qidx, device=Q.device)].cpu().numpy(), 10)
+        got = ids_dev[torch.as_tensor(qidx, device=ids_dev.device)][:, :10].cpu().numpy()
+        hits = 0
+        for r in range(len(qidx)):
+            gs = set(gi[r].tolist())
+            for i in got[r]:
+                if i >= 0 and (int(i) in gs or float(((X[int(i)].double() - Q[int(qidx[r])].double()) ** 2).sum())
+                               <= float(gd[r, 9]) * (1 + 1e-5)):
+                    hits += 1
+        return hits / (10.0 * len(qidx)), f"{len(qidx)} queries, oracle fp64 brute force (computed in this run)"
     if not os.path.exists(path):
         return None, "no ground-truth file"
     g = np.load(path)
@@ -224,7 +250,7 @@ def run_ours(a):
     gen_s = time.time() - t0
     t0 = time.time()
     ix = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, quantizer=cfg.quantizer,
-                         rank=rank, world=world)
+                         rank=rank, world=world, n_tables=cfg.L)
     sh = ShardedIndex(ix) if world > 1 else None
     torch.cuda.synchronize()
     build_s = time.time() - t0
@@ -352,7 +378,7 @@ def run_ours(a):
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic (seeded Gaussian mixture, torch Philox on device; synth/)",
-            "config": {"workload": wl, "n": cfg.n, "d": cfg.d, "nq": nq, "k": k, "G": cfg.G, "M": cfg.M,
+            "config": {"workload": wl, "n": cfg.n, "d": cfg.d, "nq": nq, "k": k, "G": cfg.G, "M": cfg.M, "L": cfg.L,
                        "W": cfg.W, "probe": cfg.probe, "T": cfg.T, "hierarchy": cfg.hierarchy,
                        "parallelism": f"leaf-shard{world}" if world > 1 else "single",
                        "l2": "no flush: table (%.1f GB) and query batch (%.0f MB) exceed the 126 MB L2"
@@ -379,7 +405,7 @@ def run_ours(a):
 def _oracle_index(cfg, Xh):
     import oracle
     t0 = time.time()
-    ox = oracle.OracleIndex(Xh, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, quantizer=cfg.quantizer)
+    ox = oracle.OracleIndex(Xh, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, quantizer=cfg.quantizer, L=cfg.L)
     return ox, time.time() - t0
 
 

@@ -75,7 +75,10 @@ typedef struct {
 
 /* Query parameters.  Defaults: blsh_query_params_default(). */
 typedef struct {
-    int32_t probe;          /* 0 standard (T = 1), 1 multiprobe on Z^M (R11), 2 lattice on E8 */
+    int32_t probe;          /* 0 standard (T = 1), 1 multiprobe on Z^M (R11), 2 lattice on E8,
+                               3 Morton-curve neighbours on Z^M (R25): the T buckets around the
+                               insertion position of the home key in the leaf's sorted keys (after, before,
+                               alternating)                                                                    */
     int32_t n_probes;       /* T >= 1 including the home bucket; <= 3^M (M <= 10) or <= 241 (E8)              */
     int32_t hierarchy;      /* 1 = Morton-prefix widening (Eq. 7-8, R17); Z^M index only               */
     int32_t hier_step_bits; /* key bits cleared per widening step: 0 = M (one Eq. 8 level), or 1..M           */

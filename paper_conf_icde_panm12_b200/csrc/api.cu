@@ -571,8 +571,10 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
     } else if (p->probe == 2) {
         if (idx->quantizer != 1) return fail(BLSH_ERR_INVALID, "lattice probing needs an E8 index");
         if (p->n_probes > 241) return fail(BLSH_ERR_INVALID, "n_probes > 241");
+    } else if (p->probe == 3) {
+        if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "Morton-curve probing needs a Z^M index");
     } else if (p->probe != 0) {
-        return fail(BLSH_ERR_INVALID, "probe must be 0, 1 or 2");
+        return fail(BLSH_ERR_INVALID, "probe must be 0, 1, 2 or 3");
     }
     if (p->n_probes > 256) return fail(BLSH_ERR_UNSUPPORTED, "n_probes > 256");
     if (p->hierarchy) {

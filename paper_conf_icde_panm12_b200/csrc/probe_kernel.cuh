@@ -236,6 +236,47 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
     return mysum;
 }
 
+// probe = 3, Morton-curve neighbours ("search within the Morton curve to
+// find the position where the query code can be inserted without violating the
+// ordering ... use the Morton codes before and after the insert position ...
+// to refer the buckets").  Reading R25: p = the insertion position of the
+// query's clamped home key among its leaf's sorted bucket keys (lower bound);
+// probe j takes bucket p + o_j with o = 0, -1, +1, -2, +2, ... (after, before,
+// alternating: T = 2 is exactly "before and after"; when the key is present,
+// bucket p is its home bucket); offsets outside the leaf are empty probes that
+// count toward T.  Every probe is one whole bucket, so the intervals are
+// disjoint (and the hierarchy's containment rule applies unchanged).
+__device__ int64_t probe_curve(const QueryArgs& a, int64_t q, int lane, int64_t ulo, int64_t uhi, uint2* ivl) {
+    const int T = a.T;
+    const Key128 k = a.qkey[q];
+    int64_t lo = ulo, hi = uhi;
+    while (lo < hi) {   // every lane runs the same search (keys L1/L2-resident)
+        const int64_t mid = (lo + hi) >> 1;
+        if (key_lt(a.ukey[mid], k)) lo = mid + 1;
+        else hi = mid;
+    }
+    const int64_t p0 = lo;
+    int64_t mysum = 0;
+    for (int p = lane; p < T; p += 32) {
+        const int64_t off = (p & 1) ? -(int64_t)((p + 1) >> 1) : (int64_t)(p >> 1);
+        const int64_t b = p0 + off;
+        const bool valid = b >= ulo && b < uhi;
+        uint2 iv = make_uint2(0, 0);
+        Key128 kb{0, 0};
+        if (valid) {
+            iv = make_uint2(a.uoff[b], a.uoff[b + 1]);
+            kb = a.ukey[b];
+        }
+        ivl[p] = iv;
+        mysum += (int64_t)(iv.y - iv.x);
+        if (a.pkey) {
+            a.pkey[(size_t)q * T + p] = kb;
+            a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
+        }
+    }
+    return mysum;
+}
+
 __global__ void __launch_bounds__(kPW * 32, 4) k_probe_lookup(QueryArgs a) {
     __shared__ ProbeSmem smem[kPW];
     const int lane = threadIdx.x & 31;
@@ -256,7 +297,9 @@ __global__ void __launch_bounds__(kPW * 32, 4) k_probe_lookup(QueryArgs a) {
     const int g = a.qleaf[q];
     const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
     int64_t mysum = 0;
-    if (a.quantizer == 1) {
+    if (a.probe == 3) {
+        mysum = probe_curve(a, q, lane, ulo, uhi, ivl);
+    } else if (a.quantizer == 1) {
         mysum = probe_e8(a, sm, q, lane, oor, ulo, uhi, ivl);
     } else {
         switch (a.M) {

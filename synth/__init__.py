@@ -54,6 +54,7 @@ class Config:
     hierarchy: int = 0
     min_cand: int = 0
     quantizer: int = 0        # 0 Z^M floor, 1 E8
+    L: int = 1                # hash tables per leaf
     zipf: float = 0.0
     between: float = 0.0
     backend: str = "numpy"
@@ -85,6 +86,13 @@ CONFIGS = {
                  k=10, G=16, M=8, W=1.2, probe=1, T=16, backend="torch",
                  seed_data=1005, seed_query=2005,
                  notes="BASELINE configs[4]: sweep base (probes 1-64, lattice vs multiprobe, batch)"),
+    # The paper's own evaluation setting: 100,000 items hashed, another
+    # 100,000 items of the same distribution as queries, L = 10 tables, M = 8,
+    # k = 500 (Tiny-Images-shaped 384-d data).
+    "p217": Config("p217", n=100_000, d=384, n_clusters=64, spread=0.02, rank=16, nq=100_000,
+                   k=500, G=16, M=8, W=1.2, probe=0, T=1, L=10, backend="torch",
+                   seed_data=1006, seed_query=2006,
+                   notes="P:217 evaluation setting: L = 10, M = 8, k = 500, 100k items / 100k queries"),
 }
 
 
