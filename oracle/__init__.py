@@ -78,6 +78,8 @@ def lib():
         L.orc_free.argtypes = [P]
         L.orc_query.restype = i32
         L.orc_query.argtypes = [P, P, i64, i32, i32, i32, i32, i32, i64, P, P, P]
+        L.orc_e8_parent.restype = None
+        L.orc_e8_parent.argtypes = [P, P]
         L.orc_query_union.restype = i32
         L.orc_query_union.argtypes = [P, i32, P, i64, i32, i32, i32, P, P, P]
         L.orc_gen_table_params.restype = None
@@ -182,6 +184,14 @@ def e8_decode(y) -> np.ndarray:
     y = _f32(y)
     out = np.empty(8, np.int32)
     lib().orc_e8_decode(_p(y), _p(out))
+    return out
+
+
+def e8_parent(c2) -> np.ndarray:
+    """Parent code in the E8 hierarchy (Eq. 10, R27), doubled coordinates: DECODE(c2 / 4)."""
+    c = np.ascontiguousarray(c2, dtype=np.int32)
+    out = np.empty(8, np.int32)
+    lib().orc_e8_parent(_p(c), _p(out))
     return out
 
 

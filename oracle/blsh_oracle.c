@@ -32,6 +32,8 @@
 
 typedef unsigned __int128 u128;
 
+#define ORC_E8_LEVELS 32   /* levels of the E8 code hierarchy searched (R27) */
+
 /* ------------------------------------------------------------------------ */
 /* R2: counter-based SplitMix64 generator.  P:43 draws a_i ~ N(0,1) and       */
 /* b_i ~ U[0,W); P:98 draws a random unit direction per RP-tree node.  The   */
@@ -250,6 +252,17 @@ void orc_e8_decode(const float *y, int32_t *c2)
     double d0 = orc_e8_dist2(y, a), d1 = orc_e8_dist2(y, b);
     if (d1 < d0) memcpy(c2, b, sizeof b);              /* ties -> integer coset */
     else memcpy(c2, a, sizeof a);
+}
+
+/* E8 hierarchy (Eq. 10; reading R27): the parent of an E8 code is
+ * DECODE of half of it, so in doubled coordinates c = 2p the parent code is
+ * DECODE(c / 4) (exact in fp32 for |c| < 2^24).  Level-j code of a bucket or
+ * query = the parent applied j times to its level-0 code. */
+void orc_e8_parent(const int32_t *c2, int32_t *out)
+{
+    float y[8];
+    for (int i = 0; i < 8; i++) y[i] = (float)c2[i] * 0.25f;
+    orc_e8_decode(y, out);
 }
 
 /* The 240 minimal vectors of E8 in canonical order (R15), doubled coords. */
@@ -805,7 +818,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     if (probe == 2 && (ix->quantizer != 1 || T > 241)) return 1;
     if (probe == 3 && ix->quantizer != 0) return 1;
     if (probe < 0 || probe > 3) return 1;
-    if (hierarchy && ix->quantizer != 0) return 1;
+    /* hierarchy: Morton prefixes on Z^M (R17), the Eq. 10 code hierarchy on E8 (R27) */
     if (min_cand < 0) return 1;
     int step = hier_step <= 0 ? M : hier_step;
     if (step > M) return 1;
@@ -827,6 +840,8 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     int64_t *be = (int64_t *)malloc(sizeof(int64_t) * nqs * T);
     int64_t *hs = (int64_t *)calloc(nqs, sizeof(int64_t));        /* hierarchy range */
     int64_t *he = (int64_t *)calloc(nqs, sizeof(int64_t));
+    int64_t **hbk = (int64_t **)calloc(nqs, sizeof(int64_t *));   /* E8 hierarchy: node buckets */
+    int64_t *nhbk = (int64_t *)calloc(nqs, sizeof(int64_t));
     u128 *hkey = (u128 *)calloc(nqs, sizeof(u128));
     int32_t roots[240 * 8];
     orc_e8_roots(roots);
@@ -913,8 +928,63 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     }
     ix->lq_tau = hierarchy ? tau : 0;
 
+    /* E8 hierarchy (R27): a node at level j = the leaf's buckets whose
+     * level-j code equals the query's; matches are closed upwards (the level-j+1
+     * code is a function of the level-j code).  The traversal descends from the
+     * root (level m_g: the first level where all the leaf's buckets share one
+     * code, <= ORC_E8_LEVELS) to the deepest node matching the query,
+     * and P:249 widens from there until the node holds >= tau points: the first
+     * level j <= m_g with a match and |node| >= tau; otherwise the whole leaf. */
+    if (hierarchy && ix->quantizer == 1) {
+        #pragma omp parallel for schedule(dynamic, 4)
+        for (int64_t q = 0; q < nq; q++) {
+            if (ix->lq_base[q] >= tau) continue;
+            int g = ix->lq_leaf[q];
+            int64_t u0 = ix->leaf_u[g], nb = ix->leaf_u[g + 1] - u0;
+            int32_t *cur = (int32_t *)malloc(sizeof(int32_t) * 8 * (size_t)(nb > 0 ? nb : 1));
+            int32_t cq[8], tmp[8];
+            memcpy(cq, ix->lq_code + q * 8, sizeof(cq));
+            for (int64_t b = 0; b < nb; b++)
+                memcpy(cur + 8 * b, ix->code + 8 * ix->perm[ix->uoff[u0 + b]], sizeof(int32_t) * 8);
+            int level = ORC_E8_LEVELS + 1;      /* whole leaf */
+            for (int jl = 0; jl <= ORC_E8_LEVELS && nb > 0; jl++) {
+                int64_t rows = 0, match = 0;
+                int same = 1;
+                for (int64_t b = 0; b < nb; b++) {
+                    if (memcmp(cur + 8 * b, cq, sizeof(cq)) == 0) {
+                        match++;
+                        rows += ix->uoff[u0 + b + 1] - ix->uoff[u0 + b];
+                    }
+                    if (memcmp(cur + 8 * b, cur, sizeof(cq)) != 0) same = 0;
+                }
+                if (match && rows >= tau) { level = jl; break; }
+                if (same) break;                 /* root reached without a large enough match */
+                for (int64_t b = 0; b < nb; b++) {
+                    orc_e8_parent(cur + 8 * b, tmp);
+                    memcpy(cur + 8 * b, tmp, sizeof(tmp));
+                }
+                orc_e8_parent(cq, tmp);
+                memcpy(cq, tmp, sizeof(cq));
+            }
+            /* node buckets */
+            int64_t *lst = (int64_t *)malloc(sizeof(int64_t) * (size_t)(nb > 0 ? nb : 1));
+            int64_t m = 0;
+            if (level > ORC_E8_LEVELS) {
+                for (int64_t b = 0; b < nb; b++) lst[m++] = u0 + b;
+            } else {
+                /* recompute the level-`level` codes (cur holds them after the loop broke there) */
+                for (int64_t b = 0; b < nb; b++)
+                    if (memcmp(cur + 8 * b, cq, sizeof(cq)) == 0) lst[m++] = u0 + b;
+            }
+            hbk[q] = lst;
+            nhbk[q] = m;
+            ix->lq_level[q] = level;
+            free(cur);
+        }
+    }
+
     /* hierarchy: widen along Morton prefixes until |R| >= tau (Eq. 8) */
-    if (hierarchy) {
+    if (hierarchy && ix->quantizer == 0) {
         const int BM = B * M;
         #pragma omp parallel for schedule(dynamic, 16)
         for (int64_t q = 0; q < nq; q++) {
@@ -946,11 +1016,15 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     #pragma omp parallel for schedule(dynamic, 16)
     for (int64_t q = 0; q < nq; q++) {
         int64_t cap = ix->lq_base[q] + (he[q] - hs[q]);
+        for (int64_t b = 0; b < nhbk[q]; b++) cap += ix->uoff[hbk[q][b] + 1] - ix->uoff[hbk[q][b]];
         int64_t *pos = (int64_t *)malloc(sizeof(int64_t) * (size_t)(cap > 0 ? cap : 1));
         int64_t np = 0;
         for (int p = 0; p < T; p++)
             for (int64_t i = bs[(size_t)q * T + p]; i < be[(size_t)q * T + p]; i++) pos[np++] = i;
         for (int64_t i = hs[q]; i < he[q]; i++) pos[np++] = i;
+        for (int64_t b = 0; b < nhbk[q]; b++)
+            for (int64_t i = ix->uoff[hbk[q][b]]; i < ix->uoff[hbk[q][b] + 1]; i++) pos[np++] = i;
+        free(hbk[q]);
         qsort(pos, (size_t)np, sizeof(int64_t), orc_cmp_i64);
         int64_t m = 0;
         for (int64_t i = 0; i < np; i++) if (m == 0 || pos[i] != pos[m - 1]) pos[m++] = pos[i];
@@ -971,7 +1045,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         memcpy(ix->lq_cand + ix->lq_coff[q], cand[q], sizeof(int64_t) * (size_t)ncand[q]);
         free(cand[q]);
     }
-    free(cand); free(ncand); free(bs); free(be); free(hs); free(he); free(hkey);
+    free(cand); free(ncand); free(bs); free(be); free(hs); free(he); free(hkey); free(hbk); free(nhbk);
     return 0;
 }
 

@@ -1,0 +1,103 @@
+"""Oracle pins for the E8 code hierarchy (Eq. 10; reading R27):
+parent(c) = DECODE(c / 2) in lattice units (doubled codes: DECODE(c2 / 4));
+P:162 scaling property (the parent of 2p is p for every lattice point p);
+the parent is a nearest lattice point of c / 2 (Voronoi test against the 240
+roots); the widening rule of P:171 + P:249 on an E8 index."""
+import numpy as np
+import pytest
+
+import synth
+
+
+def _random_e8(rng, n, scale=6):
+    """Random E8 points in doubled coordinates (D8 or D8 + 1/2)."""
+    out = []
+    while len(out) < n:
+        z = rng.integers(-scale, scale + 1, 8)
+        if rng.random() < 0.5:
+            if z.sum() % 2:
+                z[0] += 1
+            out.append(2 * z)
+        else:
+            h = 2 * z + 1                      # odd doubled coordinates = half-integers
+            if (h.sum() // 2) % 2:             # sum of the half-integer coordinates must be even
+                h[0] += 2
+            out.append(h)
+    return np.array(out, np.int32)
+
+
+def _is_e8(c2):
+    c2 = np.asarray(c2)
+    if np.all(c2 % 2 == 0):
+        return (c2 // 2).sum() % 2 == 0
+    if np.all(c2 % 2 != 0):
+        return (c2.sum() // 2) % 2 == 0
+    return False
+
+
+def test_scaling_property(orc):
+    """the integer scaling of E8 is E8, so the parent of the code of 2p is p."""
+    rng = np.random.default_rng(1)
+    for c in _random_e8(rng, 300):
+        assert _is_e8(c)
+        assert np.array_equal(orc.e8_parent(2 * c), c)
+
+
+def test_parent_is_nearest(orc):
+    rng = np.random.default_rng(2)
+    roots = orc.e8_roots().astype(np.float64) / 2.0
+    for c in _random_e8(rng, 300, scale=40):
+        par = orc.e8_parent(c)
+        assert _is_e8(par)
+        y = c.astype(np.float64) / 4.0        # half of the lattice point c / 2
+        x = par.astype(np.float64) / 2.0
+        d0 = ((y - x) ** 2).sum()
+        d = ((y[None, :] - x[None, :] - roots) ** 2).sum(1)
+        assert d0 <= d.min() + 1e-12
+        # chains shrink to the origin's neighbourhood: |parent| <= |c| / 2 + covering radius
+        assert np.sqrt((x ** 2).sum()) <= np.sqrt(((c / 2.0) ** 2).sum()) / 2 + 1.0 + 1e-9
+
+
+def _chain(orc, c, j):
+    for _ in range(j):
+        c = orc.e8_parent(c)
+    return c
+
+
+@pytest.mark.parametrize("tau", [0, 400, 2000])
+def test_e8_hierarchy_widening_rule(orc, tau):
+    X, Q = synth.make_dataset(synth.CONFIGS["c1"])
+    Q = Q[:30]
+    ix = orc.OracleIndex(X, G=4, M=8, W=2.0, seed=42, quantizer=1)
+    ix.query(Q, 10, probe=2, T=4, hierarchy=1, min_cand=tau)
+    tau_used = ix.tau
+    base, lvl, ql, code = ix.get("q_base"), ix.get("q_level"), ix.get("q_leaf"), ix.get("q_code")
+    uleaf, uoff, perm, pcode = ix.get("uleaf"), ix.get("uoff"), ix.get("perm"), ix.get("code")
+    cands = ix.candidates()
+    full = orc.OracleIndex(X, G=4, M=8, W=2.0, seed=42, quantizer=1)
+    full.query(Q, 10, probe=2, T=4)
+    a0 = full.candidates()
+    for q in range(len(Q)):
+        if base[q] >= tau_used:
+            assert lvl[q] == 0 and np.array_equal(cands[q], a0[q])
+            continue
+        bks = np.nonzero(uleaf == ql[q])[0]
+        bcode = [pcode[perm[uoff[u]]] for u in bks]
+        if lvl[q] > 32:                      # whole leaf
+            want = set(np.nonzero(ix.get("leaf") == ql[q])[0].tolist())
+        else:
+            L = int(lvl[q])
+            cq = _chain(orc, code[q], L)
+            node = [u for u, c in zip(bks, bcode) if np.array_equal(_chain(orc, c, L), cq)]
+            rows = sum(int(uoff[u + 1] - uoff[u]) for u in node)
+            assert node and rows >= tau_used
+            if L > 0:                        # the level below is not enough (no match or too small)
+                cq1 = _chain(orc, code[q], L - 1)
+                node1 = [u for u, c in zip(bks, bcode) if np.array_equal(_chain(orc, c, L - 1), cq1)]
+                assert set(node1) <= set(node)
+                assert sum(int(uoff[u + 1] - uoff[u]) for u in node1) < tau_used
+            want = set()
+            for u in node:
+                want |= set(perm[uoff[u]:uoff[u + 1]].tolist())
+        want |= set(a0[q].tolist())
+        assert set(cands[q].tolist()) == want
