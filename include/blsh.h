@@ -173,7 +173,9 @@ typedef enum {
     BLSH_EX_Q_BASE = 37,    /* int64 [nq]       |A0| before widening                          */
     BLSH_EX_Q_LEVEL = 38,   /* int32 [nq]       key bits cleared by the hierarchy (0 = none)  */
     BLSH_EX_Q_TAU = 39,     /* int64 [1]        threshold used                                */
-    BLSH_EX_Q_INTERVALS = 40/* int64 [nq][T+1][2] candidate intervals [start, end) in table positions */
+    BLSH_EX_Q_INTERVALS = 40,/* int64 [nq][T+1][2] candidate intervals [start, end) in table positions */
+    BLSH_EX_Q_CAND_OFF = 41,/* int64 [nq+1]     list path (L > 1 or E8 hierarchy): offsets into Q_CAND      */
+    BLSH_EX_Q_CAND = 42     /* int64 [sum|A(q)|] list path: candidate ids of every query, ascending           */
 } blsh_export_what;
 /* Table l of an L-table index (n_tables > 1): what = BLSH_EX_TABLE(l, item) for
  * the per-table items A, B, PERM (original ids in table-l order), UKEY, ULEAF,

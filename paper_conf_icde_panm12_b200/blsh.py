@@ -22,7 +22,8 @@ _STATUS = {0: "OK", 1: "INVALID", 2: "OOM", 3: "CUDA", 4: "RANGE", 5: "UNSUPPORT
 
 EX = dict(A=0, B=1, W=2, DIRS=3, MU=4, THETA=5, NTYPE=6, DIAM2=7, DA2=8, PERM=10, UKEY=11, ULEAF=12,
           UOFF=13, LEAF_U=14, POINT_LEAF=20, POINT_CODE=21, POINT_KEY=22, Q_LEAF=30, Q_T=31, Q_CODE=32,
-          Q_OOR=33, Q_KEY=34, Q_PKEY=35, Q_PVALID=36, Q_BASE=37, Q_LEVEL=38, Q_TAU=39, Q_INTERVALS=40)
+          Q_OOR=33, Q_KEY=34, Q_PKEY=35, Q_PVALID=36, Q_BASE=37, Q_LEVEL=38, Q_TAU=39, Q_INTERVALS=40,
+          Q_CAND_OFF=41, Q_CAND=42)
 
 
 class BuildParams(C.Structure):
@@ -265,7 +266,7 @@ _EX_DT = {"A": np.float32, "B": np.float32, "W": np.float32, "DIRS": np.float32,
           "POINT_CODE": np.int32, "POINT_KEY": np.uint64, "Q_LEAF": np.int32, "Q_T": np.float32,
           "Q_CODE": np.int32, "Q_OOR": np.int32, "Q_KEY": np.uint64, "Q_PKEY": np.uint64,
           "Q_PVALID": np.int32, "Q_BASE": np.int64, "Q_LEVEL": np.int32, "Q_TAU": np.int64,
-          "Q_INTERVALS": np.int64}
+          "Q_INTERVALS": np.int64, "Q_CAND_OFF": np.int64, "Q_CAND": np.int64}
 
 
 def blsh_export(index: "Index", what: str, table: int = 0) -> np.ndarray:

@@ -244,6 +244,8 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         ix->leaf_pos.alloc((G + 1) * sizeof(int64_t));
         BLSH_CUDA(cudaMemcpyAsync(ix->leaf_pos.p, ix->leaf_pos_h.data(), (G + 1) * sizeof(int64_t),
                                   cudaMemcpyHostToDevice, s));
+        // E8 index: the code hierarchy of P:162-173 over the primary table's buckets
+        if (ix->quantizer == 1) blsh::build_e8_hierarchy(*ix, s);
         // tables 1..L-1: own (a, b), same tree and rows
         ix->L = p->n_tables;
         std::vector<const uint32_t*> tab_pos(ix->L, nullptr);
@@ -322,7 +324,10 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         add((size_t)nq * (T + 1), 8); add(nq, 8); add(nq, 8);
         if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
     }
-    if (L > 1) { add(nq + 1, 8); add(nq, 8); add(L, 8); add(L, 8); }
+    const bool e8h = p.hierarchy && ix.quantizer == 1;   // E8 code hierarchy
+    const bool list_path = L > 1 || e8h;                   // candidates as deduplicated position lists
+    if (list_path) { add(nq + 1, 8); add(nq, 8); add(L, 8); add(L, 8); }
+    if (e8h) { add(nq, 8); add(nq, 8); add(nq, 8); }
     if (out_host) { add((size_t)nq * k, 8); add((size_t)nq * k, 4); add(nq, 8); add((size_t)nq * k, 8); }
     w.arena.ensure(need);
     Arena ar{w.arena.as<char>(), 0, w.arena.bytes};
@@ -362,11 +367,17 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t* raw = nullptr;
     const uint2** ivl_ptrs = nullptr;
     const int64_t** cnt_ptrs = nullptr;
-    if (L > 1) {
+    if (list_path) {
         w.raw_off = ar.take<int64_t>(nq + 1);
         raw = ar.take<int64_t>(nq);
         ivl_ptrs = ar.take<const uint2*>(L);
         cnt_ptrs = ar.take<const int64_t*>(L);
+    }
+    int64_t *h_s = nullptr, *h_e = nullptr, *h_rows = nullptr;
+    if (e8h) {
+        h_s = ar.take<int64_t>(nq);
+        h_e = ar.take<int64_t>(nq);
+        h_rows = ar.take<int64_t>(nq);
     }
     int64_t* d_ids = out_ids;
     float* d_d2 = out_d2;
@@ -418,25 +429,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     // a3+a4
     launch_probe_lookup(a, s); ++launches;
     for (int l = 1; l < L; ++l) { launch_probe_lookup(table_args(l), s); ++launches; }
-    int64_t total_raw = 0;
-    if (L > 1) {   // a4 across tables: deduplicated union of the L tables' buckets (R24)
-        std::vector<const uint2*> iv(L);
-        std::vector<const int64_t*> cn(L);
-        for (int l = 0; l < L; ++l) { iv[l] = w.tq[l].ivl; cn[l] = w.tq[l].cnt; }
-        BLSH_CUDA(cudaMemcpyAsync(ivl_ptrs, iv.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
-        BLSH_CUDA(cudaMemcpyAsync(cnt_ptrs, cn.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
-        UnionArgs u{};
-        u.nq = nq; u.L = L; u.T = T; u.qleaf = w.qleaf; u.qoor = w.qoor; u.ivl = ivl_ptrs; u.cnt = cnt_ptrs;
-        u.pos = ix.tab_pos.as<const uint32_t*>(); u.leaf_pos = ix.leaf_pos.as<int64_t>();
-        u.raw_off = w.raw_off; u.raw = raw; u.out_cnt = w.cnt;
-        launch_raw_counts(u, s); ++launches;
-        scan_exclusive_i64(raw, w.raw_off, nq, w.scan, s); launches += 3;
-        BLSH_CUDA(cudaMemcpyAsync(&total_raw, w.raw_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        BLSH_CUDA(cudaStreamSynchronize(s));
-        w.listbuf.ensure((size_t)std::max<int64_t>(total_raw, 1) * sizeof(uint32_t));
-        u.list = w.listbuf.as<uint32_t>();
-        launch_union_tables(u, ix.max_leaf_rows, s); ++launches;
-    }
+
     if (out_base) {   // blsh_query_base_counts: a1-a4 only
         BLSH_CUDA(cudaMemcpyAsync(out_base, w.base, (size_t)nq * 8, out_host ? cudaMemcpyDeviceToHost
                                                                               : cudaMemcpyDeviceToDevice, s));
@@ -456,15 +449,51 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
             launch_median(p.global_base ? p.global_base : w.base, nq, w.tau, s);
             ++launches;
         }
-        launch_widen(a, w.tau, p.min_cand, s); ++launches;
+        if (e8h) {
+            E8WidenArgs ew{};
+            ew.nq = nq; ew.B = ix.B; ew.qleaf = w.qleaf; ew.qoor = w.qoor; ew.qcode = w.qcode; ew.base = w.base;
+            ew.ukey = ix.ukey.as<Key128>(); ew.uoff = ix.uoff.as<uint32_t>(); ew.leaf_u = ix.leaf_u.as<int64_t>();
+            ew.root = ix.e8_root.as<int32_t>();
+            ew.lv_key = reinterpret_cast<const Key128* const*>(ix.e8_ptrs.as<char>());
+            ew.lv_cum = reinterpret_cast<const int64_t* const*>(ix.e8_ptrs.as<char>() + 2 * (kE8Levels + 1) * sizeof(void*));
+            ew.hlevel = w.level; ew.hs = h_s; ew.he = h_e; ew.hrows = h_rows;
+            launch_e8_widen(ew, w.tau, p.min_cand, s); ++launches;
+        } else {
+            launch_widen(a, w.tau, p.min_cand, s); ++launches;
+        }
     }
+    int64_t total_raw = 0;
+    if (list_path) {   // a4 across tables / with the E8 node: deduplicated union (R24, R27)
+        std::vector<const uint2*> iv(L);
+        std::vector<const int64_t*> cn(L);
+        for (int l = 0; l < L; ++l) { iv[l] = w.tq[l].ivl; cn[l] = w.tq[l].cnt; }
+        BLSH_CUDA(cudaMemcpyAsync(ivl_ptrs, iv.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
+        BLSH_CUDA(cudaMemcpyAsync(cnt_ptrs, cn.data(), L * sizeof(void*), cudaMemcpyHostToDevice, s));
+        UnionArgs u{};
+        u.nq = nq; u.L = L; u.T = T; u.qleaf = w.qleaf; u.qoor = w.qoor; u.ivl = ivl_ptrs; u.cnt = cnt_ptrs;
+        u.pos = ix.tab_pos.as<const uint32_t*>(); u.leaf_pos = ix.leaf_pos.as<int64_t>();
+        u.raw_off = w.raw_off; u.raw = raw; u.out_cnt = w.cnt;
+        if (e8h) {
+            u.hlevel = w.level; u.hs = h_s; u.he = h_e; u.hrows = h_rows;
+            u.lv_bu = reinterpret_cast<const uint32_t* const*>(ix.e8_ptrs.as<char>() + (kE8Levels + 1) * sizeof(void*));
+            u.uoff = ix.uoff.as<uint32_t>();
+        }
+        launch_raw_counts(u, s); ++launches;
+        scan_exclusive_i64(raw, w.raw_off, nq, w.scan, s); launches += 3;
+        BLSH_CUDA(cudaMemcpyAsync(&total_raw, w.raw_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        w.listbuf.ensure((size_t)std::max<int64_t>(total_raw, 1) * sizeof(uint32_t));
+        u.list = w.listbuf.as<uint32_t>();
+        launch_union_tables(u, ix.max_leaf_rows, s); ++launches;
+    }
+    w.list_valid = list_path;
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[3], s));
     // plan: chunking of the candidate lists
     scan_exclusive_i64(w.cnt, cand_off, nq, w.scan, s); launches += 3;
     int64_t total = 0;
     BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    const int kind = L > 1 ? 0 : shortlist_kind(ds, T, k);   // L > 1: warp short-list over the position lists
+    const int kind = list_path ? 0 : shortlist_kind(ds, T, k);   // lists: warp short-list over the positions
     const bool tiled = kind > 0;
     int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0;
     double qload_rows = 0.0;
@@ -498,8 +527,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
         sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
         sa.cand_off = cand_off;
-        sa.list = L > 1 ? w.listbuf.as<uint32_t>() : nullptr;
-        sa.list_off = L > 1 ? w.raw_off : nullptr;
+        sa.list = list_path ? w.listbuf.as<uint32_t>() : nullptr;
+        sa.list_off = list_path ? w.raw_off : nullptr;
         sa.cand_keys = large_k ? w.partials.as<unsigned long long>() : nullptr;
         launch_shortlist(sa, s); if (n_items) ++launches;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
@@ -579,7 +608,6 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
     if (p->n_probes > 256) return fail(BLSH_ERR_UNSUPPORTED, "n_probes > 256");
     if (p->hierarchy) {
         if (idx->L > 1) return fail(BLSH_ERR_UNSUPPORTED, "the Morton hierarchy is defined for one table (R24)");
-        if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "the Morton hierarchy needs a Z^M index");
         if (p->hier_step_bits < 0 || p->hier_step_bits > idx->M) return fail(BLSH_ERR_INVALID, "hier_step_bits must be in [0, M]");
         if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");
         if (p->min_cand == 0 && idx->world > 1 && !p->global_base)
@@ -803,6 +831,35 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
         }
         default: break;
+    }
+    if (what == BLSH_EX_Q_CAND_OFF || what == BLSH_EX_Q_CAND) {
+        if (!need_q() || !w.list_valid) return fail(BLSH_ERR_INVALID, "last query without keep_stages or without lists");
+        std::vector<int64_t> roff(nq + 1), cnt(nq);
+        if (cudaMemcpy(roff.data(), w.raw_off, (nq + 1) * 8, cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(cnt.data(), w.cnt, nq * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+            return fail(BLSH_ERR_CUDA, "export copy failed");
+        int64_t tot = 0;
+        for (int64_t q = 0; q < nq; ++q) tot += cnt[q];
+        bytes = what == BLSH_EX_Q_CAND_OFF ? (size_t)(nq + 1) * 8 : (size_t)tot * 8;
+        if (needed) *needed = bytes;
+        if (!dst || cap < bytes) return fail(BLSH_ERR_INVALID, "dst too small");
+        int64_t* o = (int64_t*)dst;
+        if (what == BLSH_EX_Q_CAND_OFF) {
+            o[0] = 0;
+            for (int64_t q = 0; q < nq; ++q) o[q + 1] = o[q] + cnt[q];
+            return BLSH_OK;
+        }
+        std::vector<uint32_t> lst((size_t)std::max<int64_t>(roff[nq], 1)), p32((size_t)std::max<int64_t>(idx->n_owned, 1));
+        if (cudaMemcpy(lst.data(), w.listbuf.p, (size_t)roff[nq] * 4, cudaMemcpyDeviceToHost) != cudaSuccess ||
+            cudaMemcpy(p32.data(), idx->perm.p, (size_t)idx->n_owned * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+            return fail(BLSH_ERR_CUDA, "export copy failed");
+        int64_t k = 0;
+        for (int64_t q = 0; q < nq; ++q) {
+            const int64_t s0 = k;
+            for (int64_t i = 0; i < cnt[q]; ++i) o[k++] = p32[lst[roff[q] + i]];
+            std::sort(o + s0, o + k);
+        }
+        return BLSH_OK;
     }
     if (what >= BLSH_EX_Q_LEAF && what <= BLSH_EX_Q_INTERVALS) {
         if (!need_q()) return fail(BLSH_ERR_INVALID, "last query without keep_stages");

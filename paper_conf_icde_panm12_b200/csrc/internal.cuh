@@ -122,6 +122,7 @@ struct QueryWork {
     std::vector<TableQuery> tq;
     DevBuf listbuf;               // deduplicated candidate positions (u32), at raw_off[q]
     int64_t* raw_off = nullptr;   // [nq+1] scan of the per-query sums of the table counts
+    bool list_valid = false;      // the last query built candidate lists (listbuf / raw_off / cnt)
 };
 
 // Hash table l >= 1 of an L-table index.  Table 0 is the primary
@@ -172,6 +173,12 @@ struct blsh_index {
     blsh::DevBuf leaf_pos;             // device copy
     blsh::DevBuf tab_pos;              // [L] const uint32_t* (pos of table l; [0] = NULL)
     int64_t max_leaf_rows = 0;         // largest owned leaf
+    // E8 code hierarchy (E8 index): levels 1..e8_levels (e8hier.cu)
+    int e8_levels = 0;
+    std::vector<std::unique_ptr<blsh::DevBuf>> e8_key, e8_bu, e8_cum;
+    std::vector<int32_t> e8_root_h;
+    blsh::DevBuf e8_root;              // [G]
+    blsh::DevBuf e8_ptrs;              // device pointer tables: keys, buckets, cum
     // kept build stages (keep_stages)
     blsh::DevBuf pt_leaf, pt_code, pt_key;
     bool has_pt = false;
@@ -216,6 +223,8 @@ void build_extra_table(const blsh_index& ix, ExtraTable& t, const unsigned long 
                        const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
                        const uint32_t* inv0, int64_t n_owned, ScanTemp& scan, cudaStream_t s);
 void invert_perm(const uint32_t* perm, int64_t n_owned, uint32_t* inv, cudaStream_t s);
+// E8 index: the code hierarchy over the primary table's buckets (e8hier.cu).
+void build_e8_hierarchy(blsh_index& ix, cudaStream_t s);
 
 // ---- query (query.cu, shortlist.cu) ----------------------------------------------
 void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,

@@ -62,7 +62,36 @@ struct UnionArgs {
     int64_t* raw;                 // [nq]
     uint32_t* list;               // [raw_off[nq]]
     int64_t* out_cnt;             // [nq] |A(q)|
+    // E8 hierarchy node (NULL hlevel: none): buckets [hs, he) of level hlevel's order
+    const int32_t* hlevel;
+    const int64_t* hs;
+    const int64_t* he;
+    const int64_t* hrows;
+    const uint32_t* const* lv_bu; // [kE8Levels + 1] bucket of each position of level j's order
+    const uint32_t* uoff;         // bucket row offsets (primary table)
 };
+
+// E8 code hierarchy (e8hier.cu, R27)
+constexpr int kE8Levels = 32;
+struct E8WidenArgs {
+    int64_t nq;
+    int B;
+    const int32_t* qleaf;
+    const int32_t* qoor;
+    const int32_t* qcode;         // [nq][8] doubled home codes
+    const int64_t* base;          // |A0(q)|
+    const Key128* ukey;           // level 0 keys (the table)
+    const uint32_t* uoff;
+    const int64_t* leaf_u;
+    const int32_t* root;          // [G] first level at which a leaf's buckets share one code
+    const Key128* const* lv_key;  // [kE8Levels + 1]
+    const int64_t* const* lv_cum; // [kE8Levels + 1] running rows of level j's order
+    int32_t* hlevel;              // out: level (kE8Levels + 1 = whole leaf; 0 = not widened)
+    int64_t* hs;
+    int64_t* he;
+    int64_t* hrows;
+};
+void launch_e8_widen(const E8WidenArgs& w, const int64_t* tau, int64_t min_cand, cudaStream_t s);
 void launch_raw_counts(const UnionArgs& u, cudaStream_t s);
 void launch_union_tables(const UnionArgs& u, int64_t max_leaf_rows, cudaStream_t s);
 void launch_median(const int64_t* base, int64_t nq, int64_t* tau, cudaStream_t s);

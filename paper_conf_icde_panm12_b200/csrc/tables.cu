@@ -27,6 +27,7 @@ __global__ void k_raw_counts(UnionArgs u) {
     if (q >= u.nq) return;
     int64_t r = 0;
     for (int l = 0; l < u.L; ++l) r += u.cnt[l][q];
+    if (u.hrows) r += u.hrows[q];
     u.raw[q] = r;
 }
 
@@ -53,6 +54,17 @@ __global__ void __launch_bounds__(kUT) k_union_tables(UnionArgs u) {
             const uint2 r = iv[p];
             for (int64_t j = (int64_t)r.x + tid; j < (int64_t)r.y; j += kUT) {
                 const int64_t x = (pos ? (int64_t)__ldg(pos + j) : j) - lb;
+                atomicOr(&bm[x >> 5], 1u << (x & 31));
+            }
+        }
+    }
+    if (u.hlevel && u.he[q] > u.hs[q]) {   // E8 hierarchy node: its buckets' rows
+        const int lv = u.hlevel[q];
+        const uint32_t* bu = (lv >= 1 && lv <= kE8Levels) ? u.lv_bu[lv] : nullptr;
+        for (int64_t b = u.hs[q] + tid; b < u.he[q]; b += kUT) {
+            const uint32_t bk = bu ? bu[b] : (uint32_t)b;
+            for (int64_t j = u.uoff[bk]; j < (int64_t)u.uoff[bk + 1]; ++j) {
+                const int64_t x = j - lb;
                 atomicOr(&bm[x >> 5], 1u << (x & 31));
             }
         }
