@@ -78,6 +78,8 @@ def lib():
         L.orc_free.argtypes = [P]
         L.orc_query.restype = i32
         L.orc_query.argtypes = [P, P, i64, i32, i32, i32, i32, i32, i64, P, P, P]
+        L.orc_e8_second_ring.restype = i32
+        L.orc_e8_second_ring.argtypes = [P]
         L.orc_e8_parent.restype = None
         L.orc_e8_parent.argtypes = [P, P]
         L.orc_query_union.restype = i32
@@ -184,6 +186,14 @@ def e8_decode(y) -> np.ndarray:
     y = _f32(y)
     out = np.empty(8, np.int32)
     lib().orc_e8_decode(_p(y), _p(out))
+    return out
+
+
+def e8_second_ring() -> np.ndarray:
+    """The 9120 second-ring E8 vectors of recursive probing (R26), doubled coordinates, canonical order."""
+    out = np.zeros((9120, 8), np.int32)
+    n = lib().orc_e8_second_ring(_p(out))
+    assert n == 9120, n
     return out
 
 

@@ -345,9 +345,52 @@ int orc_multiprobe_deltas(const float *t, int M, int T, int32_t *deltas, double 
 
 /* Lattice probe order (R15): the 240 neighbours c + r of the  */
 /* home E8 point c, ordered by (fp64 |y - c - r|^2, root index).            */
+/* Recursive E8 probing ("If the number of candidates computed is not
+ * enough, we recursively probe the adjacent buckets of the 240 probed
+ * buckets"; reading R26): the second ring S2 = {r + r'} minus {0} and the roots
+ * = the E8 vectors of norm^2 4 (2160), 6 (6720) and 8 (the 240 vectors 2r),
+ * in doubled coordinates, ordered by (norm^2, coordinates lexicographically as
+ * signed integers).  Probes 242.. of a lattice sequence take them by
+ * (distance to the query, this order). */
+#define ORC_E8_S2 9120
+static int orc_vec8_cmp(const void *pa, const void *pb)
+{
+    const int32_t *a = (const int32_t *)pa, *b = (const int32_t *)pb;
+    int32_t na = 0, nb = 0;
+    for (int j = 0; j < 8; j++) { na += a[j] * a[j]; nb += b[j] * b[j]; }
+    if (na != nb) return na < nb ? -1 : 1;
+    for (int j = 0; j < 8; j++) if (a[j] != b[j]) return a[j] < b[j] ? -1 : 1;
+    return 0;
+}
+
+int orc_e8_second_ring(int32_t *out /* [ORC_E8_S2][8] */)
+{
+    int32_t roots[240 * 8];
+    orc_e8_roots(roots);
+    int32_t *all = (int32_t *)malloc(sizeof(int32_t) * 8 * 240 * 240);
+    int m = 0;
+    for (int r = 0; r < 240; r++)
+        for (int q = 0; q < 240; q++) {
+            int32_t v[8], n2 = 0;
+            for (int j = 0; j < 8; j++) { v[j] = roots[r * 8 + j] + roots[q * 8 + j]; n2 += v[j] * v[j]; }
+            if (n2 < 16) continue;              /* 0 (r' = -r) and the roots themselves (norm^2 2 = 8 doubled) */
+            memcpy(all + 8 * m, v, sizeof(v));
+            m++;
+        }
+    qsort(all, (size_t)m, sizeof(int32_t) * 8, orc_vec8_cmp);
+    int u = 0;
+    for (int i = 0; i < m; i++)
+        if (u == 0 || orc_vec8_cmp(all + 8 * i, out + 8 * (u - 1)) != 0) {
+            if (u < ORC_E8_S2) memcpy(out + 8 * u, all + 8 * i, sizeof(int32_t) * 8);
+            u++;
+        }
+    free(all);
+    return u;
+}
+
 int orc_lattice_order(const float *y, const int32_t *c2, int T, int32_t *root_idx)
 {
-    if (T < 1 || T > 241) return -1;
+    if (T < 1 || T > 256) return -1;
     int32_t roots[240 * 8];
     orc_e8_roots(roots);
     orc_probe all[240];
@@ -358,7 +401,22 @@ int orc_lattice_order(const float *y, const int32_t *c2, int T, int32_t *root_id
         all[r].enc = r;
     }
     qsort(all, 240, sizeof(orc_probe), orc_probe_cmp);
-    for (int r = 0; r < T - 1; r++) root_idx[r] = all[r].enc;
+    for (int r = 0; r < T - 1 && r < 240; r++) root_idx[r] = all[r].enc;
+    if (T > 241) {           /* recursive probing: the second ring, index 240 + i */
+        int32_t *s2 = (int32_t *)malloc(sizeof(int32_t) * 8 * ORC_E8_S2);
+        orc_e8_second_ring(s2);
+        orc_probe *ring = (orc_probe *)malloc(sizeof(orc_probe) * ORC_E8_S2);
+        for (int i = 0; i < ORC_E8_S2; i++) {
+            int32_t p[8];
+            for (int j = 0; j < 8; j++) p[j] = c2[j] + s2[i * 8 + j];
+            ring[i].score = orc_e8_dist2(y, p);
+            ring[i].enc = i;
+        }
+        qsort(ring, ORC_E8_S2, sizeof(orc_probe), orc_probe_cmp);
+        for (int r = 240; r < T - 1; r++) root_idx[r] = 240 + (int32_t)ring[r - 240].enc;
+        free(ring);
+        free(s2);
+    }
     return 0;
 }
 
@@ -815,7 +873,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     if (k < 1 || T < 1) return 1;
     if (probe == 0 && T != 1) return 1;
     if (probe == 1 && (ix->quantizer != 0 || M > 10 || T > orc_pow3(M))) return 1;
-    if (probe == 2 && (ix->quantizer != 1 || T > 241)) return 1;
+    if (probe == 2 && (ix->quantizer != 1 || T > 256)) return 1;
     if (probe == 3 && ix->quantizer != 0) return 1;
     if (probe < 0 || probe > 3) return 1;
     /* hierarchy: Morton prefixes on Z^M (R17), the Eq. 10 code hierarchy on E8 (R27) */
@@ -845,6 +903,11 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     u128 *hkey = (u128 *)calloc(nqs, sizeof(u128));
     int32_t roots[240 * 8];
     orc_e8_roots(roots);
+    int32_t *ring2 = NULL;           /* recursive E8 probing (R26) */
+    if (probe == 2 && T > 241) {
+        ring2 = (int32_t *)malloc(sizeof(int32_t) * 8 * ORC_E8_S2);
+        orc_e8_second_ring(ring2);
+    }
 
     /* a1-a4: route, hash, probe sequence, bucket lookup, base count |A0| */
     #pragma omp parallel for schedule(dynamic, 16)
@@ -862,7 +925,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         ix->lq_key[2 * q] = (uint64_t)(hk >> 64);
         ix->lq_key[2 * q + 1] = (uint64_t)hk;
         int32_t *deltas = (int32_t *)malloc(sizeof(int32_t) * (size_t)T * 16);
-        int32_t ridx[240];
+        int32_t ridx[256];
         if (probe == 1 && T > 1) orc_multiprobe_deltas(t, M, T, deltas, NULL);
         if (probe == 2 && T > 1 && ok) orc_lattice_order(t, code, T, ridx);
         const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
@@ -900,7 +963,9 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
             } else {
                 /* E8: home c, then c + r for the selected roots */
                 valid = ok;
-                for (int i = 0; i < 8; i++) pc[i] = code[i] + (p == 0 ? 0 : roots[ridx[p - 1] * 8 + i]);
+                for (int i = 0; i < 8; i++)
+                    pc[i] = code[i] + (p == 0 ? 0 : (ridx[p - 1] < 240 ? roots[ridx[p - 1] * 8 + i]
+                                                                        : ring2[(ridx[p - 1] - 240) * 8 + i]));
                 if (valid && !orc_code_in_range(pc, 8, B)) valid = 0;
             }
             u128 pk = valid ? orc_morton(pc, M, B) : 0;
@@ -1045,7 +1110,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         memcpy(ix->lq_cand + ix->lq_coff[q], cand[q], sizeof(int64_t) * (size_t)ncand[q]);
         free(cand[q]);
     }
-    free(cand); free(ncand); free(bs); free(be); free(hs); free(he); free(hkey); free(hbk); free(nhbk);
+    free(cand); free(ncand); free(bs); free(be); free(hs); free(he); free(hkey); free(hbk); free(nhbk); free(ring2);
     return 0;
 }
 

@@ -101,3 +101,35 @@ def test_e8_hierarchy_widening_rule(orc, tau):
                 want |= set(perm[uoff[u]:uoff[u + 1]].tolist())
         want |= set(a0[q].tolist())
         assert set(cands[q].tolist()) == want
+
+
+def test_second_ring_is_the_e8_shells(orc):
+    """Recursive probing (R26): the neighbours of the 240 neighbours are
+    exactly the E8 vectors of norm^2 4 and 6 (theta series: 2160 and 6720, every
+    one of them) and the 240 vectors 2r of norm^2 8."""
+    s2 = orc.e8_second_ring()
+    roots = orc.e8_roots()
+    n2 = (s2.astype(np.int64) ** 2).sum(1)          # doubled coordinates: 4x the norm^2
+    assert (n2 == 16).sum() == 2160 and (n2 == 24).sum() == 6720 and (n2 == 32).sum() == 240
+    assert len({tuple(v) for v in s2}) == 9120
+    assert all(_is_e8(v) for v in s2[::7])
+    assert {tuple(v) for v in s2[n2 == 32]} == {tuple(2 * r) for r in roots}
+    # canonical order: by norm, then lexicographic
+    keys = [(int(n), tuple(int(x) for x in v)) for n, v in zip(n2, s2)]
+    assert keys == sorted(keys)
+
+
+def test_recursive_lattice_order(orc):
+    rng = np.random.default_rng(4)
+    s2 = orc.e8_second_ring().astype(np.float64) / 2.0
+    for _ in range(20):
+        y = (rng.standard_normal(8) * 3).astype(np.float32)
+        c = orc.e8_decode(y)
+        o241 = orc.lattice_order(y, c, 241)
+        o256 = orc.lattice_order(y, c, 256)
+        assert np.array_equal(o256[:240], o241)                  # the first ring first, unchanged
+        ring = o256[240:] - 240
+        assert np.all(ring >= 0)
+        d = ((y.astype(np.float64) - c / 2.0 - s2) ** 2).sum(1)
+        want = np.lexsort((np.arange(9120), d))[:15]
+        assert np.array_equal(ring, want)
