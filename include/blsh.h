@@ -79,7 +79,9 @@ typedef struct {
                                3 Morton-curve neighbours on Z^M (R25): the T buckets around the
                                insertion position of the home key in the leaf's sorted keys (after, before,
                                alternating)                                                                    */
-    int32_t n_probes;       /* T >= 1 including the home bucket; <= 3^M (M <= 10) or <= 241 (E8)              */
+    int32_t n_probes;       /* T >= 1 including the home bucket; <= 3^M (M <= 10), <= 256 (Morton curve) or
+                               <= 256 (E8: home, the 240 roots, then probes 242..256 from the second ring of
+                               recursive probing, R26)                                                */
     int32_t hierarchy;      /* 1 = Morton-prefix widening (Eq. 7-8, R17); Z^M index only               */
     int32_t hier_step_bits; /* key bits cleared per widening step: 0 = M (one Eq. 8 level), or 1..M           */
     int64_t min_cand;       /* tau (R18); 0 = lower median of the base counts of this batch           */

@@ -599,7 +599,7 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
         if (p->n_probes > ipow3(idx->M)) return fail(BLSH_ERR_INVALID, "n_probes > 3^M");
     } else if (p->probe == 2) {
         if (idx->quantizer != 1) return fail(BLSH_ERR_INVALID, "lattice probing needs an E8 index");
-        if (p->n_probes > 241) return fail(BLSH_ERR_INVALID, "n_probes > 241");
+        if (p->n_probes > 256) return fail(BLSH_ERR_INVALID, "n_probes > 256");
     } else if (p->probe == 3) {
         if (idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "Morton-curve probing needs a Z^M index");
     } else if (p->probe != 0) {

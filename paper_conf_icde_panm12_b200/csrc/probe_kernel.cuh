@@ -206,15 +206,22 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
     const int T = a.T, B = a.B;
     const float* t = a.qt + (size_t)q * 8;
     const int32_t* code = a.qcode + (size_t)q * 8;
+    if (a.probe == 2 && T > 241 && !(oor & 1)) {   // recursive probing (R26): the second ring
+        warp_select(sm, 9120u, 0xFFFFFFFFu, T - 241, [&](uint32_t x) { return ring2_score(t, code, x); });
+        if (lane < T - 241) sm.order2[lane] = sm.order[lane];
+        __syncwarp();
+    }
     if (a.probe == 2 && T > 1 && !(oor & 1))
-        warp_select(sm, 240u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat_score(t, code, x); });
+        warp_select(sm, 240u, 0xFFFFFFFFu, min(T - 1, 240), [&](uint32_t x) { return lat_score(t, code, x); });
     int64_t mysum = 0;
     for (int p = lane; p < T; p += 32) {
         int32_t pc[8];
         bool valid = !(oor & 1);
-        const uint32_t r = (p > 0 && valid) ? sm.order[p - 1] : 0u;
+        const bool ring = p > 240;
+        const uint32_t r = (p > 0 && valid) ? (ring ? sm.order2[p - 241] : sm.order[p - 1]) : 0u;
 #pragma unroll
-        for (int i = 0; i < 8; ++i) pc[i] = code[i] + (p > 0 ? (int32_t)c_e8_roots[r][i] : 0);
+        for (int i = 0; i < 8; ++i)
+            pc[i] = code[i] + (p > 0 ? (ring ? (int32_t)g_e8_ring2[r][i] : (int32_t)c_e8_roots[r][i]) : 0);
         const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
         if (valid)
             for (int i = 0; i < 8; ++i)

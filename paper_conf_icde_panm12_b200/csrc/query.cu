@@ -7,6 +7,10 @@
 //                  intervals of the position-sorted table + |A0|.
 //   k_median       tau = lower median of |A0| over the batch (R18).
 //   k_widen        Morton-prefix widening until |R| >= tau (Eq. 7-8, R17).
+#include <algorithm>
+#include <array>
+#include <vector>
+
 #include "hashcore.cuh"
 #include "internal.cuh"
 #include "query_kernels.cuh"
@@ -14,6 +18,7 @@
 namespace blsh {
 
 __constant__ int8_t c_e8_roots[240][8];   // doubled coordinates, canonical order (R15)
+__device__ int8_t g_e8_ring2[9120][8];     // recursive probing: the second ring, canonical order (R26)
 
 namespace {
 
@@ -213,6 +218,7 @@ struct ProbeSmem {
     unsigned long long sbits[kMaxSel];
     uint32_t sx[kMaxSel];
     uint32_t order[kMaxSel];
+    uint32_t order2[16];        // recursive E8 probing: the selected second-ring vectors
     double fs[2][kFCap];        // frontier: partial scores
     uint32_t fe[2][kFCap];      // frontier: partial enc (base-3 digits delta_i + 1, i = 0 most significant)
 };
@@ -238,6 +244,13 @@ __device__ __forceinline__ double mp_score(const MPPool& P, uint32_t x, int8_t* 
         if (dv != 0) s = __dadd_rn(s, P.sq[i][dv > 0 ? 1 : 0]);
     }
     return s;
+}
+
+__device__ __forceinline__ double ring2_score(const float* y, const int32_t* c2, uint32_t r) {
+    int32_t p[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) p[j] = c2[j] + (int32_t)g_e8_ring2[r][j];
+    return e8_dist2(y, p);
 }
 
 __device__ __forceinline__ double lat_score(const float* y, const int32_t* c2, uint32_t r) {
@@ -635,6 +648,32 @@ void upload_e8_roots() {
         ++r;
     }
     BLSH_CUDA(cudaMemcpyToSymbol(c_e8_roots, roots, sizeof(roots)));
+    // the second ring (R26): r + r' of norm^2 4, 6, 8 (doubled 16, 24, 32), sorted by (norm^2, lexicographic)
+    std::vector<std::array<int8_t, 8>> ring;
+    ring.reserve(240 * 240);
+    for (int i = 0; i < 240; ++i)
+        for (int j = 0; j < 240; ++j) {
+            std::array<int8_t, 8> v{};
+            int n2 = 0;
+            for (int t = 0; t < 8; ++t) {
+                v[t] = (int8_t)(roots[i][t] + roots[j][t]);
+                n2 += v[t] * v[t];
+            }
+            if (n2 >= 16) ring.push_back(v);
+        }
+    auto norm2 = [](const std::array<int8_t, 8>& v) {
+        int n = 0;
+        for (int t = 0; t < 8; ++t) n += v[t] * v[t];
+        return n;
+    };
+    std::sort(ring.begin(), ring.end(), [&](const std::array<int8_t, 8>& x, const std::array<int8_t, 8>& y) {
+        const int nx = norm2(x), ny = norm2(y);
+        if (nx != ny) return nx < ny;
+        return x < y;   // lexicographic on signed coordinates
+    });
+    ring.erase(std::unique(ring.begin(), ring.end()), ring.end());
+    if (ring.size() != 9120) throw Error(BLSH_ERR_CUDA, "E8 second ring size");
+    BLSH_CUDA(cudaMemcpyToSymbol(g_e8_ring2, ring.data(), ring.size() * 8));
     done = true;
 }
 

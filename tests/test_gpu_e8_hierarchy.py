@@ -87,3 +87,14 @@ def test_e8_hierarchy_sharded_global_median(blsh, orc, c1):
     torch.cuda.synchronize()
     assert torch.equal(mi, i1) and torch.equal(md.view(torch.int32), d1.view(torch.int32))
     assert torch.equal(ncs[0] + ncs[1], n1)
+
+
+@pytest.mark.parametrize("T", [242, 250, 256])
+def test_recursive_e8_probing(blsh, orc, c1, T):
+    """after the 240 neighbours, the second ring (R26), probe keys and
+    candidate sets bit-exact, with and without the hierarchy."""
+    from test_gpu_parity import run_query_pair
+    X, Q = c1
+    ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=1.0, seed=42, quantizer=1)
+    run_query_pair(ix, ox, X, Q, 10, probe=2, T=T)
+    run_e8h(ix, ox, X, Q, 10, 2, T, 0)
