@@ -388,6 +388,42 @@ int orc_e8_second_ring(int32_t *out /* [ORC_E8_S2][8] */)
     return u;
 }
 
+int orc_lattice_order(const float *y, const int32_t *c2, int T, int32_t *root_idx);
+
+/* Lattice probing with M = 16 (two E8 blocks, R28): the neighbours of the
+ * home code c change one block by one root; candidate x = blk * 240 + r,
+ * ordered by (fp64 sum over all M coordinates of (y_j - c'_j / 2)^2, x). */
+static double orc_e8_dist2_m(const float *y, const int32_t *c2, int M)
+{
+    double s = 0.0;
+    for (int j = 0; j < M; j++) {
+        double e = (double)y[j] - 0.5 * (double)c2[j];
+        s = fma(e, e, s);
+    }
+    return s;
+}
+
+int orc_lattice_order_blocks(const float *y, const int32_t *c2, int M, int T, int32_t *idx)
+{
+    if (M == 8) return orc_lattice_order(y, c2, T, idx);
+    const int P = 240 * (M / 8);
+    if (T < 1 || T > 1 + P || T > 256) return -1;
+    int32_t roots[240 * 8];
+    orc_e8_roots(roots);
+    orc_probe *all = (orc_probe *)malloc(sizeof(orc_probe) * (size_t)P);
+    for (int x = 0; x < P; x++) {
+        int32_t p[16];
+        memcpy(p, c2, sizeof(int32_t) * M);
+        for (int j = 0; j < 8; j++) p[8 * (x / 240) + j] += roots[(x % 240) * 8 + j];
+        all[x].score = orc_e8_dist2_m(y, p, M);
+        all[x].enc = x;
+    }
+    qsort(all, (size_t)P, sizeof(orc_probe), orc_probe_cmp);
+    for (int r = 0; r < T - 1; r++) idx[r] = all[r].enc;
+    free(all);
+    return 0;
+}
+
 int orc_lattice_order(const float *y, const int32_t *c2, int T, int32_t *root_idx)
 {
     if (T < 1 || T > 256) return -1;
@@ -650,14 +686,15 @@ static int orc_hash(const orc_index *ix, int g, const float *x, float *t, int32_
             if (clamped) clamped[i] = (int32_t)c;
         }
     } else {
-        for (int i = 0; i < 8; i++)
+        /* E8 (Eq. 6); M = 16: two E8 blocks decoded independently (R28) */
+        for (int i = 0; i < M; i++)
             if (!(fabsf(t[i]) < 16000.0f)) ok = 0;
         if (ok) {
-            orc_e8_decode(t, code);
-            if (!orc_code_in_range(code, 8, B)) ok = 0;
+            for (int blk = 0; blk < M / 8; blk++) orc_e8_decode(t + 8 * blk, code + 8 * blk);
+            if (!orc_code_in_range(code, M, B)) ok = 0;
         }
-        if (!ok) for (int i = 0; i < 8; i++) code[i] = 0;
-        if (clamped) memcpy(clamped, code, sizeof(int32_t) * 8);
+        if (!ok) for (int i = 0; i < M; i++) code[i] = 0;
+        if (clamped) memcpy(clamped, code, sizeof(int32_t) * M);
     }
     return ok;
 }
@@ -705,7 +742,7 @@ orc_index *orc_build(const float *X, int64_t n, int d, int G, int M, int quantiz
     *err = 1;
     if (n < 0 || d < 1 || G < 1 || G > 4096 || (G & (G - 1)) || M < 1 || M > 16) return NULL;
     if (table < 0 || table > 255) return NULL;
-    if (quantizer == 1 && M != 8) return NULL;
+    if (quantizer == 1 && M != 8 && M != 16) return NULL;   /* ceil(M/8) E8 blocks, R28 */
     if (!(W > 0.0f)) return NULL;
     orc_index *ix = (orc_index *)calloc(1, sizeof(orc_index));
     ix->n = n; ix->d = d; ix->G = G; ix->M = M; ix->quantizer = quantizer;
@@ -873,7 +910,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     if (k < 1 || T < 1) return 1;
     if (probe == 0 && T != 1) return 1;
     if (probe == 1 && (ix->quantizer != 0 || M > 10 || T > orc_pow3(M))) return 1;
-    if (probe == 2 && (ix->quantizer != 1 || T > 256)) return 1;
+    if (probe == 2 && (ix->quantizer != 1 || T > 256 || (M == 16 && T > 481))) return 1;
     if (probe == 3 && ix->quantizer != 0) return 1;
     if (probe < 0 || probe > 3) return 1;
     /* hierarchy: Morton prefixes on Z^M (R17), the Eq. 10 code hierarchy on E8 (R27) */
@@ -904,7 +941,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     int32_t roots[240 * 8];
     orc_e8_roots(roots);
     int32_t *ring2 = NULL;           /* recursive E8 probing (R26) */
-    if (probe == 2 && T > 241) {
+    if (probe == 2 && T > 241 && M == 8) {
         ring2 = (int32_t *)malloc(sizeof(int32_t) * 8 * ORC_E8_S2);
         orc_e8_second_ring(ring2);
     }
@@ -927,7 +964,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         int32_t *deltas = (int32_t *)malloc(sizeof(int32_t) * (size_t)T * 16);
         int32_t ridx[256];
         if (probe == 1 && T > 1) orc_multiprobe_deltas(t, M, T, deltas, NULL);
-        if (probe == 2 && T > 1 && ok) orc_lattice_order(t, code, T, ridx);
+        if (probe == 2 && T > 1 && ok) orc_lattice_order_blocks(t, code, M, T, ridx);
         const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
         int64_t base = 0;
         if (probe == 3) {
@@ -963,10 +1000,15 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
             } else {
                 /* E8: home c, then c + r for the selected roots */
                 valid = ok;
-                for (int i = 0; i < 8; i++)
-                    pc[i] = code[i] + (p == 0 ? 0 : (ridx[p - 1] < 240 ? roots[ridx[p - 1] * 8 + i]
-                                                                        : ring2[(ridx[p - 1] - 240) * 8 + i]));
-                if (valid && !orc_code_in_range(pc, 8, B)) valid = 0;
+                for (int i = 0; i < M; i++) pc[i] = code[i];
+                if (p > 0 && M == 8) {
+                    for (int i = 0; i < 8; i++)
+                        pc[i] += ridx[p - 1] < 240 ? roots[ridx[p - 1] * 8 + i] : ring2[(ridx[p - 1] - 240) * 8 + i];
+                } else if (p > 0) {     /* M = 16: one block moved by one root (R28) */
+                    const int blk = ridx[p - 1] / 240, r = ridx[p - 1] % 240;
+                    for (int i = 0; i < 8; i++) pc[8 * blk + i] += roots[r * 8 + i];
+                }
+                if (valid && !orc_code_in_range(pc, M, B)) valid = 0;
             }
             u128 pk = valid ? orc_morton(pc, M, B) : 0;
             ix->lq_pkey[((size_t)q * T + p) * 2] = (uint64_t)(pk >> 64);
@@ -1006,30 +1048,31 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
             if (ix->lq_base[q] >= tau) continue;
             int g = ix->lq_leaf[q];
             int64_t u0 = ix->leaf_u[g], nb = ix->leaf_u[g + 1] - u0;
-            int32_t *cur = (int32_t *)malloc(sizeof(int32_t) * 8 * (size_t)(nb > 0 ? nb : 1));
-            int32_t cq[8], tmp[8];
-            memcpy(cq, ix->lq_code + q * 8, sizeof(cq));
+            int32_t *cur = (int32_t *)malloc(sizeof(int32_t) * M * (size_t)(nb > 0 ? nb : 1));
+            int32_t cq[16], tmp[16];
+            const size_t cb = sizeof(int32_t) * (size_t)M;
+            memcpy(cq, ix->lq_code + q * M, cb);
             for (int64_t b = 0; b < nb; b++)
-                memcpy(cur + 8 * b, ix->code + 8 * ix->perm[ix->uoff[u0 + b]], sizeof(int32_t) * 8);
+                memcpy(cur + M * b, ix->code + M * ix->perm[ix->uoff[u0 + b]], cb);
             int level = ORC_E8_LEVELS + 1;      /* whole leaf */
             for (int jl = 0; jl <= ORC_E8_LEVELS && nb > 0; jl++) {
                 int64_t rows = 0, match = 0;
                 int same = 1;
                 for (int64_t b = 0; b < nb; b++) {
-                    if (memcmp(cur + 8 * b, cq, sizeof(cq)) == 0) {
+                    if (memcmp(cur + M * b, cq, cb) == 0) {
                         match++;
                         rows += ix->uoff[u0 + b + 1] - ix->uoff[u0 + b];
                     }
-                    if (memcmp(cur + 8 * b, cur, sizeof(cq)) != 0) same = 0;
+                    if (memcmp(cur + M * b, cur, cb) != 0) same = 0;
                 }
                 if (match && rows >= tau) { level = jl; break; }
                 if (same) break;                 /* root reached without a large enough match */
                 for (int64_t b = 0; b < nb; b++) {
-                    orc_e8_parent(cur + 8 * b, tmp);
-                    memcpy(cur + 8 * b, tmp, sizeof(tmp));
+                    for (int k2 = 0; k2 < M / 8; k2++) orc_e8_parent(cur + M * b + 8 * k2, tmp + 8 * k2);
+                    memcpy(cur + M * b, tmp, cb);
                 }
-                orc_e8_parent(cq, tmp);
-                memcpy(cq, tmp, sizeof(cq));
+                for (int k2 = 0; k2 < M / 8; k2++) orc_e8_parent(cq + 8 * k2, tmp + 8 * k2);
+                memcpy(cq, tmp, cb);
             }
             /* node buckets */
             int64_t *lst = (int64_t *)malloc(sizeof(int64_t) * (size_t)(nb > 0 ? nb : 1));
@@ -1039,7 +1082,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
             } else {
                 /* recompute the level-`level` codes (cur holds them after the loop broke there) */
                 for (int64_t b = 0; b < nb; b++)
-                    if (memcmp(cur + 8 * b, cq, sizeof(cq)) == 0) lst[m++] = u0 + b;
+                    if (memcmp(cur + M * b, cq, cb) == 0) lst[m++] = u0 + b;
             }
             hbk[q] = lst;
             nhbk[q] = m;

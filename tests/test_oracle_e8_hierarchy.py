@@ -133,3 +133,68 @@ def test_recursive_lattice_order(orc):
         d = ((y.astype(np.float64) - c / 2.0 - s2) ** 2).sum(1)
         want = np.lexsort((np.arange(9120), d))[:15]
         assert np.array_equal(ring, want)
+
+
+def _leaf_points_with_key(ix, g, k2):
+    leaf, key = ix.get("leaf"), ix.get("key")
+    return set(np.nonzero((leaf == g) & (key[:, 0] == k2[0]) & (key[:, 1] == k2[1]))[0].tolist())
+
+
+def test_two_block_e8_hash_and_probes(orc):
+    """M = 16 (ceil(M/8) E8 lattices, R28): the code is the two blocks'
+    DECODEs; lattice probes move one block by one root, ordered by the fp64
+    distance over all 16 coordinates (brute force over the 480 candidates)."""
+    rng = np.random.default_rng(6)
+    X = (rng.standard_normal((3000, 24)) * 0.5).astype(np.float32)
+    Q = (X[:25] + 0.05 * rng.standard_normal((25, 24))).astype(np.float32)
+    ix = orc.OracleIndex(X, G=2, M=16, W=1.0, seed=3, quantizer=1)
+    assert ix.B == 8
+    T = 40
+    ix.query(Q, 10, probe=2, T=T)
+    t, code, pk, pv, ql = ix.get("q_t"), ix.get("q_code"), ix.get("q_pkey"), ix.get("q_pvalid"), ix.get("q_leaf")
+    roots = orc.e8_roots()
+    cands = ix.candidates()
+    for q in range(len(Q)):
+        c = np.concatenate([orc.e8_decode(t[q, :8]), orc.e8_decode(t[q, 8:])])
+        assert np.array_equal(code[q], c) and _is_e8(c[:8]) and _is_e8(c[8:])
+        cand = []
+        for x in range(480):
+            p = c.copy()
+            p[8 * (x // 240):8 * (x // 240) + 8] += roots[x % 240]
+            cand.append(p)
+        cand = np.array(cand)
+        d = ((t[q].astype(np.float64)[None, :] - cand / 2.0) ** 2).sum(1)
+        order = np.lexsort((np.arange(480), d))[:T - 1]
+        want = set(_leaf_points_with_key(ix, ql[q], pk[q, 0]))
+        for p in range(1, T):
+            assert orc.morton_encode(cand[order[p - 1]]) == (int(pk[q, p, 0]) << 64) | int(pk[q, p, 1])
+            if pv[q, p]:
+                want |= _leaf_points_with_key(ix, ql[q], pk[q, p])
+        assert set(cands[q].tolist()) == want
+
+
+def test_two_block_e8_hierarchy(orc):
+    """The E8 hierarchy with two blocks: parents per block (R27, R28)."""
+    rng = np.random.default_rng(7)
+    X = (rng.standard_normal((3000, 24)) * 0.5).astype(np.float32)
+    Q = (X[:25] + 0.05 * rng.standard_normal((25, 24))).astype(np.float32)
+    ix = orc.OracleIndex(X, G=2, M=16, W=1.0, seed=3, quantizer=1)
+    ix.query(Q, 10, probe=2, T=8, hierarchy=1, min_cand=200)
+    base, lvl, ql, code = ix.get("q_base"), ix.get("q_level"), ix.get("q_leaf"), ix.get("q_code")
+    uleaf, uoff, perm, pcode = ix.get("uleaf"), ix.get("uoff"), ix.get("perm"), ix.get("code")
+
+    def chain(c, j):
+        for _ in range(j):
+            c = np.concatenate([orc.e8_parent(c[:8]), orc.e8_parent(c[8:])])
+        return c
+
+    seen = set()
+    for q in range(len(Q)):
+        if base[q] >= 200 or lvl[q] > 32:
+            continue
+        L = int(lvl[q])
+        seen.add(L)
+        bks = np.nonzero(uleaf == ql[q])[0]
+        node = [u for u in bks if np.array_equal(chain(pcode[perm[uoff[u]]], L), chain(code[q], L))]
+        assert node and sum(int(uoff[u + 1] - uoff[u]) for u in node) >= 200
+    assert seen
