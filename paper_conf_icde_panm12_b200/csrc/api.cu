@@ -121,7 +121,8 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
     if (G < 1 || G > 4096 || (G & (G - 1))) return fail(BLSH_ERR_INVALID, "n_leaves must be a power of two in [1, 4096]");
     if (p->M < 1 || p->M > 16) return fail(BLSH_ERR_INVALID, "M must be in [1, 16]");
     if (p->quantizer != 0 && p->quantizer != 1) return fail(BLSH_ERR_INVALID, "quantizer must be 0 or 1");
-    if (p->quantizer == 1 && p->M != 8) return fail(BLSH_ERR_INVALID, "E8 quantizer needs M = 8");
+    if (p->quantizer == 1 && p->M != 8 && p->M != 16)
+        return fail(BLSH_ERR_INVALID, "E8 quantizer needs M = 8 or 16 (ceil(M/8) E8 blocks, P:175)");
     if (!(p->W > 0.0f) || !std::isfinite(p->W)) return fail(BLSH_ERR_INVALID, "W must be > 0");
     if (p->rp_rule != 0 && p->rp_rule != 1) return fail(BLSH_ERR_INVALID, "rp_rule must be 0 or 1");
     if (p->ek_iters < 1) return fail(BLSH_ERR_INVALID, "ek_iters must be >= 1");
@@ -451,7 +452,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         }
         if (e8h) {
             E8WidenArgs ew{};
-            ew.nq = nq; ew.B = ix.B; ew.qleaf = w.qleaf; ew.qoor = w.qoor; ew.qcode = w.qcode; ew.base = w.base;
+            ew.nq = nq; ew.M = ix.M; ew.B = ix.B; ew.qleaf = w.qleaf; ew.qoor = w.qoor; ew.qcode = w.qcode; ew.base = w.base;
             ew.ukey = ix.ukey.as<Key128>(); ew.uoff = ix.uoff.as<uint32_t>(); ew.leaf_u = ix.leaf_u.as<int64_t>();
             ew.root = ix.e8_root.as<int32_t>();
             ew.lv_key = reinterpret_cast<const Key128* const*>(ix.e8_ptrs.as<char>());

@@ -46,23 +46,21 @@ __device__ __forceinline__ void e8_parent(const int32_t* c2, int32_t* out) {
 }
 
 // level 0 codes of every bucket
-__global__ void k_bucket_codes(const Key128* __restrict__ ukey, int64_t nu, int B, int32_t* __restrict__ codes) {
+__global__ void k_bucket_codes(const Key128* __restrict__ ukey, int64_t nu, int M, int B, int32_t* __restrict__ codes) {
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < nu; u += (int64_t)gridDim.x * blockDim.x)
-        morton_decode(ukey[u], 8, B, codes + 8 * u);
+        morton_decode(ukey[u], M, B, codes + (size_t)M * u);
 }
 
 // one level up: codes <- parent(codes); sort entries (leaf, key, u)
-__global__ void k_parent_level(int32_t* __restrict__ codes, const int32_t* __restrict__ uleaf, int64_t nu, int B,
+__global__ void k_parent_level(int32_t* __restrict__ codes, const int32_t* __restrict__ uleaf, int64_t nu, int M, int B,
                                unsigned long long* __restrict__ hi, unsigned long long* __restrict__ lo,
                                uint32_t* __restrict__ leaf, uint32_t* __restrict__ id) {
     for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < nu; u += (int64_t)gridDim.x * blockDim.x) {
-        int32_t c[8], p[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) c[i] = codes[8 * u + i];
-        e8_parent(c, p);
-#pragma unroll
-        for (int i = 0; i < 8; ++i) codes[8 * u + i] = p[i];
-        const Key128 k = morton_key(p, 8, B);
+        int32_t c[16], p[16];
+        for (int i = 0; i < M; ++i) c[i] = codes[(size_t)M * u + i];
+        for (int blk = 0; blk < M / 8; ++blk) e8_parent(c + 8 * blk, p + 8 * blk);   // per block (R28)
+        for (int i = 0; i < M; ++i) codes[(size_t)M * u + i] = p[i];
+        const Key128 k = morton_key(p, M, B);
         hi[u] = k.hi;
         lo[u] = k.lo;
         leaf[u] = (uint32_t)uleaf[u];
@@ -109,13 +107,13 @@ __global__ void k_e8_widen(E8WidenArgs w, const int64_t* __restrict__ tau_p, int
     if ((w.qoor[q] & 2) || w.base[q] >= tau) return;
     const int g = w.qleaf[q];
     const int64_t u0 = w.leaf_u[g], u1 = w.leaf_u[g + 1];
-    int32_t c[8], p[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) c[i] = w.qcode[8 * q + i];
+    const int M = w.M;
+    int32_t c[16], p[16];
+    for (int i = 0; i < M; ++i) c[i] = w.qcode[(size_t)M * q + i];
     int level = kE8Levels + 1;
     int64_t s = 0, e = 0, rows = 0;
     for (int j = 0; j <= kE8Levels && u1 > u0; ++j) {
-        const Key128 k = morton_key(c, 8, w.B);
+        const Key128 k = morton_key(c, M, w.B);
         const Key128* K = j == 0 ? w.ukey : w.lv_key[j];
         const int64_t a = lower_k(K, u0, u1, k);
         const int64_t b = upper_k(K, a, u1, k);
@@ -124,9 +122,8 @@ __global__ void k_e8_widen(E8WidenArgs w, const int64_t* __restrict__ tau_p, int
             if (r >= tau) { level = j; s = a; e = b; rows = r; break; }
         }
         if (j >= w.root[g]) break;                 // root: every bucket of the leaf shares a_j
-        e8_parent(c, p);
-#pragma unroll
-        for (int i = 0; i < 8; ++i) c[i] = p[i];
+        for (int blk = 0; blk < M / 8; ++blk) e8_parent(c + 8 * blk, p + 8 * blk);
+        for (int i = 0; i < M; ++i) c[i] = p[i];
     }
     if (level > kE8Levels) {                       // the whole leaf
         s = u0;
@@ -151,8 +148,8 @@ void build_e8_hierarchy(blsh_index& ix, cudaStream_t s) {
         return;
     }
     DevBuf codes;
-    codes.alloc((size_t)nu * 8 * sizeof(int32_t));
-    k_bucket_codes<<<592, 256, 0, s>>>(ix.ukey.as<Key128>(), nu, ix.B, codes.as<int32_t>());
+    codes.alloc((size_t)nu * ix.M * sizeof(int32_t));
+    k_bucket_codes<<<592, 256, 0, s>>>(ix.ukey.as<Key128>(), nu, ix.M, ix.B, codes.as<int32_t>());
     BLSH_LAUNCH_CHECK();
     SortBufs sb;
     for (int i = 0; i < 2; ++i) {
@@ -186,7 +183,7 @@ void build_e8_hierarchy(blsh_index& ix, cudaStream_t s) {
     ScanTemp scan;
     int passes = 0;
     for (int j = 1; j <= kE8Levels && open > 0; ++j) {
-        k_parent_level<<<592, 256, 0, s>>>(codes.as<int32_t>(), ix.uleaf.as<int32_t>(), nu, ix.B,
+        k_parent_level<<<592, 256, 0, s>>>(codes.as<int32_t>(), ix.uleaf.as<int32_t>(), nu, ix.M, ix.B,
                                            sb.hi[0].as<unsigned long long>(), sb.lo[0].as<unsigned long long>(),
                                            sb.leaf[0].as<uint32_t>(), sb.id[0].as<uint32_t>());
         BLSH_LAUNCH_CHECK();

@@ -75,19 +75,19 @@ __device__ __forceinline__ bool quantise(const float* t, int M, int B, int quant
             if (c != f) ok = false;
             code[i] = (int32_t)c;
         }
-    } else if (M != 8) {
+    } else if (M != 8 && M != 16) {
         ok = false;
-    } else {
-        for (int i = 0; i < 8; ++i)
+    } else {   // E8 (Eq. 6); M = 16: two E8 blocks decoded independently (R28)
+        for (int i = 0; i < M; ++i)
             if (!(fabsf(t[i]) < 16000.0f)) ok = false;
         if (ok) {
-            e8_decode(t, code);
+            for (int blk = 0; blk < M / 8; ++blk) e8_decode(t + 8 * blk, code + 8 * blk);
             const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
-            for (int i = 0; i < 8; ++i)
+            for (int i = 0; i < M; ++i)
                 if (code[i] < lo || code[i] > hi) ok = false;
         }
         if (!ok)
-            for (int i = 0; i < 8; ++i) code[i] = 0;
+            for (int i = 0; i < M; ++i) code[i] = 0;
     }
     return ok;
 }

@@ -203,33 +203,43 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
 
 __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int lane, int oor, int64_t ulo,
                             int64_t uhi, uint2* ivl) {
-    const int T = a.T, B = a.B;
-    const float* t = a.qt + (size_t)q * 8;
-    const int32_t* code = a.qcode + (size_t)q * 8;
-    if (a.probe == 2 && T > 241 && !(oor & 1)) {   // recursive probing (R26): the second ring
+    const int T = a.T, B = a.B, M = a.M;   // M = 8, or 16 = two E8 blocks (R28)
+    const float* t = a.qt + (size_t)q * M;
+    const int32_t* code = a.qcode + (size_t)q * M;
+    if (M == 8 && a.probe == 2 && T > 241 && !(oor & 1)) {   // recursive probing (R26): the second ring
         warp_select(sm, 9120u, 0xFFFFFFFFu, T - 241, [&](uint32_t x) { return ring2_score(t, code, x); });
         if (lane < T - 241) sm.order2[lane] = sm.order[lane];
         __syncwarp();
     }
-    if (a.probe == 2 && T > 1 && !(oor & 1))
-        warp_select(sm, 240u, 0xFFFFFFFFu, min(T - 1, 240), [&](uint32_t x) { return lat_score(t, code, x); });
+    if (a.probe == 2 && T > 1 && !(oor & 1)) {
+        if (M == 8) warp_select(sm, 240u, 0xFFFFFFFFu, min(T - 1, 240), [&](uint32_t x) { return lat_score(t, code, x); });
+        else warp_select(sm, 480u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat2_score(t, code, x); });
+    }
     int64_t mysum = 0;
     for (int p = lane; p < T; p += 32) {
-        int32_t pc[8];
+        int32_t pc[16];
         bool valid = !(oor & 1);
-        const bool ring = p > 240;
-        const uint32_t r = (p > 0 && valid) ? (ring ? sm.order2[p - 241] : sm.order[p - 1]) : 0u;
+        for (int i = 0; i < M; ++i) pc[i] = code[i];
+        if (p > 0 && valid) {
+            if (M == 8) {
+                const bool ring = p > 240;
+                const uint32_t r = ring ? sm.order2[p - 241] : sm.order[p - 1];
 #pragma unroll
-        for (int i = 0; i < 8; ++i)
-            pc[i] = code[i] + (p > 0 ? (ring ? (int32_t)g_e8_ring2[r][i] : (int32_t)c_e8_roots[r][i]) : 0);
+                for (int i = 0; i < 8; ++i) pc[i] += ring ? (int32_t)g_e8_ring2[r][i] : (int32_t)c_e8_roots[r][i];
+            } else {
+                const uint32_t x = sm.order[p - 1], blk = x / 240u, r = x - blk * 240u;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) pc[8 * blk + i] += (int32_t)c_e8_roots[r][i];
+            }
+        }
         const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
         if (valid)
-            for (int i = 0; i < 8; ++i)
+            for (int i = 0; i < M; ++i)
                 if (pc[i] < lo || pc[i] > hi) valid = false;
         Key128 k{0, 0};
         uint2 iv = make_uint2(0, 0);
         if (valid) {
-            k = morton_key(pc, 8, B);
+            k = morton_key(pc, M, B);
             const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
             if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
         }

@@ -253,6 +253,20 @@ __device__ __forceinline__ double ring2_score(const float* y, const int32_t* c2,
     return e8_dist2(y, p);
 }
 
+// M = 16 (two E8 blocks, R28): candidate x moves block x / 240 by root x % 240;
+// fp64 distance over all 16 coordinates (fma-accumulated, ascending j).
+__device__ __forceinline__ double lat2_score(const float* y, const int32_t* c2, uint32_t x) {
+    const uint32_t blk = x / 240u, r = x - blk * 240u;
+    double s = 0.0;
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+        const int32_t c = c2[j] + ((uint32_t)(j >> 3) == blk ? (int32_t)c_e8_roots[r][j & 7] : 0);
+        const double e = __dsub_rn((double)y[j], __dmul_rn(0.5, (double)c));
+        s = __fma_rn(e, e, s);
+    }
+    return s;
+}
+
 __device__ __forceinline__ double lat_score(const float* y, const int32_t* c2, uint32_t r) {
     int32_t p[8];
 #pragma unroll

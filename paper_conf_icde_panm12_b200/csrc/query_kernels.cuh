@@ -75,10 +75,10 @@ struct UnionArgs {
 constexpr int kE8Levels = 32;
 struct E8WidenArgs {
     int64_t nq;
-    int B;
+    int M, B;                     // M = 8 or 16 (E8 blocks)
     const int32_t* qleaf;
     const int32_t* qoor;
-    const int32_t* qcode;         // [nq][8] doubled home codes
+    const int32_t* qcode;         // [nq][M] doubled home codes
     const int64_t* base;          // |A0(q)|
     const Key128* ukey;           // level 0 keys (the table)
     const uint32_t* uoff;

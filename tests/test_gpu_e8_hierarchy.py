@@ -98,3 +98,19 @@ def test_recursive_e8_probing(blsh, orc, c1, T):
     ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=1.0, seed=42, quantizer=1)
     run_query_pair(ix, ox, X, Q, 10, probe=2, T=T)
     run_e8h(ix, ox, X, Q, 10, 2, T, 0)
+
+
+def test_two_block_e8(blsh, orc):
+    """M = 16: two E8 blocks (R28) -- build, lattice probes over 480
+    one-block moves, the hierarchy with per-block parents."""
+    from test_gpu_parity import compare_build, run_query_pair
+    rng = np.random.default_rng(6)
+    X = (rng.standard_normal((3000, 24)) * 0.5).astype(np.float32)
+    Q = (X[:40] + 0.05 * rng.standard_normal((40, 24))).astype(np.float32)
+    ix, ox = build_pair(blsh, orc, X, G=2, M=16, W=1.0, seed=3, quantizer=1)
+    compare_build(ix, ox)
+    run_query_pair(ix, ox, X, Q, 10, probe=0, T=1)
+    run_query_pair(ix, ox, X, Q, 10, probe=2, T=40)
+    run_query_pair(ix, ox, X, Q, 100, probe=2, T=256)
+    run_e8h(ix, ox, X, Q, 10, 2, 8, 200)
+    run_e8h(ix, ox, X, Q, 10, 0, 1, 0)
