@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -407,6 +408,10 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.nq = nq; a.d = ix.d; a.ds = ds; a.G = ix.G; a.M = M; a.B = ix.B; a.depth = ix.depth;
     a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi;
     a.probe = p.probe; a.T = T; a.hstep = p.hier_step_bits > 0 ? p.hier_step_bits : M;
+    {
+        const char* rh = std::getenv("BLSH_RH_STAGE");   // ablation: 1 = stage query rows in shared memory
+        a.rh_direct = (rh && rh[0] == '1') ? 0 : 1;
+    }
     a.Q = w.Qd; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
     a.ntype = ix.ntype.as<int32_t>(); a.A = ix.A.as<float>(); a.bvec = ix.b.as<float>(); a.Wl = ix.W.as<float>();
     a.ukey = ix.ukey.as<Key128>(); a.uoff = ix.uoff.as<uint32_t>(); a.leaf_u = ix.leaf_u.as<int64_t>();

@@ -55,11 +55,13 @@ __global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict
     const int64_t q0 = blockIdx.x * (int64_t)kRHQ;
     const int nrow = (int)min((int64_t)kRHQ, a.nq - q0);
     float4* rows4 = reinterpret_cast<float4*>(rh_rows);
-    stage_rows(a, rows4, nullptr, q0, nrow, lane);
+    if (!a.rh_direct) stage_rows(a, rows4, nullptr, q0, nrow, lane);
     __syncwarp();
     if (lane >= nrow) return;
     const int64_t q = q0 + lane;
-    const float4* x4 = rows4 + lane * ((a.ds >> 2) + 1);
+    // rh_direct: each lane reads its own row through L1 (no staging: more blocks per SM)
+    const float4* x4 = a.rh_direct ? reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds)
+                                   : rows4 + lane * ((a.ds >> 2) + 1);
     const int d = a.d;
     const int nfull = d >> 2, rem = d & 3;
     int v = 0;
@@ -149,15 +151,16 @@ __global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __re
     const int nrow = (int)min((int64_t)kRHQ, a.nq - p0);
     const int d = a.d;
     float4* rows4 = reinterpret_cast<float4*>(rh_rows);
-    float* As = rh_rows + (size_t)kRHQ * (a.ds + 4);     // [MM][d] of the block's first leaf
+    float* As = rh_rows + (a.rh_direct ? (size_t)0 : (size_t)kRHQ * (a.ds + 4));   // [MM][d] of the block's first leaf
     const int g0 = a.qleaf[lperm[p0]];
     const float* Ag0 = a.A + (size_t)g0 * MM * d;
     for (int i = lane; i < MM * d; i += 32) As[i] = __ldg(Ag0 + i);
-    stage_rows(a, rows4, lperm, p0, nrow, lane);
+    if (!a.rh_direct) stage_rows(a, rows4, lperm, p0, nrow, lane);
     __syncwarp();
     if (lane >= nrow) return;
     const int64_t q = lperm[p0 + lane];
-    const float4* x4 = rows4 + lane * ((a.ds >> 2) + 1);
+    const float4* x4 = a.rh_direct ? reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds)
+                                   : rows4 + lane * ((a.ds >> 2) + 1);
     const int g = a.qleaf[q];
     const bool active = g >= a.leaf_lo && g < a.leaf_hi;
     const float* Ag = g == g0 ? As : a.A + (size_t)g * MM * d;   // generic: shared (broadcast) or global
@@ -694,8 +697,8 @@ void upload_e8_roots() {
 int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    const size_t smem_r = (size_t)kRHQ * (a.ds + 4) * sizeof(float);
-    const size_t smem_h = smem_r + (size_t)a.M * a.d * sizeof(float);
+    const size_t smem_r = a.rh_direct ? 16 : (size_t)kRHQ * (a.ds + 4) * sizeof(float);
+    const size_t smem_h = (a.rh_direct ? 0 : smem_r) + (size_t)a.M * a.d * sizeof(float);
     int32_t* lcnt = a.lcnt;
     int32_t* lcur = a.lcnt + a.G;
     BLSH_CUDA(cudaMemsetAsync(lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
@@ -726,7 +729,7 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
 void launch_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    const size_t smem_h = (size_t)kRHQ * (a.ds + 4) * sizeof(float) + (size_t)a.M * a.d * sizeof(float);
+    const size_t smem_h = (a.rh_direct ? 0 : (size_t)kRHQ * (a.ds + 4) * sizeof(float)) + (size_t)a.M * a.d * sizeof(float);
 #define BLSH_H_CASE(MMV)                                                                                    \
     case MMV:                                                                                              \
         BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \

@@ -11,6 +11,7 @@ struct QueryArgs {
     int64_t nq;
     int d, ds, G, M, B, depth, quantizer, leaf_lo, leaf_hi;
     int probe, T, hstep;
+    int rh_direct;           // a1/a2 read query rows through L1 instead of staging them in shared memory
     // queries
     const float* Q;          // [nq][ds]
     // tree + params

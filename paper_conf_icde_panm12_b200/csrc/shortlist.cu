@@ -321,7 +321,7 @@ __device__ void block_select_write(const SelSrc& src, int k, int64_t q, int64_t*
     }
     __syncthreads();
     if (tid == 0) s_cnt = 0;
-    for (int i = tid; i < kSelCap; i += kSelThreads) buf[i] = kEmpty;
+    for (int i = tid; i < kSelCap; i += kSelThreads) buf[i] = kEmpty;   // (only the sorted prefix is read)
     __syncthreads();
     const bool take_all = len <= k;
     for (int64_t i = tid; i < len; i += kSelThreads) {
@@ -338,10 +338,14 @@ __device__ void block_select_write(const SelSrc& src, int k, int64_t q, int64_t*
             if (base + i < kSelCap) buf[base + i] = thr_eq;
         __syncthreads();
     }
-    // bitonic sort of kSelCap keys (padding kEmpty sorts last)
-    for (int size = 2; size <= kSelCap; size <<= 1) {
+    // bitonic sort of the first npow keys (npow = the power of two >= the selected
+    // count, >= 64; padding kEmpty sorts last)
+    const int nsel = (int)min((int64_t)k, len);
+    int npow = 64;
+    while (npow < nsel) npow <<= 1;
+    for (int size = 2; size <= npow; size <<= 1) {
         for (int stride = size >> 1; stride > 0; stride >>= 1) {
-            for (int i = tid; i < kSelCap / 2; i += kSelThreads) {
+            for (int i = tid; i < npow / 2; i += kSelThreads) {
                 const int lo = 2 * i - (i & (stride - 1));
                 const int hi = lo + stride;
                 const bool up = (lo & size) == 0;
