@@ -294,6 +294,35 @@ __device__ int64_t probe_curve(const QueryArgs& a, int64_t q, int lane, int64_t 
     return mysum;
 }
 
+// T = 1 (standard probing): one thread per query -- the home key (the
+// clamped home key equals the probe key whenever the code is in range) and
+// one binary search; same outputs as k_probe_lookup.
+__global__ void __launch_bounds__(256) k_lookup_home(QueryArgs a) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= a.nq) return;
+    const int oor = a.qoor[q];
+    uint2* ivl = a.ivl + (size_t)q * 2;
+    uint2 iv = make_uint2(0, 0);
+    Key128 k{0, 0};
+    const bool valid = !(oor & 3);
+    if (valid) {
+        const int g = a.qleaf[q];
+        k = a.qkey[q];
+        const int64_t u = find_bucket(a.ukey, a.leaf_u[g], a.leaf_u[g + 1], k);
+        if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
+    }
+    ivl[0] = iv;
+    ivl[1] = make_uint2(0, 0);
+    if (a.pkey) {
+        a.pkey[q] = (oor & 2) ? Key128{0, 0} : k;
+        a.pvalid[q] = valid ? 1 : 0;
+    }
+    const int64_t c = (int64_t)(iv.y - iv.x);
+    a.base[q] = c;
+    a.cnt[q] = c;
+    if (a.level) a.level[q] = 0;
+}
+
 __global__ void __launch_bounds__(kPW * 32, 4) k_probe_lookup(QueryArgs a) {
     __shared__ ProbeSmem smem[kPW];
     const int lane = threadIdx.x & 31;

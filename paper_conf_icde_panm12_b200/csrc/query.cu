@@ -747,6 +747,11 @@ void launch_hash(const QueryArgs& a, cudaStream_t s) {
 }
 
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s) {
+    if (a.T == 1 && a.probe != 3) {   // standard probing: thread per query
+        k_lookup_home<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a);
+        BLSH_LAUNCH_CHECK();
+        return;
+    }
     k_probe_lookup<<<(unsigned)((a.nq + kPW - 1) / kPW), kPW * 32, 0, s>>>(a);
     BLSH_LAUNCH_CHECK();
 }
