@@ -38,10 +38,16 @@ constexpr int kTcChunk = 64;               // K columns per A chunk
 constexpr int kTcSlots = 4;                // A chunk ring
 constexpr int kTcAhead = 3;                // staged chunks in flight ahead of the conversion (< kTcSlots)
 constexpr int kTcBlk = 4;                  // TMEM / metadata slots
-constexpr int kTcConv = 8;                 // converter warps
-constexpr int kTcMmaWarp = 8;
-constexpr int kTcEpi0 = 9;                 // first epilogue warp
-constexpr int kTcThreads = 13 * 32;
+#ifndef BLSH_TC_Q
+#define BLSH_TC_Q 2
+#endif
+constexpr int kTcQ = BLSH_TC_Q;            // column parts of a 64-column chunk (one converter warp each per quadrant)
+constexpr int kTcCols = 64 / kTcQ;         // columns per converter warp and chunk (32 or 16)
+constexpr int kTcPieces = kTcCols / 4;     // 16-byte pieces per staged row
+constexpr int kTcConv = 4 * kTcQ;          // converter warps
+constexpr int kTcMmaWarp = kTcConv;
+constexpr int kTcEpi0 = kTcConv + 1;       // first epilogue warp
+constexpr int kTcThreads = (kTcConv + 5) * 32;
 constexpr int kTcMaxK = 16;                // k supported by the TC path
 constexpr int kTcScap = 96;                // buffered pairs per (item, query, epilogue warp)
 constexpr uint32_t kTcStageBytes = kTcRows * kTcChunk * 4;   // 32 KB staging per chunk
@@ -94,6 +100,15 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t* r) {
     asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
 
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* r) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};"
+        ::"r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+        "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+        : "memory");
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
     uint32_t r[32];
     asm volatile(
@@ -116,7 +131,7 @@ struct TcSmem {
     alignas(16) float qn[QT];                // |q'|^2
     uint32_t rpos[kTcBlk][kTcRows];          // table row of each block row
     uint32_t rmask[kTcBlk][kTcRows];         // query mask of each block row (0 = padding)
-    float xn2[kTcBlk][2][kTcRows];           // |x'|^2, per column half
+    float xn2[kTcBlk][kTcQ][kTcRows];        // |x'|^2, per column part
     alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
     unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
@@ -288,10 +303,13 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         // writes the 32 TF32 operands to the A ring in tensor memory (tcgen05.st).  Staging is
         // warp-private (cp.async.wait_group orders it), so only the TMEM A slots and the block
         // metadata need cross-warp barriers.
-        const int qd = warp & 3, hf = warp >> 2;
+        const int qd = warp & 3, hf = warp >> 2;   // quadrant, column part
         const int nch_total = nblk * nchunk;
         const uint2* RI = a.rowinfo + a.rows_off[tile];
-        unsigned char* stg = Aop + (size_t)warp * 4096;   // + slot * kTcStageBytes
+        unsigned char* stg = Aop + (size_t)warp * (32 * kTcCols * 4);   // + slot * kTcStageBytes
+        // 16-byte piece p of staged row r lives at r * kTcCols * 4 + ((p ^ swz(r)) << 4): conflict-free
+        // for the copies and for the row-per-lane reads (8-lane phases see 8 distinct bank groups)
+        auto swz = [](int r) { return kTcPieces == 8 ? (r & 7) : ((r >> 1) & 3); };
         auto fetch = [&](int b) {                          // this lane's row entry of block b
             const int64_t r = r0 + (int64_t)b * kTcRows + 32 * qd + lane;
             return (b < nblk && r < r1) ? RI[r] : make_uint2(0u, 0u);
@@ -314,14 +332,14 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 }
                 const uint32_t sb = smem_u32(stg + (size_t)(g % kTcSlots) * kTcStageBytes);
                 const bool nol = (a.dbgmode & 2) != 0;
-                const int p = lane & 7;
+                const int p = lane % kTcPieces;
 #pragma unroll
-                for (int it = 0; it < 8; ++it) {
-                    const int r = it * 4 + (lane >> 3);
+                for (int it = 0; it < kTcPieces; ++it) {   // 32 / kTcPieces rows per instruction
+                    const int r = it * (32 / kTcPieces) + lane / kTcPieces;
                     const uint32_t pos = __shfl_sync(BLSH_FULL, e_iss.x, r);
                     const uint32_t msk = __shfl_sync(BLSH_FULL, e_iss.y, r);
-                    const float* src = a.Xp + (size_t)pos * ds + c * kTcChunk + hf * 32 + p * 4;
-                    const uint32_t dst = sb + (uint32_t)(r * 128 + ((p ^ (r & 7)) << 4));
+                    const float* src = a.Xp + (size_t)pos * ds + c * kTcChunk + hf * kTcCols + p * 4;
+                    const uint32_t dst = sb + (uint32_t)(r * kTcCols * 4 + ((p ^ swz(r)) << 4));
                     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src),
                                  "r"((msk != 0u && !nol) ? 16u : 0u)
                                  : "memory");
@@ -337,12 +355,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             asm volatile("cp.async.wait_group %0;" ::"n"(kTcAhead) : "memory");   // chunk g has landed
             const int b = g / nchunk, c = g - b * nchunk;
             const int slot = g % kTcSlots;
-            const unsigned char* row = stg + (size_t)slot * kTcStageBytes + lane * 128;
-            uint32_t v[32];
+            const unsigned char* row = stg + (size_t)slot * kTcStageBytes + lane * (kTcCols * 4);
+            uint32_t v[kTcCols];
 #pragma unroll
-            for (int p = 0; p < 8; ++p) {
-                float4 x = *reinterpret_cast<const float4*>(row + ((p ^ (lane & 7)) << 4));
-                const float4 cc = reinterpret_cast<const float4*>(cen)[(c * kTcChunk + hf * 32) / 4 + p];
+            for (int p = 0; p < kTcPieces; ++p) {
+                float4 x = *reinterpret_cast<const float4*>(row + ((p ^ swz(lane)) << 4));
+                const float4 cc = reinterpret_cast<const float4*>(cen)[(c * kTcChunk + hf * kTcCols) / 4 + p];
                 x.x -= cc.x; x.y -= cc.y; x.z -= cc.z; x.w -= cc.w;
                 xs = fmaf(x.x, x.x, xs);
                 xs = fmaf(x.y, x.y, xs);
@@ -356,7 +374,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             const int as = g % kTcASlots;
             if (g >= kTcASlots) mbar_wait(&S.aempty[as], (uint32_t)((g / kTcASlots - 1) & 1));
             tc_fence_after();
-            tmem_st32(tbase + tl + kTcACol0 + (uint32_t)(as * kTcChunk + hf * 32), v);
+            if (kTcCols == 32) tmem_st32(tbase + tl + kTcACol0 + (uint32_t)(as * kTcChunk + hf * kTcCols), v);
+            else tmem_st16(tbase + tl + kTcACol0 + (uint32_t)(as * kTcChunk + hf * kTcCols), v);
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&S.afull[as]);
@@ -430,7 +449,9 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             tmem_ld32(tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 32u, dot);
             tc_fence_before();
             const uint32_t msk = S.rmask[ts][brow];
-            const float xn = S.xn2[ts][0][brow] + S.xn2[ts][1][brow];
+            float xn = S.xn2[ts][0][brow];
+#pragma unroll
+            for (int h = 1; h < kTcQ; ++h) xn += S.xn2[ts][h][brow];
             const uint32_t prow = S.rpos[ts][brow];
             __syncwarp();
             if (lane == 0) {
