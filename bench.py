@@ -311,6 +311,12 @@ def run_ours(a):
     total_cand = sum(s.total_cand for s in stats) / max(len(stats), 1)
     launches = sum(s.launches for s in stats) + extra
     recall, recall_note = (None, "sharded") if world > 1 and rank != 0 else recall_from_gt(cfg, X, Q, out_ids)
+    shard_load = None
+    if world > 1:   # query skew across leaves -> per-rank load of the last step
+        ld = sh.load_stats()
+        cands = [c for _, c in ld]
+        shard_load = {"queries": [q for q, _ in ld], "candidates": cands,
+                      "imbalance": max(cands) / max(1e-9, sum(cands) / len(cands))}
 
     # end to end through the C ABI with host buffers (pinned), copies inside the timed region
     e2e = None
@@ -390,6 +396,7 @@ def run_ours(a):
             "stage_ms": {k2: avg(k2) for k2 in ("ms_route_hash", "ms_probe", "ms_plan", "ms_shortlist", "ms_screen",
                                                  "ms_rescore", "ms_merge", "ms_total")},
             "gpu_launches": launches,
+            "shard_load": shard_load,
             "e2e": e2e,
             "cpu_baseline": cpu,
             "clocks": clocks,

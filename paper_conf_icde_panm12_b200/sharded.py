@@ -48,6 +48,7 @@ class ShardedIndex:
             merge = blsh.blsh_merge_topk
         self._merge = merge
         self._gathered = None
+        self.last_ncand = None
 
     @classmethod
     def build(cls, X, group=None, **build_kw) -> "ShardedIndex":
@@ -67,6 +68,18 @@ class ShardedIndex:
             self.dist.all_reduce(base, op=self.dist.ReduceOp.SUM, group=self.group)
         return base
 
+    def load_stats(self, ncand=None):
+        """Per-rank load of the last query (SURVEY §8(e) scaling risk: query skew across
+        leaves): [[queries with candidates, sum |A(q)|] for every rank], all-gathered."""
+        import torch
+        nc = self.last_ncand if ncand is None else ncand
+        mine = torch.stack([(nc > 0).sum(), nc.sum()]).to(torch.int64)
+        if self.world == 1:
+            return [mine.tolist()]
+        allv = [torch.empty_like(mine) for _ in range(self.world)]
+        self.dist.all_gather(allv, mine, group=self.group)
+        return [v.tolist() for v in allv]
+
     def query(self, Q, k: int, out=None, timing: bool = False, packed_out=None, **kw):
         """-> (ids [nq,k] int64, dist2 [nq,k] fp32): the merged top-k of the whole sharded index.
 
@@ -78,7 +91,8 @@ class ShardedIndex:
             kw["global_base"] = self.global_base_counts(Q, kw.get("probe", 0), kw.get("n_probes", 1))
         if packed_out is not None:
             kw["out"] = packed_out
-        pk, _ = self.index.query_packed(Q, k, timing=timing, **kw)
+        pk, nc = self.index.query_packed(Q, k, timing=timing, **kw)
+        self.last_ncand = nc
         if self.world == 1:
             return self._merge(pk, 1, nq, k, out=out)
         shape = (self.world * nq, k)

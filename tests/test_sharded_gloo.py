@@ -67,7 +67,10 @@ class _OracleShard:
             tau = int(gb[(len(gb) - 1) // 2])         # lower median (R18)
         ids, d2, nc = self.ox.query(Q, k, probe=probe, T=n_probes, hierarchy=hierarchy, min_cand=tau)
         pk = _pack(ids, d2)
-        pk[~self._owned(len(Q))] = PAD
+        own = self._owned(len(Q))
+        pk[~own] = PAD
+        nc = nc.copy()
+        nc[~own] = 0                                  # blsh_query_packed: 0 for queries of other shards
         return torch.from_numpy(pk.view(np.int64)), torch.from_numpy(nc)
 
 
@@ -88,6 +91,7 @@ def _worker(rank, world, port, outdir, probe, T, hierarchy):
         if hierarchy:
             gb = sh.global_base_counts(Q, probe, T).numpy()
             np.save(os.path.join(outdir, f"gb{rank}.npy"), gb)
+        np.save(os.path.join(outdir, f"load{rank}.npy"), np.array(sh.load_stats(), np.int64))
         np.save(os.path.join(outdir, f"ids{rank}.npy"), ids)
         np.save(os.path.join(outdir, f"d2{rank}.npy"), d2)
     finally:
@@ -104,7 +108,7 @@ def test_sharded_exchange_equals_single_index(orc, probe, T, hierarchy):
         cfg = synth.CONFIGS["c1"]
         X, Q = synth.make_dataset(cfg, n=3000, nq=96)
         ox = orc.OracleIndex(X, G=4, M=8, W=4.0, seed=11)
-        ids_ref, d2_ref, _ = ox.query(Q, 10, probe=probe, T=T, hierarchy=hierarchy)
+        ids_ref, d2_ref, nc_ref = ox.query(Q, 10, probe=probe, T=T, hierarchy=hierarchy)
         if hierarchy:
             base_ref = ox.get("q_base")
         for r in range(world):
@@ -114,6 +118,11 @@ def test_sharded_exchange_equals_single_index(orc, probe, T, hierarchy):
             assert np.array_equal(d2.view(np.uint32), d2_ref.view(np.uint32)), f"rank {r}: merged d2 differ"
             if hierarchy:
                 assert np.array_equal(np.load(os.path.join(td, f"gb{r}.npy")), base_ref)
+            # per-rank load (all-gathered, the same on every rank): the shards split the batch's work
+            load = np.load(os.path.join(td, f"load{r}.npy"))
+            assert load.shape == (world, 2)
+            assert load[:, 0].sum() == int((nc_ref > 0).sum()) and load[:, 1].sum() == int(nc_ref.sum())
+            assert np.array_equal(load, np.load(os.path.join(td, "load0.npy")))
         # the exchange was not vacuous: both shards own queries
         ql = ox.get("q_leaf")
         assert 0 < int((ql < 2).sum()) < len(ql)
