@@ -135,7 +135,7 @@ struct TcSmem {
     alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
     unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
-    int lock[QT];                            // guards tk[q] during overflow rescoring
+    int lock[QT];                            // (unused: the screen no longer rescores inside the kernel)
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
     float tr[4][32 * 33];                    // per epilogue warp: transposed dots [query][row], padded
     uint4 rinfo[4][32];                      // per epilogue warp: (|x'|^2 bits, query mask, table row) per row
@@ -147,47 +147,6 @@ __device__ __forceinline__ void tk_insert(unsigned long long* L, int k, unsigned
         while (p > 0 && L[p - 1] > key) { L[p] = L[p - 1]; --p; }
         L[p] = key;
     }
-}
-
-// The warp short-list's fp32 direct form (k_shortlist, k_tc_rescore: lane l sums the
-// float4 columns l, l+32, .. in one fmaf chain, then a 5-level xor butterfly) evaluated
-// by ONE thread, so every distance the TC path reports has the same bits.
-__device__ __noinline__ float warp_order_d2_thread(const float4* __restrict__ x, const float4* __restrict__ q, int nv4) {
-    float p[32];
-#pragma unroll
-    for (int l = 0; l < 32; ++l) {
-        float acc = 0.0f;
-        for (int v = l; v < nv4; v += 32) {
-            const float4 xv = __ldg(x + v), qq = q[v];
-            const float dx = qq.x - xv.x, dy = qq.y - xv.y, dz = qq.z - xv.z, dw = qq.w - xv.w;
-            acc = fmaf(dx, dx, acc);
-            acc = fmaf(dy, dy, acc);
-            acc = fmaf(dz, dz, acc);
-            acc = fmaf(dw, dw, acc);
-        }
-        p[l] = acc;
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1)
-#pragma unroll
-        for (int l = 0; l < o; ++l) p[l] = p[l] + p[l + o];
-    return p[0];
-}
-
-// Overflow (screen phase, lane = query): the pair's exact d^2 by this thread,
-// inserted into the query's shared top-k under its lock.  Only when a pair buffer is
-// still full after dropping what the current bound excludes.
-__device__ __noinline__ void tc_overflow_lane(const TiledArgs& a, unsigned long long* tk, int* lock, const float* qq,
-                                              uint32_t prow) {
-    const float d2 = warp_order_d2_thread(reinterpret_cast<const float4*>(a.Xp + (size_t)prow * a.ds),
-                                          reinterpret_cast<const float4*>(qq), a.ds >> 2);
-    const unsigned long long key = pack_entry(d2, __ldg(a.perm + prow));
-    while (atomicCAS(lock, 0, 1) != 0) {
-    }
-    __threadfence_block();
-    tk_insert(tk, a.k, key);
-    __threadfence_block();
-    atomicExch(lock, 0);
 }
 
 __device__ __forceinline__ void tc_stamp(const TiledArgs& a, int64_t item, int p) {
@@ -437,6 +396,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
 #pragma unroll
         for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
         int my_cnt = 0;                         // buffered pairs of query j in this warp's buffer
+        bool my_fail = false;                   // buffer overflowed: k_tc_rescore scans all of j's rows exactly
         unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * 4 + ew) * kTcScap;
         float* Tt = S.tr[ew];
         const bool screen = !(a.dbgmode & 1);
@@ -479,7 +439,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                 const uint4 ri = S.rinfo[ew][i];                   // broadcast
                 const float t2 = -2.0f * Tt[j * 33 + i];
                 const float lo = (qa + __uint_as_float(ri.x)) + t2;
-                if (((ri.z >> j) & 1u) && lo <= U) {               // rare: keep the pair
+                if (((ri.z >> j) & 1u) && lo <= U && !my_fail) {   // rare: keep the pair (failed: nothing to keep)
                     const float up = (qb + __uint_as_float(ri.y)) + t2;
                     if (up < U) {                                  // sorted insert; only bounds below U matter
 #pragma unroll
@@ -495,15 +455,17 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
                             if (__uint_as_float((uint32_t)(f >> 32)) <= U) SBj[c2++] = f;
                         }
                         my_cnt = c2;
+                        // compaction freed < 1/4: the screen cannot separate this query's candidates
+                        // (further compactions would rescan the buffer per pair) -> exact scan later
+                        if (my_cnt > 3 * kTcScap / 4) my_fail = true;
                     }
-                    if (my_cnt < kTcScap) SBj[my_cnt++] = e;
-                    else tc_overflow_lane(a, S.tk[j], &S.lock[j], a.Q + (size_t)a.qorder[q0 + j] * ds, ri.w);
+                    if (!my_fail) SBj[my_cnt++] = e;
                 }
             }
             if (ulr[KT - 1] < kth0) atomicMin(&S.umin[j], __float_as_uint(ulr[KT - 1]));
             __syncwarp();                                          // Tt / rinfo reused by the next block
         }
-        S.scnt[ew][j] = my_cnt;
+        S.scnt[ew][j] = my_fail ? -1 : my_cnt;
         if (a.counters && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
         if (warp == kTcEpi0 && lane == 0) tc_stamp(a, item, 4);
     }
@@ -519,17 +481,20 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         const int j = threadIdx.x;
         a.ufin[(size_t)item * QT + j] = j < nqt ? S.umin[j] : 0u;   // 0.0f: nothing to rescore for padding slots
 #pragma unroll
-        for (int w = 0; w < 4; ++w) a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
+        for (int w = 0; w < 4; ++w)   // -1: this warp's buffer for j overflowed (full exact scan of j's rows)
+            a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
     }
     for (int i = threadIdx.x; i < nqt * k; i += kTcThreads)
-        a.partials[((size_t)item * QT + i / k) * k + i % k] = S.tk[i / k][i % k];   // overflow-path results
+        a.partials[((size_t)item * QT + i / k) * k + i % k] = S.tk[i / k][i % k];   // (empty lists: the start of k_tc_rescore)
 }
 
 // Exact rescoring of the TC screen's survivors, at full occupancy (one warp per
 // (item, query)): the buffered pairs whose lower bound is <= the final U_j get the
 // fp32 direct-form distance of k_shortlist (lane l: float4 columns l, l+32, ..,
 // per-lane fmaf chain, butterfly; bit-identical to the warp short-list), four rows
-// at a time, and a warp top-k that starts from the TC kernel's overflow results.
+// at a time, and a warp top-k.  A query whose pair buffer overflowed in the screen (its
+// candidates are too close together for the TF32 bound to separate them) gets the exact
+// distance to every row of the item that its query mask selects instead.
 template <int NV>
 __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     const int lane = threadIdx.x & 31;
@@ -558,15 +523,8 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
         qv[u] = v < nv ? __ldg(qrow + v) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
     int rescored = 0;
-    for (int w = 0; w < 4; ++w) {
-        const int cnt = a.scnt[unit * 4 + w];
-        const unsigned long long* Bf = a.sbuf + ((size_t)unit * 4 + w) * kTcScap;
-        for (int base = 0; base < cnt; base += 32) {
-            const int i = base + lane;
-            const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
-            const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
-            unsigned nm = __ballot_sync(BLSH_FULL, need);
-            rescored += __popc(nm);
+    // rows of the set bits of nm: lane i of the warp holds row position rpos (from its entry)
+    auto score_rows = [&](unsigned nm, uint32_t rpos) {
             while (nm) {
                 uint32_t row[4];
                 int nr = 0;
@@ -576,7 +534,7 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
                     if (nm) {
                         const int src = __ffs(nm) - 1;
                         nm &= nm - 1;
-                        row[r] = (uint32_t)__shfl_sync(BLSH_FULL, (unsigned)(e & 0xFFFFFFFFull), src);
+                        row[r] = (uint32_t)__shfl_sync(BLSH_FULL, rpos, src);
                         nr = r + 1;
                     }
                 }
@@ -618,6 +576,34 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
                         }
                     }
                 }
+            }
+    };
+    bool failed = false;
+    for (int w = 0; w < 4; ++w) failed |= a.scnt[unit * 4 + w] < 0;
+    if (failed) {
+        // The screen could not separate this query's candidates (a buffer overflowed):
+        // exact distance to every row of the item whose query mask has bit j.
+        const int64_t r0 = (item - a.item_off[lo]) * a.chr;
+        const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[lo]);
+        const uint2* RI = a.rowinfo + a.rows_off[lo];
+        for (int64_t base = r0; base < r1; base += 32) {
+            const int64_t i = base + lane;
+            const uint2 e = i < r1 ? RI[i] : make_uint2(0u, 0u);
+            const unsigned nm = __ballot_sync(BLSH_FULL, (e.y >> j) & 1u);
+            rescored += __popc(nm);
+            score_rows(nm, e.x);
+        }
+    } else {
+        for (int w = 0; w < 4; ++w) {
+            const int cnt = a.scnt[unit * 4 + w];
+            const unsigned long long* Bf = a.sbuf + ((size_t)unit * 4 + w) * kTcScap;
+            for (int base = 0; base < cnt; base += 32) {
+                const int i = base + lane;
+                const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
+                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+                const unsigned nm = __ballot_sync(BLSH_FULL, need);
+                rescored += __popc(nm);
+                score_rows(nm, (uint32_t)(e & 0xFFFFFFFFull));
             }
         }
     }
