@@ -61,7 +61,8 @@ typedef struct {
     float   W;              /* bucket width > 0                                                       */
     const float* W_leaf;    /* optional HOST array [G] of per-leaf widths (R3); NULL = W everywhere  */
     uint64_t seed;          /* seed of the counter-based generator (R2)                                     */
-    int32_t rank, world;    /* shard: this index keeps leaves [rank*G/world, (rank+1)*G/world) (default 0,1)*/
+    int32_t rank, world;    /* shard: this index keeps leaves [rank*G/world, (rank+1)*G/world) (default 0,1),
+                               or the leaf_split ranges below                                                */
     void*   stream;         /* cudaStream_t                                                                 */
     int32_t keep_stages;    /* 1 = keep per-point leaf/code/key for blsh_export (parity tests)              */
     int32_t n_tables;       /* L hash tables per leaf, 1..64 ("L hash tables ... each constructed
@@ -71,6 +72,11 @@ typedef struct {
                                probed buckets over the L tables, deduplicated (R24).  L > 1 needs every
                                owned leaf to hold <= 1,600,000 points (the per-query dedup bitmap lives
                                in shared memory) and excludes the Morton hierarchy.                      */
+    const int32_t* leaf_split; /* optional HOST array [world+1]: rank r keeps leaves [leaf_split[r],
+                               leaf_split[r+1]) -- a load-aware contiguous assignment (SURVEY §8(e):
+                               query skew across leaves); leaf_split[0] = 0, leaf_split[world] = G,
+                               non-decreasing, identical on every rank.  NULL = G/world leaves each
+                               (then world must divide G).                                                */
 } blsh_build_params;
 
 /* Query parameters.  Defaults: blsh_query_params_default(). */

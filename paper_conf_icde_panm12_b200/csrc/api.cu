@@ -127,8 +127,16 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
     if (!(p->W > 0.0f) || !std::isfinite(p->W)) return fail(BLSH_ERR_INVALID, "W must be > 0");
     if (p->rp_rule != 0 && p->rp_rule != 1) return fail(BLSH_ERR_INVALID, "rp_rule must be 0 or 1");
     if (p->ek_iters < 1) return fail(BLSH_ERR_INVALID, "ek_iters must be >= 1");
-    if (p->world < 1 || p->rank < 0 || p->rank >= p->world || G % p->world != 0)
-        return fail(BLSH_ERR_INVALID, "rank/world must satisfy 0 <= rank < world and world | n_leaves");
+    if (p->world < 1 || p->rank < 0 || p->rank >= p->world)
+        return fail(BLSH_ERR_INVALID, "rank/world must satisfy 0 <= rank < world");
+    if (p->leaf_split) {
+        if (p->leaf_split[0] != 0 || p->leaf_split[p->world] != G)
+            return fail(BLSH_ERR_INVALID, "leaf_split must start at 0 and end at n_leaves");
+        for (int r = 0; r < p->world; ++r)
+            if (p->leaf_split[r + 1] < p->leaf_split[r]) return fail(BLSH_ERR_INVALID, "leaf_split must be non-decreasing");
+    } else if (G % p->world != 0) {
+        return fail(BLSH_ERR_INVALID, "world must divide n_leaves (or pass leaf_split)");
+    }
     if (p->n_tables < 1 || p->n_tables > 64) return fail(BLSH_ERR_INVALID, "n_tables must be in [1, 64]");
     if (p->W_leaf)
         for (int g = 0; g < G; ++g)
@@ -153,8 +161,8 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         ix->seed = p->seed;
         ix->rank = p->rank;
         ix->world = p->world;
-        ix->leaf_lo = p->rank * (G / p->world);
-        ix->leaf_hi = (p->rank + 1) * (G / p->world);
+        ix->leaf_lo = p->leaf_split ? p->leaf_split[p->rank] : p->rank * (G / p->world);
+        ix->leaf_hi = p->leaf_split ? p->leaf_split[p->rank + 1] : (p->rank + 1) * (G / p->world);
         int depth = 0;
         while ((1 << depth) < G) ++depth;
         ix->depth = depth;

@@ -33,6 +33,45 @@ def leaf_range(G: int, rank: int, world: int):
     return rank * per, (rank + 1) * per
 
 
+def balanced_leaf_split(weights, world: int):
+    """Load-aware leaf -> rank assignment (query skew across leaves):
+    the contiguous partition of the leaves into `world` ranges whose largest load
+    sum is minimal (binary search on that bound + greedy fill).  Returns the
+    [world + 1] boundaries blsh_build takes as `leaf_split`."""
+    w = [int(x) for x in weights]
+    if world < 1 or any(x < 0 for x in w):
+        raise ValueError("need world >= 1 and non-negative weights")
+    G = len(w)
+
+    def ranges_needed(cap):
+        n, acc = 1, 0
+        for x in w:
+            if acc + x > cap:
+                n, acc = n + 1, x
+            else:
+                acc += x
+        return n
+
+    lo, hi = max(w) if w else 0, sum(w)
+    while lo < hi:
+        mid = (lo + hi) // 2
+        if ranges_needed(mid) <= world:
+            hi = mid
+        else:
+            lo = mid + 1
+    bounds, acc = [0], 0
+    for g, x in enumerate(w):
+        if acc + x > lo and len(bounds) < world:
+            bounds.append(g)
+            acc = x
+        else:
+            acc += x
+    while len(bounds) < world:
+        bounds.append(G)
+    bounds.append(G)
+    return bounds
+
+
 class ShardedIndex:
     """One leaf shard of a Bi-level LSH index per process of `group`."""
 
@@ -67,6 +106,26 @@ class ShardedIndex:
         if self.world > 1:
             self.dist.all_reduce(base, op=self.dist.ReduceOp.SUM, group=self.group)
         return base
+
+    def leaf_loads(self, Q, k: int, **kw):
+        """Per-leaf work of a (sample) batch on the whole sharded index: sum of |A(q)| over
+        the queries routed to each leaf (this rank's leaves from its own answers, the rest
+        from the other ranks: SUM all-reduce).  Feeds balanced_leaf_split."""
+        import numpy as np
+        import torch
+        self.index.query_packed(Q, k, keep_stages=True, **kw)
+        leaf = self.index.export("Q_LEAF")
+        nc = self.index.export("Q_BASE") if not kw.get("hierarchy") else None
+        if nc is None:
+            raise ValueError("leaf_loads: use a probe configuration without the hierarchy")
+        G = int(self.index.info().G)
+        loads = np.bincount(leaf, weights=nc.astype(np.float64), minlength=G).astype(np.int64)
+        t = torch.from_numpy(loads)
+        if torch.cuda.is_available():
+            t = t.cuda()
+        if self.world > 1:
+            self.dist.all_reduce(t, op=self.dist.ReduceOp.SUM, group=self.group)
+        return t.cpu().numpy()
 
     def load_stats(self, ncand=None):
         """Per-rank load of the last query (SURVEY §8(e) scaling risk: query skew across

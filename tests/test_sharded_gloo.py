@@ -137,3 +137,25 @@ def test_leaf_range_partition():
         assert len({h - l for l, h in got}) == 1
     with pytest.raises(ValueError):
         leaf_range(64, 0, 3)
+
+
+def test_balanced_leaf_split_is_optimal():
+    """balanced_leaf_split = the best contiguous partition (brute force over all of them)."""
+    import itertools
+    from paper_conf_icde_panm12_b200.sharded import balanced_leaf_split
+    rng = np.random.default_rng(2)
+    for _ in range(60):
+        G = int(rng.integers(1, 9))
+        world = int(rng.integers(1, 5))
+        w = rng.integers(0, 50, G).tolist()
+        b = balanced_leaf_split(w, world)
+        assert len(b) == world + 1 and b[0] == 0 and b[-1] == G and all(x <= y for x, y in zip(b, b[1:]))
+        got = max(sum(w[b[r]:b[r + 1]]) for r in range(world))
+        best = None
+        for cuts in itertools.combinations_with_replacement(range(G + 1), world - 1):
+            bb = [0, *cuts, G]
+            m = max(sum(w[bb[r]:bb[r + 1]]) for r in range(world))
+            best = m if best is None else min(best, m)
+        assert got == best
+    # a skewed batch: the hot leaf gets a rank of its own
+    assert balanced_leaf_split([100, 1, 1, 1, 1, 1, 1, 1], 2) == [0, 1, 8]
