@@ -72,7 +72,7 @@ def lib():
         L.orc_diameter_estimate.restype = f32
         L.orc_diameter_estimate.argtypes = [P, i32, P, i64, i32, P, P]
         L.orc_build.restype = P
-        L.orc_build.argtypes = [P, i64, i32, i32, i32, i32, f32, P, i32, f64, f64, i32, u64, i32,
+        L.orc_build.argtypes = [P, i64, i32, i32, i32, i32, f32, P, i32, f64, f64, i32, u64, i32, i32,
                                 C.POINTER(C.c_int)]
         L.orc_free.restype = None
         L.orc_free.argtypes = [P]
@@ -304,7 +304,7 @@ class OracleIndex:
 
     def __init__(self, X, G: int, M: int = 8, W: float = 4.0, seed: int = 42, quantizer: int = 0,
                  W_leaf=None, rp_rule: int = 0, rp_mean_c: float = 10.0,
-                 rp_max_jitter: float = 0.0, ek_iters: int = 40, L: int = 1):
+                 rp_max_jitter: float = 0.0, ek_iters: int = 40, L: int = 1, W_rule: int = 0):
         """L > 1: L independent hash tables over the same RP-tree; table l
         is the single-table index built with table = l (its own (a, b))."""
         self.X = _f32(X)
@@ -315,7 +315,7 @@ class OracleIndex:
             err = C.c_int(0)
             h = lib().orc_build(_p(self.X), n, d, G, M, quantizer, float(W),
                                 _p(Wl) if Wl is not None else None, rp_rule, float(rp_mean_c),
-                                float(rp_max_jitter), ek_iters, seed, l, C.byref(err))
+                                float(rp_max_jitter), ek_iters, seed, l, W_rule, C.byref(err))
             if not h:
                 self.close()
                 raise OracleError(f"orc_build failed (code {err.value})", err.value)

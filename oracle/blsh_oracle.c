@@ -737,11 +737,13 @@ static int orc_entry_cmp(const void *pa, const void *pb)
  * *err: 1 invalid argument, 4 code outside the Morton range (R9). */
 orc_index *orc_build(const float *X, int64_t n, int d, int G, int M, int quantizer, float W,
                      const float *Wleaf, int rp_rule, double rp_mean_c, double rp_max_jitter,
-                     int ek_iters, uint64_t seed, int table, int *err)
+                     int ek_iters, uint64_t seed, int table, int W_rule, int *err)
 {
     *err = 1;
     if (n < 0 || d < 1 || G < 1 || G > 4096 || (G & (G - 1)) || M < 1 || M > 16) return NULL;
     if (table < 0 || table > 255) return NULL;
+    if (W_rule != 0 && W_rule != 1) return NULL;
+    if (W_rule == 1 && Wleaf) return NULL;
     if (quantizer == 1 && M != 8 && M != 16) return NULL;   /* ceil(M/8) E8 blocks, R28 */
     if (!(W > 0.0f)) return NULL;
     orc_index *ix = (orc_index *)calloc(1, sizeof(orc_index));
@@ -797,6 +799,44 @@ orc_index *orc_build(const float *X, int64_t n, int d, int G, int M, int quantiz
     ix->leaf = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     for (int g = 0; g < G; g++)
         for (int64_t i = seg[g]; i < seg[g + 1]; i++) ix->leaf[order[i]] = g;
+
+    /* P:107 "different LSH parameters (e.g. bucket size W) ... for each cell"
+     * (R29): W_g = fp32(W sqrt(D_g / D_med)), D_g = Delta_A^2 of leaf g with
+     * the R7 reductions (members in ascending id), D_med = lower median of the
+     * D_g; W_g = W when D_g = 0.  (a, b) are redrawn with the new widths. */
+    if (W_rule == 1) {
+        double *D = (double *)calloc((size_t)G, sizeof(double));
+        double *tot = (double *)malloc(sizeof(double) * (size_t)d);
+        float *mu = (float *)malloc(sizeof(float) * (size_t)d);
+        for (int g = 0; g < G; g++) {
+            int64_t nS = seg[g + 1] - seg[g];
+            if (nS == 0) continue;
+            const int64_t *S = order + seg[g];
+            orc_chunked_colsum(X, d, S, nS, tot);
+            for (int j = 0; j < d; j++) mu[j] = (float)(tot[j] / (double)nS);
+            float *e = (float *)malloc(sizeof(float) * (size_t)nS);
+            for (int64_t i = 0; i < nS; i++) e[i] = orc_dist2c(X + S[i] * (int64_t)d, mu, d);
+            D[g] = 2.0 * orc_chunked_sum_vals(e, nS) / (double)nS;
+            free(e);
+        }
+        double *srt = (double *)malloc(sizeof(double) * (size_t)G);
+        memcpy(srt, D, sizeof(double) * (size_t)G);
+        for (int a = 1; a < G; a++) {          /* insertion sort: G <= 4096 */
+            double v = srt[a];
+            int b = a - 1;
+            while (b >= 0 && srt[b] > v) { srt[b + 1] = srt[b]; b--; }
+            srt[b + 1] = v;
+        }
+        double med = srt[(G - 1) / 2];
+        for (int g = 0; g < G; g++) {
+            float wg = (D[g] > 0.0 && med > 0.0) ? (float)((double)W * sqrt(D[g] / med)) : W;
+            if (!(wg > 0.0f) || !isfinite(wg)) wg = W;
+            ix->Wl[g] = wg;
+        }
+        orc_gen_params(seed, G, M, d, ix->Wl, ix->A, ix->b, ix->dirs, ix->jit);
+        if (table > 0) orc_gen_table_params(seed, table, G, M, d, ix->Wl, ix->A, ix->b);
+        free(D); free(tot); free(mu); free(srt);
+    }
     free(tmp); free(s); free(seg); free(nseg); free(order);
 
     /* b3: hash every point with its leaf's parameters */
