@@ -77,6 +77,11 @@ typedef struct {
                                query skew across leaves); leaf_split[0] = 0, leaf_split[world] = G,
                                non-decreasing, identical on every rank.  NULL = G/world leaves each
                                (then world must divide G).                                                */
+    int32_t W_rule;         /* 0 = W (or W_leaf) for every leaf; 1 = per-leaf width adapted to the leaf's
+                               spread ("different LSH parameters (e.g. bucket size W) that are optimal
+                               for each cell"; R29): W_g = fp32(W * sqrt(D_g / D_med)), D_g = Delta_A^2 of
+                               leaf g (R7), D_med = the lower median of D over the leaves; W_g = W for leaves
+                               with D_g = 0.  Exported as BLSH_EX_W.  Excludes W_leaf.                       */
 } blsh_build_params;
 
 /* Query parameters.  Defaults: blsh_query_params_default(). */

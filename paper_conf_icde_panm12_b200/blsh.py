@@ -31,7 +31,8 @@ class BuildParams(C.Structure):
                 ("rp_max_jitter", C.c_double), ("ek_iters", C.c_int32), ("M", C.c_int32),
                 ("quantizer", C.c_int32), ("W", C.c_float), ("W_leaf", C.c_void_p), ("seed", C.c_uint64),
                 ("rank", C.c_int32), ("world", C.c_int32), ("stream", C.c_void_p),
-                ("keep_stages", C.c_int32), ("n_tables", C.c_int32), ("leaf_split", C.c_void_p)]
+                ("keep_stages", C.c_int32), ("n_tables", C.c_int32), ("leaf_split", C.c_void_p),
+                ("W_rule", C.c_int32)]
 
 
 class QueryParams(C.Structure):
@@ -158,7 +159,7 @@ def _f32(a):
 def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42, quantizer: int = 0,
                rp_rule: int = 0, rp_mean_c: float = 10.0, rp_max_jitter: float = 0.0, ek_iters: int = 40,
                W_leaf=None, rank: int = 0, world: int = 1, keep_stages: bool = False,
-               n_tables: int = 1, leaf_split=None) -> "Index":
+               n_tables: int = 1, leaf_split=None, W_rule: int = 0) -> "Index":
     X = _f32(X)
     n, d = int(X.shape[0]), int(X.shape[1])
     p = BuildParams()
@@ -167,6 +168,7 @@ def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42,
     p.rp_rule, p.rp_mean_c, p.rp_max_jitter, p.ek_iters = rp_rule, rp_mean_c, rp_max_jitter, ek_iters
     p.rank, p.world, p.keep_stages = rank, world, int(bool(keep_stages))
     p.n_tables = n_tables
+    p.W_rule = W_rule
     ls = None
     if leaf_split is not None:   # load-aware contiguous leaf -> rank assignment [world+1]
         ls = np.ascontiguousarray(np.asarray(leaf_split, dtype=np.int32))

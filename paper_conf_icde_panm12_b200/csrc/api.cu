@@ -138,6 +138,8 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         return fail(BLSH_ERR_INVALID, "world must divide n_leaves (or pass leaf_split)");
     }
     if (p->n_tables < 1 || p->n_tables > 64) return fail(BLSH_ERR_INVALID, "n_tables must be in [1, 64]");
+    if (p->W_rule != 0 && p->W_rule != 1) return fail(BLSH_ERR_INVALID, "W_rule must be 0 or 1");
+    if (p->W_rule == 1 && p->W_leaf) return fail(BLSH_ERR_INVALID, "W_rule = 1 derives the per-leaf widths (no W_leaf)");
     if (p->W_leaf)
         for (int g = 0; g < G; ++g)
             if (!(p->W_leaf[g] > 0.0f) || !std::isfinite(p->W_leaf[g])) return fail(BLSH_ERR_INVALID, "W_leaf must be > 0");
@@ -199,6 +201,25 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         order.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(uint32_t));
         std::vector<int64_t> seg;
         blsh::build_rptree(*ix, Xs.as<float>(), order.as<uint32_t>(), seg, s);
+        if (p->W_rule == 1) {
+            // P:107 / R29: per-leaf widths from the leaves' spread, then (a, b) redrawn with them
+            // (b = W_g U depends on W_g; a and the tree do not)
+            blsh::leaf_spread(*ix, Xs.as<float>(), order.as<uint32_t>(), seg, ix->leaf_da2_h, s);
+            std::vector<double> srt(ix->leaf_da2_h);
+            std::sort(srt.begin(), srt.end());
+            const double med = srt[(G - 1) / 2];
+            for (int g = 0; g < G; ++g) {
+                const double dg = ix->leaf_da2_h[g];
+                ix->W_h[g] = (dg > 0.0 && med > 0.0) ? (float)((double)p->W * std::sqrt(dg / med)) : p->W;
+                if (!(ix->W_h[g] > 0.0f) || !std::isfinite(ix->W_h[g])) ix->W_h[g] = p->W;
+            }
+            blsh::gen_params(p->seed, G, M, d, ix->W_h.data(), ix->A_h.data(), ix->b_h.data(), ix->dirs_h.data(),
+                             ix->jit_h.data());
+            BLSH_CUDA(cudaMemcpyAsync(ix->A.p, ix->A_h.data(), ix->A_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+            BLSH_CUDA(cudaMemcpyAsync(ix->b.p, ix->b_h.data(), ix->b_h.size() * sizeof(float), cudaMemcpyHostToDevice, s));
+            BLSH_CUDA(cudaMemcpyAsync(ix->W.p, ix->W_h.data(), G * sizeof(float), cudaMemcpyHostToDevice, s));
+            BLSH_CUDA(cudaStreamSynchronize(s));
+        }
         const int64_t pos_lo = seg[ix->leaf_lo], pos_hi = seg[ix->leaf_hi];
         const int64_t no = pos_hi - pos_lo;
         ix->n_owned = no;

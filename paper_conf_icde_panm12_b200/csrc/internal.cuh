@@ -156,6 +156,7 @@ struct blsh_index {
     std::vector<float> A_h, b_h, W_h, dirs_h, mu_h, theta_h;
     std::vector<int32_t> ntype_h;
     std::vector<double> diam2_h, da2_h, jit_h;
+    std::vector<double> leaf_da2_h;    // [G] W rule 1: Delta_A^2 of every leaf (R29)
     std::vector<int64_t> leaf_u_h;     // [G+1]
     // device: parameters and tree
     blsh::DevBuf A, b, W, dirs, mu, theta, ntype;
@@ -203,6 +204,11 @@ void gen_table_params(uint64_t seed, int table, int G, int M, int d, const float
 // seg [G+1] (host).
 void build_rptree(blsh_index& ix, const float* Xs, uint32_t* order_dev,
                   std::vector<int64_t>& seg, cudaStream_t s);
+
+// Delta_A^2 of every leaf (R7 reductions over the members in ascending id), for
+// the per-leaf W rule (R29).
+void leaf_spread(const blsh_index& ix, const float* Xs, const uint32_t* order, const std::vector<int64_t>& seg,
+                 std::vector<double>& da2_out, cudaStream_t s);
 
 // Hash the points order[lo..hi) (grouped by leaf) with their leaf's params;
 // writes sort entries; returns false when a code leaves the Morton range.

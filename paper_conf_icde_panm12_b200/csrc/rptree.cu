@@ -595,4 +595,52 @@ void build_rptree(blsh_index& ix, const float* Xs, uint32_t* order_dev, std::vec
         for (int j = 0; j < d; ++j) ix.mu_h[(size_t)v * d + j] = mup[(size_t)v * ds + j];
 }
 
+// Per-leaf spread for the W rule of P:107 (reading R29): Delta_A^2(g) =
+// 2 sum dist2c(x, mu_g) / |g| over the leaf's members in ascending id, with the
+// same R7 reductions (chunks of 4096, fp64, in order) as the tree's nodes.
+void leaf_spread(const blsh_index& ix, const float* Xs, const uint32_t* order, const std::vector<int64_t>& seg,
+                 std::vector<double>& da2_out, cudaStream_t s) {
+    const int G = ix.G, d = ix.d, ds = ix.ds;
+    da2_out.assign(G, 0.0);
+    std::vector<Tile> tiles;
+    std::vector<Chunk> chunks;
+    std::vector<int64_t> chunk_off(G + 1, 0), nsz(G);
+    for (int k = 0; k < G; ++k) {
+        const int64_t a = seg[k], e = seg[k + 1];
+        nsz[k] = e - a;
+        for (int64_t p = a; p < e; p += kTR) tiles.push_back(Tile{k, (int32_t)std::min<int64_t>(kTR, e - p), p});
+        chunk_off[k] = (int64_t)chunks.size();
+        for (int64_t p = a; p < e; p += kChunk) chunks.push_back(Chunk{k, (int32_t)std::min<int64_t>(kChunk, e - p), p});
+    }
+    chunk_off[G] = (int64_t)chunks.size();
+    const int ntiles = (int)tiles.size(), nchunks = (int)chunks.size();
+    if (ntiles == 0) return;
+    DevBuf tiles_d, chunks_d, chunk_off_d, nsz_d, part, mu, vals, csum, da;
+    upload(tiles_d, tiles, s);
+    upload(chunks_d, chunks, s);
+    upload(chunk_off_d, chunk_off, s);
+    upload(nsz_d, nsz, s);
+    part.alloc((size_t)nchunks * d * sizeof(double));
+    mu.alloc((size_t)G * ds * sizeof(float));
+    BLSH_CUDA(cudaMemsetAsync(mu.p, 0, (size_t)G * ds * sizeof(float), s));
+    vals.alloc((size_t)std::max<int64_t>(ix.n, 1) * sizeof(float));
+    csum.alloc((size_t)nchunks * sizeof(double));
+    da.alloc((size_t)G * sizeof(double));
+    k_colsum<<<dim3(nchunks, (d + 127) / 128), 128, 0, s>>>(Xs, ds, d, order, chunks_d.as<Chunk>(), part.as<double>());
+    BLSH_LAUNCH_CHECK();
+    k_mean_final<<<dim3(G, (d + 127) / 128), 128, 0, s>>>(part.as<double>(), chunk_off_d.as<int64_t>(),
+                                                          nsz_d.as<int64_t>(), 0, d, ds, mu.as<float>());
+    BLSH_LAUNCH_CHECK();
+    k_rowchain<RC_DIST><<<ntiles, kTR, 0, s>>>(Xs, ds, d, order, tiles_d.as<Tile>(), mu.as<float>(), nullptr, nullptr,
+                                               nullptr, vals.as<float>());
+    BLSH_LAUNCH_CHECK();
+    k_chunksum<<<(nchunks + 127) / 128, 128, 0, s>>>(vals.as<float>(), chunks_d.as<Chunk>(), nchunks, csum.as<double>());
+    BLSH_LAUNCH_CHECK();
+    k_da_final<<<(G + 127) / 128, 128, 0, s>>>(csum.as<double>(), chunk_off_d.as<int64_t>(), nsz_d.as<int64_t>(), G,
+                                               da.as<double>());
+    BLSH_LAUNCH_CHECK();
+    BLSH_CUDA(cudaMemcpyAsync(da2_out.data(), da.p, G * sizeof(double), cudaMemcpyDeviceToHost, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+}
+
 }  // namespace blsh

@@ -58,3 +58,23 @@ def test_leaf_split_validation(blsh):
         blsh.blsh_build(Xd, n_leaves=4, rank=0, world=2, leaf_split=[0, 3, 2])    # decreasing
     with pytest.raises(blsh.BlshError):
         blsh.blsh_build(Xd, n_leaves=4, rank=0, world=2, leaf_split=[1, 2, 4])    # not from 0
+
+
+@pytest.mark.parametrize("G,L", [(4, 1), (8, 1), (4, 3)])
+def test_w_rule_parity(blsh, orc, G, L):
+    """W_rule = 1 (R29): per-leaf widths, redrawn (a, b), tables and queries bit-exact."""
+    from parity_utils import check_topk
+    X, Q = synth.make_dataset(synth.CONFIGS["c1"])
+    ix = blsh.blsh_build(torch.from_numpy(X).cuda(), n_leaves=G, M=8, W=3.0, seed=5, W_rule=1, n_tables=L,
+                         keep_stages=True)
+    ox = orc.OracleIndex(X, G=G, M=8, W=3.0, seed=5, W_rule=1, L=L)
+    assert np.array_equal(ix.export("W").view(np.uint32), ox.get("W").view(np.uint32)), "per-leaf W differs"
+    assert len(set(ix.export("W").tolist())) > 1
+    for l in range(L):
+        for a, b in [("A", "A"), ("B", "b"), ("PERM", "perm"), ("UKEY", "ukey"), ("UOFF", "uoff")]:
+            assert np.array_equal(ix.export(a, table=l).view(np.uint8), ox.get(b, l).ravel().view(np.uint8)), a
+    ids, d2, nc = ix.query(torch.from_numpy(Q).cuda(), 10, probe=1, n_probes=8)
+    torch.cuda.synchronize()
+    oi, od, onc = ox.query(Q, 10, probe=1, T=8)
+    assert np.array_equal(nc.cpu().numpy(), onc)
+    check_topk(ids.cpu().numpy(), d2.cpu().numpy(), oi, od, X, Q, cands=ox.candidates())
