@@ -11,6 +11,8 @@
 // a warp-distributed sorted top-k of packed (d^2 bits << 32 | id) keys (lane l
 // holds entries l and l+32).  Results per item go to a private slot, so the
 // outcome never depends on scheduling.
+#include <algorithm>
+
 #include "internal.cuh"
 #include "query_kernels.cuh"
 
@@ -49,11 +51,17 @@ __device__ __forceinline__ void topk_insert(TopK& t, unsigned long long v, int l
 // a.list[a.list_off[q] ..] that k_union_tables wrote (ascending positions).
 // The distance arithmetic is the same in every mode (R22), so the modes agree
 // bit for bit.
+constexpr int kRG = 4;   // rows per distance group (loads in flight per lane: kRG x NV float4)
+
 template <int NV, bool EMIT, bool LIST>
 __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int lane = threadIdx.x & 31;
-    const int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5);
-    if (item >= a.n_items) return;
+    // grid-stride over the work items (a warp takes the next item as soon as it is done:
+    // items differ in length, and a block would otherwise hold its slot until its slowest warp ends)
+    // (list mode; the interval mode keeps one item per warp: neighbouring items, which share
+    // rows in L2, then run together)
+    for (int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5); item < a.n_items;
+         item += LIST ? (int64_t)gridDim.x * kSLWarps : a.n_items) {
     // query of this item: last q with item_off[q] <= item
     int64_t lo = 0, hi = a.nq;
     while (hi - lo > 1) {
@@ -76,10 +84,10 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int k = a.k;
     unsigned long long thr = kEmpty;
     // Rows r[0..nr) (table positions) that are candidates c, c+1, .. of q.
-    auto group = [&](const int64_t (&r)[4], int nr, int64_t c) {
-        float part[4];
+    auto group = [&](const int64_t (&r)[kRG], int nr, int64_t c) {
+        float part[kRG];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < kRG; ++j) {
             part[j] = 0.0f;
             if (j < nr) {
                 const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
@@ -100,23 +108,23 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) part[j] += __shfl_xor_sync(BLSH_FULL, part[j], o);
+            for (int j = 0; j < kRG; ++j) part[j] += __shfl_xor_sync(BLSH_FULL, part[j], o);
         }
         int64_t rl = r[0];
 #pragma unroll
-        for (int j = 1; j < 4; ++j) rl = lane == j ? r[j] : rl;
+        for (int j = 1; j < kRG; ++j) rl = lane == j ? r[j] : rl;
         const uint32_t idl = (lane < nr) ? __ldg(a.perm + rl) : 0u;
         if (EMIT) {
             if (lane < nr) {
                 float pj = part[0];
 #pragma unroll
-                for (int j = 1; j < 4; ++j) pj = lane == j ? part[j] : pj;
+                for (int j = 1; j < kRG; ++j) pj = lane == j ? part[j] : pj;
                 a.cand_keys[a.cand_off[q] + c + lane] = pack_entry(pj, idl);
             }
             return;
         }
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < kRG; ++j) {
             const uint32_t id = __shfl_sync(BLSH_FULL, idl, j);
             if (j < nr) {
                 const unsigned long long key = pack_entry(part[j], id);
@@ -129,11 +137,11 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     };
     if (LIST) {
         const uint32_t* L = a.list + a.list_off[q];
-        for (int64_t c = c0; c < c1; c += 4) {
-            const int nr = (int)min((int64_t)4, c1 - c);
-            int64_t r[4];
+        for (int64_t c = c0; c < c1; c += kRG) {
+            const int nr = (int)min((int64_t)kRG, c1 - c);
+            int64_t r[kRG];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) r[j] = j < nr ? (int64_t)__ldg(L + c + j) : 0;
+            for (int j = 0; j < kRG; ++j) r[j] = j < nr ? (int64_t)__ldg(L + c + j) : 0;
             group(r, nr, c);
         }
     } else {
@@ -146,19 +154,23 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
             const int64_t s = max(c0, acc), e = min(c1, acc + len);
             if (s < e) {
                 const int64_t pa = (int64_t)iv.x + (s - acc), pb = (int64_t)iv.x + (e - acc);
-                for (int64_t r0 = pa; r0 < pb; r0 += 4) {
-                    const int nr = (int)min((int64_t)4, pb - r0);
-                    const int64_t r[4] = {r0, r0 + 1, r0 + 2, r0 + 3};
+                for (int64_t r0 = pa; r0 < pb; r0 += kRG) {
+                    const int nr = (int)min((int64_t)kRG, pb - r0);
+                    int64_t r[kRG];
+#pragma unroll
+                    for (int j = 0; j < kRG; ++j) r[j] = r0 + j;
                     group(r, nr, acc + (r0 - (int64_t)iv.x));
                 }
             }
             acc += len;
         }
     }
-    if (EMIT) return;
-    unsigned long long* out = a.partials + (size_t)item * k;
-    if (lane < k) out[lane] = tk.e0;
-    if (lane + 32 < k) out[lane + 32] = tk.e1;
+    if (!EMIT) {
+        unsigned long long* out = a.partials + (size_t)item * k;
+        if (lane < k) out[lane] = tk.e0;
+        if (lane + 32 < k) out[lane + 32] = tk.e1;
+    }
+    }   // item loop
 }
 
 __global__ void k_items(const int64_t* __restrict__ cnt, int64_t nq, int chunk, int64_t* __restrict__ items) {
@@ -394,7 +406,8 @@ void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cud
 
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     if (a.n_items == 0) return;
-    const unsigned grid = (unsigned)((a.n_items + kSLWarps - 1) / kSLWarps);
+    const int64_t blocks = (a.n_items + kSLWarps - 1) / kSLWarps;
+    const unsigned grid = (unsigned)(a.list ? std::min<int64_t>(blocks, 148 * 8) : blocks);
     const int nvl = ((a.ds >> 2) + 31) / 32;
 
 #define BLSH_SL_CASE(V)                                                                             \
