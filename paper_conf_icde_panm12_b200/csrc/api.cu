@@ -459,7 +459,17 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         al.pvalid = t.pvalid; al.ivl = t.ivl; al.base = t.base; al.cnt = t.cnt; al.level = nullptr;
         return al;
     };
-    for (int l = 1; l < L; ++l) { launch_hash(table_args(l), s); ++launches; }
+    if (L > 1) {   // tables 1..L-1: one launch
+        HashTables ht{};
+        ht.n = L - 1;
+        for (int l = 1; l < L; ++l) {
+            const QueryArgs al = table_args(l);
+            ht.A[l - 1] = al.A; ht.b[l - 1] = al.bvec; ht.qt[l - 1] = al.qt; ht.qcode[l - 1] = al.qcode;
+            ht.qoor[l - 1] = al.qoor; ht.qkey[l - 1] = al.qkey;
+        }
+        launch_hash_tables(a, ht, s);
+        ++launches;
+    }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // a3+a4
     launch_probe_lookup(a, s); ++launches;

@@ -144,8 +144,7 @@ __global__ void k_leaf_scatter(const int32_t* __restrict__ qleaf, int64_t nq, in
 }
 
 template <int MM>
-__global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __restrict__ lperm) {
-    extern __shared__ __align__(16) float rh_rows[];
+__device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __restrict__ lperm, float* rh_rows) {
     const int lane = threadIdx.x;
     const int64_t p0 = blockIdx.x * (int64_t)kRHQ;
     const int nrow = (int)min((int64_t)kRHQ, a.nq - p0);
@@ -193,6 +192,23 @@ __global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __re
     a.qoor[q] = ok ? 0 : 1;
     a.qkey[q] = morton_key(code, MM, a.B);   // clamped home key (hierarchy uses it)
     if (!active) a.qoor[q] |= 2;
+}
+
+template <int MM>
+__global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __restrict__ lperm) {
+    extern __shared__ __align__(16) float rh_rows[];
+    hash_body<MM>(a, lperm, rh_rows);
+}
+
+// a2 of hash tables 1..L-1 in one launch (blockIdx.y = table - 1): the tables'
+// blocks run together instead of one latency-bound launch per table.
+template <int MM>
+__global__ void __launch_bounds__(kRHQ) k_hash_tables(QueryArgs a, const __grid_constant__ HashTables ht) {
+    extern __shared__ __align__(16) float rh_rows[];
+    const int t = blockIdx.y;
+    QueryArgs b = a;
+    b.A = ht.A[t]; b.bvec = ht.b[t]; b.qt = ht.qt[t]; b.qcode = ht.qcode[t]; b.qoor = ht.qoor[t]; b.qkey = ht.qkey[t];
+    hash_body<MM>(b, a.lperm, rh_rows);
 }
 
 // ---------------------------------------------------------------------------
@@ -743,6 +759,26 @@ void launch_hash(const QueryArgs& a, cudaStream_t s) {
         default: throw Error(BLSH_ERR_INVALID, "M out of range");
     }
 #undef BLSH_H_CASE
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_hash_tables(const QueryArgs& a, const HashTables& ht, cudaStream_t s) {
+    if (a.nq == 0 || ht.n == 0) return;
+    const dim3 grid((unsigned)((a.nq + kRHQ - 1) / kRHQ), (unsigned)ht.n);
+    const size_t smem_h = (a.rh_direct ? 0 : (size_t)kRHQ * (a.ds + 4) * sizeof(float)) + (size_t)a.M * a.d * sizeof(float);
+#define BLSH_HT_CASE(MMV)                                                                                     \
+    case MMV:                                                                                                \
+        BLSH_CUDA(cudaFuncSetAttribute(k_hash_tables<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        k_hash_tables<MMV><<<grid, kRHQ, smem_h, s>>>(a, ht);                                                 \
+        break;
+    switch (a.M) {
+        BLSH_HT_CASE(1) BLSH_HT_CASE(2) BLSH_HT_CASE(3) BLSH_HT_CASE(4)
+        BLSH_HT_CASE(5) BLSH_HT_CASE(6) BLSH_HT_CASE(7) BLSH_HT_CASE(8)
+        BLSH_HT_CASE(9) BLSH_HT_CASE(10) BLSH_HT_CASE(11) BLSH_HT_CASE(12)
+        BLSH_HT_CASE(13) BLSH_HT_CASE(14) BLSH_HT_CASE(15) BLSH_HT_CASE(16)
+        default: throw Error(BLSH_ERR_INVALID, "M out of range");
+    }
+#undef BLSH_HT_CASE
     BLSH_LAUNCH_CHECK();
 }
 

@@ -47,6 +47,18 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s);   // returns kernels 
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s);
 // a2 only (queries already routed and grouped by leaf in a.lperm): hash with a.A / a.bvec
 void launch_hash(const QueryArgs& a, cudaStream_t s);
+// a2 of several hash tables in one launch (tables 1..L-1 of an L-table index)
+constexpr int kMaxTables = 64;
+struct HashTables {
+    int n;
+    const float* A[kMaxTables];
+    const float* b[kMaxTables];
+    float* qt[kMaxTables];
+    int32_t* qcode[kMaxTables];
+    int32_t* qoor[kMaxTables];
+    Key128* qkey[kMaxTables];
+};
+void launch_hash_tables(const QueryArgs& a, const HashTables& ht, cudaStream_t s);
 
 // L > 1 tables (tables.cu): raw[q] = sum over tables of |A0_l(q)|, then the
 // deduplicated union of the L tables' intervals as ascending table-0 positions.
