@@ -336,11 +336,23 @@ __device__ void block_select_write(const SelSrc& src, int k, int64_t q, int64_t*
     for (int i = tid; i < kSelCap; i += kSelThreads) buf[i] = kEmpty;   // (only the sorted prefix is read)
     __syncthreads();
     const bool take_all = len <= k;
-    for (int64_t i = tid; i < len; i += kSelThreads) {
-        const unsigned long long v = src.get(i);
-        if (take_all || v <= thr_le) {
-            const int slot = atomicAdd(&s_cnt, 1);
-            if (slot < kSelCap) buf[slot] = v;
+    if (take_all) {   // every key is selected: position = index, no counter
+        for (int64_t i = tid; i < len; i += kSelThreads) buf[i] = src.get(i);
+        if (tid == 0) s_cnt = (int)len;
+    } else {          // warp-aggregated slots: one shared atomic per warp and pass
+        const int lane = tid & 31;
+        for (int64_t b0 = 0; b0 < len; b0 += kSelThreads) {
+            const int64_t i = b0 + tid;
+            const unsigned long long v = i < len ? src.get(i) : kEmpty;
+            const bool take = i < len && v <= thr_le;
+            const unsigned m = __ballot_sync(BLSH_FULL, take);
+            int base = 0;
+            if (lane == 0 && m) base = atomicAdd(&s_cnt, __popc(m));
+            base = __shfl_sync(BLSH_FULL, base, 0);
+            if (take) {
+                const int slot = base + __popc(m & lanemask_lt());
+                if (slot < kSelCap) buf[slot] = v;
+            }
         }
     }
     __syncthreads();
