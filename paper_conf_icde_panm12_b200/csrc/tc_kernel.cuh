@@ -600,7 +600,10 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
             for (int base = 0; base < cnt; base += 32) {
                 const int i = base + lane;
                 const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
-                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+                // the k-th exact distance found so far bounds the final one too: once the list is
+                // full, pairs whose lower bound exceeds it are skipped (ties: <= keeps them)
+                const float dk = thr == kEmpty ? U : fminf(U, __uint_as_float((uint32_t)(thr >> 32)));
+                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= dk;
                 const unsigned nm = __ballot_sync(BLSH_FULL, need);
                 rescored += __popc(nm);
                 score_rows(nm, (uint32_t)(e & 0xFFFFFFFFull));
