@@ -471,6 +471,16 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         ++launches;
     }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
+    // query-tiled short-list ahead: fork the query sort + tile formation (a1/a2 outputs only)
+    const int kind_pre = (list_path || out_base) ? 0 : shortlist_kind(ds, T, k);
+    if (kind_pre > 0) {
+        if (!w.side) {
+            BLSH_CUDA(cudaStreamCreateWithFlags(&w.side, cudaStreamNonBlocking));
+            BLSH_CUDA(cudaEventCreateWithFlags(&w.ev_fork, cudaEventDisableTiming));
+            BLSH_CUDA(cudaEventCreateWithFlags(&w.ev_join, cudaEventDisableTiming));
+        }
+        BLSH_CUDA(cudaEventRecord(w.ev_fork, s));
+    }
     // a3+a4
     launch_probe_lookup(a, s); ++launches;
     for (int l = 1; l < L; ++l) { launch_probe_lookup(table_args(l), s); ++launches; }
@@ -532,13 +542,21 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         launch_union_tables(u, ix.max_leaf_rows, s); ++launches;
     }
     w.list_valid = list_path;
+    int64_t ntiles_pre = 0;
+    if (kind_pre > 0) {   // side stream, overlapping a3/a4 already queued on s
+        BLSH_CUDA(cudaStreamWaitEvent(w.side, w.ev_fork, 0));
+        sort_queries(a, w.qsort, qorder, w.side, &launches);
+        ntiles_pre = plan_tiles(a, qorder, w.tilebuf, w.scan2, w.side, &launches);
+        BLSH_CUDA(cudaEventRecord(w.ev_join, w.side));
+        BLSH_CUDA(cudaStreamWaitEvent(s, w.ev_join, 0));
+    }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[3], s));
     // plan: chunking of the candidate lists
     scan_exclusive_i64(w.cnt, cand_off, nq, w.scan, s); launches += 3;
     int64_t total = 0;
     BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    const int kind = list_path ? 0 : shortlist_kind(ds, T, k);   // lists: warp short-list over the positions
+    const int kind = kind_pre;   // lists: warp short-list over the positions
     const bool tiled = kind > 0;
     int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0;
     double qload_rows = 0.0;
@@ -546,12 +564,11 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t ch = 0;
     if (tiled) {
         // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
-        sort_queries(a, w.qsort, qorder, s, &launches);
         int chr = 0;
         run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
                             tm ? ix.ev[4] : nullptr, tm ? ix.ev[8] : nullptr, tm ? ix.ev[5] : nullptr, &pairs,
-                            &kept, &qload_rows, kind);
+                            &kept, &qload_rows, kind, ntiles_pre);
         ch = chr;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {

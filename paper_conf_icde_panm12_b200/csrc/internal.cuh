@@ -123,6 +123,18 @@ struct QueryWork {
     DevBuf listbuf;               // deduplicated candidate positions (u32), at raw_off[q]
     int64_t* raw_off = nullptr;   // [nq+1] scan of the per-query sums of the table counts
     bool list_valid = false;      // the last query built candidate lists (listbuf / raw_off / cnt)
+    // side stream: the query sort and tile formation run while a3/a4 run on the caller's stream
+    ScanTemp scan2;
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    QueryWork() = default;
+    QueryWork(const QueryWork&) = delete;
+    QueryWork& operator=(const QueryWork&) = delete;
+    ~QueryWork() {
+        if (ev_fork) cudaEventDestroy(ev_fork);
+        if (ev_join) cudaEventDestroy(ev_join);
+        if (side) cudaStreamDestroy(side);
+    }
 };
 
 // Hash table l >= 1 of an L-table index.  Table 0 is the primary

@@ -132,12 +132,14 @@ struct ShortlistArgs {
 // BLSH_SHORTLIST=warp|simt forces the others.
 int shortlist_kind(int ds, int T, int k);
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
+int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, ScanTemp& scan, cudaStream_t s,
+                   int* launches);
 void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
                          cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
-                         int64_t* kept_out, double* qload_rows_out, int kind);
+                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles);
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s);
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s);

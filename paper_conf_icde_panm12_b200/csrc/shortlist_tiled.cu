@@ -580,15 +580,12 @@ void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream
     BLSH_CUDA(cudaMemcpyAsync(qorder, sb.id[cur].p, (size_t)nq * 4, cudaMemcpyDeviceToDevice, s));
 }
 
-void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
-                         DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
-                         unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
-                         cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
-                         cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
-                         int64_t* kept_out, double* qload_rows_out, int kind) {
+// Query tiles (DESIGN §7 "Tiling"): consecutive sorted queries cut at leaf changes and
+// large jumps.  Needs only a1/a2 outputs, so run_query issues it on a side stream while
+// a3/a4 run; returns the tile count (host-synchronised on `s`).
+int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, ScanTemp& scan, cudaStream_t s,
+                   int* launches) {
     const int64_t nq = a.nq;
-    const int T = a.T;
-    const int segcap = 2 * QT * (T + 1);
     // tile arrays are sized for the worst case (one query per tile)
     const size_t slot = (((size_t)(nq + 1) * 8) + 255) & ~size_t(255);
     tilebuf.ensure(slot * 13 + 256);
@@ -627,6 +624,23 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int64_t ntiles = 0;
     BLSH_CUDA(cudaMemcpyAsync(&ntiles, fexcl + nq, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
+    return ntiles;
+}
+
+void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
+                         DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
+                         unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
+                         cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
+                         cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
+                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles) {
+    const int64_t nq = a.nq;
+    const int T = a.T;
+    const int segcap = 2 * QT * (T + 1);
+    const size_t slot = (((size_t)(nq + 1) * 8) + 255) & ~size_t(255);
+    char* tb = tilebuf.as<char>();
+    unsigned long long* counters = reinterpret_cast<unsigned long long*>(tb + 5 * slot);
+    int64_t* tile_off = reinterpret_cast<int64_t*>(tb + 6 * slot);
+    int32_t* tile_of = reinterpret_cast<int32_t*>(tb + 7 * slot);
     segbuf.ensure((size_t)std::max<int64_t>(ntiles, 1) * segcap * sizeof(Seg));
     int32_t* nseg = reinterpret_cast<int32_t*>(tb);
     int64_t* rows = reinterpret_cast<int64_t*>(tb + slot);
