@@ -502,14 +502,15 @@ __global__ void k_consec_d2(const float* __restrict__ Q, int ds, const uint32_t*
 
 __global__ void k_tile_flags(const int64_t* __restrict__ d2bits, const int64_t* __restrict__ med,
                              const int32_t* __restrict__ qleaf, const int32_t* __restrict__ qoor,
-                             const uint32_t* __restrict__ qorder, int64_t nq, uint8_t* __restrict__ brk) {
+                             const uint32_t* __restrict__ qorder, int64_t nq, uint8_t* __restrict__ brk,
+                             float jump) {
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i >= nq) return;
     if (i == 0) { brk[0] = 1; return; }
     const uint32_t a = qorder[i], b = qorder[i - 1];
     const uint32_t la = (qoor[a] & 2) ? 0xFFFFu : (uint32_t)qleaf[a];
     const uint32_t lb = (qoor[b] & 2) ? 0xFFFFu : (uint32_t)qleaf[b];
-    const float lim = 16.0f * __uint_as_float((uint32_t)*med);
+    const float lim = jump * __uint_as_float((uint32_t)*med);
     brk[i] = (la != lb || __uint_as_float((uint32_t)d2bits[i - 1]) > lim) ? 1 : 0;
 }
 
@@ -609,7 +610,9 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
             launch_median(d2bits, nq - 1, med, s);
             *launches += 2;
         }
-        k_tile_flags<<<g256, 256, 0, s>>>(d2bits, med, a.qleaf, a.qoor, qorder, nq, brk);
+        float jump = 16.0f;   // cut a tile where consecutive queries are > 16x the median squared step apart
+        if (const char* e = std::getenv("BLSH_TILE_JUMP")) jump = (float)std::atof(e);   // (experiments)
+        k_tile_flags<<<g256, 256, 0, s>>>(d2bits, med, a.qleaf, a.qoor, qorder, nq, brk, jump);
         BLSH_LAUNCH_CHECK();
         scan_exclusive_u8(brk, fexcl, nq, scan, s);
         k_run_start<<<g256, 256, 0, s>>>(brk, fexcl, nq, run_start);
