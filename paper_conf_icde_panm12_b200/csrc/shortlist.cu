@@ -249,6 +249,7 @@ __global__ void __launch_bounds__(256) k_merge_lists(const unsigned long long* _
 //   key; stop early when that bin is taken whole.  Then the selected keys
 //   (<= k) are collected into shared memory and bitonic-sorted.
 constexpr int kSelThreads = 512;
+constexpr int kSmallSel = 512;  // queries with at most this many candidates: warp-register sort
 constexpr int kSelCap = 1024;   // max k
 
 struct SelSrc {
@@ -394,9 +395,76 @@ __global__ void __launch_bounds__(kSelThreads) k_select(const unsigned long long
                                                         int64_t* out_ids, float* out_d2, unsigned long long* out_packed,
                                                         int64_t* out_ncand) {
     const int64_t q = blockIdx.x;
+    if (cand_off[q + 1] - cand_off[q] <= kSmallSel) return;   // k_select_small's query
     SelSrc src{cand_keys, cand_off[q], cand_off[q + 1] - cand_off[q], 0, nq, q, k};
     block_select_write(src, k, q, out_ids, out_d2, out_packed);
     if (threadIdx.x == 0 && out_ncand) out_ncand[q] = (qoor[q] & 2) ? 0 : cnt[q];
+}
+
+// a5, large k, queries with <= 512 candidates (all of them are in the answer or the
+// answer is their sorted prefix): one warp per query sorts its keys in registers -- key
+// i = 32 r + lane in v[r]; bitonic strides < 32 by shuffles, >= 32 between a lane's own
+// registers -- no shared memory, no barriers.
+__global__ void __launch_bounds__(256) k_select_small(const unsigned long long* __restrict__ cand_keys,
+                                                      const int64_t* __restrict__ cand_off, int64_t nq, int k,
+                                                      const int32_t* __restrict__ qoor, const int64_t* __restrict__ cnt,
+                                                      int64_t* out_ids, float* out_d2, unsigned long long* out_packed,
+                                                      int64_t* out_ncand) {
+    constexpr int R = kSmallSel / 32;   // keys per lane
+    const int lane = threadIdx.x & 31;
+    const int64_t q = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (q >= nq) return;
+    const int64_t off = cand_off[q], len = cand_off[q + 1] - off;
+    if (len > kSmallSel) return;        // k_select's query
+    unsigned long long v[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int i = 32 * r + lane;
+        v[r] = i < len ? cand_keys[off + i] : kEmpty;
+    }
+#pragma unroll
+    for (int size = 2; size <= kSmallSel; size <<= 1) {
+#pragma unroll
+        for (int stride = size >> 1; stride > 0; stride >>= 1) {
+            if (stride >= 32) {
+                const int rs = stride >> 5;
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    if (r & rs) continue;   // (r, r | rs): the lower index keeps the min when ascending
+                    const int i = 32 * r + lane;
+                    const bool up = (i & size) == 0;
+                    const unsigned long long x = v[r], y = v[r | rs];
+                    const bool sw = (x > y) == up;
+                    v[r] = sw ? y : x;
+                    v[r | rs] = sw ? x : y;
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < R; ++r) {
+                    const unsigned long long o = __shfl_xor_sync(BLSH_FULL, v[r], stride);
+                    const int i = 32 * r + lane;
+                    const bool take_min = ((lane & stride) == 0) == ((i & size) == 0);
+                    v[r] = take_min ? (v[r] < o ? v[r] : o) : (v[r] < o ? o : v[r]);
+                }
+            }
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int i = 32 * r + lane;
+        if (i < k) {
+            const unsigned long long e = v[r];
+            if (out_packed) out_packed[(size_t)q * k + i] = e == kEmpty ? kPadPacked : e;
+            if (out_ids) out_ids[(size_t)q * k + i] = e == kEmpty ? -1 : (int64_t)(uint32_t)(e & 0xFFFFFFFFull);
+            if (out_d2) out_d2[(size_t)q * k + i] = e == kEmpty ? __int_as_float(0x7F800000) : __uint_as_float((uint32_t)(e >> 32));
+        }
+    }
+    for (int i = kSmallSel + lane; i < k; i += 32) {   // k > 512: padding beyond the sorted keys
+        if (out_packed) out_packed[(size_t)q * k + i] = kPadPacked;
+        if (out_ids) out_ids[(size_t)q * k + i] = -1;
+        if (out_d2) out_d2[(size_t)q * k + i] = __int_as_float(0x7F800000);
+    }
+    if (lane == 0 && out_ncand) out_ncand[q] = (qoor[q] & 2) ? 0 : cnt[q];
 }
 
 // a6, large k: per query, the k smallest over n_lists packed lists.
@@ -465,6 +533,9 @@ void launch_select(const unsigned long long* cand_keys, const int64_t* cand_off,
                    unsigned long long* out_packed, int64_t* out_ncand, cudaStream_t s) {
     if (nq == 0) return;
     if (k > kSelCap) throw Error(BLSH_ERR_UNSUPPORTED, "k > 1024");
+    k_select_small<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(cand_keys, cand_off, nq, k, qoor, cnt, out_ids, out_d2,
+                                                             out_packed, out_ncand);
+    BLSH_LAUNCH_CHECK();
     k_select<<<(unsigned)nq, kSelThreads, 0, s>>>(cand_keys, cand_off, nq, k, qoor, cnt, out_ids, out_d2, out_packed,
                                                   out_ncand);
     BLSH_LAUNCH_CHECK();
