@@ -179,9 +179,22 @@ def traffic_for(workload: str, kernel: str):
     return None
 
 
-def recall_from_gt(cfg, X, Q, ids_dev):
-    """recall@10 on the committed oracle ground-truth sample (tools/make_gt.py), tie-aware (C9)."""
+def error_ratio(gt_d2, our_d2):
+    """Eq. 4: kappa = (1/k) sum_i |v - N(v)_i| / |v - I(v)_i| over the sample
+    (0/0 = 1; a padded answer contributes 0), from fp64 ground-truth and reported d^2."""
+    g = np.sqrt(np.maximum(np.asarray(gt_d2, np.float64), 0.0))
+    o = np.sqrt(np.maximum(np.asarray(our_d2, np.float64), 0.0))
+    with np.errstate(divide="ignore", invalid="ignore"):
+        r = np.where(o > 0, g / o, np.where(g == 0, 1.0, 0.0))
+    r[~np.isfinite(o)] = 0.0
+    return float(r.mean())
+
+
+def recall_from_gt(cfg, X, Q, ids_dev, d2_dev=None):
+    """recall@10 on the committed oracle ground-truth sample (tools/make_gt.py), tie-aware (C9);
+    with d2_dev, also the error ratio of Eq. 4 on the same sample (stored as self.kappa)."""
     import torch
+    recall_from_gt.kappa = None
     path = os.path.join(ROOT, "bench_data", f"{cfg.name}_gt.npz")
     if not os.path.exists(path) and X.shape[0] <= 2_000_000 and ids_dev.shape[1] >= 10:
         # no committed ground truth: exact 10-NN of a fixed 200-query sample by the oracle's fp64 brute force
@@ -189,6 +202,8 @@ def recall_from_gt(cfg, X, Q, ids_dev):
         qidx = np.arange(0, Q.shape[0], max(1, Q.shape[0] // 200))[:200]
         gi, gd = oracle.bruteforce(X.cpu().numpy(), Q[torch.as_tensor(qidx, device=Q.device)].cpu().numpy(), 10)
         got = ids_dev[torch.as_tensor(qidx, device=ids_dev.device)][:, :10].cpu().numpy()
+        if d2_dev is not None:
+            recall_from_gt.kappa = error_ratio(gd, d2_dev[torch.as_tensor(qidx, device=d2_dev.device)][:, :10].cpu().numpy())
         hits = 0
         for r in range(len(qidx)):
             gs = set(gi[r].tolist())
@@ -210,6 +225,8 @@ def recall_from_gt(cfg, X, Q, ids_dev):
         return None, "ground-truth fingerprint mismatch"
     gi, gd = g["ids"][:, :10], g["d2"][:, :10].astype(np.float64)
     got = ids_dev[qidx][:, :10].cpu().numpy()
+    if d2_dev is not None:
+        recall_from_gt.kappa = error_ratio(gd, d2_dev[qidx][:, :10].cpu().numpy())
     Xs = X
     hits = 0
     for r in range(len(gi)):
@@ -310,7 +327,8 @@ def run_ours(a):
     sl_bytes = sum(s.shortlist_bytes for s in stats) / max(len(stats), 1)
     total_cand = sum(s.total_cand for s in stats) / max(len(stats), 1)
     launches = sum(s.launches for s in stats) + extra
-    recall, recall_note = (None, "sharded") if world > 1 and rank != 0 else recall_from_gt(cfg, X, Q, out_ids)
+    recall, recall_note = (None, "sharded") if world > 1 and rank != 0 else recall_from_gt(cfg, X, Q, out_ids, out_d2)
+    kappa = getattr(recall_from_gt, "kappa", None)
     shard_load = None
     if world > 1:   # query skew across leaves -> per-rank load of the last step
         ld = sh.load_stats()
@@ -389,7 +407,7 @@ def run_ours(a):
                        "parallelism": f"leaf-shard{world}" if world > 1 else "single",
                        "l2": "no flush: table (%.1f GB) and query batch (%.0f MB) exceed the 126 MB L2"
                              % (cfg.n * info.d_stride * 4 / 1e9, nq * cfg.d * 4 / 1e6)},
-            "recall@10": recall, "recall_note": recall_note,
+            "recall@10": recall, "recall_note": recall_note, "error_ratio@10": kappa,
             "selectivity": total_cand / nq / cfg.n, "mean_candidates": total_cand / nq,
             "build_s": build_s, "datagen_s": gen_s,
             "roofline": roof,
