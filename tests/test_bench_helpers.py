@@ -1,5 +1,4 @@
-"""bench.py host helpers (no GPU): the error ratio of Eq. 4 and the
-balanced leaf split used by the multi-GPU line."""
+"""bench.py host helpers (no GPU): the error ratio of Eq. 4."""
 import os
 import sys
 
