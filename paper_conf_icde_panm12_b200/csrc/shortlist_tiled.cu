@@ -719,7 +719,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_tc) {
-            auto kern = k <= 8 ? k_shortlist_tc<8> : (k <= 12 ? k_shortlist_tc<12> : k_shortlist_tc<16>);
+            auto kern = k <= 8 ? k_shortlist_tc<8>
+                      : (k <= 12 ? k_shortlist_tc<12> : (k <= 16 ? k_shortlist_tc<16> : k_shortlist_tc<32>));
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
             BLSH_LAUNCH_CHECK();

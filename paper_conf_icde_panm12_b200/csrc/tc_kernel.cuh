@@ -48,7 +48,7 @@ constexpr int kTcConv = 4 * kTcQ;          // converter warps
 constexpr int kTcMmaWarp = kTcConv;
 constexpr int kTcEpi0 = kTcConv + 1;       // first epilogue warp
 constexpr int kTcThreads = (kTcConv + 5) * 32;
-constexpr int kTcMaxK = 16;                // k supported by the TC path
+constexpr int kTcMaxK = 32;                // k supported by the TC path
 constexpr int kTcScap = 96;                // buffered pairs per (item, query, epilogue warp)
 constexpr uint32_t kTcStageBytes = kTcRows * kTcChunk * 4;   // 32 KB staging per chunk
 constexpr uint32_t kTcChunkBytes = kTcStageBytes;
@@ -134,7 +134,6 @@ struct TcSmem {
     float xn2[kTcBlk][kTcQ][kTcRows];        // |x'|^2, per column part
     alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
-    unsigned long long tk[QT][kTcMaxK];      // per query exact top-k (final)
     int lock[QT];                            // (unused: the screen no longer rescores inside the kernel)
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
     float tr[4][32 * 33];                    // per epilogue warp: transposed dots [query][row], padded
@@ -226,7 +225,6 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
             S.lock[n] = 0;
         }
     }
-    for (int i = threadIdx.x; i < QT * kTcMaxK; i += kTcThreads) (&S.tk[0][0])[i] = kEmpty;
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
     if (threadIdx.x == 0) {
         for (int s = 0; s < kTcASlots; ++s) {
@@ -484,8 +482,6 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         for (int w = 0; w < 4; ++w)   // -1: this warp's buffer for j overflowed (full exact scan of j's rows)
             a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
     }
-    for (int i = threadIdx.x; i < nqt * k; i += kTcThreads)
-        a.partials[((size_t)item * QT + i / k) * k + i % k] = S.tk[i / k][i % k];   // (empty lists: the start of k_tc_rescore)
 }
 
 // Exact rescoring of the TC screen's survivors, at full occupancy (one warp per
@@ -512,7 +508,7 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     if (j >= (int)(a.tile_off[lo + 1] - q0)) return;
     const int k = a.k, nv = a.ds >> 2;
     unsigned long long* out = a.partials + (size_t)unit * k;
-    TopK tk{lane < k ? out[lane] : kEmpty, kEmpty};
+    TopK tk{kEmpty, kEmpty};
     unsigned long long thr = topk_thr(tk, k);
     const float U = __uint_as_float(a.ufin[unit]);
     const float4* qrow = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + j] * a.ds);

@@ -331,7 +331,7 @@ def test_tiled_shortlist_variants(blsh, orc, c1, monkeypatch, mode):
     else:
         monkeypatch.setenv("BLSH_SHORTLIST", "tc")
     ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=4.0, seed=21)
-    for k, T in [(1, 1), (10, 16), (16, 64)]:
+    for k, T in [(1, 1), (10, 16), (16, 64)] + ([(32, 16)] if mode == "tc" else []):
         run_query_pair(ix, ox, X, Q, k, probe=1 if T > 1 else 0, T=T)
         assert ix.stats().tiled == (1 if mode == "simt" else 2)
 
@@ -371,7 +371,7 @@ def test_tc_screen_equals_warp(blsh, orc, monkeypatch, shape):
         Q = synth.sample_points(mix, 100, 53)
         G, W, T = 2, 3.0, 4
     ix, ox = build_pair(blsh, orc, X, G=G, M=8, W=W, seed=5)
-    for k in (1, 10, 16):
+    for k in (1, 10, 16, 17, 24, 32):
         a = _query_mode(ix, Q, k, "warp", monkeypatch, probe=1, n_probes=T)
         b = _query_mode(ix, Q, k, "tc", monkeypatch, probe=1, n_probes=T)
         assert a[3] == 0 and b[3] == 2
