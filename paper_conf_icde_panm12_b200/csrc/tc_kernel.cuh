@@ -607,5 +607,6 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
         }
     }
     if (lane < k) out[lane] = tk.e0;
+    if (lane + 32 < k) out[lane + 32] = tk.e1;
     if (lane == 0 && a.counters && rescored) atomicAdd(a.counters + 1, (unsigned long long)rescored);
 }
