@@ -128,7 +128,7 @@ struct ShortlistArgs {
 
 // query-tiled short-list (shortlist_tiled.cu)
 // 0: warp short-list, 1: SIMT query-tiled, 2: tensor-core screened query-tiled.  The TC
-// kernel is the default where it applies (k <= 16, d_stride a multiple of 64 and <= 512);
+// kernel is the default where it applies (k <= 32, d_stride a multiple of 64 and <= 512);
 // BLSH_SHORTLIST=warp|simt forces the others.
 int shortlist_kind(int ds, int T, int k);
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
