@@ -134,7 +134,6 @@ struct TcSmem {
     float xn2[kTcBlk][kTcQ][kTcRows];        // |x'|^2, per column part
     alignas(16) uint32_t umin[QT];           // per query: smallest k-th upper bound over the epilogue warps (bits)
     int scnt[4][QT];                         // per (epilogue warp, query): buffered pairs
-    int lock[QT];                            // (unused: the screen no longer rescores inside the kernel)
     alignas(16) float cen[512];              // centre of the tile (mean of its queries)
     float tr[4][32 * 33];                    // per epilogue warp: transposed dots [query][row], padded
     uint4 rinfo[4][32];                      // per epilogue warp: (|x'|^2 bits, query mask, table row) per row
@@ -222,7 +221,6 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(BLSH_FULL, s, o);
         if (lane == 0) {
             S.qn[n] = s;
-            S.lock[n] = 0;
         }
     }
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
