@@ -37,9 +37,25 @@ __host__ __device__ __forceinline__ int bits_per_coord(int M) {
 
 // Morton interleave (R9): bit p of u_i = code_i + 2^(B-1) goes to key
 // bit p*M + (M-1-i).  Caller guarantees the code is inside the range.
+// Bits 0..7 of b to bit 0 of bytes 0..7 (multiply-replicate, mask bit j of
+// byte j, carry it to bit 7 with +0x7F, which never carries across bytes).
+__device__ __forceinline__ unsigned long long spread8(uint32_t b) {
+    const unsigned long long r = ((unsigned long long)(b & 0xFFu) * 0x0101010101010101ull) & 0x8040201008040201ull;
+    return ((r + 0x7F7F7F7F7F7F7F7Full) & 0x8080808080808080ull) >> 7;
+}
+
 __device__ __forceinline__ Key128 morton_key(const int32_t* code, int M, int B) {
     unsigned long long hi = 0ull, lo = 0ull;
     const int off = 1 << (B - 1);
+    if (M == 8 && B == 16) {   // bit p of u_i -> key byte p, bit 7-i: the same interleave, 2 spreads per coordinate
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const uint32_t u = (uint32_t)(code[i] + off);
+            lo |= spread8(u) << (7 - i);
+            hi |= spread8(u >> 8) << (7 - i);
+        }
+        return Key128{hi, lo};
+    }
     for (int i = 0; i < M; ++i) {
         uint32_t u = (uint32_t)(code[i] + off);
         const int base = M - 1 - i;

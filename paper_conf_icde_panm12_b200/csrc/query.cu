@@ -418,7 +418,28 @@ __device__ void warp_select_impl(ProbeSmem& sm, uint32_t P, uint32_t skip, int R
         }
     }
     __syncwarp();
-    // sort the R selected entries by (score bits, index): rank by counting
+    // sort the R selected entries by (score bits, index): R <= 32 by a register
+    // bitonic network over the lanes (keys are distinct: x is unique), else
+    // rank by counting
+    if (R <= 32) {
+        unsigned long long b = lane < R ? sm.sbits[lane] : ~0ull;
+        uint32_t x = lane < R ? sm.sx[lane] : 0xFFFFFFFFu;
+#pragma unroll
+        for (int kk = 2; kk <= 32; kk <<= 1) {
+#pragma unroll
+            for (int j = kk >> 1; j > 0; j >>= 1) {
+                const unsigned long long pb = __shfl_xor_sync(BLSH_FULL, b, j);
+                const uint32_t px = __shfl_xor_sync(BLSH_FULL, x, j);
+                const bool p_lt = pb < b || (pb == b && px < x);
+                const bool m_lt = b < pb || (b == pb && x < px);
+                const bool keep_min = ((lane & j) == 0) == ((lane & kk) == 0);
+                if (keep_min ? p_lt : m_lt) { b = pb; x = px; }
+            }
+        }
+        if (lane < R) sm.order[lane] = x;
+        __syncwarp();
+        return;
+    }
     for (int e = lane; e < R; e += 32) {
         const unsigned long long b = sm.sbits[e];
         const uint32_t x = sm.sx[e];
