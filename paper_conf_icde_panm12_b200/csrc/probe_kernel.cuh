@@ -115,17 +115,27 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
             v[2 * i] = pl.sqm[i];
             v[2 * i + 1] = pl.sqp[i];
         }
-        // bound B': sum of the J smallest terms, J minimal with >= T-1 valid subsets
+        // bound B': sum of the J smallest terms, J minimal with >= T-1 valid subsets.
+        // Lane j < 2M holds term j and its rank in the order (value, index); the
+        // J-th smallest is then one ballot away (the same sequence a selection
+        // by smallest value, lowest index first, takes).
+        double vme = 0.0;
+#pragma unroll
+        for (int j = 0; j < 2 * MM; ++j)
+            if (lane == j) vme = v[j];
+        int rank = 0;
+#pragma unroll
+        for (int j = 0; j < 2 * MM; ++j) {
+            const double vj = __shfl_sync(0xFFFFFFFFu, vme, j);
+            rank += (vj < vme || (vj == vme && j < lane)) ? 1 : 0;
+        }
+        if (lane >= 2 * MM) rank = 64;
         uint32_t used = 0;            // 2 bits per coordinate
-        unsigned long long taken = 0ull;
         double Bsum = 0.0;
         for (int J = 0; J < 2 * MM; ++J) {
-            int jb = -1;
-            double vb = 0.0;
-#pragma unroll
-            for (int j = 0; j < 2 * MM; ++j)
-                if (!((taken >> j) & 1ull) && (jb < 0 || v[j] < vb)) { jb = j; vb = v[j]; }
-            taken |= 1ull << jb;
+            const int jb = __ffs(__ballot_sync(0xFFFFFFFFu, rank == J)) - 1;
+            if (jb < 0) break;   // NaN terms (no rank J): stop at the terms ranked so far
+            const double vb = __shfl_sync(0xFFFFFFFFu, vme, jb);
             used += 1u << (2 * (jb >> 1));
             Bsum = __dadd_rn(Bsum, vb);
             uint32_t prod = 1;
