@@ -217,6 +217,17 @@ __global__ void __launch_bounds__(kRHQ) k_hash_tables(QueryArgs a, const __grid_
 __device__ __forceinline__ int64_t find_bucket(const Key128* __restrict__ ukey, int64_t lo, int64_t hi,
                                                const Key128& k) {
     const int64_t end = hi;
+    // lower bound, 4-ary while the range is wide: the three pivot loads are
+    // independent, so the dependent-load chain is half the binary one
+    while (hi - lo > 3) {
+        const int64_t n = hi - lo;
+        const int64_t m1 = lo + (n >> 2), m2 = lo + (n >> 1), m3 = lo + ((3 * n) >> 2);
+        const Key128 k1 = ukey[m1], k2 = ukey[m2], k3 = ukey[m3];
+        if (key_lt(k3, k)) lo = m3 + 1;
+        else if (key_lt(k2, k)) { lo = m2 + 1; hi = m3; }
+        else if (key_lt(k1, k)) { lo = m1 + 1; hi = m2; }
+        else hi = m1;
+    }
     while (lo < hi) {
         const int64_t mid = (lo + hi) >> 1;
         const Key128 m = ukey[mid];
