@@ -76,10 +76,29 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
         if (tid == 0) { nseg[t] = 0; rows[t] = 0; }
         return;
     }
-    int np2 = 1;
+    int np2 = 32;                                   // >= one warp of (padding) keys; npow >= 2 * QT
     while (np2 < cnt) np2 <<= 1;
-    for (int k2 = 2; k2 <= np2; k2 <<= 1) {          // bitonic sort of bnd[0..np2)
-        for (int j = k2 >> 1; j > 0; j >>= 1) {
+    // bitonic sort of bnd[0..np2): steps with j >= 32 in shared memory, the
+    // j <= 16 steps of each merge in registers (element i in lane i & 31, its
+    // partner i ^ j one shuffle away), so a merge costs one barrier per
+    // shared-memory step plus one for its register tail
+    auto reg_steps = [&](int k2lo, int k2hi) {
+        for (int i = tid; i < np2; i += kPrepThreads) {
+            uint32_t v = bnd[i];
+            for (int k2 = k2lo; k2 <= k2hi; k2 <<= 1) {
+                const bool up = (i & k2) == 0;
+                for (int j = min(k2 >> 1, 16); j > 0; j >>= 1) {
+                    const uint32_t o = __shfl_xor_sync(BLSH_FULL, v, j);
+                    v = (((i & j) == 0) == up) ? min(v, o) : max(v, o);
+                }
+            }
+            bnd[i] = v;
+        }
+        __syncthreads();
+    };
+    reg_steps(2, 32);
+    for (int k2 = 64; k2 <= np2; k2 <<= 1) {
+        for (int j = k2 >> 1; j >= 32; j >>= 1) {
             for (int i = tid; i < np2; i += kPrepThreads) {
                 const int ixj = i ^ j;
                 if (ixj > i) {
@@ -89,6 +108,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
             }
             __syncthreads();
         }
+        reg_steps(k2, k2);
     }
     // unique boundaries (exclusive scan of first-occurrence flags by warp 0)
     if (tid < 32) {
