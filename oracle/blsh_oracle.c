@@ -995,16 +995,20 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         int32_t *code = ix->lq_code + q * M;
         int32_t clamped[16];
         int ok = orc_hash(ix, g, x, t, code, clamped);
+        /* R30: a non-finite projection (NaN/Inf in the query) has no
+         * probe order (its scores are NaN): no probes, no candidates.           */
+        int nonfin = 0;
+        for (int i = 0; i < M; i++) if (!isfinite(t[i])) nonfin = 1;
         ix->lq_leaf[q] = g;
-        ix->lq_oor[q] = !ok;
+        ix->lq_oor[q] = nonfin ? 5 : !ok;
         hkey[q] = orc_morton(clamped, M, B);
         u128 hk = ok ? orc_morton(code, M, B) : 0;
         ix->lq_key[2 * q] = (uint64_t)(hk >> 64);
         ix->lq_key[2 * q + 1] = (uint64_t)hk;
         int32_t *deltas = (int32_t *)malloc(sizeof(int32_t) * (size_t)T * 16);
         int32_t ridx[256];
-        if (probe == 1 && T > 1) orc_multiprobe_deltas(t, M, T, deltas, NULL);
-        if (probe == 2 && T > 1 && ok) orc_lattice_order_blocks(t, code, M, T, ridx);
+        if (probe == 1 && T > 1 && !nonfin) orc_multiprobe_deltas(t, M, T, deltas, NULL);
+        if (probe == 2 && T > 1 && ok && !nonfin) orc_lattice_order_blocks(t, code, M, T, ridx);
         const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
         int64_t base = 0;
         if (probe == 3) {
@@ -1017,7 +1021,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
             for (int p = 0; p < T; p++) {
                 int64_t off = (p % 2 == 1) ? -(int64_t)((p + 1) / 2) : (int64_t)(p / 2);
                 int64_t b = p0 + off;
-                int valid = b >= ix->leaf_u[g] && b < ix->leaf_u[g + 1];
+                int valid = !nonfin && b >= ix->leaf_u[g] && b < ix->leaf_u[g + 1];
                 u128 pk = valid ? ix->ukey[b] : 0;
                 ix->lq_pkey[((size_t)q * T + p) * 2] = (uint64_t)(pk >> 64);
                 ix->lq_pkey[((size_t)q * T + p) * 2 + 1] = (uint64_t)pk;
@@ -1030,7 +1034,9 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         for (int p = 0; p < T && probe != 3; p++) {
             int32_t pc[16];
             int valid = 1;
-            if (ix->quantizer == 0) {
+            if (nonfin) {
+                valid = 0;
+            } else if (ix->quantizer == 0) {
                 /* Z^M: probe code = floor(t) + delta, empty if outside the range (R9) */
                 for (int i = 0; i < M; i++) {
                     float f = floorf(t[i]) + (p == 0 ? 0.0f : (float)deltas[(p - 1) * M + i]);
@@ -1085,7 +1091,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     if (hierarchy && ix->quantizer == 1) {
         #pragma omp parallel for schedule(dynamic, 4)
         for (int64_t q = 0; q < nq; q++) {
-            if (ix->lq_base[q] >= tau) continue;
+            if (ix->lq_base[q] >= tau || (ix->lq_oor[q] & 4)) continue;
             int g = ix->lq_leaf[q];
             int64_t u0 = ix->leaf_u[g], nb = ix->leaf_u[g + 1] - u0;
             int32_t *cur = (int32_t *)malloc(sizeof(int32_t) * M * (size_t)(nb > 0 ? nb : 1));
@@ -1136,7 +1142,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         const int BM = B * M;
         #pragma omp parallel for schedule(dynamic, 16)
         for (int64_t q = 0; q < nq; q++) {
-            if (ix->lq_base[q] >= tau) continue;
+            if (ix->lq_base[q] >= tau || (ix->lq_oor[q] & 4)) continue;
             int g = ix->lq_leaf[q];
             for (int l = 1;; l++) {
                 int cb = l * step < BM ? l * step : BM;

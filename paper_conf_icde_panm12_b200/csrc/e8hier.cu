@@ -104,7 +104,7 @@ __global__ void k_e8_widen(E8WidenArgs w, const int64_t* __restrict__ tau_p, int
     w.hrows[q] = 0;
     w.hs[q] = 0;
     w.he[q] = 0;
-    if ((w.qoor[q] & 2) || w.base[q] >= tau) return;
+    if ((w.qoor[q] & 6) || w.base[q] >= tau) return;
     const int g = w.qleaf[q];
     const int64_t u0 = w.leaf_u[g], u1 = w.leaf_u[g + 1];
     const int M = w.M;

@@ -173,7 +173,9 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
         int8_t dl[MM];
 #pragma unroll
         for (int i = 0; i < MM; ++i) dl[i] = 0;
-        if (p > 0) {
+        bool sel_ok = true;
+        if (p > 0 && sm.order[p - 1] == 0xFFFFFFFFu) sel_ok = false;   // short pool (warp_select)
+        else if (p > 0) {
             if (fbuf >= 0) {
                 uint32_t en = sm.fe[fbuf][sm.order[p - 1]];
 #pragma unroll
@@ -187,7 +189,7 @@ __device__ int64_t probe_zm(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
             }
         }
         int32_t pc[MM];
-        bool valid = true;
+        bool valid = sel_ok;
 #pragma unroll
         for (int i = 0; i < MM; ++i) {
             const float f = __fadd_rn(fl[i], (float)dl[i]);
@@ -234,12 +236,18 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
             if (M == 8) {
                 const bool ring = p > 240;
                 const uint32_t r = ring ? sm.order2[p - 241] : sm.order[p - 1];
+                if (r == 0xFFFFFFFFu) valid = false;   // short pool (warp_select)
+                else {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) pc[i] += ring ? (int32_t)g_e8_ring2[r][i] : (int32_t)c_e8_roots[r][i];
+                    for (int i = 0; i < 8; ++i) pc[i] += ring ? (int32_t)g_e8_ring2[r][i] : (int32_t)c_e8_roots[r][i];
+                }
             } else {
                 const uint32_t x = sm.order[p - 1], blk = x / 240u, r = x - blk * 240u;
+                if (x == 0xFFFFFFFFu) valid = false;
+                else {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) pc[8 * blk + i] += (int32_t)c_e8_roots[r][i];
+                    for (int i = 0; i < 8; ++i) pc[8 * blk + i] += (int32_t)c_e8_roots[r][i];
+                }
             }
         }
         const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
@@ -314,7 +322,7 @@ __global__ void __launch_bounds__(256) k_lookup_home(QueryArgs a) {
     uint2* ivl = a.ivl + (size_t)q * 2;
     uint2 iv = make_uint2(0, 0);
     Key128 k{0, 0};
-    const bool valid = !(oor & 3);
+    const bool valid = !(oor & 7);
     if (valid) {
         const int g = a.qleaf[q];
         k = a.qkey[q];
@@ -343,7 +351,7 @@ __global__ void __launch_bounds__(kPW * 32, 4) k_probe_lookup(QueryArgs a) {
     const int T = a.T;
     const int oor = a.qoor[q];
     uint2* ivl = a.ivl + (size_t)q * (T + 1);
-    if (oor & 2) {   // leaf not owned by this shard
+    if (oor & 6) {   // leaf not owned by this shard, or a non-finite projection (R30): no probes
         for (int p = lane; p <= T; p += 32) ivl[p] = make_uint2(0, 0);
         if (a.pkey)
             for (int p = lane; p < T; p += 32) { a.pkey[(size_t)q * T + p] = Key128{0, 0}; a.pvalid[(size_t)q * T + p] = 0; }

@@ -9,6 +9,7 @@
 //   k_widen        Morton-prefix widening until |R| >= tau (Eq. 7-8, R17).
 #include <algorithm>
 #include <array>
+#include <mutex>
 #include <vector>
 
 #include "hashcore.cuh"
@@ -189,7 +190,10 @@ __device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __
     const bool ok = quantise(t, MM, a.B, a.quantizer, code);
 #pragma unroll
     for (int i = 0; i < MM; ++i) a.qcode[(size_t)q * MM + i] = code[i];
-    a.qoor[q] = ok ? 0 : 1;
+    bool fin = true;   // R30: a non-finite projection (NaN/Inf query) has no probes and no candidates
+#pragma unroll
+    for (int i = 0; i < MM; ++i) fin = fin && isfinite(t[i]);
+    a.qoor[q] = !fin ? 5 : (ok ? 0 : 1);
     a.qkey[q] = morton_key(code, MM, a.B);   // clamped home key (hierarchy uses it)
     if (!active) a.qoor[q] |= 2;
 }
@@ -253,29 +257,6 @@ struct ProbeSmem {
     uint32_t fe[2][kFCap];      // frontier: partial enc (base-3 digits delta_i + 1, i = 0 most significant)
 };
 
-// Multiprobe pool (R11 + the pruning bound in DESIGN.md "Probe generation"):
-// per coordinate the admissible options among {-1, 0, +1}.
-struct MPPool {
-    int M;
-    uint32_t P;                 // pool size (mixed radix product)
-    uint32_t home;              // pool index of delta = 0
-    int nopt[10];
-    int8_t opt[10][3];
-    uint32_t stride[10];
-    double sq[10][2];           // [i][0] = x_i(-1)^2, [i][1] = x_i(+1)^2
-};
-
-__device__ __forceinline__ double mp_score(const MPPool& P, uint32_t x, int8_t* delta) {
-    double s = 0.0;
-    for (int i = 0; i < P.M; ++i) {
-        const uint32_t dg = (x / P.stride[i]) % (uint32_t)P.nopt[i];
-        const int8_t dv = P.opt[i][dg];
-        delta[i] = dv;
-        if (dv != 0) s = __dadd_rn(s, P.sq[i][dv > 0 ? 1 : 0]);
-    }
-    return s;
-}
-
 __device__ __forceinline__ double ring2_score(const float* y, const int32_t* c2, uint32_t r) {
     int32_t p[8];
 #pragma unroll
@@ -327,6 +308,24 @@ __device__ void warp_select_impl(ProbeSmem& sm, uint32_t P, uint32_t skip, int R
         for (int c = 0; c < kSelCache; ++c) {
             const uint32_t x = lane + 32u * c;
             sc[c] = (x < P && x != skip) ? (unsigned long long)__double_as_longlong(score(x)) : ~0ull;
+        }
+    }
+    // a pool with fewer than R keys (only possible for non-finite scores, R30): select what
+    // there is and mark the remaining slots invalid (0xFFFFFFFF: an empty probe)
+    {
+        int nvalid = 0;
+#pragma unroll
+        for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
+            for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
+                nvalid += __popc(__ballot_sync(BLSH_FULL, key(c, lane + 32u * cc) != ~0ull));
+                if (CACHED) break;
+            }
+        }
+        if (nvalid < R) {
+            for (int e = nvalid + lane; e < R; e += 32) sm.order[e] = 0xFFFFFFFFu;
+            R = nvalid;
+            __syncwarp();
+            if (R == 0) return;
         }
     }
     unsigned long long prefix = 0ull, mask = 0ull;
@@ -470,133 +469,6 @@ __device__ void warp_select(ProbeSmem& sm, uint32_t P, uint32_t skip, int R, Sco
     else warp_select_impl<false>(sm, P, skip, R, score);
 }
 
-#if 0   // superseded by probe_kernel.cuh (kept until the next cleanup)
-__global__ void __launch_bounds__(kPW * 32) k_probe_lookup_v1(QueryArgs a) {
-    __shared__ ProbeSmem smem[kPW];
-    const int lane = threadIdx.x & 31;
-    const int w = threadIdx.x >> 5;
-    const int64_t q = blockIdx.x * (int64_t)kPW + w;
-    if (q >= a.nq) return;
-    ProbeSmem& sm = smem[w];
-    const int T = a.T, M = a.M;
-    const int oor = a.qoor[q];
-    uint2* ivl = a.ivl + (size_t)q * (T + 1);
-    if (oor & 2) {   // leaf not owned by this shard
-        for (int p = lane; p <= T; p += 32) ivl[p] = make_uint2(0, 0);
-        if (a.pkey)
-            for (int p = lane; p < T; p += 32) { a.pkey[(size_t)q * T + p] = Key128{0, 0}; a.pvalid[(size_t)q * T + p] = 0; }
-        if (lane == 0) { a.base[q] = 0; a.cnt[q] = 0; if (a.level) a.level[q] = 0; }
-        return;
-    }
-    const int g = a.qleaf[q];
-    const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
-    const float* t = a.qt + (size_t)q * M;
-    const int32_t* code = a.qcode + (size_t)q * M;
-    const int B = a.B;
-    MPPool pool;
-    if (a.probe == 1 && T > 1) {
-        // pruned pool of perturbations
-        pool.M = M;
-        double v[20];
-        for (int i = 0; i < M; ++i) {
-            const float xm = __fsub_rn(t[i], floorf(t[i]));
-            const float xp = __fsub_rn(1.0f, xm);
-            pool.sq[i][0] = (double)xm * (double)xm;
-            pool.sq[i][1] = (double)xp * (double)xp;
-            v[2 * i] = pool.sq[i][0];
-            v[2 * i + 1] = pool.sq[i][1];
-        }
-        // smallest J terms (ascending value, ties by index) until the valid subsets number >= T-1
-        int used[10];
-        for (int i = 0; i < M; ++i) used[i] = 0;
-        unsigned long long taken = 0ull;
-        double Bsum = 0.0;
-        for (int J = 0; J < 2 * M; ++J) {
-            int jb = -1;
-            for (int j = 0; j < 2 * M; ++j)
-                if (!((taken >> j) & 1ull) && (jb < 0 || v[j] < v[jb])) jb = j;
-            taken |= 1ull << jb;
-            used[jb >> 1] += 1;
-            Bsum = __dadd_rn(Bsum, v[jb]);
-            double prod = 1.0;
-            for (int i = 0; i < M; ++i) prod *= (double)(1 + used[i]);
-            if (prod - 1.0 >= (double)(T - 1)) break;
-        }
-        const double Bp = __dmul_ru(Bsum, 1.0 + 0x1p-40);
-        uint32_t P = 1;
-        for (int i = M - 1; i >= 0; --i) {
-            int n = 0;
-            if (pool.sq[i][0] <= Bp) pool.opt[i][n++] = -1;
-            pool.opt[i][n++] = 0;
-            if (pool.sq[i][1] <= Bp) pool.opt[i][n++] = 1;
-            pool.nopt[i] = n;
-            pool.stride[i] = P;
-            P *= (uint32_t)n;
-        }
-        pool.P = P;
-        uint32_t home = 0;
-        for (int i = 0; i < M; ++i) {
-            const int zi = pool.opt[i][0] == 0 ? 0 : 1;
-            home += (uint32_t)zi * pool.stride[i];
-        }
-        pool.home = home;
-        warp_select(sm, P, home, T - 1, [&](uint32_t x) {
-            int8_t dl[10];
-            return mp_score(pool, x, dl);
-        });
-    } else if (a.probe == 2 && T > 1) {
-        if (!(oor & 1)) {
-            warp_select(sm, 240u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat_score(t, code, x); });
-        }
-    }
-    // keys + binary search, one probe per lane
-    int64_t mysum = 0;
-    for (int p = lane; p < T; p += 32) {
-        int32_t pc[16];
-        bool valid = true;
-        if (a.quantizer == 0) {
-            int8_t dl[10];
-            if (p > 0) mp_score(pool, sm.order[p - 1], dl);
-            const float lo = -(float)(1 << (B - 1)), hi = (float)((1 << (B - 1)) - 1);
-            for (int i = 0; i < M; ++i) {
-                const float f = __fadd_rn(floorf(t[i]), p == 0 ? 0.0f : (float)dl[i]);
-                if (!(f >= lo && f <= hi)) valid = false;
-                else pc[i] = (int32_t)f;
-            }
-        } else {
-            valid = !(oor & 1);
-            const uint32_t r = (p > 0 && valid) ? sm.order[p - 1] : 0u;
-            for (int i = 0; i < 8; ++i) pc[i] = code[i] + (p > 0 ? (int32_t)c_e8_roots[r][i] : 0);
-            const int32_t lo = -(1 << (B - 1)), hi = (1 << (B - 1)) - 1;
-            if (valid)
-                for (int i = 0; i < 8; ++i)
-                    if (pc[i] < lo || pc[i] > hi) valid = false;
-        }
-        Key128 k{0, 0};
-        uint2 iv = make_uint2(0, 0);
-        if (valid) {
-            k = morton_key(pc, M, B);
-            const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
-            if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
-        }
-        ivl[p] = iv;
-        mysum += (int64_t)(iv.y - iv.x);
-        if (a.pkey) {
-            a.pkey[(size_t)q * T + p] = k;
-            a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
-        }
-    }
-    if (lane == 0) ivl[T] = make_uint2(0, 0);
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) mysum += __shfl_xor_sync(BLSH_FULL, mysum, o);
-    if (lane == 0) {
-        a.base[q] = mysum;
-        a.cnt[q] = mysum;
-        if (a.level) a.level[q] = 0;
-    }
-}
-
-#endif
 
 #include "probe_kernel.cuh"
 
@@ -652,7 +524,7 @@ __global__ void k_widen(QueryArgs a, const int64_t* __restrict__ tau_p, int64_t 
     const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (q >= a.nq) return;
     const int64_t tau = min_cand > 0 ? min_cand : *tau_p;
-    if ((a.qoor[q] & 2) || a.base[q] >= tau) return;
+    if ((a.qoor[q] & 6) || a.base[q] >= tau) return;
     const int g = a.qleaf[q];
     const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
     const int BM = a.B * a.M;
@@ -695,8 +567,13 @@ __global__ void k_widen(QueryArgs a, const int64_t* __restrict__ tau_p, int64_t 
 }  // namespace
 
 void upload_e8_roots() {
-    static bool done = false;   // per process; roots are a constant table of this library
-    if (done) return;
+    // __constant__ / __device__ tables are per device: track the upload per device, under a lock
+    static std::mutex mu;
+    static std::vector<bool> done_dev;
+    int dev = 0;
+    BLSH_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(mu);
+    if ((size_t)dev < done_dev.size() && done_dev[dev]) return;
     int8_t roots[240][8] = {};
     int r = 0;
     for (int i = 0; i < 8; ++i)
@@ -739,7 +616,8 @@ void upload_e8_roots() {
     ring.erase(std::unique(ring.begin(), ring.end()), ring.end());
     if (ring.size() != 9120) throw Error(BLSH_ERR_CUDA, "E8 second ring size");
     BLSH_CUDA(cudaMemcpyToSymbol(g_e8_ring2, ring.data(), ring.size() * 8));
-    done = true;
+    if ((size_t)dev >= done_dev.size()) done_dev.resize(dev + 1, false);
+    done_dev[dev] = true;
 }
 
 int launch_route_hash(const QueryArgs& a, cudaStream_t s) {

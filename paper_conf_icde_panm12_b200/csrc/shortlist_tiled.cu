@@ -302,145 +302,6 @@ __device__ __forceinline__ void topk_offer(TopK& tk, unsigned long long& thr, un
     }
 }
 
-#if 0   // superseded by tiled_kernel.cuh (kept until the next cleanup)
-__global__ void __launch_bounds__(kTW * 32, 1) k_shortlist_tiled_v1(TiledArgs a) {
-    extern __shared__ __align__(128) unsigned char smraw[];
-    const int nv4 = a.ds >> 2;
-    const int pitch = a.ds + 4;                              // floats per staged row
-    uint64_t* bar = reinterpret_cast<uint64_t*>(smraw);      // [2]
-    uint32_t* rmask = reinterpret_cast<uint32_t*>(smraw + 16);   // [2][kRows]
-    uint32_t* rid = rmask + 2 * kRows;                            // [2][kRows]
-    int* nrows = reinterpret_cast<int*>(rid + 2 * kRows);         // [2]
-    float* qs = reinterpret_cast<float*>(smraw + 1024);           // [QT][ds]
-    float* rws = qs + (size_t)QT * a.ds;                          // [2][kRows][pitch]
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int64_t item = blockIdx.x;
-    int64_t lo = 0, hi = a.ntiles;
-    while (hi - lo > 1) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (a.item_off[mid] <= item) lo = mid;
-        else hi = mid;
-    }
-    const int64_t tile = lo;
-    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
-    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
-    const Seg* S = a.segs + (size_t)tile * a.segcap;
-    const int ns = a.nseg[tile];
-    for (int i = threadIdx.x; i < QT * nv4; i += kTW * 32) {
-        const int slot = i / nv4, v = i % nv4;
-        const int64_t qp = tile * QT + slot;
-        float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (qp < a.nq) x = reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[qp] * a.ds)[v];
-        reinterpret_cast<float4*>(qs)[(size_t)slot * nv4 + v] = x;
-    }
-    if (threadIdx.x == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    const uint32_t rowbytes = (uint32_t)a.ds * 4u;
-    // warp 0: stage rows [rs, rs + kRows) of the union into buffer st (one row per lane)
-    auto issue = [&](int st, int64_t rs) {
-        if (warp != 0) return;
-        const int64_t r = rs + lane;
-        const bool v = r < r1;
-        const int64_t left = r1 - rs;
-        const int n = left <= 0 ? 0 : (left < kRows ? (int)left : kRows);
-        uint32_t row = 0, msk = 0;
-        if (v) {
-            int l2 = 0, h2 = ns;                // last segment with off <= r
-            while (h2 - l2 > 1) {
-                const int m = (l2 + h2) >> 1;
-                if ((int64_t)S[m].off <= r) l2 = m;
-                else h2 = m;
-            }
-            const Seg sg = S[l2];
-            row = sg.start + (uint32_t)(r - sg.off);
-            msk = sg.mask;
-        }
-        rmask[st * kRows + lane] = msk;
-        rid[st * kRows + lane] = row;
-        if (lane == 0) nrows[st] = n;
-        if (n > 0) {
-            if (lane == 0) {
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&bar[st], (uint32_t)n * rowbytes);
-            }
-            __syncwarp();
-            if (v) bulk_g2s(rws + (size_t)(st * kRows + lane) * pitch, a.Xp + (size_t)row * a.ds, rowbytes, &bar[st]);
-        }
-        __syncwarp();
-    };
-    TopK tk[4];
-    unsigned long long thr[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) { tk[j] = TopK{kEmpty, kEmpty}; thr[j] = kEmpty; }
-    const int k = a.k;
-    uint32_t phase0 = 0u, phase1 = 0u;
-    unsigned long long evaluated = 0ull;
-    int st = 0;
-    issue(0, r0);
-    __syncthreads();
-    int64_t rs = r0;
-    const float4* q4 = reinterpret_cast<const float4*>(qs) + (size_t)(warp * 4) * nv4;
-    while (true) {
-        const int n = nrows[st];
-        if (n == 0) break;
-        issue(st ^ 1, rs + n);                   // prefetch the next stage into the other buffer
-        mbar_wait(&bar[st], st ? phase1 : phase0);
-        if (st) phase1 ^= 1u; else phase0 ^= 1u;
-        const bool valid = lane < n;
-        const uint32_t msk = valid ? rmask[st * kRows + lane] : 0u;
-        const uint32_t prow = rid[st * kRows + lane];
-        const uint32_t myq = (msk >> (warp * 4)) & 15u;
-        const unsigned need = __ballot_sync(BLSH_FULL, myq != 0u);
-        if (need) {
-            evaluated += 4 * 32;
-            const uint32_t id = valid ? __ldg(a.perm + prow) : 0u;
-            const float4* xr = reinterpret_cast<const float4*>(rws + (size_t)(st * kRows + lane) * pitch);
-            // fp32 direct form in partial sums of <= 64 terms (16 float4), then summed (R22)
-            float tot[4] = {0.f, 0.f, 0.f, 0.f};
-            for (int vb = 0; vb < nv4; vb += 16) {
-                const int ve = min(nv4, vb + 16);
-                float acc[4] = {0.f, 0.f, 0.f, 0.f};
-#pragma unroll 4
-                for (int v = vb; v < ve; ++v) {
-                    const float4 x = xr[v];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const float4 q = q4[(size_t)j * nv4 + v];
-                        const float dx = q.x - x.x, dy = q.y - x.y, dz = q.z - x.z, dw = q.w - x.w;
-                        acc[j] = fmaf(dx, dx, acc[j]);
-                        acc[j] = fmaf(dy, dy, acc[j]);
-                        acc[j] = fmaf(dz, dz, acc[j]);
-                        acc[j] = fmaf(dw, dw, acc[j]);
-                    }
-                }
-#pragma unroll
-                for (int j = 0; j < 4; ++j) tot[j] += acc[j];
-            }
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const bool mine = (myq >> j) & 1u;
-                const unsigned long long key = mine ? pack_entry(tot[j], id) : kEmpty;
-                topk_offer(tk[j], thr[j], key, k, lane);
-            }
-        }
-        __syncthreads();                          // buffer st fully consumed before it is refilled
-        rs += n;
-        st ^= 1;
-    }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        if (j == 0 && lane == 0 && a.counters) atomicAdd(a.counters, evaluated);
-        unsigned long long* out = a.partials + ((size_t)item * QT + warp * 4 + j) * k;
-        if (lane < k) out[lane] = tk[j].e0;
-        if (lane + 32 < k) out[lane + 32] = tk[j].e1;
-    }
-}
-
-#endif
 
 #include "tiled_kernel.cuh"
 #include "tc_kernel.cuh"
@@ -492,7 +353,7 @@ __global__ void k_qsort_keys(const Key128* __restrict__ qkey, const int32_t* __r
     const Key128 k = qkey[q];
     hi[q] = 0ull;
     lo[q] = k.lo;
-    leaf[q] = (qoor[q] & 2) ? 0xFFFFu : (uint32_t)qleaf[q];
+    leaf[q] = (qoor[q] & 6) ? 0xFFFFu : (uint32_t)qleaf[q];   // not owned / non-finite (R30): own tiles
     id[q] = (uint32_t)q;
 }
 
@@ -528,8 +389,8 @@ __global__ void k_tile_flags(const int64_t* __restrict__ d2bits, const int64_t* 
     if (i >= nq) return;
     if (i == 0) { brk[0] = 1; return; }
     const uint32_t a = qorder[i], b = qorder[i - 1];
-    const uint32_t la = (qoor[a] & 2) ? 0xFFFFu : (uint32_t)qleaf[a];
-    const uint32_t lb = (qoor[b] & 2) ? 0xFFFFu : (uint32_t)qleaf[b];
+    const uint32_t la = (qoor[a] & 6) ? 0xFFFFu : (uint32_t)qleaf[a];
+    const uint32_t lb = (qoor[b] & 6) ? 0xFFFFu : (uint32_t)qleaf[b];
     const float lim = jump * __uint_as_float((uint32_t)*med);
     brk[i] = (la != lb || __uint_as_float((uint32_t)d2bits[i - 1]) > lim) ? 1 : 0;
 }

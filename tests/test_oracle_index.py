@@ -286,3 +286,64 @@ def test_invalid_arguments(orc, c1):
     with pytest.raises(orc.OracleError) as e:
         orc.OracleIndex(X[:500] * 1e4, G=2, M=8, W=1e-3)
     assert e.value.args[1] == 4
+
+
+@pytest.mark.parametrize("probe,T,hier", [(1, 16, 0), (0, 1, 1), (3, 4, 0)])
+def test_nonfinite_queries_have_no_candidates(orc, c1, c1_index, probe, T, hier):
+    """R30: a query whose projection is non-finite has no probes and no candidates;
+    the rest of the batch is answered exactly as without it (min_cand fixed, so the
+    batch median does not move)."""
+    X, Q = c1
+    Qb = Q.copy()
+    Qb[2, 0] = np.nan
+    Qb[5, 3] = np.inf
+    ids_b, d2_b, nc_b = c1_index.query(Qb, 10, probe=probe, T=T, hierarchy=hier, min_cand=50)
+    oor = c1_index.get("q_oor")
+    assert oor[2] == 5 and oor[5] == 5
+    assert nc_b[2] == 0 and nc_b[5] == 0
+    assert np.all(ids_b[[2, 5]] == -1) and np.all(np.isinf(d2_b[[2, 5]]))
+    assert not np.any(c1_index.get("q_pvalid").reshape(len(Q), T)[[2, 5]])
+    ids, d2, nc = c1_index.query(Q, 10, probe=probe, T=T, hierarchy=hier, min_cand=50)
+    good = [q for q in range(len(Q)) if q not in (2, 5)]
+    assert np.array_equal(ids[good], ids_b[good]) and np.array_equal(nc[good], nc_b[good])
+
+
+def test_max_rule_jitter_closed_form(orc):
+    """R4 max rule with jitter ([20]): theta_j - theta_0 = (2u - 1) j |x0 - y| / sqrt(d),
+    u = U(seed, stream (4, 0, v), 0) (R2, pinned by the SplitMix64 known answers), x0 the
+    node's lowest-id member, y its farthest member from x0 (ties -> lowest id).  The node
+    membership and |x0 - y| are recomputed here in numpy fp64; a sign, index or scale error
+    in the oracle's jitter branch moves theta by far more than the fp32 tolerance."""
+    rng = np.random.default_rng(11)
+    n, d, j, seed = 3000, 24, 0.25, 77   # [20]'s j = 6 empties one child at this size (SURVEY C3)
+    X = rng.standard_normal((n, d)).astype(np.float32)
+    o0 = orc.OracleIndex(X, G=4, M=4, W=1.0, seed=seed, rp_rule=1, rp_max_jitter=0.0)
+    oj = orc.OracleIndex(X, G=4, M=4, W=1.0, seed=seed, rp_rule=1, rp_max_jitter=j)
+    dirs = oj.get("dirs").astype(np.float64)
+    assert np.array_equal(o0.get("dirs"), oj.get("dirs"))
+    th0, thj = o0.get("theta"), oj.get("theta")
+    leaf = oj.get("leaf")
+    members = {0: np.arange(n), 1: np.nonzero(leaf < 2)[0], 2: np.nonzero(leaf >= 2)[0]}
+    X64 = X.astype(np.float64)
+    shifts = []
+    for v, S in members.items():
+        x0 = X64[S[0]]
+        dist2 = ((X64[S] - x0) ** 2).sum(1)
+        y = S[int(np.argmax(dist2))]
+        u = orc.rng_uniform(seed, (4 << 24) + v, 0)
+        delta = (2.0 * u - 1.0) * j * math.sqrt(dist2.max()) / math.sqrt(d)
+        # the jitter-free median of the SAME node (node v's members under the jittered tree)
+        s = np.sort(np.array([np.float32(np.dot(dirs[v], X64[i])) for i in S]))
+        med = float(s[(len(S) - 1) // 2])
+        if v == 0:
+            assert float(th0[0]) == pytest.approx(med, rel=1e-5, abs=1e-5)
+            assert float(thj[0]) - float(th0[0]) == pytest.approx(delta, rel=1e-4, abs=4e-6)
+        else:
+            assert float(thj[v]) - med == pytest.approx(delta, rel=1e-4, abs=5e-5)
+        shifts.append(delta)
+    assert len(set(np.round(shifts, 9))) == 3, "each node draws its own u"
+    # balance moves by exactly the points between the two thetas at the root
+    s_root = X64 @ dirs[0]
+    lo, hi = sorted([float(th0[0]), float(thj[0])])
+    moved = np.count_nonzero((s_root > lo) & (s_root <= hi))
+    assert abs(np.count_nonzero(leaf < 2) - np.count_nonzero(o0.get("leaf") < 2)) == moved
