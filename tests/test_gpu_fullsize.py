@@ -6,12 +6,17 @@ batch (the median is a batch statistic), so the table is compared bit for bit, t
 candidate counts of every query, and candidate sets + top-k on a sample.
 
 c4 (configs[3], 10M x 384, 100k queries, k = 10, multiprobe T = 32; the bench
-workload): too large for the oracle's index in a test, so it is checked through
-properties that hold at any size: the default (tensor-core screened) short-list
-equals the warp short-list (oracle-checked at small sizes) bit for bit on the whole
-batch; reported distances are the exact fp64 distances of the reported ids within
-1e-5; lists are sorted and duplicate-free; recall@10 against the committed oracle
-brute-force ground truth (bench_data/c4_gt.npz, tools/make_gt.py) is >= 0.9.
+workload, in bench.py's launch configuration):
+* against the oracle: the oracle builds the same 10M-point index (~2.5 min on the
+  box's host cores) and the table (perm, bucket keys, offsets, leaf ranges) is
+  compared bit for bit; 400 sampled queries go through the oracle's query phase and
+  their leaf, codes, out-of-range flags, probe-key sequences, |A(q)|, candidate sets
+  and top-k (check_topk) are compared with the GPU's answers to the whole batch;
+* properties over the whole batch: the default (tensor-core screened) short-list
+  equals the warp short-list bit for bit; reported distances are the exact fp64
+  distances of the reported ids within 1e-5; lists are sorted and duplicate-free;
+  recall@10 against the committed oracle brute-force ground truth on 1000 queries
+  (bench_data/c4_gt.npz, tools/make_gt.py --sample 1000) is >= 0.9.
 """
 import os
 
@@ -61,10 +66,53 @@ def test_c3_full_size_parity(blsh, orc):
     check_topk(ids[sample], d2[sample], oi[sample], od[sample], X, Q[sample], cands=[oc[q] for q in sample])
 
 
-def test_c4_full_size_properties(blsh, monkeypatch):
+@pytest.fixture(scope="module")
+def c4_gpu(blsh):
     cfg = synth.CONFIGS["c4"]
     Xd, Qd = synth.make_dataset(cfg, backend="torch", device="cuda")
-    ix = blsh.blsh_build(Xd, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
+    ix = blsh.blsh_build(Xd, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, keep_stages=True)
+    yield cfg, Xd, Qd, ix
+    ix.close()
+
+
+def test_c4_full_size_oracle_parity(c4_gpu, orc):
+    cfg, Xd, Qd, ix = c4_gpu
+    kw = dict(probe=cfg.probe, n_probes=cfg.T, hierarchy=cfg.hierarchy, min_cand=cfg.min_cand)
+    ids, d2, nc = ix.query(Qd, cfg.k, keep_stages=True, **kw)
+    torch.cuda.synchronize()
+    assert ix.stats().tiled == 2, "the bench launch configuration runs the tensor-core short-list"
+    ids, d2, nc = ids.cpu().numpy(), d2.cpu().numpy(), nc.cpu().numpy()
+    T = cfg.T
+    g_leaf, g_code, g_oor = ix.export("Q_LEAF"), ix.export("Q_CODE").reshape(-1, cfg.M), ix.export("Q_OOR")
+    g_pkey = ix.export("Q_PKEY").reshape(cfg.nq, T, 2)
+    g_pval = ix.export("Q_PVALID").reshape(cfg.nq, T)
+    iv = ix.export("Q_INTERVALS").reshape(-1, T + 1, 2)
+    perm = ix.export("PERM")
+    X = Xd.cpu().numpy()
+    ox = orc.OracleIndex(X, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
+    for g, o in [("PERM", "perm"), ("UKEY", "ukey"), ("UOFF", "uoff"), ("LEAF_U", "leaf_u")]:
+        assert np.array_equal(ix.export(g), ox.get(o).ravel()), f"{g} differs at full size"
+    rng = np.random.default_rng(44)
+    sample = np.sort(rng.choice(cfg.nq, 400, replace=False))
+    Qs = Qd[torch.as_tensor(sample, device="cuda")].cpu().numpy()
+    oi, od, onc = ox.query(Qs, cfg.k, probe=cfg.probe, T=T, hierarchy=cfg.hierarchy, min_cand=cfg.min_cand)
+    assert np.array_equal(g_leaf[sample], ox.get("q_leaf")), "query leaves differ"
+    assert np.array_equal(g_code[sample].ravel(), ox.get("q_code").ravel()), "query codes differ"
+    assert np.array_equal(g_oor[sample], ox.get("q_oor")), "out-of-range flags differ"
+    assert np.array_equal(g_pval[sample].ravel(), ox.get("q_pvalid").ravel()), "probe validity differs"
+    assert np.array_equal(g_pkey[sample].ravel(), ox.get("q_pkey").ravel()), "probe-key sequences differ"
+    assert np.array_equal(nc[sample], onc), "|A(q)| differs"
+    oc = ox.candidates()
+    for r, q in enumerate(sample):
+        parts = [perm[a:b] for a, b in iv[q] if b > a]
+        gq = np.sort(np.concatenate(parts)) if parts else np.zeros(0, np.int64)
+        assert np.array_equal(gq, oc[r]), f"candidate set of query {q} differs"
+    check_topk(ids[sample], d2[sample], oi, od, X, Qs, cands=oc)
+    ox.close()
+
+
+def test_c4_full_size_properties(c4_gpu, monkeypatch):
+    cfg, Xd, Qd, ix = c4_gpu
     kw = dict(probe=cfg.probe, n_probes=cfg.T, hierarchy=cfg.hierarchy, min_cand=cfg.min_cand)
     ids, d2, nc = ix.query(Qd, cfg.k, **kw)
     torch.cuda.synchronize()
@@ -99,6 +147,7 @@ def test_c4_full_size_properties(blsh, monkeypatch):
     assert abs(fpx - float(g["fp_x"])) <= 1e-6 * max(1.0, abs(float(g["fp_x"]))), "ground truth for other data"
     got = ids[qidx][:, :10].cpu().numpy()
     kth = g["d2"][:, 9].astype(np.float64)
+    assert len(got) >= 1000, "SURVEY D5: recall on a 1000-query oracle sample"
     hits = 0
     for r in range(len(got)):
         gs = set(g["ids"][r, :10].tolist())
