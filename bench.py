@@ -164,19 +164,74 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def source_sha() -> str:
+    """sha256 (16 hex) of the library's CUDA/C++ sources: ties an ncu capture to the build it measured."""
+    import glob
+    import hashlib
+    h = hashlib.sha256()
+    for f in sorted(glob.glob(os.path.join(ROOT, "paper_conf_icde_panm12_b200", "csrc", "*"))):
+        with open(f, "rb") as fh:
+            h.update(os.path.basename(f).encode())
+            h.update(fh.read())
+    return h.hexdigest()[:16]
+
+
 def traffic_for(workload: str, kernel: str):
-    """dram read+write bytes per launch from a committed ncu --set full capture of this kernel/workload."""
+    """(dram read+write bytes per launch, entry) from a committed ncu --set full capture of this
+    kernel and workload, ONLY if the capture was taken on the current sources (source_sha);
+    otherwise (None, reason)."""
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             entries = json.load(f)
-        hit = None
-        for t in entries if isinstance(entries, list) else [entries]:
-            if t.get("workload") == workload and t.get("kernel", "").split("<")[0] == kernel:
-                hit = t.get("bytes_per_launch")   # the latest capture of this kernel wins
-        return hit
     except Exception:
-        pass
-    return None
+        return None, "no profiles/traffic.json"
+    cur = source_sha()
+    hit, stale = None, None
+    for t in entries if isinstance(entries, list) else [entries]:
+        if t.get("workload") == workload and t.get("kernel", "").split("<")[0] == kernel:
+            if t.get("source_sha") == cur:
+                hit = t
+            else:
+                stale = t
+    if hit:
+        return hit.get("bytes_per_launch"), hit
+    if stale:
+        return None, f"latest ncu capture of {kernel} is of another build ({stale.get('source_sha', 'untagged')})"
+    return None, f"no ncu capture of {kernel} on this workload"
+
+
+def distinct_candidate_rows(ix, T: int, n_owned: int) -> int:
+    """Table rows that are candidates of at least one query of the last (keep_stages) query:
+    the union of every query's intervals, by a difference array (torch, measurement only)."""
+    import torch
+    iv = torch.as_tensor(ix.export("Q_INTERVALS").reshape(-1, 2).astype(np.int64), device="cuda")
+    iv = iv[iv[:, 1] > iv[:, 0]]
+    diff = torch.zeros(n_owned + 1, dtype=torch.int32, device="cuda")
+    ones = torch.ones(iv.shape[0], dtype=torch.int32, device="cuda")
+    diff.index_add_(0, iv[:, 0], ones)
+    diff.index_add_(0, iv[:, 1], -ones)
+    return int((torch.cumsum(diff[:-1], 0) > 0).sum().item())
+
+
+def l2_copy_gbs() -> float:
+    """L2-resident copy bandwidth (read + write bytes / time) of a 24 MB torch copy, best of 50:
+    the denominator for short-lists whose table fits in the 126 MB L2."""
+    import torch
+    a = torch.empty(6 * 1024 * 1024, dtype=torch.float32, device="cuda")
+    b = torch.empty_like(a)
+    for _ in range(5):
+        b.copy_(a)
+    best = None
+    for _ in range(50):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(20):
+            b.copy_(a)
+        e1.record()
+        torch.cuda.synchronize()
+        t = e0.elapsed_time(e1) / 20
+        best = t if best is None else min(best, t)
+    return 2 * a.numel() * 4 / (best * 1e-3) / 1e9
 
 
 def error_ratio(gt_d2, our_d2):
@@ -377,26 +432,52 @@ def run_ours(a):
         wl = workload_str(cfg)
         kind = stats[0].tiled if stats else 0
         avg = lambda f: sum(getattr(s, f) for s in stats) / max(len(stats), 1)
+        skind = stats[0].screen_kind if stats else 0
         kname = {0: "k_shortlist", 1: "k_shortlist_tiled", 2: "k_shortlist_tc"}[kind]
+        if kind == 2 and skind == 1:
+            kname = "k_screen_f16"
         if kind:
-            # query-tiled short-list: one launch streams, per work item, the union
-            # of its tile's candidate rows once (+ the (row, query-mask) metadata and the tile's
-            # queries); those bytes are the kernel's algorithmic traffic, against HBM.  The
-            # per-query figure sum|A(q)| d 4 is the "effective gather" rate (exceeds peak: reuse).
             k_ms = avg("ms_screen")
-            k_bytes = avg("union_bytes")
+            union_bytes = avg("union_bytes")
+            row_bytes = stats[0].screen_row_bytes
         else:
             k_ms = sl_ms
-            k_bytes = sl_bytes
-        achieved = k_bytes / (k_ms * 1e-3) / 1e9 if k_ms > 0 else None
-        roof = {"kernel": kname, "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": (achieved / peak) if achieved else None, "traffic": traffic_for(wl, kname),
-                "peak_source": peak_src, "algorithmic_bytes_per_launch": k_bytes, "kernel_ms_per_launch": k_ms,
-                "kernel_share_of_step": k_ms / (ms / a.steps),
+            union_bytes = sl_bytes
+            row_bytes = 4 * cfg.d + 4
+        # Algorithmic bytes of one launch (SURVEY §8(d) D4 with reuse): every table row that is a
+        # candidate of some query of the batch has to reach the SMs at least once, at the width the
+        # kernel reads it (fp16 screen: 2 dr + 16 B; fp32 kernels: 4 d_stride (+ metadata)); plus
+        # the query batch once.  Bytes served again from L2 (tiles sharing rows) are NOT counted.
+        distinct = None
+        if cfg.L == 1 and world == 1:
+            ix.query(Q, k, keep_stages=True, **kw)
+            distinct = distinct_candidate_rows(ix, cfg.T, info.n_owned)
+        if distinct is None:
+            distinct = min(total_cand, info.n_owned)
+        per_row = (row_bytes - 16) if (kind == 2 and skind == 1) else row_bytes   # rowinfo is per union row, not per table row
+        alg_bytes = distinct * per_row + nq * 4 * info.d_stride
+        achieved = alg_bytes / (k_ms * 1e-3) / 1e9 if k_ms > 0 else None
+        traffic, tnote = traffic_for(wl, kname)
+        l2_resident = info.n_owned * per_row <= 96e6
+        l2_peak = l2_copy_gbs() if l2_resident else None
+        bound, pk = ("l2", l2_peak) if l2_resident else ("hbm", peak)
+        roof = {"kernel": kname, "bound": bound, "achieved": achieved, "peak": pk, "unit": "GB/s",
+                "frac": (achieved / pk) if achieved else None, "traffic": traffic,
+                "peak_source": ("measured in this run: L2-resident 24 MB torch copy" if l2_resident else peak_src),
+                "algorithmic_bytes_per_launch": alg_bytes,
+                "algorithmic_note": f"{distinct} distinct candidate rows x {per_row} B + the query batch",
+                "floor_ms": alg_bytes / (pk * 1e9) * 1e3 if pk else None,
+                "kernel_ms_per_launch": k_ms, "kernel_share_of_step": k_ms / (ms / a.steps),
+                "dram_gbs": traffic / (k_ms * 1e-3) / 1e9 if traffic else None,
+                "dram_frac": traffic / (k_ms * 1e-3) / 1e9 / peak if traffic else None,
+                "traffic_note": tnote if traffic is None else tnote.get("source"),
+                "union_bytes_per_launch": union_bytes,
+                "union_gbs": union_bytes / (k_ms * 1e-3) / 1e9 if k_ms > 0 else None,
                 "effective_gather_gbs": sl_bytes / (k_ms * 1e-3) / 1e9 if k_ms > 0 else None,
                 "union_rows_per_step": avg("union_rows"), "pairs_algorithmic": total_cand,
                 "pairs_kept": avg("pairs_kept"), "pairs_rescored": avg("pairs_scored") if kind == 2 else None,
-                "rescore_ms": avg("ms_rescore") if kind == 2 else None}
+                "rescore_ms": avg("ms_rescore") if kind == 2 else None,
+                "k_slots": avg("k_slots") if kind == 2 else None}
         res = {
             "metric": METRIC, "value": nq * a.steps / (ms * 1e-3), "unit": UNIT, "n_gpus": world,
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps, "higher_is_better": True,

@@ -227,6 +227,9 @@ typedef struct {
     double  union_bytes;              /* tiled: algorithmic bytes of the streaming kernel: union rows x (4 d_stride + 8)
                                          + the tile queries each work item loads (4 d_stride per query)              */
     int64_t pairs_kept;               /* TC: (row, query) pairs that passed the running screen and were buffered   */
+    int64_t k_slots;                  /* fp16 screen: (tile, anchor block) pairs of the K table                    */
+    int32_t screen_row_bytes;         /* bytes per union row the screen kernel reads (rows + metadata)            */
+    int32_t screen_kind;              /* 0 none, 1 fp16 compact-table screen (k_screen_f16), 2 TF32 (k_shortlist_tc) */
 } blsh_stats;
 
 blsh_status blsh_last_stats(const blsh_index* idx, blsh_stats* out);

@@ -58,7 +58,8 @@ class Stats(C.Structure):
                 ("tiled", C.c_int32), ("pad_", C.c_int32), ("union_rows", C.c_int64),
                 ("pairs_scored", C.c_int64), ("shortlist_flops", C.c_double),
                 ("ms_screen", C.c_float), ("ms_rescore", C.c_float), ("union_bytes", C.c_double),
-                ("pairs_kept", C.c_int64)]
+                ("pairs_kept", C.c_int64), ("k_slots", C.c_int64), ("screen_row_bytes", C.c_int32),
+                ("screen_kind", C.c_int32)]
 
 
 class BlshError(RuntimeError):

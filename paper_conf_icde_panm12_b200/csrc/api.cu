@@ -264,6 +264,7 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
         const int cur = blsh::radix_sort_entries(sb, no, s, &passes);
         blsh::build_table(*ix, Xs.as<float>(), sb.hi[cur].as<unsigned long long>(), sb.lo[cur].as<unsigned long long>(),
                           sb.leaf[cur].as<uint32_t>(), sb.id[cur].as<uint32_t>(), no, sb.scan, s);
+        blsh::build_screen_rows(*ix, s);   // the short-list screen's fp16 residual rows (resid.cu)
         BLSH_CUDA(cudaStreamSynchronize(s));
         // leaves as table position ranges (the same in every table: entries sort by leaf first)
         ix->leaf_pos_h.assign(G + 1, 0);
@@ -447,6 +448,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.qleaf = w.qleaf; a.qt = w.qt; a.qcode = w.qcode; a.qoor = w.qoor; a.qkey = w.qkey;
     a.pkey = w.pkey; a.pvalid = w.pvalid; a.ivl = w.ivl; a.base = w.base; a.cnt = w.cnt; a.level = w.level;
     a.lperm = lperm; a.lcnt = lcnt;
+    a.dr = ix.dr; a.Rh = ix.Rh.p; a.rconst = ix.rconst.as<float4>(); a.bscale = ix.bscale.as<float>();
+    a.anc = ix.anc.as<float>();
     // a1+a2
     launches += launch_route_hash(a, s);
     auto table_args = [&](int l) {   // QueryArgs of hash table l
@@ -472,7 +475,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // query-tiled short-list ahead: fork the query sort + tile formation (a1/a2 outputs only)
-    const int kind_pre = (list_path || out_base) ? 0 : shortlist_kind(ds, T, k);
+    const int kind_pre = (list_path || out_base) ? 0 : shortlist_kind(ds, ix.dr, T, k);
     if (kind_pre > 0) {
         if (!w.side) {
             BLSH_CUDA(cudaStreamCreateWithFlags(&w.side, cudaStreamNonBlocking));
@@ -558,7 +561,8 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     BLSH_CUDA(cudaStreamSynchronize(s));
     const int kind = kind_pre;   // lists: warp short-list over the positions
     const bool tiled = kind > 0;
-    int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0;
+    int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0, kslots = 0;
+    int screen_kind = 0;
     double qload_rows = 0.0;
     const int tcpath = kind == 2 ? 1 : 0;
     int64_t ch = 0;
@@ -568,7 +572,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
                             tm ? ix.ev[4] : nullptr, tm ? ix.ev[8] : nullptr, tm ? ix.ev[5] : nullptr, &pairs,
-                            &kept, &qload_rows, kind, ntiles_pre);
+                            &kept, &qload_rows, kind, ntiles_pre, &kslots, &screen_kind);
         ch = chr;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {
@@ -617,7 +621,14 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     stt.tiled = tiled ? (tcpath ? 2 : 1) : 0;
     stt.union_rows = union_rows;
     stt.pairs_kept = kept;
-    stt.union_bytes = tiled ? (double)union_rows * (4.0 * ds + 8.0) + qload_rows * 4.0 * ds : stt.shortlist_bytes;
+    // bytes the streaming kernel reads per union row: fp16 screen: the fp16 row (2 dr), its (row, mask, K slot)
+    // entry and its bound constants (16 + 16); TF32 screen / SIMT tiled: the fp32 row + its entry
+    const int row_bytes = screen_kind == 1 ? 2 * ix.dr + 32 : 4 * ds + (screen_kind == 2 ? 16 : 8);
+    stt.k_slots = kslots;
+    stt.screen_kind = screen_kind;
+    stt.screen_row_bytes = tiled ? row_bytes : 4 * ix.d + 4;
+    stt.union_bytes = tiled ? (double)union_rows * row_bytes + qload_rows * 4.0 * ds + (double)kslots * 32.0 * 4.0
+                            : stt.shortlist_bytes;
     stt.pairs_scored = pairs;
     stt.shortlist_flops = 3.0 * ix.d * (double)total;
     if (p.hierarchy) {

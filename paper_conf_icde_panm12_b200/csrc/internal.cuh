@@ -155,6 +155,10 @@ struct ExtraTable {
 
 }  // namespace blsh
 
+namespace blsh {
+constexpr int kAnchorShift = 9;   // rows per anchor block of the screen's compact table = 512
+}
+
 struct blsh_index {
     // metadata
     int64_t n = 0, n_owned = 0, nu = 0;
@@ -179,6 +183,13 @@ struct blsh_index {
     blsh::DevBuf uleaf;   // [nu] int32
     blsh::DevBuf uoff;    // [nu+1] uint32
     blsh::DevBuf leaf_u;  // [G+1] int64
+    // device: the short-list screen's compact rows (resid.cu): anchor blocks of 2^kAnchorShift rows
+    int dr = 0;                 // fp16 columns per row (ds rounded up to 64)
+    int64_t nanchor = 0;        // anchor blocks
+    blsh::DevBuf anc;           // [nanchor][dr] fp32 anchors a_b
+    blsh::DevBuf bscale;        // [nanchor] fp32 power-of-two scale s_b
+    blsh::DevBuf Rh;            // [n_owned][dr] fp16 residuals r = (x - a_b) / s_b
+    blsh::DevBuf rconst;        // [n_owned] float4 (|s_b r|^2, a_b . s_b r, |s_b r|, G)
     // L > 1 hash tables
     int L = 1;
     std::vector<std::unique_ptr<blsh::ExtraTable>> xt;   // tables 1..L-1
@@ -234,6 +245,11 @@ bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order,
 void build_table(blsh_index& ix, const float* Xs, const unsigned long long* key_hi,
                  const unsigned long long* key_lo, const uint32_t* leaf, const uint32_t* id,
                  int64_t n_owned, ScanTemp& scan, cudaStream_t s);
+
+// The short-list screen's compact copy of the table: anchors, fp16 residual rows and
+// per-row bound constants (resid.cu).  Call after build_table.
+void build_screen_rows(blsh_index& ix, cudaStream_t s);
+int screen_cols(int ds);
 
 // Table l >= 1 (sorted entries of that table): bucket directory + pos via the
 // inverse of table 0's permutation (inv0[id] = table-0 position).

@@ -40,6 +40,12 @@ struct QueryArgs {
     int32_t* level;          // nullable
     uint32_t* lperm;         // [nq] queries grouped by leaf (a1 -> a2)
     int32_t* lcnt;           // [2G] leaf counts, scatter cursors
+    // short-list screen's compact table (resid.cu)
+    int dr;
+    const void* Rh;          // [n][dr] fp16
+    const float4* rconst;
+    const float* bscale;
+    const float* anc;        // [anchor blocks][dr]
 };
 
 void upload_e8_roots();
@@ -130,7 +136,7 @@ struct ShortlistArgs {
 // 0: warp short-list, 1: SIMT query-tiled, 2: tensor-core screened query-tiled.  The TC
 // kernel is the default where it applies (k <= 32, d_stride a multiple of 64 and <= 512);
 // BLSH_SHORTLIST=warp|simt forces the others.
-int shortlist_kind(int ds, int T, int k);
+int shortlist_kind(int ds, int dr, int T, int k);
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
 int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, ScanTemp& scan, cudaStream_t s,
                    int* launches);
@@ -139,7 +145,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
                          cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
-                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles);
+                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles,
+                         int64_t* kslots_out, int* screen_kind_out);
 
 void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cudaStream_t s);
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s);

@@ -1,0 +1,465 @@
+// screen_kernel.cuh -- the short-list screen on the compact fp16 table (a5), included
+// by shortlist_tiled.cu inside its anonymous namespace after tc_kernel.cuh.
+//
+// Work item = (query tile of <= QT = 32 queries, range of the tile's candidate union).
+// For a 128-row block of the union, one tcgen05.mma chain (kind::f16, M = 128,
+// N = 48, K = dr in steps of 16, fp32 accumulators in TMEM) computes, per row i,
+//   D_ij = r_i . u_j   (j < 32)   u_j = fp16((q_j - c) / S): the tile's centred queries
+//   D_i,hi / D_i,lo = r_i . c_hi / r_i . c_lo   c = c_hi + c_lo (fp16 split of c / S_c)
+// straight from the fp16 residual rows r_i in shared memory (no conversion pass: the
+// rows are copied by cp.async into the 128-byte-swizzled K-major layout the tensor core
+// reads).  With x~ = a + s r (resid.cu) and K_aj = |q_j - a|^2 (k_anchor_k):
+//   |q_j - x~|^2 = K_aj - 2 (q_j - c).(s r) - 2 (c - a).(s r) + |s r|^2
+//               ~ K_aj + beta_i + m_i D_ij,
+//   beta_i = nu_i - 2 (s S_c (D_i,hi + D_i,lo) - rho_i),   m_i = -2 S s.
+// Every rounding in that chain is bounded (DESIGN.md §7 "Screen bound"):
+//   |d2(q_j, x_i) - d~2| <= delta d~2 + E_i + eta_j n_i,
+// so lo = d~2 (1 - delta) - (E_i + eta_j n_i) <= d2 <= d~2 (1 + delta) + (E_i + eta_j n_i) = up.
+// From there the epilogue is the one of k_shortlist_tc: lane j keeps query j's k smallest
+// upper bounds (U_j), buffers every pair with lo <= U_j, and k_tc_rescore computes the
+// exact fp32 distance of the survivors from the fp32 rows.  The screen only decides
+// which pairs get exact work; results equal the warp short-list's.
+//
+// Warp roles (9 warps): 0-3 producers (cp.async of the block's rows, 16 B per lane),
+// 4 MMA issuer + TMEM allocation, 5-8 epilogue (TMEM lane quadrant = warp % 4).
+
+constexpr int kSxProd = 4;                  // producer warps
+constexpr int kSxMma = 4;                   // MMA warp index
+constexpr int kSxEpi0 = 5;                  // first epilogue warp
+constexpr int kSxThreads = 9 * 32;
+constexpr int kSxN = 48;                    // MMA N: 32 queries + c_hi + c_lo + 14 zero columns
+constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
+constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 48 rows x 64 fp16 columns (6 KB)
+constexpr int kSxMaxDr = 640;
+constexpr int kSxNst = 8;                   // A ring stages
+constexpr int kSxAhead = kSxNst - 2;        // stages in flight ahead of the MMA
+// instruction descriptor: D f32, A/B f16, K-major both, N = 48, M = 128
+constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u >> 4) << 24);
+// error model (DESIGN.md §7 "Screen bound")
+constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, relative to sum |a_k b_k|
+constexpr float kSxDelta = 0x1p-11f;        // relative slack on d~2 (AM-GM split 2^-12, K table 2^-13, fp32 ops)
+
+struct SxSmem {
+    uint64_t afull[kSxNst], aempty[kSxNst];
+    uint64_t tfull[4], tempty[4];
+    uint32_t tmem_base;
+    float S, Sc, Cc;
+    float red[16];
+    alignas(16) float eta[QT];
+    uint32_t umin[QT];
+    int scnt[4][QT];
+    float tr[4][32 * 33];           // per epilogue warp: transposed dots [query][row]
+    float4 rf[4][32];               // per epilogue warp and row: beta, m, E, n
+    uint4 ru[4][32];                // per epilogue warp and row: mask, table row, K slot
+    float cen[kSxMaxDr];            // tile centre c
+};
+
+__device__ __forceinline__ uint64_t sw128_desc(uint32_t saddr) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+    d |= (uint64_t)1u << 16;                  // LBO (unused for swizzled K-major)
+    d |= (uint64_t)(1024u >> 4) << 32;        // SBO: 8-row groups 1024 B apart
+    d |= 1ull << 46;                          // descriptor version (sm_100)
+    d |= 2ull << 61;                          // SWIZZLE_128B
+    return d;
+}
+__device__ __forceinline__ void sx_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t accum) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(kSxIdesc), "r"(accum)
+        : "memory");
+}
+__device__ __forceinline__ void tmem_ld2(uint32_t taddr, float& a, float& b) {
+    uint32_t r0, r1;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0,%1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+    a = __uint_as_float(r0);
+    b = __uint_as_float(r1);
+}
+// byte offset of 16-byte chunk ch of row n in a 128B-swizzled K-major panel
+__device__ __forceinline__ uint32_t sw128_off(int n, int ch) {
+    return (uint32_t)((n >> 3) * 1024 + (n & 7) * 128 + ((ch ^ (n & 7)) << 4));
+}
+
+size_t screen_smem_bytes(int dr) {
+    return ((sizeof(SxSmem) + 1023) & ~size_t(1023)) + (size_t)(dr / 64) * kSxPanelB + (size_t)kSxNst * kSxStage;
+}
+
+template <int KT>
+__global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
+    extern __shared__ __align__(1024) unsigned char smraw[];
+    SxSmem& S = *reinterpret_cast<SxSmem*>(smraw);
+    const int ds = a.ds, dr = a.dr, np = dr >> 6;
+    constexpr int nst = kSxNst;
+    unsigned char* Bop = smraw + ((sizeof(SxSmem) + 1023) & ~size_t(1023));
+    unsigned char* Aop = Bop + (size_t)np * kSxPanelB;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t item = blockIdx.x;
+    int64_t lo = 0, hi = a.ntiles;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (a.item_off[mid] <= item) lo = mid;
+        else hi = mid;
+    }
+    const int64_t tile = lo;
+    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
+    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    const int nblk = (int)((r1 - r0 + 127) / 128);
+    const int k = a.k;
+    const int64_t q0 = a.tile_off[tile];
+    const int nqt = (int)(a.tile_off[tile + 1] - q0);
+    const uint4* RI = a.rowinfo + a.rows_off[tile];
+    // ---- setup: centre c, scales, B operand (u_j, c_hi, c_lo), per-query eta ----
+    for (int j = threadIdx.x; j < dr; j += kSxThreads) {
+        float s = 0.f;
+        if (j < ds)
+            for (int n = 0; n < nqt; ++n) s += __ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j);
+        S.cen[j] = j < ds ? s / (float)nqt : 0.f;
+    }
+    __syncthreads();
+    {   // max |c_k|, max |q_jk - c_k|, |c|^2
+        float mc = 0.f, mq = 0.f, c2 = 0.f;
+        for (int j = threadIdx.x; j < ds; j += kSxThreads) {
+            const float c = S.cen[j];
+            mc = fmaxf(mc, fabsf(c));
+            c2 = fmaf(c, c, c2);
+            for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(__ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j) - c));
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            mc = fmaxf(mc, __shfl_xor_sync(BLSH_FULL, mc, o));
+            mq = fmaxf(mq, __shfl_xor_sync(BLSH_FULL, mq, o));
+            c2 += __shfl_xor_sync(BLSH_FULL, c2, o);
+        }
+        if (lane == 0) S.red[warp] = mc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            float m = 0.f;
+            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
+            int e = 0;
+            if (m > 0.f) { frexpf(m, &e); e -= 15; }
+            S.Sc = ldexpf(1.0f, max(-120, min(120, e)));
+        }
+        __syncthreads();
+        if (lane == 0) S.red[warp] = mq;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            float m = 0.f;
+            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
+            int e = 0;
+            if (m > 0.f) { frexpf(m, &e); e -= 15; }
+            S.S = ldexpf(1.0f, max(-120, min(120, e)));
+        }
+        __syncthreads();
+        if (lane == 0) S.red[warp] = c2;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            float t = 0.f;
+            for (int w = 0; w < 9; ++w) t += S.red[w];
+            const float cn = sqrtf(t) * (1.0f + 0x1p-20f);
+            // C_c: accumulation of c.r (hi + lo), the hi/lo split, fp16 underflow of c_lo
+            S.Cc = (kSxEpsAcc * (1.0f + 0x1p-9f) * cn + 0x1p-22f * cn + sqrtf((float)ds) * 0x1p-25f * S.Sc) *
+                   (1.0f + 0x1p-10f);
+        }
+        __syncthreads();
+    }
+    const float Sq = S.S, Sc = S.Sc;
+    const float iSq = 1.0f / Sq, iSc = 1.0f / Sc;   // powers of two: exact
+    for (int i = threadIdx.x; i < kSxN * (dr >> 3); i += kSxThreads) {
+        const int n = i % kSxN, cc = i / kSxN;      // row n of B, 16-byte chunk cc (8 columns)
+        __align__(16) __half h[8];
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            const int j = cc * 8 + e;
+            float v = 0.f;
+            if (j < ds) {
+                const float c = S.cen[j];
+                if (n < nqt) v = (__ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j) - c) * iSq;
+                else if (n == 32 || n == 33) {
+                    const float cs = c * iSc;
+                    const __half chi = __float2half_rn(cs);
+                    v = n == 32 ? __half2float(chi) : cs - __half2float(chi);
+                }
+            }
+            h[e] = __float2half_rn(v);
+        }
+        *reinterpret_cast<uint4*>(Bop + (size_t)(cc >> 3) * kSxPanelB + sw128_off(n, cc & 7)) =
+            *reinterpret_cast<const uint4*>(h);
+    }
+    // per query: qn = |q_j - c|, un = S |u_j| (of the fp16 values), eta_j
+    for (int n = warp; n < QT; n += kSxThreads / 32) {
+        float sq = 0.f, su = 0.f;
+        if (n < nqt) {
+            const float* qq = a.Q + (size_t)a.qorder[q0 + n] * ds;
+            for (int j = lane; j < ds; j += 32) {
+                const float e = __ldg(qq + j) - S.cen[j];
+                sq = fmaf(e, e, sq);
+                const float u = __half2float(__float2half_rn(e * iSq));
+                su = fmaf(u, u, su);
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            sq += __shfl_xor_sync(BLSH_FULL, sq, o);
+            su += __shfl_xor_sync(BLSH_FULL, su, o);
+        }
+        if (lane == 0) {
+            const float qn = sqrtf(sq) * (1.0f + 0x1p-18f);
+            const float un = sqrtf(su) * Sq * (1.0f + 0x1p-18f);
+            const float om = (0x1p-11f + 0x1p-23f) * qn + sqrtf((float)ds) * 0x1p-25f * Sq;
+            S.eta[n] = (2.0f * kSxEpsAcc * un + 2.0f * om + 0x1p-19f * (qn + om)) * (1.0f + 0x1p-10f);
+        }
+    }
+    if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < nst; ++s) {
+            mbar_init(&S.afull[s], kSxProd);
+            mbar_init(&S.aempty[s], 1);
+        }
+        for (int s = 0; s < 4; ++s) {
+            mbar_init(&S.tfull[s], 1);
+            mbar_init(&S.tempty[s], 4);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == kSxMma) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(smem_u32(&S.tmem_base)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B operand visible to the tensor core
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tbase = S.tmem_base;
+    const int nstage = nblk * np;
+
+    if (warp < kSxProd) {
+        // ======================= producers =======================
+        // thread t: 16-byte chunk pc = t & 7 of rows rr + 16 i (i < 8), rr = t >> 3; a warp
+        // instruction copies 4 whole 128-byte row segments (coalesced) into 4 swizzled
+        // shared-memory lines (conflict-free).  Rows with an empty query mask are zero-filled.
+        const int t = threadIdx.x, pc = t & 7, rr = t >> 3;
+        constexpr int ahead = kSxAhead;
+        uint32_t pos[8];
+        bool ok[8];
+        auto issue = [&](int g) {
+            if (g < nstage) {
+                const int b = g / np, p = g - b * np;
+                if (p == 0) {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const int64_t r = r0 + (int64_t)b * 128 + rr + 16 * i;
+                        uint2 e = make_uint2(0u, 0u);
+                        if (r < r1) { const uint4 f = RI[r]; e = make_uint2(f.x, f.y); }
+                        pos[i] = e.x;
+                        ok[i] = e.y != 0u;
+                    }
+                }
+                const int slot = g % nst;
+                if (g >= nst) mbar_wait(&S.aempty[slot], (uint32_t)((g / nst - 1) & 1));
+                const uint32_t sb = smem_u32(Aop + (size_t)slot * kSxStage);
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int r = rr + 16 * i;
+                    const __half* src = a.Rh + (size_t)(ok[i] ? pos[i] : 0u) * dr + p * 64 + pc * 8;
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sb + sw128_off(r, pc)),
+                                 "l"(src), "r"(ok[i] ? 16u : 0u)
+                                 : "memory");
+                }
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");   // (possibly empty: uniform group count)
+        };
+        for (int g = 0; g < ahead; ++g) issue(g);
+        for (int g = 0; g < nstage; ++g) {
+            issue(g + ahead);
+            asm volatile("cp.async.wait_group %0;" ::"n"(kSxAhead) : "memory");
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.afull[g % nst]);
+        }
+    } else if (warp == kSxMma) {
+        // ======================= MMA issuer =======================
+        for (int b = 0; b < nblk; ++b) {
+            const int ts = b & 3;
+            if (b >= 4) mbar_wait(&S.tempty[ts], (uint32_t)(((b >> 2) - 1) & 1));
+            tc_fence_after();
+            const uint32_t dt = tbase + (uint32_t)ts * 64u;
+            for (int p = 0; p < np; ++p) {
+                const int g = b * np + p;
+                const int slot = g % nst;
+                mbar_wait(&S.afull[slot], (uint32_t)((g / nst) & 1));
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t as = smem_u32(Aop + (size_t)slot * kSxStage);
+                    const uint32_t bs = smem_u32(Bop + (size_t)p * kSxPanelB);
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk)
+                        sx_mma(dt, sw128_desc(as + 32u * kk), sw128_desc(bs + 32u * kk), (p > 0 || kk > 0) ? 1u : 0u);
+                    tc_commit(&S.aempty[slot]);
+                    if (p == np - 1) tc_commit(&S.tfull[ts]);
+                }
+                __syncwarp();
+            }
+        }
+    } else {
+        // ======================= epilogue =======================
+        const int ew = warp - kSxEpi0;          // 0..3
+        const int quad = warp & 3;              // TMEM lane quadrant of this warp
+        const int j = lane;                     // query of this lane (screen phase)
+        const float Cc = S.Cc;
+        const float eta = S.eta[j];
+        float ulr[KT];
+#pragma unroll
+        for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
+        int my_cnt = 0;
+        bool my_fail = false;
+        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * 4 + ew) * kTcScap;
+        float* Tt = S.tr[ew];
+        // this lane's row of block b (row phase)
+        auto row_meta = [&](int b, uint4& ri, float4& rc, float& sb) {
+            const int64_t r = r0 + (int64_t)b * 128 + quad * 32 + lane;
+            ri = r < r1 ? RI[r] : make_uint4(0u, 0u, 0u, 0u);
+            rc = make_float4(0.f, 0.f, 0.f, 0.f);
+            sb = 0.f;
+            if (ri.y != 0u) {
+                rc = __ldg(a.rconst + ri.x);
+                sb = __ldg(a.bscale + (ri.x >> kAnchorShift));
+            }
+        };
+        uint4 ri_n;
+        float4 rc_n;
+        float sb_n;
+        if (nblk > 0) row_meta(0, ri_n, rc_n, sb_n);
+        for (int b = 0; b < nblk; ++b) {
+            const uint4 ri = ri_n;
+            const float4 rc = rc_n;
+            const float sbv = sb_n;
+            if (b + 1 < nblk) row_meta(b + 1, ri_n, rc_n, sb_n);
+            const int ts = b & 3;
+            mbar_wait(&S.tfull[ts], (uint32_t)((b >> 2) & 1));
+            tc_fence_after();
+            float dot[32], dch, dcl;
+            const uint32_t ta = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 64u;
+            tmem_ld32(ta, dot);
+            tmem_ld2(ta + 32u, dch, dcl);
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.tempty[ts]);
+            // per-row terms (lane = row)
+            const float cr = sbv * Sc * (dch + dcl);
+            const float beta = rc.x - 2.0f * (cr - rc.y);
+            const float m = -2.0f * Sq * sbv;
+            const float E = (2.0f * rc.z * Cc + 0x1p-22f * fabsf(cr) + rc.w + 0x1p-21f * fabsf(beta)) * (1.0f + 0x1p-10f);
+            if (a.dbg && item == 0 && b == 0) {
+                const int row = quad * 32 + lane;
+                for (int jj = 0; jj < 32; ++jj) a.dbg[row * 32 + jj] = dot[jj];
+                a.dbg[4096 + row] = dch;
+                a.dbg[4096 + 128 + row] = dcl;
+                a.dbg[4096 + 256 + row] = beta;
+                a.dbg[4096 + 384 + row] = m;
+                a.dbg[4096 + 512 + row] = E;
+                a.dbg[4096 + 640 + row] = __uint_as_float(ri.x);
+                a.dbg[4096 + 768 + row] = __uint_as_float(ri.y);
+                a.dbg[4096 + 896 + row] = __uint_as_float(ri.z);
+                if (row < 32) a.dbg[4096 + 1024 + row] = S.eta[row];
+                a.dbg[4096 + 1152 + row] = rc.z;
+                a.dbg[4096 + 1280 + row] = sbv;
+                if (row == 0) {
+                    a.dbg[4096 + 1056] = Sq; a.dbg[4096 + 1057] = Sc; a.dbg[4096 + 1058] = Cc;
+                    a.dbg[4096 + 1059] = (float)nqt;
+                }
+            }
+            // transpose: row lane writes its 32 dots, column j -> Tt[j][lane]
+#pragma unroll
+            for (int jj = 0; jj < 32; ++jj) Tt[jj * 33 + lane] = dot[jj];
+            S.rf[ew][lane] = make_float4(beta, m, E, rc.z);
+            S.ru[ew][lane] = make_uint4(ri.y, ri.x, ri.z, 0u);
+            __syncwarp();
+            const float kth0 = ulr[KT - 1];
+            float U = fminf(kth0, __uint_as_float(S.umin[j]));    // any warp's bound is valid
+#pragma unroll 8
+            for (int i = 0; i < 32; ++i) {
+                const uint4 ru = S.ru[ew][i];                      // broadcast
+                const float4 rf = S.rf[ew][i];
+                const float Kv = __ldg(a.ktab + (size_t)ru.z * QT + j);
+                const float d2 = Kv + fmaf(rf.y, Tt[j * 33 + i], rf.x);
+                const float err = fmaf(eta, rf.w, rf.z);
+                const float lo = fmaf(d2, 1.0f - kSxDelta, -err);
+                if (((ru.x >> j) & 1u) && lo <= U && !my_fail) {   // rare: keep the pair
+                    const float up = fmaf(d2, 1.0f + kSxDelta, err);
+                    if (up < U) {                                  // sorted insert; only bounds below U matter
+#pragma unroll
+                        for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
+                        ulr[0] = fminf(ulr[0], up);
+                        U = fminf(U, ulr[KT - 1]);
+                    }
+                    const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
+                    if (my_cnt == kTcScap) {                       // full: drop what the tighter U excludes
+                        int c2 = 0;
+                        for (int t = 0; t < kTcScap; ++t) {
+                            const unsigned long long f = SBj[t];
+                            if (__uint_as_float((uint32_t)(f >> 32)) <= U) SBj[c2++] = f;
+                        }
+                        my_cnt = c2;
+                        if (my_cnt > 3 * kTcScap / 4) my_fail = true;   // exact scan of j's rows later
+                    }
+                    if (!my_fail) SBj[my_cnt++] = e;
+                }
+            }
+            if (ulr[KT - 1] < kth0) atomicMin(&S.umin[j], __float_as_uint(ulr[KT - 1]));
+            __syncwarp();                                          // Tt / rf / ru reused by the next block
+        }
+        S.scnt[ew][j] = my_fail ? -1 : my_cnt;
+        if (a.counters && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == kSxMma) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 256;" ::"r"(tbase));
+    }
+    // ---- hand-off to k_tc_rescore: final bound U_j, buffered pair counts ----
+    if (threadIdx.x < QT) {
+        const int j = threadIdx.x;
+        a.ufin[(size_t)item * QT + j] = j < nqt ? S.umin[j] : 0u;
+#pragma unroll
+        for (int w = 0; w < 4; ++w)
+            a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
+    }
+}
+
+// K_aj = |q_j - a|^2 for every (tile, anchor slot): one CTA per tile, the tile's queries
+// staged in shared memory (row pitch ds + 4 floats: conflict-free float4 reads), one warp
+// per anchor slot, lane j = query j, fp32 direct form in 4 partial chains.
+__global__ void __launch_bounds__(256) k_anchor_k(const float* __restrict__ Q, int ds, const uint32_t* __restrict__ qorder,
+                                                  const int64_t* __restrict__ tile_off, const int64_t* __restrict__ aoff,
+                                                  const uint32_t* __restrict__ slot_anchor, const float* __restrict__ anc,
+                                                  int dr, float* __restrict__ ktab) {
+    extern __shared__ float4 qs4[];
+    const int64_t t = blockIdx.x;
+    const int64_t q0 = tile_off[t];
+    const int nqt = (int)(tile_off[t + 1] - q0);
+    const int nv = ds >> 2, pitch = nv + 1;
+    for (int i = threadIdx.x; i < QT * nv; i += 256) {
+        const int n = i / nv, v = i - n * nv;
+        qs4[n * pitch + v] = n < nqt ? __ldg(reinterpret_cast<const float4*>(Q + (size_t)qorder[q0 + n] * ds) + v)
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    __syncthreads();
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const float4* qr = qs4 + lane * pitch;
+    for (int64_t sl = aoff[t] + warp; sl < aoff[t + 1]; sl += 8) {
+        const float4* ar = reinterpret_cast<const float4*>(anc + (size_t)slot_anchor[sl] * dr);
+        float s0 = 0.f, s1 = 0.f, s2 = 0.f, s3 = 0.f;
+        for (int v = 0; v < nv; ++v) {
+            const float4 x = __ldg(ar + v), q = qr[v];
+            const float e0 = q.x - x.x, e1 = q.y - x.y, e2 = q.z - x.z, e3 = q.w - x.w;
+            s0 = fmaf(e0, e0, s0);
+            s1 = fmaf(e1, e1, s1);
+            s2 = fmaf(e2, e2, s2);
+            s3 = fmaf(e3, e3, s3);
+        }
+        ktab[(size_t)sl * QT + lane] = lane < nqt ? (s0 + s1) + (s2 + s3) : 0.f;
+    }
+}

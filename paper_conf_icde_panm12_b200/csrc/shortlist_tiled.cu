@@ -20,6 +20,8 @@
 #include <cstdlib>
 #include <cstring>
 
+#include <cuda_fp16.h>
+
 #include "internal.cuh"
 #include "query_kernels.cuh"
 
@@ -34,6 +36,7 @@ constexpr int kTW = 8;            // warps per CTA (each owns 4 tile queries)
 
 struct Seg {
     uint32_t start, len, mask, off;   // table rows [start, start+len), query mask, rows before it in the union
+    uint32_t abase;                   // tile-local index of the anchor block of row `start` (screen K table)
 };
 
 // ---------------------------------------------------------------------------
@@ -44,7 +47,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
                                                             const int64_t* __restrict__ tile_off,
                                                             int segcap, Seg* __restrict__ segs,
                                                             int32_t* __restrict__ nseg,
-                                                            int64_t* __restrict__ rows) {
+                                                            int64_t* __restrict__ rows,
+                                                            int64_t* __restrict__ nanch) {
     extern __shared__ uint32_t sm[];
     const int cap = 2 * QT * (T + 1);
     int npow = 1;
@@ -73,7 +77,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
     __syncthreads();
     const int cnt = s_cnt;
     if (cnt == 0) {
-        if (tid == 0) { nseg[t] = 0; rows[t] = 0; }
+        if (tid == 0) { nseg[t] = 0; rows[t] = 0; nanch[t] = 0; }
         return;
     }
     int np2 = 32;                                   // >= one warp of (padding) keys; npow >= 2 * QT
@@ -184,28 +188,66 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
                 const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
                 if (tid >= o) inc += y;
             }
-            if (v) S[out + __popc(bm & lanemask_lt())] = Seg{bnd[i], len, tog[i], off + inc - len};
+            if (v) S[out + __popc(bm & lanemask_lt())] = Seg{bnd[i], len, tog[i], off + inc - len, 0u};
             off += __shfl_sync(BLSH_FULL, inc, 31);
             out += __popc(bm);
         }
-        if (tid == 0) { nseg[t] = out; rows[t] = off; }
+        __syncwarp();
+        // anchor blocks (2^kAnchorShift table rows) of the union, numbered in row order:
+        // segment i covers blocks [a0, a1]; it shares a0 with segment i-1 when that one ends in it
+        uint32_t na = 0, prev_last = 0xFFFFFFFFu;
+        for (int base = 0; base < out; base += 32) {
+            const int i = base + tid;
+            uint32_t a0 = 0, a1 = 0, pl = 0xFFFFFFFFu;
+            if (i < out) {
+                const Seg sg = S[i];
+                a0 = sg.start >> kAnchorShift;
+                a1 = (sg.start + sg.len - 1) >> kAnchorShift;
+            }
+            const uint32_t up = __shfl_up_sync(BLSH_FULL, a1, 1);
+            pl = tid == 0 ? prev_last : up;
+            const uint32_t shared = (i < out && pl == a0) ? 1u : 0u;
+            const uint32_t c = i < out ? a1 - a0 + 1u - shared : 0u;
+            uint32_t inc = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+                if (tid >= o) inc += y;
+            }
+            if (i < out) S[i].abase = na + inc - c - shared;
+            na += __shfl_sync(BLSH_FULL, inc, 31);
+            prev_last = __shfl_sync(BLSH_FULL, a1, min(31, out - 1 - base));
+        }
+        if (tid == 0) { nseg[t] = out; rows[t] = off; nanch[t] = na; }
     }
 }
 
 // Expand the tiles' segment lists to one (table row, query mask) entry per union row,
 // at rows_off[tile] + (row index within the tile's union): the TC short-list reads its
 // block metadata with one coalesced load instead of walking the segment list.
+// Each entry also carries the row's K-table slot (aoff[tile] + the tile-local index of
+// its anchor block); the first row of every (segment, anchor block) records the slot's
+// anchor block (a block shared by two segments is written twice with the same value).
 __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ segs, const int32_t* __restrict__ nseg,
                                                      int segcap, const int64_t* __restrict__ rows_off,
-                                                     uint2* __restrict__ rowinfo) {
+                                                     const int64_t* __restrict__ aoff, uint4* __restrict__ rowinfo,
+                                                     uint32_t* __restrict__ slot_anchor) {
     const int64_t t = blockIdx.x;
     const Seg* S = segs + (size_t)t * segcap;
-    uint2* out = rowinfo + rows_off[t];
+    uint4* out = rowinfo + rows_off[t];
+    const int64_t ab = aoff[t];
     const int ns = nseg[t];
     const int lane = threadIdx.x & 31;
     for (int sI = threadIdx.x >> 5; sI < ns; sI += 8) {
         const Seg sg = S[sI];
-        for (uint32_t i = lane; i < sg.len; i += 32) out[sg.off + i] = make_uint2(sg.start + i, sg.mask);
+        const uint32_t a0 = sg.start >> kAnchorShift;
+        for (uint32_t i = lane; i < sg.len; i += 32) {
+            const uint32_t row = sg.start + i;
+            const uint32_t blk = row >> kAnchorShift;
+            const int64_t slot = ab + sg.abase + (blk - a0);
+            out[sg.off + i] = make_uint4(row, sg.mask, (uint32_t)slot, 0u);
+            if (slot_anchor && (i == 0 || (row & ((1u << kAnchorShift) - 1u)) == 0u)) slot_anchor[slot] = blk;
+        }
     }
 }
 
@@ -264,7 +306,12 @@ struct TiledArgs {
     int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA, 32 phase timers
     unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
     const int64_t* rows_off;        // [ntiles + 1] union rows before each tile
-    const uint2* rowinfo;           // TC: [total rows] (table row, query mask) per union row
+    const uint4* rowinfo;           // TC: [total rows] (table row, query mask, K slot, 0) per union row
+    int dr;                         // screen: fp16 columns of the compact rows
+    const __half* Rh;               // screen: [n][dr] fp16 residual rows (resid.cu)
+    const float4* rconst;           // screen: [n] per-row bound constants
+    const float* bscale;            // screen: [anchor blocks] scale s_b
+    const float* ktab;              // screen: [K slots][QT] K_aj = |q_j - a|^2
     uint32_t* ufin;                 // TC -> k_tc_rescore: [n_items][QT] final screen bound U_j (fp32 bits)
     int32_t* scnt;                  // TC -> k_tc_rescore: [n_items][QT][4] buffered pairs per epilogue warp
 };
@@ -305,6 +352,7 @@ __device__ __forceinline__ void topk_offer(TopK& tk, unsigned long long& thr, un
 
 #include "tiled_kernel.cuh"
 #include "tc_kernel.cuh"
+#include "screen_kernel.cuh"
 
 __global__ void __launch_bounds__(256) k_merge_tiled(TiledArgs a, const int32_t* __restrict__ qoor,
                                                      const int64_t* __restrict__ cnt, int64_t* out_ids, float* out_d2,
@@ -427,7 +475,17 @@ size_t tc_smem_bytes(int ds) {
     return ((sizeof(TcSmem) + 1023) & ~size_t(1023)) + (size_t)QT * ds * 4 + (size_t)kTcSlots * kTcChunkBytes;
 }
 
-int shortlist_kind(int ds, int T, int k) {
+// BLSH_SCREEN=tf32: the round-1 TF32 screen (k_shortlist_tc, converter warps) instead of
+// the fp16 compact-table screen (k_screen_f16); read once per process.
+static int screen_variant() {
+    static const int v = [] {
+        const char* e = std::getenv("BLSH_SCREEN");
+        return (e && std::strcmp(e, "tf32") == 0) ? 1 : 0;
+    }();
+    return v;
+}
+
+int shortlist_kind(int ds, int dr, int T, int k) {
     const char* mode = std::getenv("BLSH_SHORTLIST");
     if (mode && std::strcmp(mode, "warp") == 0) return 0;
     if (k > 64) return 0;   // large k: warp short-list emitting every key + k_select
@@ -435,7 +493,9 @@ int shortlist_kind(int ds, int T, int k) {
     while (npow < cap) npow <<= 1;
     if ((size_t)3 * npow * 4 > 227 * 1024) return 0;   // tile prep does not fit
     const bool simt_ok = tiled_smem_bytes(ds) <= 227 * 1024;
-    const bool tc_ok = k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024;
+    const bool tc_ok = screen_variant() == 1
+                           ? (k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024)
+                           : (k <= kTcMaxK && dr >= 64 && dr <= kSxMaxDr && screen_smem_bytes(dr) <= 227 * 1024);
     if (mode && std::strcmp(mode, "simt") == 0) return simt_ok ? 1 : 0;
     if (tc_ok) return 2;
     return simt_ok ? 1 : 0;
@@ -470,7 +530,7 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
     const int64_t nq = a.nq;
     // tile arrays are sized for the worst case (one query per tile)
     const size_t slot = (((size_t)(nq + 1) * 8) + 255) & ~size_t(255);
-    tilebuf.ensure(slot * 13 + 256);
+    tilebuf.ensure(slot * 15 + 256);
     char* tb = tilebuf.as<char>();
     unsigned long long* counters = reinterpret_cast<unsigned long long*>(tb + 5 * slot);
     BLSH_CUDA(cudaMemsetAsync(counters, 0, 16, s));
@@ -516,7 +576,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
                          cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
-                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles) {
+                         int64_t* kept_out, double* qload_rows_out, int kind, int64_t ntiles,
+                         int64_t* kslots_out, int* screen_kind_out) {
     const int64_t nq = a.nq;
     const int T = a.T;
     const int segcap = 2 * QT * (T + 1);
@@ -534,16 +595,26 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int npow = 1;
     while (npow < segcap) npow <<= 1;
     const size_t prep_smem = (size_t)3 * npow * 4;
+    int64_t* nanch = reinterpret_cast<int64_t*>(tb + 13 * slot);   // anchor blocks per tile (screen K table)
+    int64_t* aoff = reinterpret_cast<int64_t*>(tb + 14 * slot);
     BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
     k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, tile_off, segcap,
-                                                                  segbuf.as<Seg>(), nseg, rows);
+                                                                  segbuf.as<Seg>(), nseg, rows, nanch);
     BLSH_LAUNCH_CHECK();
     ++*launches;
     scan_exclusive_i64(rows, rows_off, ntiles, scan, s);
     *launches += 3;
-    int64_t total_rows = 0;
-    BLSH_CUDA(cudaMemcpyAsync(&total_rows, rows_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
+    const bool use_tc = kind == 2;   // chosen by shortlist_kind()
+    const bool use_f16 = use_tc && screen_variant() == 0;
+    if (use_f16) {
+        scan_exclusive_i64(nanch, aoff, ntiles, scan, s);
+        *launches += 3;
+    }
+    int64_t tot2[2] = {0, 0};   // union rows, K slots
+    BLSH_CUDA(cudaMemcpyAsync(&tot2[0], rows_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
+    if (use_f16) BLSH_CUDA(cudaMemcpyAsync(&tot2[1], aoff + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
+    const int64_t total_rows = tot2[0], total_slots = tot2[1];
     const int64_t target = 148 * 4;
     int64_t chr = (total_rows + target - 1) / target;
     chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 31) / 32 * 32));
@@ -558,9 +629,12 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
-    const size_t rinfo_bytes = ((size_t)std::max<int64_t>(total_rows, 1) * 8 + 255) & ~size_t(255);
+    const size_t rinfo_bytes = ((size_t)std::max<int64_t>(total_rows, 1) * 16 + 255) & ~size_t(255);
     const size_t ufin_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 4 + 255) & ~size_t(255);
-    partials.ensure(part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes + (size_t)std::max<int64_t>(n_items, 1) * QT * 16);
+    const size_t scnt_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 16 + 255) & ~size_t(255);
+    const size_t ktab_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * QT * 4 + 255) & ~size_t(255);
+    const size_t slot_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * 4 + 255) & ~size_t(255);
+    partials.ensure(part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes + scnt_bytes + ktab_bytes + slot_bytes);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
@@ -573,15 +647,23 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.rows_off = rows_off;
     ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes);
     ta.scnt = reinterpret_cast<int32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes);
+    float* ktab = reinterpret_cast<float*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes +
+                                           scnt_bytes);
+    uint32_t* slot_anchor = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ktab) + ktab_bytes);
+    ta.dr = a.dr;
+    ta.Rh = reinterpret_cast<const __half*>(a.Rh);
+    ta.rconst = a.rconst;
+    ta.bscale = a.bscale;
+    ta.ktab = ktab;
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
-    const size_t tc_smem = tc_smem_bytes(a.ds);
-    const bool use_tc = kind == 2;   // chosen by shortlist_kind()
+    const size_t tc_smem = use_f16 ? screen_smem_bytes(a.dr) : tc_smem_bytes(a.ds);
     const char* dbg_path = std::getenv("BLSH_TC_DEBUG");
     DevBuf dbgbuf;
+    constexpr int kDbgN = 4096 + 2048;
     if (use_tc && dbg_path) {
-        dbgbuf.alloc((4096 + 512) * sizeof(float));
-        BLSH_CUDA(cudaMemsetAsync(dbgbuf.p, 0, (4096 + 512) * sizeof(float), s));
+        dbgbuf.alloc(kDbgN * sizeof(float));
+        BLSH_CUDA(cudaMemsetAsync(dbgbuf.p, 0, kDbgN * sizeof(float), s));
         ta.dbg = dbgbuf.as<float>();
     }
     DevBuf tsbuf;
@@ -591,19 +673,36 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         ta.tstamp = tsbuf.as<unsigned long long>();
     }
     if (use_tc && ntiles > 0) {
-        uint2* ri = reinterpret_cast<uint2*>(partials.as<char>() + part_bytes + sbuf_bytes);
-        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(ta.segs, nseg, segcap, rows_off, ri);
+        uint4* ri = reinterpret_cast<uint4*>(partials.as<char>() + part_bytes + sbuf_bytes);
+        if (!use_f16) BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
+        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(ta.segs, nseg, segcap, rows_off, aoff, ri,
+                                                       use_f16 ? slot_anchor : nullptr);
         BLSH_LAUNCH_CHECK();
         ++*launches;
         ta.rowinfo = ri;
+        if (use_f16 && total_slots > 0) {
+            const size_t ks = (size_t)QT * (a.ds / 4 + 1) * sizeof(float4);
+            BLSH_CUDA(cudaFuncSetAttribute(k_anchor_k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ks));
+            k_anchor_k<<<(unsigned)ntiles, 256, ks, s>>>(a.Q, a.ds, qorder, tile_off, aoff, slot_anchor, a.anc, a.dr,
+                                                        ktab);
+            BLSH_LAUNCH_CHECK();
+            ++*launches;
+        }
     }
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
-        if (use_tc) {
+        if (use_f16) {
+            auto kern = k <= 8 ? k_screen_f16<8>
+                      : (k <= 12 ? k_screen_f16<12> : (k <= 16 ? k_screen_f16<16> : k_screen_f16<32>));
+            BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
+            kern<<<(unsigned)n_items, kSxThreads, tc_smem, s>>>(ta);
+        } else if (use_tc) {
             auto kern = k <= 8 ? k_shortlist_tc<8>
                       : (k <= 12 ? k_shortlist_tc<12> : (k <= 16 ? k_shortlist_tc<16> : k_shortlist_tc<32>));
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
+        }
+        if (use_tc) {
             BLSH_LAUNCH_CHECK();
             ++*launches;
             if (ev_mid) BLSH_CUDA(cudaEventRecord(ev_mid, s));
@@ -633,6 +732,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     BLSH_CUDA(cudaStreamSynchronize(s));
     *pairs_out = (int64_t)(use_tc ? ev[1] : ev[0]);   // TC: exact rescorings after the screen
     *kept_out = use_tc ? (int64_t)ev[0] : 0;
+    *kslots_out = use_f16 ? total_slots : 0;
+    *screen_kind_out = use_f16 ? 1 : (use_tc ? 2 : 0);
     // every work item loads its tile's queries: sum over tiles of |tile| x items(tile) ~ n_items x nq / ntiles
     *qload_rows_out = ntiles > 0 ? (double)n_items * (double)nq / (double)ntiles : 0.0;
     if (use_tc && std::getenv("BLSH_TC_MODE"))
@@ -655,7 +756,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
                      acc[6] / n_items, acc[8] / n_items, acc[7] / n_items, (double)psum / n_items, pmax);
     }
     if (ta.dbg) {
-        std::vector<float> h(4096 + 512);
+        std::vector<float> h(kDbgN);
         BLSH_CUDA(cudaMemcpy(h.data(), ta.dbg, h.size() * sizeof(float), cudaMemcpyDeviceToHost));
         std::vector<uint32_t> q0(QT);
         BLSH_CUDA(cudaMemcpy(q0.data(), qorder, QT * sizeof(uint32_t), cudaMemcpyDeviceToHost));

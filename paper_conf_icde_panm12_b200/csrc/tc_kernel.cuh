@@ -260,14 +260,15 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
         // metadata need cross-warp barriers.
         const int qd = warp & 3, hf = warp >> 2;   // quadrant, column part
         const int nch_total = nblk * nchunk;
-        const uint2* RI = a.rowinfo + a.rows_off[tile];
+        const uint4* RI = a.rowinfo + a.rows_off[tile];
         unsigned char* stg = Aop + (size_t)warp * (32 * kTcCols * 4);   // + slot * kTcStageBytes
         // 16-byte piece p of staged row r lives at r * kTcCols * 4 + ((p ^ swz(r)) << 4): conflict-free
         // for the copies and for the row-per-lane reads (8-lane phases see 8 distinct bank groups)
         auto swz = [](int r) { return kTcPieces == 8 ? (r & 7) : ((r >> 1) & 3); };
         auto fetch = [&](int b) {                          // this lane's row entry of block b
             const int64_t r = r0 + (int64_t)b * kTcRows + 32 * qd + lane;
-            return (b < nblk && r < r1) ? RI[r] : make_uint2(0u, 0u);
+            if (b < nblk && r < r1) { const uint4 f = RI[r]; return make_uint2(f.x, f.y); }
+            return make_uint2(0u, 0u);
         };
         uint2 e_next = fetch(0), e_iss = make_uint2(0u, 0u);
         auto issue = [&](int g) {                          // cp.async of chunk g (this warp's part)
@@ -579,10 +580,10 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
         // exact distance to every row of the item whose query mask has bit j.
         const int64_t r0 = (item - a.item_off[lo]) * a.chr;
         const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[lo]);
-        const uint2* RI = a.rowinfo + a.rows_off[lo];
+        const uint4* RI = a.rowinfo + a.rows_off[lo];
         for (int64_t base = r0; base < r1; base += 32) {
             const int64_t i = base + lane;
-            const uint2 e = i < r1 ? RI[i] : make_uint2(0u, 0u);
+            const uint4 e = i < r1 ? RI[i] : make_uint4(0u, 0u, 0u, 0u);
             const unsigned nm = __ballot_sync(BLSH_FULL, (e.y >> j) & 1u);
             rescored += __popc(nm);
             score_rows(nm, e.x);
