@@ -430,9 +430,15 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     w.k = k;
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[0], s));
     // ---- queries into the padded layout ----
-    if (ds != ix.d) BLSH_CUDA(cudaMemsetAsync(w.Qd, 0, (size_t)nq * ds * sizeof(float), s));
-    BLSH_CUDA(cudaMemcpy2DAsync(w.Qd, ds * sizeof(float), Q, ix.d * sizeof(float), ix.d * sizeof(float), nq,
-                                q_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, s));
+    // device queries already in the kernels' layout (d a multiple of 4, 16-byte aligned rows) are
+    // read in place; otherwise they are copied (host -> device, or padded to d_stride)
+    const bool q_direct = !q_host && ds == ix.d && (reinterpret_cast<uintptr_t>(Q) & 15u) == 0;
+    if (!q_direct) {
+        if (ds != ix.d) BLSH_CUDA(cudaMemsetAsync(w.Qd, 0, (size_t)nq * ds * sizeof(float), s));
+        BLSH_CUDA(cudaMemcpy2DAsync(w.Qd, ds * sizeof(float), Q, ix.d * sizeof(float), ix.d * sizeof(float), nq,
+                                    q_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, s));
+    }
+    const float* Qdev = q_direct ? Q : w.Qd;
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[1], s));
     QueryArgs a{};
     a.nq = nq; a.d = ix.d; a.ds = ds; a.G = ix.G; a.M = M; a.B = ix.B; a.depth = ix.depth;
@@ -442,7 +448,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         const char* rh = std::getenv("BLSH_RH_STAGE");   // ablation: 1 = stage query rows in shared memory
         a.rh_direct = (rh && rh[0] == '1') ? 0 : 1;
     }
-    a.Q = w.Qd; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
+    a.Q = Qdev; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
     a.ntype = ix.ntype.as<int32_t>(); a.A = ix.A.as<float>(); a.bvec = ix.b.as<float>(); a.Wl = ix.W.as<float>();
     a.ukey = ix.ukey.as<Key128>(); a.uoff = ix.uoff.as<uint32_t>(); a.leaf_u = ix.leaf_u.as<int64_t>();
     a.qleaf = w.qleaf; a.qt = w.qt; a.qcode = w.qcode; a.qoor = w.qoor; a.qkey = w.qkey;
@@ -569,7 +575,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     if (tiled) {
         // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
         int chr = 0;
-        run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
+        run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.rowbuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
                             tm ? ix.ev[4] : nullptr, tm ? ix.ev[8] : nullptr, tm ? ix.ev[5] : nullptr, &pairs,
                             &kept, &qload_rows, kind, ntiles_pre, &kslots, &screen_kind);
@@ -590,7 +596,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         // a5, one warp per (query, chunk)
         ShortlistArgs sa{};
         sa.nq = nq; sa.n_items = n_items; sa.d = ix.d; sa.ds = ds; sa.T = T; sa.k = k; sa.chunk = (int)ch;
-        sa.Q = w.Qd; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
+        sa.Q = Qdev; sa.Xp = ix.Xp.as<float>(); sa.perm = ix.perm.as<uint32_t>(); sa.ivl = w.ivl; sa.cnt = w.cnt;
         sa.item_off = w.item_off; sa.partials = w.partials.as<unsigned long long>();
         sa.cand_off = cand_off;
         sa.list = list_path ? w.listbuf.as<uint32_t>() : nullptr;

@@ -192,7 +192,7 @@ __device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __
     for (int i = 0; i < MM; ++i) a.qcode[(size_t)q * MM + i] = code[i];
     bool fin = true;   // R30: a non-finite projection (NaN/Inf query) has no probes and no candidates
 #pragma unroll
-    for (int i = 0; i < MM; ++i) fin = fin && isfinite(t[i]);
+    for (int i = 0; i < MM; ++i) fin = fin && (__float_as_uint(t[i]) & 0x7F800000u) != 0x7F800000u;   // exponent bits
     a.qoor[q] = !fin ? 5 : (ok ? 0 : 1);
     a.qkey[q] = morton_key(code, MM, a.B);   // clamped home key (hierarchy uses it)
     if (!active) a.qoor[q] |= 2;
@@ -310,28 +310,10 @@ __device__ void warp_select_impl(ProbeSmem& sm, uint32_t P, uint32_t skip, int R
             sc[c] = (x < P && x != skip) ? (unsigned long long)__double_as_longlong(score(x)) : ~0ull;
         }
     }
-    // a pool with fewer than R keys (only possible for non-finite scores, R30): select what
-    // there is and mark the remaining slots invalid (0xFFFFFFFF: an empty probe)
-    {
-        int nvalid = 0;
-#pragma unroll
-        for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
-            for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
-                nvalid += __popc(__ballot_sync(BLSH_FULL, key(c, lane + 32u * cc) != ~0ull));
-                if (CACHED) break;
-            }
-        }
-        if (nvalid < R) {
-            for (int e = nvalid + lane; e < R; e += 32) sm.order[e] = 0xFFFFFFFFu;
-            R = nvalid;
-            __syncwarp();
-            if (R == 0) return;
-        }
-    }
     unsigned long long prefix = 0ull, mask = 0ull;
-    int r = R - 1;
     // bits common to every key are skipped: start at the byte of the highest differing bit
     unsigned long long kmin = ~0ull, kmax = 0ull;
+    int nvalid = 0;
 #pragma unroll
     for (int c = 0; c < (CACHED ? kSelCache : 1); ++c) {
         for (int cc = c; cc < nslot; cc += (CACHED ? nslot : 1)) {
@@ -340,10 +322,22 @@ __device__ void warp_select_impl(ProbeSmem& sm, uint32_t P, uint32_t skip, int R
             if (b != ~0ull) {
                 kmin = b < kmin ? b : kmin;
                 kmax = b > kmax ? b : kmax;
+                ++nvalid;
             }
             if (CACHED) break;
         }
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) nvalid += __shfl_xor_sync(BLSH_FULL, nvalid, o);
+    // a pool with fewer than R keys (only for non-finite scores, R30): select what there is and
+    // mark the remaining slots invalid (0xFFFFFFFF: an empty probe)
+    if (nvalid < R) {
+        for (int e = nvalid + lane; e < R; e += 32) sm.order[e] = 0xFFFFFFFFu;
+        R = nvalid;
+        __syncwarp();
+        if (R == 0) return;
+    }
+    int r = R - 1;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         const unsigned long long a0 = __shfl_xor_sync(BLSH_FULL, kmin, o);

@@ -7,8 +7,8 @@
 // fp16 residual r = fp16_rn((x - a_b) / s_b), padded with zeros to dr (a multiple of
 // 64) columns.  x~ = a_b + s_b r is the screen's stand-in for x; per row the library
 // keeps, from fp64 sums,
-//   nu  = |s_b r|^2,  rho = a_b . (s_b r),  n = |s_b r| (rounded up),
-//   G   = the row's share of the screen's error bound (rounding of nu and rho, the
+//   nu  = |s_b r|^2,  rho = a_b . (s_b r) (diagnostic),  n = |s_b r| (rounded up),
+//   G   = the row's share of the screen's error bound (rounding of nu, the
 //         distance between x and x~: 4097 |x - x~|^2 for the 2^-12 AM-GM split, and
 //         2^-13 n^2 for the K table's relative error),
 // so the screen never needs the fp32 row: it reads 2 bytes per coordinate, and the
@@ -111,8 +111,7 @@ __global__ void __launch_bounds__(kAT) k_anchor_rows(const float* __restrict__ X
         e2 = warp_sum_d(e2);
         if (lane == 0) {
             const double nrm = sqrt(nu) * (1.0 + 0x1p-40);
-            const double G = 0x1p-23 * nu + 0x1p-22 * fabs(rho) + 0x1p-39 * anorm * nrm + 4097.0 * e2 * (1.0 + 0x1p-20) +
-                             0x1p-13 * nu;
+            const double G = 0x1p-23 * nu + 4097.0 * e2 * (1.0 + 0x1p-20) + 0x1p-13 * nu;
             float4 v;
             v.x = (float)nu;
             v.y = (float)rho;

@@ -3,15 +3,18 @@
 //
 // Work item = (query tile of <= QT = 32 queries, range of the tile's candidate union).
 // For a 128-row block of the union, one tcgen05.mma chain (kind::f16, M = 128,
-// N = 48, K = dr in steps of 16, fp32 accumulators in TMEM) computes, per row i,
-//   D_ij = r_i . u_j   (j < 32)   u_j = fp16((q_j - c) / S): the tile's centred queries
-//   D_i,hi / D_i,lo = r_i . c_hi / r_i . c_lo   c = c_hi + c_lo (fp16 split of c / S_c)
+// N = 80, K = dr in steps of 16, fp32 accumulators in TMEM) computes, per row i,
+//   D_ij = r_i . u_j   (j < 32)    u_j = fp16((q_j - c) / S): the tile's centred queries
+//   D_ia = r_i . v_a   (a < 48)    v_a = fp16((c - a) / S_v): the item's anchors seen from c
 // straight from the fp16 residual rows r_i in shared memory (no conversion pass: the
 // rows are copied by cp.async into the 128-byte-swizzled K-major layout the tensor core
-// reads).  With x~ = a + s r (resid.cu) and K_aj = |q_j - a|^2 (k_anchor_k):
+// reads).  Every operand is a small difference vector (queries and anchors near c, rows
+// near their anchor), so the tensor core's fp32 accumulation error stays far below the
+// distances.  With x~ = a + s r (resid.cu) and K_aj = |q_j - a|^2 (k_anchor_k):
 //   |q_j - x~|^2 = K_aj - 2 (q_j - c).(s r) - 2 (c - a).(s r) + |s r|^2
 //               ~ K_aj + beta_i + m_i D_ij,
-//   beta_i = nu_i - 2 (s S_c (D_i,hi + D_i,lo) - rho_i),   m_i = -2 S s.
+//   beta_i = nu_i - 2 S_v s D_i,a(i),   m_i = -2 S s.
+// An item spans < 48 anchor blocks (k_tile_items), so every row's anchor has a column.
 // Every rounding in that chain is bounded (DESIGN.md §7 "Screen bound"):
 //   |d2(q_j, x_i) - d~2| <= delta d~2 + E_i + eta_j n_i,
 // so lo = d~2 (1 - delta) - (E_i + eta_j n_i) <= d2 <= d~2 (1 + delta) + (E_i + eta_j n_i) = up.
@@ -27,13 +30,14 @@ constexpr int kSxProd = 4;                  // producer warps
 constexpr int kSxMma = 4;                   // MMA warp index
 constexpr int kSxEpi0 = 5;                  // first epilogue warp
 constexpr int kSxThreads = 9 * 32;
-constexpr int kSxN = 48;                    // MMA N: 32 queries + c_hi + c_lo + 14 zero columns
+constexpr int kSxAnc = 48;                  // anchor columns per item
+constexpr int kSxN = 32 + kSxAnc;           // MMA N: 32 queries + the item's anchors
 constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
-constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 48 rows x 64 fp16 columns (6 KB)
+constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 80 rows x 64 fp16 columns (10 KB)
 constexpr int kSxMaxDr = 640;
 constexpr int kSxNst = 8;                   // A ring stages
 constexpr int kSxAhead = kSxNst - 2;        // stages in flight ahead of the MMA
-// instruction descriptor: D f32, A/B f16, K-major both, N = 48, M = 128
+// instruction descriptor: D f32, A/B f16, K-major both, N = 80, M = 128
 constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u >> 4) << 24);
 // error model (DESIGN.md §7 "Screen bound")
 constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, relative to sum |a_k b_k|
@@ -43,8 +47,9 @@ struct SxSmem {
     uint64_t afull[kSxNst], aempty[kSxNst];
     uint64_t tfull[4], tempty[4];
     uint32_t tmem_base;
-    float S, Sc, Cc;
+    float S, Sv;
     float red[16];
+    float ca[kSxAnc];               // per anchor column: error constant of the D_ia term
     alignas(16) float eta[QT];
     uint32_t umin[QT];
     int scnt[4][QT];
@@ -70,12 +75,11 @@ __device__ __forceinline__ void sx_mma(uint32_t d_tmem, uint64_t adesc, uint64_t
         "l"(adesc), "l"(bdesc), "r"(kSxIdesc), "r"(accum)
         : "memory");
 }
-__device__ __forceinline__ void tmem_ld2(uint32_t taddr, float& a, float& b) {
-    uint32_t r0, r1;
-    asm volatile("tcgen05.ld.sync.aligned.32x32b.x2.b32 {%0,%1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(taddr));
+__device__ __forceinline__ void tmem_ld1(uint32_t taddr, float& a) {
+    uint32_t r0;
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x1.b32 {%0}, [%1];" : "=r"(r0) : "r"(taddr));
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
     a = __uint_as_float(r0);
-    b = __uint_as_float(r1);
 }
 // byte offset of 16-byte chunk ch of row n in a 128B-swizzled K-major panel
 __device__ __forceinline__ uint32_t sw128_off(int n, int ch) {
@@ -96,21 +100,14 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     unsigned char* Aop = Bop + (size_t)np * kSxPanelB;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t item = blockIdx.x;
-    int64_t lo = 0, hi = a.ntiles;
-    while (hi - lo > 1) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (a.item_off[mid] <= item) lo = mid;
-        else hi = mid;
-    }
-    const int64_t tile = lo;
-    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
-    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    int64_t r0, r1;
+    const int64_t tile = item_tile_rows(a, item, &r0, &r1);
     const int nblk = (int)((r1 - r0 + 127) / 128);
     const int k = a.k;
     const int64_t q0 = a.tile_off[tile];
     const int nqt = (int)(a.tile_off[tile + 1] - q0);
     const uint4* RI = a.rowinfo + a.rows_off[tile];
-    // ---- setup: centre c, scales, B operand (u_j, c_hi, c_lo), per-query eta ----
+    // ---- setup: centre c, scales, B operand (u_j, v_a), per-query eta ----
     for (int j = threadIdx.x; j < dr; j += kSxThreads) {
         float s = 0.f;
         if (j < ds)
@@ -118,30 +115,22 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         S.cen[j] = j < ds ? s / (float)nqt : 0.f;
     }
     __syncthreads();
-    {   // max |c_k|, max |q_jk - c_k|, |c|^2
-        float mc = 0.f, mq = 0.f, c2 = 0.f;
+    // the item's anchor slots: RI[r].z is non-decreasing; slot0 = its first, na <= kSxAnc
+    const uint32_t slot0 = r1 > r0 ? RI[r0].z : 0u;
+    const int na = r1 > r0 ? (int)(RI[r1 - 1].z - slot0) + 1 : 0;
+    {   // S: max |q_jk - c_k|, S_v: max |c_k - a_k| over the item's anchors
+        float mq = 0.f, mv = 0.f;
         for (int j = threadIdx.x; j < ds; j += kSxThreads) {
             const float c = S.cen[j];
-            mc = fmaxf(mc, fabsf(c));
-            c2 = fmaf(c, c, c2);
             for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(__ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j) - c));
+            for (int la = 0; la < na; ++la)
+                mv = fmaxf(mv, fabsf(c - __ldg(a.anc + (size_t)a.slot_anchor[slot0 + la] * dr + j)));
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
-            mc = fmaxf(mc, __shfl_xor_sync(BLSH_FULL, mc, o));
             mq = fmaxf(mq, __shfl_xor_sync(BLSH_FULL, mq, o));
-            c2 += __shfl_xor_sync(BLSH_FULL, c2, o);
+            mv = fmaxf(mv, __shfl_xor_sync(BLSH_FULL, mv, o));
         }
-        if (lane == 0) S.red[warp] = mc;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            float m = 0.f;
-            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
-            int e = 0;
-            if (m > 0.f) { frexpf(m, &e); e -= 15; }
-            S.Sc = ldexpf(1.0f, max(-120, min(120, e)));
-        }
-        __syncthreads();
         if (lane == 0) S.red[warp] = mq;
         __syncthreads();
         if (threadIdx.x == 0) {
@@ -152,40 +141,56 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             S.S = ldexpf(1.0f, max(-120, min(120, e)));
         }
         __syncthreads();
-        if (lane == 0) S.red[warp] = c2;
+        if (lane == 0) S.red[warp] = mv;
         __syncthreads();
         if (threadIdx.x == 0) {
-            float t = 0.f;
-            for (int w = 0; w < 9; ++w) t += S.red[w];
-            const float cn = sqrtf(t) * (1.0f + 0x1p-20f);
-            // C_c: accumulation of c.r (hi + lo), the hi/lo split, fp16 underflow of c_lo
-            S.Cc = (kSxEpsAcc * (1.0f + 0x1p-9f) * cn + 0x1p-22f * cn + sqrtf((float)ds) * 0x1p-25f * S.Sc) *
-                   (1.0f + 0x1p-10f);
+            float m = 0.f;
+            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
+            int e = 0;
+            if (m > 0.f) { frexpf(m, &e); e -= 15; }
+            S.Sv = ldexpf(1.0f, max(-120, min(120, e)));
         }
         __syncthreads();
     }
-    const float Sq = S.S, Sc = S.Sc;
-    const float iSq = 1.0f / Sq, iSc = 1.0f / Sc;   // powers of two: exact
+    const float Sq = S.S, Sv = S.Sv;
+    const float iSq = 1.0f / Sq, iSv = 1.0f / Sv;   // powers of two: exact
     for (int i = threadIdx.x; i < kSxN * (dr >> 3); i += kSxThreads) {
         const int n = i % kSxN, cc = i / kSxN;      // row n of B, 16-byte chunk cc (8 columns)
         __align__(16) __half h[8];
+        const float* src = nullptr;
+        if (n < nqt) src = a.Q + (size_t)a.qorder[q0 + n] * ds;
+        else if (n >= 32 && n - 32 < na) src = a.anc + (size_t)a.slot_anchor[slot0 + (n - 32)] * dr;
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
             const int j = cc * 8 + e;
             float v = 0.f;
-            if (j < ds) {
+            if (j < ds && src) {
                 const float c = S.cen[j];
-                if (n < nqt) v = (__ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j) - c) * iSq;
-                else if (n == 32 || n == 33) {
-                    const float cs = c * iSc;
-                    const __half chi = __float2half_rn(cs);
-                    v = n == 32 ? __half2float(chi) : cs - __half2float(chi);
-                }
+                v = n < 32 ? (__ldg(src + j) - c) * iSq : (c - __ldg(src + j)) * iSv;
             }
             h[e] = __float2half_rn(v);
         }
         *reinterpret_cast<uint4*>(Bop + (size_t)(cc >> 3) * kSxPanelB + sw128_off(n, cc & 7)) =
             *reinterpret_cast<const uint4*>(h);
+    }
+    // per anchor column: |c - a| -> ca = error constant of 2 S_v s D_ia (accumulation, fp16
+    // rounding of (c - a) / S_v, fp32 rounding of c - a, fp16 underflow)
+    for (int la = warp; la < kSxAnc; la += kSxThreads / 32) {
+        float sv = 0.f;
+        if (la < na) {
+            const float* ar = a.anc + (size_t)a.slot_anchor[slot0 + la] * dr;
+            for (int j = lane; j < ds; j += 32) {
+                const float e = S.cen[j] - __ldg(ar + j);
+                sv = fmaf(e, e, sv);
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sv += __shfl_xor_sync(BLSH_FULL, sv, o);
+        if (lane == 0) {
+            const float cn = sqrtf(sv) * (1.0f + 0x1p-18f);
+            S.ca[la] = ((kSxEpsAcc + 0x1p-11f + 0x1p-23f) * (1.0f + 0x1p-9f) * cn + sqrtf((float)ds) * 0x1p-25f * Sv) *
+                       (1.0f + 0x1p-10f);
+        }
     }
     // per query: qn = |q_j - c|, un = S |u_j| (of the fp16 values), eta_j
     for (int n = warp; n < QT; n += kSxThreads / 32) {
@@ -224,7 +229,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == kSxMma) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 256;" ::"r"(smem_u32(&S.tmem_base)));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&S.tmem_base)));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // B operand visible to the tensor core
@@ -284,7 +289,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             const int ts = b & 3;
             if (b >= 4) mbar_wait(&S.tempty[ts], (uint32_t)(((b >> 2) - 1) & 1));
             tc_fence_after();
-            const uint32_t dt = tbase + (uint32_t)ts * 64u;
+            const uint32_t dt = tbase + (uint32_t)ts * 128u;
             for (int p = 0; p < np; ++p) {
                 const int g = b * np + p;
                 const int slot = g % nst;
@@ -307,7 +312,6 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         const int ew = warp - kSxEpi0;          // 0..3
         const int quad = warp & 3;              // TMEM lane quadrant of this warp
         const int j = lane;                     // query of this lane (screen phase)
-        const float Cc = S.Cc;
         const float eta = S.eta[j];
         float ulr[KT];
 #pragma unroll
@@ -339,23 +343,36 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             const int ts = b & 3;
             mbar_wait(&S.tfull[ts], (uint32_t)((b >> 2) & 1));
             tc_fence_after();
-            float dot[32], dch, dcl;
-            const uint32_t ta = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 64u;
+            float dot[32];
+            const uint32_t ta = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 128u;
             tmem_ld32(ta, dot);
-            tmem_ld2(ta + 32u, dch, dcl);
+            // this row's anchor column 32 + la: one tcgen05.ld per distinct anchor among the 32 rows
+            const bool live = ri.y != 0u;
+            const int myla = (int)(ri.z - slot0);
+            float Da = 0.f;
+            unsigned pend = __ballot_sync(BLSH_FULL, live);
+            while (pend) {
+                const int la = __shfl_sync(BLSH_FULL, myla, __ffs(pend) - 1);
+                float v;
+                tmem_ld1(ta + 32u + (uint32_t)la, v);
+                const bool mine = live && myla == la;
+                if (mine) Da = v;
+                pend &= ~__ballot_sync(BLSH_FULL, mine);
+            }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&S.tempty[ts]);
             // per-row terms (lane = row)
-            const float cr = sbv * Sc * (dch + dcl);
-            const float beta = rc.x - 2.0f * (cr - rc.y);
+            const float t2 = 2.0f * Sv * sbv * Da;
+            const float beta = rc.x - t2;
             const float m = -2.0f * Sq * sbv;
-            const float E = (2.0f * rc.z * Cc + 0x1p-22f * fabsf(cr) + rc.w + 0x1p-21f * fabsf(beta)) * (1.0f + 0x1p-10f);
+            const float E = (2.0f * rc.z * (live ? S.ca[myla] : 0.f) + rc.w + 0x1p-21f * (fabsf(beta) + fabsf(t2))) *
+                            (1.0f + 0x1p-10f);
             if (a.dbg && item == 0 && b == 0) {
                 const int row = quad * 32 + lane;
                 for (int jj = 0; jj < 32; ++jj) a.dbg[row * 32 + jj] = dot[jj];
-                a.dbg[4096 + row] = dch;
-                a.dbg[4096 + 128 + row] = dcl;
+                a.dbg[4096 + row] = Da;
+                a.dbg[4096 + 128 + row] = (float)myla;
                 a.dbg[4096 + 256 + row] = beta;
                 a.dbg[4096 + 384 + row] = m;
                 a.dbg[4096 + 512 + row] = E;
@@ -366,7 +383,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                 a.dbg[4096 + 1152 + row] = rc.z;
                 a.dbg[4096 + 1280 + row] = sbv;
                 if (row == 0) {
-                    a.dbg[4096 + 1056] = Sq; a.dbg[4096 + 1057] = Sc; a.dbg[4096 + 1058] = Cc;
+                    a.dbg[4096 + 1056] = Sq; a.dbg[4096 + 1057] = Sv; a.dbg[4096 + 1058] = (float)na;
                     a.dbg[4096 + 1059] = (float)nqt;
                 }
             }
@@ -417,7 +434,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     __syncthreads();
     if (warp == kSxMma) {
         tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 256;" ::"r"(tbase));
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
     }
     // ---- hand-off to k_tc_rescore: final bound U_j, buffered pair counts ----
     if (threadIdx.x < QT) {

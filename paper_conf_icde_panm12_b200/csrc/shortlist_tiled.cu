@@ -251,9 +251,39 @@ __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ seg
     }
 }
 
-__global__ void k_tile_items(const int64_t* __restrict__ rows, int64_t ntiles, int chr, int64_t* __restrict__ items) {
+// Work items of a tile: consecutive row ranges of <= chr union rows; with the fp16 screen
+// (rowinfo != NULL) an item also spans < amax anchor blocks (its anchor columns of the
+// MMA, k_screen_f16).  One thread per tile walks its rows; the anchor slot (rowinfo.z) is
+// non-decreasing along a tile's rows.  Pass 1 (item_r0 == NULL) counts, pass 2 writes
+// every item's first row (item_r0[item_off[t] + i], tile-relative).
+__global__ void k_tile_items(const int64_t* __restrict__ rows, const int64_t* __restrict__ rows_off,
+                             const uint4* __restrict__ rowinfo, int64_t ntiles, int chr, int amax,
+                             int64_t* __restrict__ items, const int64_t* __restrict__ item_off,
+                             int64_t* __restrict__ item_r0) {
     const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    if (t < ntiles) items[t] = (rows[t] + chr - 1) / chr;
+    if (t >= ntiles) return;
+    const int64_t R = rows[t];
+    const uint4* RI = rowinfo ? rowinfo + rows_off[t] : nullptr;
+    int64_t r = 0, it = 0;
+    while (r < R) {
+        int64_t e = min(r + (int64_t)chr, R);
+        if (RI) {
+            const uint32_t lim = RI[r].z + (uint32_t)amax;   // first slot that no longer fits
+            if (RI[e - 1].z >= lim) {
+                int64_t lo = r + 1, hi = e - 1;                // smallest row with slot >= lim
+                while (lo < hi) {
+                    const int64_t m = (lo + hi) >> 1;
+                    if (RI[m].z >= lim) hi = m;
+                    else lo = m + 1;
+                }
+                e = lo;
+            }
+        }
+        if (item_r0) item_r0[item_off[t] + it] = r;
+        ++it;
+        r = e;
+    }
+    if (!item_r0) items[t] = it;
 }
 
 // ---------------------------------------------------------------------------
@@ -296,6 +326,8 @@ struct TiledArgs {
     const int32_t* nseg;
     const int64_t* rows;       // [ntiles] union rows per tile
     const int64_t* item_off;   // [ntiles+1]
+    const int64_t* item_r0;    // [n_items] first union row of each item (tile-relative); the item ends at
+                               // the next item's first row (or the tile's last row)
     unsigned long long* partials;   // [n_items][QT][k]
     const int64_t* tile_off;        // [ntiles+1] sorted-query positions of each tile
     const int32_t* tile_of;         // [nq] tile of each sorted position
@@ -312,9 +344,24 @@ struct TiledArgs {
     const float4* rconst;           // screen: [n] per-row bound constants
     const float* bscale;            // screen: [anchor blocks] scale s_b
     const float* ktab;              // screen: [K slots][QT] K_aj = |q_j - a|^2
+    const float* anc;               // screen: [anchor blocks][dr] fp32 anchors
+    const uint32_t* slot_anchor;    // screen: [K slots] anchor block of each slot
     uint32_t* ufin;                 // TC -> k_tc_rescore: [n_items][QT] final screen bound U_j (fp32 bits)
     int32_t* scnt;                  // TC -> k_tc_rescore: [n_items][QT][4] buffered pairs per epilogue warp
 };
+
+// Tile of a work item (binary search over item_off) and the item's union rows [r0, r1).
+__device__ __forceinline__ int64_t item_tile_rows(const TiledArgs& a, int64_t item, int64_t* r0, int64_t* r1) {
+    int64_t lo = 0, hi = a.ntiles;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (a.item_off[mid] <= item) lo = mid;
+        else hi = mid;
+    }
+    *r0 = a.item_r0[item];
+    *r1 = item + 1 < a.item_off[lo + 1] ? a.item_r0[item + 1] : a.rows[lo];
+    return lo;
+}
 
 struct TopK {
     unsigned long long e0, e1;
@@ -572,6 +619,7 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
 }
 
 void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
+                         DevBuf& rowbuf,
                          DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
@@ -615,26 +663,45 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (use_f16) BLSH_CUDA(cudaMemcpyAsync(&tot2[1], aoff + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     const int64_t total_rows = tot2[0], total_slots = tot2[1];
+    // per-union-row entries (TC paths), the fp16 screen's K table and anchor list, item first rows
+    const size_t rinfo_bytes = ((size_t)std::max<int64_t>(total_rows, 1) * 16 + 255) & ~size_t(255);
+    const size_t ktab_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * QT * 4 + 255) & ~size_t(255);
+    const size_t slot_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * 4 + 255) & ~size_t(255);
     const int64_t target = 148 * 4;
     int64_t chr = (total_rows + target - 1) / target;
     chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 31) / 32 * 32));
-    k_tile_items<<<(unsigned)((ntiles + 255) / 256), 256, 0, s>>>(rows, ntiles, (int)chr, items);
+    // items <= rows / chr + (anchor splits: at most one per kSxAnc anchor slots) + one per tile
+    const int64_t items_max = (total_rows + chr - 1) / chr + total_slots / kSxAnc + ntiles + 1;
+    const size_t ir0_bytes = ((size_t)items_max * 8 + 255) & ~size_t(255);
+    rowbuf.ensure(rinfo_bytes + ktab_bytes + slot_bytes + ir0_bytes);
+    uint4* ri = use_tc ? reinterpret_cast<uint4*>(rowbuf.as<char>()) : nullptr;
+    float* ktab = reinterpret_cast<float*>(rowbuf.as<char>() + rinfo_bytes);
+    uint32_t* slot_anchor = reinterpret_cast<uint32_t*>(rowbuf.as<char>() + rinfo_bytes + ktab_bytes);
+    int64_t* item_r0 = reinterpret_cast<int64_t*>(rowbuf.as<char>() + rinfo_bytes + ktab_bytes + slot_bytes);
+    if (use_tc && ntiles > 0) {
+        if (!use_f16) BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
+        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(segbuf.as<Seg>(), nseg, segcap, rows_off, aoff, ri,
+                                                       use_f16 ? slot_anchor : nullptr);
+        BLSH_LAUNCH_CHECK();
+        ++*launches;
+    }
+    const unsigned gt = (unsigned)((ntiles + 255) / 256);
+    const uint4* ri_split = use_f16 ? ri : nullptr;
+    k_tile_items<<<gt, 256, 0, s>>>(rows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, nullptr, nullptr);
     BLSH_LAUNCH_CHECK();
-    ++*launches;
     scan_exclusive_i64(items, item_off, ntiles, scan, s);
-    *launches += 3;
+    k_tile_items<<<gt, 256, 0, s>>>(rows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, item_off, item_r0);
+    BLSH_LAUNCH_CHECK();
+    *launches += 5;
     int64_t n_items = 0;
     BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
-    const size_t rinfo_bytes = ((size_t)std::max<int64_t>(total_rows, 1) * 16 + 255) & ~size_t(255);
     const size_t ufin_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 4 + 255) & ~size_t(255);
     const size_t scnt_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 16 + 255) & ~size_t(255);
-    const size_t ktab_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * QT * 4 + 255) & ~size_t(255);
-    const size_t slot_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * 4 + 255) & ~size_t(255);
-    partials.ensure(part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes + scnt_bytes + ktab_bytes + slot_bytes);
+    partials.ensure(part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
@@ -645,16 +712,17 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
     ta.rows_off = rows_off;
-    ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes);
-    ta.scnt = reinterpret_cast<int32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes);
-    float* ktab = reinterpret_cast<float*>(partials.as<char>() + part_bytes + sbuf_bytes + rinfo_bytes + ufin_bytes +
-                                           scnt_bytes);
-    uint32_t* slot_anchor = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(ktab) + ktab_bytes);
+    ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes);
+    ta.scnt = reinterpret_cast<int32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + ufin_bytes);
+    ta.item_r0 = item_r0;
+    ta.rowinfo = ri;
+    ta.anc = a.anc;
     ta.dr = a.dr;
     ta.Rh = reinterpret_cast<const __half*>(a.Rh);
     ta.rconst = a.rconst;
     ta.bscale = a.bscale;
     ta.ktab = ktab;
+    ta.slot_anchor = slot_anchor;
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
     const size_t tc_smem = use_f16 ? screen_smem_bytes(a.dr) : tc_smem_bytes(a.ds);
@@ -672,22 +740,12 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         BLSH_CUDA(cudaMemsetAsync(tsbuf.p, 0, (size_t)n_items * 16 * 8, s));
         ta.tstamp = tsbuf.as<unsigned long long>();
     }
-    if (use_tc && ntiles > 0) {
-        uint4* ri = reinterpret_cast<uint4*>(partials.as<char>() + part_bytes + sbuf_bytes);
-        if (!use_f16) BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
-        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(ta.segs, nseg, segcap, rows_off, aoff, ri,
-                                                       use_f16 ? slot_anchor : nullptr);
+    if (use_f16 && total_slots > 0) {
+        const size_t ks = (size_t)QT * (a.ds / 4 + 1) * sizeof(float4);
+        BLSH_CUDA(cudaFuncSetAttribute(k_anchor_k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ks));
+        k_anchor_k<<<(unsigned)ntiles, 256, ks, s>>>(a.Q, a.ds, qorder, tile_off, aoff, slot_anchor, a.anc, a.dr, ktab);
         BLSH_LAUNCH_CHECK();
         ++*launches;
-        ta.rowinfo = ri;
-        if (use_f16 && total_slots > 0) {
-            const size_t ks = (size_t)QT * (a.ds / 4 + 1) * sizeof(float4);
-            BLSH_CUDA(cudaFuncSetAttribute(k_anchor_k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ks));
-            k_anchor_k<<<(unsigned)ntiles, 256, ks, s>>>(a.Q, a.ds, qorder, tile_off, aoff, slot_anchor, a.anc, a.dr,
-                                                        ktab);
-            BLSH_LAUNCH_CHECK();
-            ++*launches;
-        }
     }
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {

@@ -169,15 +169,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_shortlist_tc(TiledArgs a) {
     const uint32_t sboB = (uint32_t)kp_total * 128u;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t item = blockIdx.x;
-    int64_t lo = 0, hi = a.ntiles;
-    while (hi - lo > 1) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (a.item_off[mid] <= item) lo = mid;
-        else hi = mid;
-    }
-    const int64_t tile = lo;
-    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
-    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    int64_t r0, r1;
+    const int64_t tile = item_tile_rows(a, item, &r0, &r1);
     const int nblk = (int)((r1 - r0 + kTcRows - 1) / kTcRows);
     const int nchunk = ds / kTcChunk;
     const int k = a.k;
@@ -497,12 +490,8 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     if (unit >= a.n_items * QT) return;
     const int64_t item = unit / QT;
     const int j = (int)(unit % QT);
-    int64_t lo = 0, hi = a.ntiles;
-    while (hi - lo > 1) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (a.item_off[mid] <= item) lo = mid;
-        else hi = mid;
-    }
+    int64_t r0, r1;
+    const int64_t lo = item_tile_rows(a, item, &r0, &r1);
     const int64_t q0 = a.tile_off[lo];
     if (j >= (int)(a.tile_off[lo + 1] - q0)) return;
     const int k = a.k, nv = a.ds >> 2;
@@ -578,8 +567,6 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     if (failed) {
         // The screen could not separate this query's candidates (a buffer overflowed):
         // exact distance to every row of the item whose query mask has bit j.
-        const int64_t r0 = (item - a.item_off[lo]) * a.chr;
-        const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[lo]);
         const uint4* RI = a.rowinfo + a.rows_off[lo];
         for (int64_t base = r0; base < r1; base += 32) {
             const int64_t i = base + lane;

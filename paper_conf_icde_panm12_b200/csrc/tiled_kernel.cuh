@@ -63,15 +63,8 @@ __global__ void __launch_bounds__(kTiledThreads, 1) k_shortlist_tiled(TiledArgs 
     float* rws = qs + (size_t)QT * ds;                          // [kStages][32][pitch]
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t item = blockIdx.x;
-    int64_t lo = 0, hi = a.ntiles;
-    while (hi - lo > 1) {
-        const int64_t mid = (lo + hi) >> 1;
-        if (a.item_off[mid] <= item) lo = mid;
-        else hi = mid;
-    }
-    const int64_t tile = lo;
-    const int64_t r0 = (item - a.item_off[tile]) * a.chr;
-    const int64_t r1 = min(r0 + (int64_t)a.chr, a.rows[tile]);
+    int64_t r0, r1;
+    const int64_t tile = item_tile_rows(a, item, &r0, &r1);
     const int nst = (int)((r1 - r0 + 31) / 32);
     for (int i = threadIdx.x; i < QT * nv4; i += kTiledThreads) {
         const int slot = i / nv4, v = i % nv4;

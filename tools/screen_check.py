@@ -45,14 +45,14 @@ def main():
     q0 = raw[(4096 + 2048) * 4:].view(np.uint32)
     dots = h[:4096].reshape(128, 32).astype(np.float64)
     t = h[4096:]
-    dch, dcl, beta, m, E = (t[0:128], t[128:256], t[256:384], t[384:512], t[512:640])
+    Da, la, beta, m, E = (t[0:128], t[128:256], t[256:384], t[384:512], t[512:640])
     pos = t[640:768].view(np.uint32)
     mask = t[768:896].view(np.uint32)
     eta = t[1024:1056].astype(np.float64)
-    Sq, Sc, Cc, nqt = t[1056], t[1057], t[1058], int(t[1059])
+    Sq, Sv, na, nqt = t[1056], t[1057], int(t[1058]), int(t[1059])
     nr = t[1152:1280].astype(np.float64)
     sb = t[1280:1408].astype(np.float64)
-    print(f"S={Sq} Sc={Sc} Cc={Cc:.3e} nqt={nqt}")
+    print(f"S={Sq} Sv={Sv} anchors={na} nqt={nqt}")
     perm = ix.export("PERM").astype(np.int64)
     Xh = X.cpu().numpy().astype(np.float64)
     Qh = Q.cpu().numpy().astype(np.float64)
@@ -60,6 +60,7 @@ def main():
     qs = Qh[q0[:nqt]]
     delta = 2.0 ** -11
     worst, widths, npairs, bad = 0.0, [], 0, 0
+    terms = {"E": [], "eta_n": [], "delta_d2": [], "d2": []}
     for i in range(128):
         if mask[i] == 0:
             continue
@@ -82,9 +83,15 @@ def main():
                 if bad < 10:
                     print(f"VIOLATION row {i} q {j}: exact {ex:.6g} lo {lo:.6g} up {up:.6g} d~ {dt:.6g}")
             widths.append((up - lo) / max(ex, 1e-30))
+            terms["E"].append(E[i]); terms["eta_n"].append(eta[j] * nr[i]); terms["delta_d2"].append(delta * dt)
+            terms["d2"].append(ex)
             worst = max(worst, abs(dt - ex) / max(ex, 1e-30))
     print(f"pairs {npairs}, violations {bad}, max |d~2 - d2|/d2 {worst:.3e}, "
           f"bound width/d2 median {np.median(widths) if widths else 0:.3e} max {max(widths) if widths else 0:.3e}")
+    for kk, v in terms.items():
+        if v:
+            print(f"  {kk}: median {np.median(v):.3e} max {np.max(v):.3e}")
+    print(f"  |s r| median {np.median(nr[mask != 0]):.3e} max {np.max(nr[mask != 0]):.3e}")
     sys.exit(1 if bad or npairs == 0 else 0)
 
 
