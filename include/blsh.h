@@ -173,13 +173,16 @@ typedef enum {
     BLSH_EX_ULEAF = 12,     /* int32 [nu]       bucket leaf                                   */
     BLSH_EX_UOFF = 13,      /* int64 [nu+1]     bucket start positions                        */
     BLSH_EX_LEAF_U = 14,    /* int64 [G+1]      first bucket of each leaf                     */
+    BLSH_EX_RGRP = 15,      /* int32 [n_owned]  screen anchor group of every table row (resid.cu) */
+    BLSH_EX_GSTART = 16,    /* int64 [groups+1] first table row of every anchor group          */
     BLSH_EX_POINT_LEAF = 20,/* int32 [n]        leaf of every point (keep_stages)             */
     BLSH_EX_POINT_CODE = 21,/* int32 [n][M]     code (Z^M floor / doubled E8), owned points   */
     BLSH_EX_POINT_KEY = 22, /* uint64 [n][2]    Morton key (hi, lo), owned points             */
     BLSH_EX_Q_LEAF = 30,    /* int32 [nq]       last query: leaf                              */
     BLSH_EX_Q_T = 31,       /* float [nq][M]    projections t                                 */
     BLSH_EX_Q_CODE = 32,    /* int32 [nq][M]    clamped home code                             */
-    BLSH_EX_Q_OOR = 33,     /* int32 [nq]       1 = home code outside the Morton range        */
+    BLSH_EX_Q_OOR = 33,     /* int32 [nq]       1 = home code outside the Morton range; 5 = non-finite
+                               projection (NaN/Inf query, R30): no probes, no candidates      */
     BLSH_EX_Q_KEY = 34,     /* uint64 [nq][2]   home key (0 when out of range)                */
     BLSH_EX_Q_PKEY = 35,    /* uint64 [nq][T][2] probe keys in probe order (0 = invalid)      */
     BLSH_EX_Q_PVALID = 36,  /* int32 [nq][T]    probe key inside the range                    */

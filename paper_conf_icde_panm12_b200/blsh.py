@@ -21,7 +21,7 @@ BLSH_OK, BLSH_ERR_INVALID, BLSH_ERR_OOM, BLSH_ERR_CUDA, BLSH_ERR_RANGE, BLSH_ERR
 _STATUS = {0: "OK", 1: "INVALID", 2: "OOM", 3: "CUDA", 4: "RANGE", 5: "UNSUPPORTED"}
 
 EX = dict(A=0, B=1, W=2, DIRS=3, MU=4, THETA=5, NTYPE=6, DIAM2=7, DA2=8, PERM=10, UKEY=11, ULEAF=12,
-          UOFF=13, LEAF_U=14, POINT_LEAF=20, POINT_CODE=21, POINT_KEY=22, Q_LEAF=30, Q_T=31, Q_CODE=32,
+          UOFF=13, LEAF_U=14, RGRP=15, GSTART=16, POINT_LEAF=20, POINT_CODE=21, POINT_KEY=22, Q_LEAF=30, Q_T=31, Q_CODE=32,
           Q_OOR=33, Q_KEY=34, Q_PKEY=35, Q_PVALID=36, Q_BASE=37, Q_LEVEL=38, Q_TAU=39, Q_INTERVALS=40,
           Q_CAND_OFF=41, Q_CAND=42)
 
@@ -271,7 +271,8 @@ def blsh_merge_topk(packed, n_lists: int, nq: int, k: int, out=None):
 
 _EX_DT = {"A": np.float32, "B": np.float32, "W": np.float32, "DIRS": np.float32, "MU": np.float32,
           "THETA": np.float32, "NTYPE": np.int32, "DIAM2": np.float64, "DA2": np.float64, "PERM": np.int64,
-          "UKEY": np.uint64, "ULEAF": np.int32, "UOFF": np.int64, "LEAF_U": np.int64, "POINT_LEAF": np.int32,
+          "UKEY": np.uint64, "ULEAF": np.int32, "UOFF": np.int64, "LEAF_U": np.int64,
+          "RGRP": np.int32, "GSTART": np.int64, "POINT_LEAF": np.int32,
           "POINT_CODE": np.int32, "POINT_KEY": np.uint64, "Q_LEAF": np.int32, "Q_T": np.float32,
           "Q_CODE": np.int32, "Q_OOR": np.int32, "Q_KEY": np.uint64, "Q_PKEY": np.uint64,
           "Q_PVALID": np.int32, "Q_BASE": np.int64, "Q_LEVEL": np.int32, "Q_TAU": np.int64,

@@ -454,7 +454,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.qleaf = w.qleaf; a.qt = w.qt; a.qcode = w.qcode; a.qoor = w.qoor; a.qkey = w.qkey;
     a.pkey = w.pkey; a.pvalid = w.pvalid; a.ivl = w.ivl; a.base = w.base; a.cnt = w.cnt; a.level = w.level;
     a.lperm = lperm; a.lcnt = lcnt;
-    a.dr = ix.dr; a.Rh = ix.Rh.p; a.rconst = ix.rconst.as<float4>(); a.bscale = ix.bscale.as<float>();
+    a.dr = ix.dr; a.Rh = ix.Rh.p; a.rconst = ix.rconst.as<float4>(); a.rgrp = ix.rgrp.as<uint32_t>();
     a.anc = ix.anc.as<float>();
     // a1+a2
     launches += launch_route_hash(a, s);
@@ -877,6 +877,8 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
             return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");
         }
         case BLSH_EX_ULEAF: dev_src = uleaf_p; bytes = (size_t)nu * 4; break;
+        case BLSH_EX_RGRP: dev_src = idx->rgrp.p; bytes = (size_t)idx->n_owned * 4; break;
+        case BLSH_EX_GSTART: dev_src = idx->gstart.p; bytes = (size_t)(idx->nanchor + 1) * 8; break;
         case BLSH_EX_UOFF: {
             bytes = (size_t)(nu + 1) * 8;
             if (dst && cap >= bytes) {
@@ -952,7 +954,7 @@ blsh_status blsh_export(const blsh_index* idx, int32_t what, void* dst, size_t c
                     if (cudaMemcpy(dst, tq.qoor, bytes, cudaMemcpyDeviceToHost) != cudaSuccess)
                         return fail(BLSH_ERR_CUDA, "export copy failed");
                     int32_t* o = (int32_t*)dst;
-                    for (int64_t i = 0; i < nq; ++i) o[i] &= 1;
+                    for (int64_t i = 0; i < nq; ++i) o[i] &= ~2;   // hide the shard bit (1 range, 4 non-finite)
                 }
                 if (needed) *needed = bytes;
                 return (dst && cap >= bytes) ? BLSH_OK : fail(BLSH_ERR_INVALID, "dst too small");

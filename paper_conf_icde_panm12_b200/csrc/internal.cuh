@@ -156,10 +156,6 @@ struct ExtraTable {
 
 }  // namespace blsh
 
-namespace blsh {
-constexpr int kAnchorShift = 9;   // rows per anchor block of the screen's compact table = 512
-}
-
 struct blsh_index {
     // metadata
     int64_t n = 0, n_owned = 0, nu = 0;
@@ -184,13 +180,15 @@ struct blsh_index {
     blsh::DevBuf uleaf;   // [nu] int32
     blsh::DevBuf uoff;    // [nu+1] uint32
     blsh::DevBuf leaf_u;  // [G+1] int64
-    // device: the short-list screen's compact rows (resid.cu): anchor blocks of 2^kAnchorShift rows
+    // device: the short-list screen's compact rows (resid.cu): anchor groups of consecutive buckets
     int dr = 0;                 // fp16 columns per row (ds rounded up to 64)
-    int64_t nanchor = 0;        // anchor blocks
-    blsh::DevBuf anc;           // [nanchor][dr] fp32 anchors a_b
-    blsh::DevBuf bscale;        // [nanchor] fp32 power-of-two scale s_b
-    blsh::DevBuf Rh;            // [n_owned][dr] fp16 residuals r = (x - a_b) / s_b
-    blsh::DevBuf rconst;        // [n_owned] float4 (|s_b r|^2, a_b . s_b r, |s_b r|, G)
+    int64_t nanchor = 0;        // anchor groups
+    float anchor_tau2 = 0.f;    // grouping threshold (squared distance between consecutive bucket means)
+    blsh::DevBuf anc;           // [nanchor][dr] fp32 anchors a_g
+    blsh::DevBuf gstart;        // [nanchor+1] int64 first table row of every group
+    blsh::DevBuf rgrp;          // [n_owned] uint32 group of every table row
+    blsh::DevBuf Rh;            // [n_owned][dr] fp16 residuals r = (x - a_g) / s_g
+    blsh::DevBuf rconst;        // [n_owned] float4 (|s_g r|^2, s_g, |s_g r|, G)
     // L > 1 hash tables
     int L = 1;
     std::vector<std::unique_ptr<blsh::ExtraTable>> xt;   // tables 1..L-1

@@ -44,7 +44,7 @@ struct QueryArgs {
     int dr;
     const void* Rh;          // [n][dr] fp16
     const float4* rconst;
-    const float* bscale;
+    const uint32_t* rgrp;    // [n_owned] anchor group of every table row
     const float* anc;        // [anchor blocks][dr]
 };
 

@@ -14,7 +14,7 @@
 //   |q_j - x~|^2 = K_aj - 2 (q_j - c).(s r) - 2 (c - a).(s r) + |s r|^2
 //               ~ K_aj + beta_i + m_i D_ij,
 //   beta_i = nu_i - 2 S_v s D_i,a(i),   m_i = -2 S s.
-// An item spans < 48 anchor blocks (k_tile_items), so every row's anchor has a column.
+// An item spans <= 48 anchor groups (k_tile_items), so every row's anchor has a column.
 // Every rounding in that chain is bounded (DESIGN.md §7 "Screen bound"):
 //   |d2(q_j, x_i) - d~2| <= delta d~2 + E_i + eta_j n_i,
 // so lo = d~2 (1 - delta) - (E_i + eta_j n_i) <= d2 <= d~2 (1 + delta) + (E_i + eta_j n_i) = up.
@@ -35,8 +35,7 @@ constexpr int kSxN = 32 + kSxAnc;           // MMA N: 32 queries + the item's an
 constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
 constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 80 rows x 64 fp16 columns (10 KB)
 constexpr int kSxMaxDr = 640;
-constexpr int kSxNst = 8;                   // A ring stages
-constexpr int kSxAhead = kSxNst - 2;        // stages in flight ahead of the MMA
+// A ring: NST stages of 16 KB (template: 8, or 6 / 4 when the B operand is large)
 // instruction descriptor: D f32, A/B f16, K-major both, N = 80, M = 128
 constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u >> 4) << 24);
 // error model (DESIGN.md §7 "Screen bound")
@@ -44,7 +43,7 @@ constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, re
 constexpr float kSxDelta = 0x1p-11f;        // relative slack on d~2 (AM-GM split 2^-12, K table 2^-13, fp32 ops)
 
 struct SxSmem {
-    uint64_t afull[kSxNst], aempty[kSxNst];
+    uint64_t afull[8], aempty[8];
     uint64_t tfull[4], tempty[4];
     uint32_t tmem_base;
     float S, Sv;
@@ -86,12 +85,20 @@ __device__ __forceinline__ uint32_t sw128_off(int n, int ch) {
     return (uint32_t)((n >> 3) * 1024 + (n & 7) * 128 + ((ch ^ (n & 7)) << 4));
 }
 
-size_t screen_smem_bytes(int dr) {
-    return ((sizeof(SxSmem) + 1023) & ~size_t(1023)) + (size_t)(dr / 64) * kSxPanelB + (size_t)kSxNst * kSxStage;
+size_t screen_smem_bytes(int dr, int nst) {
+    return ((sizeof(SxSmem) + 1023) & ~size_t(1023)) + (size_t)(dr / 64) * kSxPanelB + (size_t)nst * kSxStage;
+}
+// the deepest A ring that fits (0: none)
+int screen_stages(int dr) {
+    for (int nst : {8, 6, 4})
+        if (screen_smem_bytes(dr, nst) <= 227 * 1024) return nst;
+    return 0;
 }
 
-template <int KT>
+template <int KT, int NST>
 __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
+    constexpr int kSxNst = NST;
+    constexpr int kSxAhead = NST - 2;          // stages in flight ahead of the MMA
     extern __shared__ __align__(1024) unsigned char smraw[];
     SxSmem& S = *reinterpret_cast<SxSmem*>(smraw);
     const int ds = a.ds, dr = a.dr, np = dr >> 6;
@@ -328,7 +335,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             sb = 0.f;
             if (ri.y != 0u) {
                 rc = __ldg(a.rconst + ri.x);
-                sb = __ldg(a.bscale + (ri.x >> kAnchorShift));
+                sb = rc.y;                      // the group's scale s_g
             }
         };
         uint4 ri_n;

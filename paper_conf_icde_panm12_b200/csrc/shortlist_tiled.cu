@@ -48,7 +48,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
                                                             int segcap, Seg* __restrict__ segs,
                                                             int32_t* __restrict__ nseg,
                                                             int64_t* __restrict__ rows,
-                                                            int64_t* __restrict__ nanch) {
+                                                            int64_t* __restrict__ nanch,
+                                                            const uint32_t* __restrict__ rgrp) {
     extern __shared__ uint32_t sm[];
     const int cap = 2 * QT * (T + 1);
     int npow = 1;
@@ -193,16 +194,16 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
             out += __popc(bm);
         }
         __syncwarp();
-        // anchor blocks (2^kAnchorShift table rows) of the union, numbered in row order:
-        // segment i covers blocks [a0, a1]; it shares a0 with segment i-1 when that one ends in it
+        // anchor groups (resid.cu: runs of table rows) of the union, numbered in row order:
+        // segment i covers groups [a0, a1]; it shares a0 with segment i-1 when that one ends in it
         uint32_t na = 0, prev_last = 0xFFFFFFFFu;
         for (int base = 0; base < out; base += 32) {
             const int i = base + tid;
             uint32_t a0 = 0, a1 = 0, pl = 0xFFFFFFFFu;
             if (i < out) {
                 const Seg sg = S[i];
-                a0 = sg.start >> kAnchorShift;
-                a1 = (sg.start + sg.len - 1) >> kAnchorShift;
+                a0 = rgrp ? rgrp[sg.start] : 0u;
+                a1 = rgrp ? rgrp[sg.start + sg.len - 1] : 0u;
             }
             const uint32_t up = __shfl_up_sync(BLSH_FULL, a1, 1);
             pl = tid == 0 ? prev_last : up;
@@ -231,7 +232,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
 __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ segs, const int32_t* __restrict__ nseg,
                                                      int segcap, const int64_t* __restrict__ rows_off,
                                                      const int64_t* __restrict__ aoff, uint4* __restrict__ rowinfo,
-                                                     uint32_t* __restrict__ slot_anchor) {
+                                                     uint32_t* __restrict__ slot_anchor,
+                                                     const uint32_t* __restrict__ rgrp) {
     const int64_t t = blockIdx.x;
     const Seg* S = segs + (size_t)t * segcap;
     uint4* out = rowinfo + rows_off[t];
@@ -240,13 +242,13 @@ __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ seg
     const int lane = threadIdx.x & 31;
     for (int sI = threadIdx.x >> 5; sI < ns; sI += 8) {
         const Seg sg = S[sI];
-        const uint32_t a0 = sg.start >> kAnchorShift;
+        const uint32_t a0 = rgrp ? rgrp[sg.start] : 0u;
         for (uint32_t i = lane; i < sg.len; i += 32) {
             const uint32_t row = sg.start + i;
-            const uint32_t blk = row >> kAnchorShift;
-            const int64_t slot = ab + sg.abase + (blk - a0);
+            const uint32_t grp = rgrp ? rgrp[row] : 0u;
+            const int64_t slot = ab + sg.abase + (grp - a0);
             out[sg.off + i] = make_uint4(row, sg.mask, (uint32_t)slot, 0u);
-            if (slot_anchor && (i == 0 || (row & ((1u << kAnchorShift) - 1u)) == 0u)) slot_anchor[slot] = blk;
+            if (slot_anchor && (i == 0 || rgrp[row - 1] != grp)) slot_anchor[slot] = grp;
         }
     }
 }
@@ -342,10 +344,9 @@ struct TiledArgs {
     int dr;                         // screen: fp16 columns of the compact rows
     const __half* Rh;               // screen: [n][dr] fp16 residual rows (resid.cu)
     const float4* rconst;           // screen: [n] per-row bound constants
-    const float* bscale;            // screen: [anchor blocks] scale s_b
     const float* ktab;              // screen: [K slots][QT] K_aj = |q_j - a|^2
-    const float* anc;               // screen: [anchor blocks][dr] fp32 anchors
-    const uint32_t* slot_anchor;    // screen: [K slots] anchor block of each slot
+    const float* anc;               // screen: [anchor groups][dr] fp32 anchors
+    const uint32_t* slot_anchor;    // screen: [K slots] anchor group of each slot
     uint32_t* ufin;                 // TC -> k_tc_rescore: [n_items][QT] final screen bound U_j (fp32 bits)
     int32_t* scnt;                  // TC -> k_tc_rescore: [n_items][QT][4] buffered pairs per epilogue warp
 };
@@ -542,7 +543,7 @@ int shortlist_kind(int ds, int dr, int T, int k) {
     const bool simt_ok = tiled_smem_bytes(ds) <= 227 * 1024;
     const bool tc_ok = screen_variant() == 1
                            ? (k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024)
-                           : (k <= kTcMaxK && dr >= 64 && dr <= kSxMaxDr && screen_smem_bytes(dr) <= 227 * 1024);
+                           : (k <= kTcMaxK && dr >= 64 && dr <= kSxMaxDr && screen_stages(dr) > 0);
     if (mode && std::strcmp(mode, "simt") == 0) return simt_ok ? 1 : 0;
     if (tc_ok) return 2;
     return simt_ok ? 1 : 0;
@@ -647,7 +648,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int64_t* aoff = reinterpret_cast<int64_t*>(tb + 14 * slot);
     BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
     k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, tile_off, segcap,
-                                                                  segbuf.as<Seg>(), nseg, rows, nanch);
+                                                                  segbuf.as<Seg>(), nseg, rows, nanch, a.rgrp);
     BLSH_LAUNCH_CHECK();
     ++*launches;
     scan_exclusive_i64(rows, rows_off, ntiles, scan, s);
@@ -681,7 +682,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (use_tc && ntiles > 0) {
         if (!use_f16) BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
         k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(segbuf.as<Seg>(), nseg, segcap, rows_off, aoff, ri,
-                                                       use_f16 ? slot_anchor : nullptr);
+                                                       use_f16 ? slot_anchor : nullptr, use_f16 ? a.rgrp : nullptr);
         BLSH_LAUNCH_CHECK();
         ++*launches;
     }
@@ -720,12 +721,12 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.dr = a.dr;
     ta.Rh = reinterpret_cast<const __half*>(a.Rh);
     ta.rconst = a.rconst;
-    ta.bscale = a.bscale;
     ta.ktab = ktab;
     ta.slot_anchor = slot_anchor;
     if (const char* dm = std::getenv("BLSH_TC_MODE")) ta.dbgmode = std::atoi(dm);
     const size_t smem = tiled_smem_bytes(a.ds);
-    const size_t tc_smem = use_f16 ? screen_smem_bytes(a.dr) : tc_smem_bytes(a.ds);
+    const int nst = use_f16 ? screen_stages(a.dr) : 0;
+    const size_t tc_smem = use_f16 ? screen_smem_bytes(a.dr, nst) : tc_smem_bytes(a.ds);
     const char* dbg_path = std::getenv("BLSH_TC_DEBUG");
     DevBuf dbgbuf;
     constexpr int kDbgN = 4096 + 2048;
@@ -750,8 +751,10 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_f16) {
-            auto kern = k <= 8 ? k_screen_f16<8>
-                      : (k <= 12 ? k_screen_f16<12> : (k <= 16 ? k_screen_f16<16> : k_screen_f16<32>));
+            auto pick = [&](auto k8, auto k12, auto k16, auto k32) { return k <= 8 ? k8 : (k <= 12 ? k12 : (k <= 16 ? k16 : k32)); };
+            auto kern = nst == 8 ? pick(k_screen_f16<8, 8>, k_screen_f16<12, 8>, k_screen_f16<16, 8>, k_screen_f16<32, 8>)
+                      : nst == 6 ? pick(k_screen_f16<8, 6>, k_screen_f16<12, 6>, k_screen_f16<16, 6>, k_screen_f16<32, 6>)
+                                 : pick(k_screen_f16<8, 4>, k_screen_f16<12, 4>, k_screen_f16<16, 4>, k_screen_f16<32, 4>);
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kSxThreads, tc_smem, s>>>(ta);
         } else if (use_tc) {

@@ -54,6 +54,10 @@ def main():
     sb = t[1280:1408].astype(np.float64)
     print(f"S={Sq} Sv={Sv} anchors={na} nqt={nqt}")
     perm = ix.export("PERM").astype(np.int64)
+    rgrp = ix.export("RGRP")
+    gstart = ix.export("GSTART")
+    sizes = np.diff(gstart)
+    print(f"anchor groups {len(sizes)}: rows per group median {np.median(sizes):.0f} mean {sizes.mean():.1f} max {sizes.max()}")
     Xh = X.cpu().numpy().astype(np.float64)
     Qh = Q.cpu().numpy().astype(np.float64)
     Xp = Xh[perm]
@@ -65,8 +69,8 @@ def main():
         if mask[i] == 0:
             continue
         p = int(pos[i])
-        b = p >> 9
-        blk = Xp[b * 512: (b + 1) * 512]
+        b = int(rgrp[p])
+        blk = Xp[gstart[b]: gstart[b + 1]]
         anc = blk.mean(0).astype(np.float32).astype(np.float64)
         x = Xp[p]
         for j in range(nqt):
