@@ -49,6 +49,10 @@ struct SxSmem {
     float S, Sv;
     float red[16];
     float ca[kSxAnc];               // per anchor column: error constant of the D_ia term
+    float cdist[kSxAnc];            // per anchor column: |c - a|
+    int arow[kSxAnc + 1];           // item rows of anchor column s: [arow[s], arow[s+1]) (item-relative)
+    int cum[kSxAnc + 1];            // stream order: anchors by |c - a|; cum[k] = rows of the k nearest
+    int aord[kSxAnc];               // anchor column of stream rank k
     alignas(16) float eta[QT];
     uint32_t umin[QT];
     int scnt[4][QT];
@@ -197,6 +201,45 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             const float cn = sqrtf(sv) * (1.0f + 0x1p-18f);
             S.ca[la] = ((kSxEpsAcc + 0x1p-11f + 0x1p-23f) * (1.0f + 0x1p-9f) * cn + sqrtf((float)ds) * 0x1p-25f * Sv) *
                        (1.0f + 0x1p-10f);
+            S.cdist[la] = la < na ? cn : __int_as_float(0x7F800000);
+        }
+    }
+    // Stream order: the item's rows grouped by anchor (contiguous), anchors nearest to c first,
+    // so the rows closest to the tile come early and the running bounds U_j tighten before most
+    // of the union has been screened (fewer buffered pairs).  Results do not depend on it.
+    __syncthreads();                                           // S.cdist from every warp
+    if (warp == 0) {
+        for (int la = lane; la <= kSxAnc; la += 32) {         // first item row of anchor column la
+            int v = (int)(r1 - r0);
+            if (la < na) {
+                int64_t lo = r0, hi = r1;
+                while (lo < hi) {
+                    const int64_t m = (lo + hi) >> 1;
+                    if (RI[m].z < slot0 + (uint32_t)la) lo = m + 1;
+                    else hi = m;
+                }
+                v = (int)(lo - r0);
+            }
+            S.arow[la] = v;
+        }
+        __syncwarp();
+        for (int la = lane; la < kSxAnc; la += 32) {          // rank by (|c - a|, column)
+            int rk = 0;
+            const float me = S.cdist[la];
+            for (int o = 0; o < na; ++o) {
+                const float x = S.cdist[o];
+                rk += (x < me || (x == me && o < la)) ? 1 : 0;
+            }
+            if (la < na) S.aord[rk] = la;
+        }
+        __syncwarp();
+        if (lane == 0) {
+            int c = 0;
+            for (int kk = 0; kk < na; ++kk) {
+                S.cum[kk] = c;
+                c += S.arow[S.aord[kk] + 1] - S.arow[S.aord[kk]];
+            }
+            S.cum[na] = c;
         }
     }
     // per query: qn = |q_j - c|, un = S |u_j| (of the fp16 values), eta_j
@@ -245,6 +288,17 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     tc_fence_after();
     const uint32_t tbase = S.tmem_base;
     const int nstage = nblk * np;
+    // stream position -> item-relative union row (anchors in |c - a| order)
+    auto srow = [&](int p) -> int64_t {
+        int lo = 0, hi = na;                                   // largest k with cum[k] <= p
+        while (hi - lo > 1) {
+            const int m = (lo + hi) >> 1;
+            if (S.cum[m] <= p) lo = m;
+            else hi = m;
+        }
+        return r0 + S.arow[S.aord[lo]] + (p - S.cum[lo]);
+    };
+    const int nrow = (int)(r1 - r0);
 
     if (warp < kSxProd) {
         // ======================= producers =======================
@@ -259,13 +313,16 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             if (g < nstage) {
                 const int b = g / np, p = g - b * np;
                 if (p == 0) {
+                    // thread pc of each 8-thread group loads the entry of row rr + 16 pc; shuffles
+                    // hand every thread of the group the entries of its 8 rows
+                    const int sp = b * 128 + rr + 16 * pc;
+                    uint4 f = make_uint4(0u, 0u, 0u, 0u);
+                    if (sp < nrow) f = RI[srow(sp)];
 #pragma unroll
                     for (int i = 0; i < 8; ++i) {
-                        const int64_t r = r0 + (int64_t)b * 128 + rr + 16 * i;
-                        uint2 e = make_uint2(0u, 0u);
-                        if (r < r1) { const uint4 f = RI[r]; e = make_uint2(f.x, f.y); }
-                        pos[i] = e.x;
-                        ok[i] = e.y != 0u;
+                        const int src = (lane & ~7) | i;
+                        pos[i] = __shfl_sync(BLSH_FULL, f.x, src);
+                        ok[i] = __shfl_sync(BLSH_FULL, f.y, src) != 0u;
                     }
                 }
                 const int slot = g % nst;
@@ -329,8 +386,8 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         float* Tt = S.tr[ew];
         // this lane's row of block b (row phase)
         auto row_meta = [&](int b, uint4& ri, float4& rc, float& sb) {
-            const int64_t r = r0 + (int64_t)b * 128 + quad * 32 + lane;
-            ri = r < r1 ? RI[r] : make_uint4(0u, 0u, 0u, 0u);
+            const int sp = b * 128 + quad * 32 + lane;
+            ri = sp < nrow ? RI[srow(sp)] : make_uint4(0u, 0u, 0u, 0u);
             rc = make_float4(0.f, 0.f, 0.f, 0.f);
             sb = 0.f;
             if (ri.y != 0u) {
@@ -421,9 +478,16 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                     const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
                     if (my_cnt == kTcScap) {                       // full: drop what the tighter U excludes
                         int c2 = 0;
-                        for (int t = 0; t < kTcScap; ++t) {
-                            const unsigned long long f = SBj[t];
-                            if (__uint_as_float((uint32_t)(f >> 32)) <= U) SBj[c2++] = f;
+                        const ulonglong2* B2 = reinterpret_cast<const ulonglong2*>(SBj);
+                        for (int t0 = 0; t0 < kTcScap / 2; t0 += 8) {   // 8 independent 16-byte loads per batch
+                            ulonglong2 f[8];
+#pragma unroll
+                            for (int u = 0; u < 8; ++u) f[u] = B2[t0 + u];
+#pragma unroll
+                            for (int u = 0; u < 8; ++u) {
+                                if (__uint_as_float((uint32_t)(f[u].x >> 32)) <= U) SBj[c2++] = f[u].x;
+                                if (__uint_as_float((uint32_t)(f[u].y >> 32)) <= U) SBj[c2++] = f[u].y;
+                            }
                         }
                         my_cnt = c2;
                         if (my_cnt > 3 * kTcScap / 4) my_fail = true;   // exact scan of j's rows later

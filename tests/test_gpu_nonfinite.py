@@ -57,7 +57,12 @@ def test_nonfinite_queries(blsh, orc, quantizer, probe, T, hier):
         assert np.all(ids[q] == -1) and np.all(np.isinf(d2[q]))
     assert np.array_equal(ix.export("Q_PVALID"), ox.get("q_pvalid").ravel())
     assert np.array_equal(ix.export("Q_PKEY"), ox.get("q_pkey").ravel())
-    gc, oc = gpu_candidates(ix, T), ox.candidates()
+    if quantizer == 1 and hier:   # E8 code hierarchy: candidates as deduplicated lists (list path)
+        off, lst = ix.export("Q_CAND_OFF"), ix.export("Q_CAND")
+        gc = [np.sort(lst[off[q]:off[q + 1]]) for q in range(len(Q))]
+    else:
+        gc = gpu_candidates(ix, T)
+    oc = ox.candidates()
     for q in range(len(Q)):
         assert np.array_equal(gc[q], oc[q]), f"candidate set of query {q} differs"
     assert np.array_equal(nc, onc)

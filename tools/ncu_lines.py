@@ -17,7 +17,7 @@ import sys
 import tempfile
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-LIB = os.path.join(ROOT, "paper_conf_icde_panm12_b200", "_lib", "libblsh.so")
+LIB = os.environ.get("BLSH_LIB") or os.path.join(ROOT, "paper_conf_icde_panm12_b200", "_lib", "libblsh.so")
 
 
 def line_map(kernel_sub):
