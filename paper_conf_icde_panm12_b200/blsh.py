@@ -15,7 +15,7 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "_lib", "libblsh.so")
+LIB_PATH = os.environ.get("BLSH_LIB_PATH") or os.path.join(_HERE, "_lib", "libblsh.so")   # (variant builds: experiments)
 
 BLSH_OK, BLSH_ERR_INVALID, BLSH_ERR_OOM, BLSH_ERR_CUDA, BLSH_ERR_RANGE, BLSH_ERR_UNSUPPORTED = range(6)
 _STATUS = {0: "OK", 1: "INVALID", 2: "OOM", 3: "CUDA", 4: "RANGE", 5: "UNSUPPORTED"}

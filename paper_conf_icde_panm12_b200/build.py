@@ -17,7 +17,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-OUT_DIR = os.path.join(HERE, "_lib")
+OUT_DIR = os.environ.get("BLSH_BUILD_DIR") or os.path.join(HERE, "_lib")   # (experiments: variant builds)
 LIB = os.path.join(OUT_DIR, "libblsh.so")
 OBJ_DIR = os.path.join(OUT_DIR, "obj")
 
@@ -25,6 +25,7 @@ NVCC = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC",
          "-Xcompiler", "-ffp-contract=off", "-Xcompiler", "-fno-fast-math", "-I", os.path.join(ROOT, "include")]
+FLAGS += os.environ.get("BLSH_NVCC_FLAGS", "").split()   # (experiments: e.g. -DBLSH_SPIN_WAIT=1)
 
 
 def sources():

@@ -455,6 +455,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.pkey = w.pkey; a.pvalid = w.pvalid; a.ivl = w.ivl; a.base = w.base; a.cnt = w.cnt; a.level = w.level;
     a.lperm = lperm; a.lcnt = lcnt;
     a.dr = ix.dr; a.Rh = ix.Rh.p; a.rconst = ix.rconst.as<float4>(); a.rgrp = ix.rgrp.as<uint32_t>();
+    a.natom = (ix.n_owned + 7) / 8;
     a.anc = ix.anc.as<float>();
     // a1+a2
     launches += launch_route_hash(a, s);

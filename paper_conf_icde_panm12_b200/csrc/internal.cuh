@@ -187,8 +187,8 @@ struct blsh_index {
     blsh::DevBuf anc;           // [nanchor][dr] fp32 anchors a_g
     blsh::DevBuf gstart;        // [nanchor+1] int64 first table row of every group
     blsh::DevBuf rgrp;          // [n_owned] uint32 group of every table row
-    blsh::DevBuf Rh;            // [n_owned][dr] fp16 residuals r = (x - a_g) / s_g
-    blsh::DevBuf rconst;        // [n_owned] float4 (|s_g r|^2, s_g, |s_g r|, G)
+    blsh::DevBuf Rh;            // fp16 residuals r = (x - a_g) / s_g in swizzled 8-row atoms (resid.cu)
+    blsh::DevBuf rconst;        // [atoms * 8] float4 (|s_g r|^2, s_g, |s_g r|, G); zero for padding rows
     // L > 1 hash tables
     int L = 1;
     std::vector<std::unique_ptr<blsh::ExtraTable>> xt;   // tables 1..L-1

@@ -42,7 +42,8 @@ struct QueryArgs {
     int32_t* lcnt;           // [2G] leaf counts, scatter cursors
     // short-list screen's compact table (resid.cu)
     int dr;
-    const void* Rh;          // [n][dr] fp16
+    const void* Rh;          // fp16 rows in swizzled 8-row atoms (resid.cu)
+    int64_t natom;           // atoms of the table
     const float4* rconst;
     const uint32_t* rgrp;    // [n_owned] anchor group of every table row
     const float* anc;        // [anchor blocks][dr]

@@ -9,6 +9,12 @@
 // a_g (fp32 mean of its rows, fp64 sums), a power-of-two scale s_g with
 // max |x - a_g| / s_g in [2^14, 2^15), and per row the fp16 residual
 // r = fp16_rn((x - a_g) / s_g), padded with zeros to dr (a multiple of 64) columns.
+// Layout of the fp16 rows ("atoms"): table rows 8a..8a+7 form atom a; panel-major: for every
+// 64-column panel p the atoms are consecutive KBs (panel p, atom a at (p * atoms + a) KB), an
+// atom's 8 x 128 bytes with 16-byte chunk ch of row r stored at chunk ch ^ r -- the
+// 128-byte-swizzled K-major layout the tensor core reads from shared memory.  A run of
+// consecutive table rows (a bucket) is then one contiguous bulk copy per panel, with no
+// per-16-byte copies and no swizzling on the device.
 // x~ = a_g + s_g r is the screen's stand-in for x; per row the library keeps, from fp64
 // sums,
 //   nu = |s_g r|^2,  s_g,  n = |s_g r| (rounded up),
@@ -101,7 +107,7 @@ __global__ void k_group_rows(const uint8_t* __restrict__ flag, const int64_t* __
 
 // One CTA per group: anchor, scale, fp16 residual rows, per-row bound constants.
 __global__ void __launch_bounds__(kAT) k_anchor_rows(const float* __restrict__ Xp, const int64_t* __restrict__ gstart,
-                                                     int ds, int dr, float* __restrict__ anc,
+                                                     int ds, int dr, int64_t natom, float* __restrict__ anc,
                                                      __half* __restrict__ Rh, float4* __restrict__ rconst) {
     extern __shared__ float a32[];          // [dr] the group's anchor
     __shared__ double red[kAT / 32];
@@ -144,7 +150,9 @@ __global__ void __launch_bounds__(kAT) k_anchor_rows(const float* __restrict__ X
     for (int64_t r = warp; r < nr; r += kAT / 32) {
         const int64_t row = r0 + r;
         const float* x = Xp + (size_t)row * ds;
-        __half* out = Rh + (size_t)row * dr;
+        // panel c >> 6, atom (row >> 3), row (row & 7), chunk ((c >> 3) & 7) ^ (row & 7), element c & 7
+        __half* out = Rh + (size_t)(row >> 3) * 512 + (row & 7) * 64;
+        const int sw = (int)(row & 7);
         double nu = 0.0, e2 = 0.0;
         for (int c = lane; c < dr; c += 32) {
             __half h = __float2half_rn(0.0f);
@@ -157,7 +165,7 @@ __global__ void __launch_bounds__(kAT) k_anchor_rows(const float* __restrict__ X
                 const double ex = diff - rr;
                 e2 += ex * ex;
             }
-            out[c] = h;
+            out[(size_t)(c >> 6) * natom * 512 + ((((c >> 3) & 7) ^ sw) << 3) + (c & 7)] = h;
         }
         nu = warp_sum_d(nu);
         e2 = warp_sum_d(e2);
@@ -182,8 +190,11 @@ void build_screen_rows(blsh_index& ix, cudaStream_t s) {
     const int64_t n = ix.n_owned, nu = ix.nu;
     const int ds = ix.ds, dr = screen_cols(ds);
     ix.dr = dr;
-    ix.Rh.alloc((size_t)std::max<int64_t>(n, 1) * dr * sizeof(__half));
-    ix.rconst.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(float4));
+    const int64_t natom = (n + 7) / 8;   // rows padded to whole atoms (zero rows)
+    ix.Rh.alloc((size_t)std::max<int64_t>(natom, 1) * 8 * dr * sizeof(__half));
+    BLSH_CUDA(cudaMemsetAsync(ix.Rh.p, 0, (size_t)std::max<int64_t>(natom, 1) * 8 * dr * sizeof(__half), s));
+    ix.rconst.alloc((size_t)std::max<int64_t>(natom, 1) * 8 * sizeof(float4));
+    BLSH_CUDA(cudaMemsetAsync(ix.rconst.p, 0, (size_t)std::max<int64_t>(natom, 1) * 8 * sizeof(float4), s));
     ix.rgrp.alloc((size_t)std::max<int64_t>(n, 1) * sizeof(uint32_t));
     if (n == 0 || nu == 0) {
         ix.nanchor = 0;
@@ -235,7 +246,7 @@ void build_screen_rows(blsh_index& ix, cudaStream_t s) {
     ix.anc.alloc((size_t)ng * dr * sizeof(float));
     const size_t smem = (size_t)dr * sizeof(float);
     BLSH_CUDA(cudaFuncSetAttribute(k_anchor_rows, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    k_anchor_rows<<<(unsigned)ng, kAT, smem, s>>>(ix.Xp.as<float>(), ix.gstart.as<int64_t>(), ds, dr,
+    k_anchor_rows<<<(unsigned)ng, kAT, smem, s>>>(ix.Xp.as<float>(), ix.gstart.as<int64_t>(), ds, dr, natom,
                                                    ix.anc.as<float>(), ix.Rh.as<__half>(), ix.rconst.as<float4>());
     BLSH_LAUNCH_CHECK();
     BLSH_CUDA(cudaStreamSynchronize(s));

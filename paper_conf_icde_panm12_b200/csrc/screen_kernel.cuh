@@ -23,18 +23,19 @@
 // exact fp32 distance of the survivors from the fp32 rows.  The screen only decides
 // which pairs get exact work; results equal the warp short-list's.
 //
-// Warp roles (9 warps): 0-3 producers (cp.async of the block's rows, 16 B per lane),
-// 4 MMA issuer + TMEM allocation, 5-8 epilogue (TMEM lane quadrant = warp % 4).
+// Warp roles (12 warps): 0 producer (bulk copies of swizzled 8-row atoms), 1 MMA issuer + TMEM
+// allocation, 2-3 setup only, 4-11 epilogue (TMEM lane quadrant = warp % 4, two warps per
+// quadrant, 16 rows each).
 
-constexpr int kSxProd = 4;                  // producer warps
-constexpr int kSxMma = 4;                   // MMA warp index
-constexpr int kSxEpi0 = 5;                  // first epilogue warp
-constexpr int kSxThreads = 9 * 32;
+constexpr int kSxMma = 1;                   // MMA warp index
+constexpr int kSxEpi0 = 4;                  // first epilogue warp
+constexpr int kSxEpiN = 8;                  // epilogue warps: 2 per TMEM lane quadrant (16 rows each)
+constexpr int kSxThreads = (kSxEpi0 + kSxEpiN) * 32;
 constexpr int kSxAnc = 48;                  // anchor columns per item
 constexpr int kSxN = 32 + kSxAnc;           // MMA N: 32 queries + the item's anchors
 constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
 constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 80 rows x 64 fp16 columns (10 KB)
-constexpr int kSxMaxDr = 640;
+constexpr int kSxMaxDr = 512;            // (the setup stages the tile's queries in the A ring)
 // A ring: NST stages of 16 KB (template: 8, or 6 / 4 when the B operand is large)
 // instruction descriptor: D f32, A/B f16, K-major both, N = 80, M = 128
 constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u >> 4) << 24);
@@ -42,23 +43,25 @@ constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u
 constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, relative to sum |a_k b_k|
 constexpr float kSxDelta = 0x1p-11f;        // relative slack on d~2 (AM-GM split 2^-12, K table 2^-13, fp32 ops)
 
+constexpr int kSxNM = 8;                    // block metadata ring (row entries + bound constants)
+constexpr int kSxMA = 4;                    // metadata fetched this many blocks ahead of the producers
+
 struct SxSmem {
     uint64_t afull[8], aempty[8];
     uint64_t tfull[4], tempty[4];
+    uint64_t mfull[kSxNM], cfull[kSxNM], mempty[kSxNM];
+    alignas(16) uint4 mrow[kSxNM][128];    // per block: (table row, query mask, K slot, -) of its 128 rows
+    alignas(16) float4 mcon[kSxNM][128];   // per block: the rows' bound constants (resid.cu)
     uint32_t tmem_base;
     float S, Sv;
     float red[16];
     float ca[kSxAnc];               // per anchor column: error constant of the D_ia term
-    float cdist[kSxAnc];            // per anchor column: |c - a|
-    int arow[kSxAnc + 1];           // item rows of anchor column s: [arow[s], arow[s+1]) (item-relative)
-    int cum[kSxAnc + 1];            // stream order: anchors by |c - a|; cum[k] = rows of the k nearest
-    int aord[kSxAnc];               // anchor column of stream rank k
     alignas(16) float eta[QT];
     uint32_t umin[QT];
-    int scnt[4][QT];
-    float tr[4][32 * 33];           // per epilogue warp: transposed dots [query][row]
-    float4 rf[4][32];               // per epilogue warp and row: beta, m, E, n
-    uint4 ru[4][32];                // per epilogue warp and row: mask, table row, K slot
+    int scnt[kSxEpiN][QT];
+    float tr[kSxEpiN][32 * 17];     // per epilogue warp: transposed dots [query][row of its 16]
+    float4 rf[kSxEpiN][16];         // per epilogue warp and row: beta, m, E, n
+    uint4 ru[kSxEpiN][16];          // per epilogue warp and row: mask, table row, K slot
     float cen[kSxMaxDr];            // tile centre c
 };
 
@@ -89,8 +92,41 @@ __device__ __forceinline__ uint32_t sw128_off(int n, int ch) {
     return (uint32_t)((n >> 3) * 1024 + (n & 7) * 128 + ((ch ^ (n & 7)) << 4));
 }
 
+// BLSH_TC_MODE & 32 (experiments): globaltimer stamps per item (0 start, 1 setup done, 2 producers done,
+// 3 MMA done, 4 epilogue done, 5 end) and clock cycles spent waiting on mbarriers (6 producers on
+// aempty, 7 MMA on afull, 8 MMA on tempty, 9 epilogue on tfull)
+__device__ __forceinline__ void sx_stamp(const TiledArgs& a, int64_t item, int p) {
+    if (a.tstamp) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        a.tstamp[item * 16 + p] = t;
+    }
+}
+// single-thread wait (no warp reconvergence: the caller is one lane)
+__device__ __forceinline__ void mbar_wait1(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT1_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT1_%=;\n\t}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void mbar_complete_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.complete_tx.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void sx_wait(const TiledArgs& a, uint64_t* bar, uint32_t parity, long long& acc) {
+    if (a.tstamp) {
+        const long long t0 = clock64();
+        mbar_wait(bar, parity);
+        acc += clock64() - t0;
+    } else {
+        mbar_wait(bar, parity);
+    }
+}
+
 size_t screen_smem_bytes(int dr, int nst) {
-    return ((sizeof(SxSmem) + 1023) & ~size_t(1023)) + (size_t)(dr / 64) * kSxPanelB + (size_t)nst * kSxStage;
+    return 1024 + ((sizeof(SxSmem) + 1023) & ~size_t(1023)) + (size_t)(dr / 64) * kSxPanelB + (size_t)nst * kSxStage;
 }
 // the deepest A ring that fits (0: none)
 int screen_stages(int dr) {
@@ -102,8 +138,10 @@ int screen_stages(int dr) {
 template <int KT, int NST>
 __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     constexpr int kSxNst = NST;
-    constexpr int kSxAhead = NST - 2;          // stages in flight ahead of the MMA
-    extern __shared__ __align__(1024) unsigned char smraw[];
+    extern __shared__ __align__(1024) unsigned char smraw_[];
+    // the 128-byte-swizzled operands need 1024-byte aligned shared memory: align the base
+    // (the launch reserves 1 KB for it) instead of trusting the declaration's alignment
+    unsigned char* smraw = smraw_ + ((1024u - (smem_u32(smraw_) & 1023u)) & 1023u);
     SxSmem& S = *reinterpret_cast<SxSmem*>(smraw);
     const int ds = a.ds, dr = a.dr, np = dr >> 6;
     constexpr int nst = kSxNst;
@@ -118,11 +156,24 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     const int64_t q0 = a.tile_off[tile];
     const int nqt = (int)(a.tile_off[tile + 1] - q0);
     const uint4* RI = a.rowinfo + a.rows_off[tile];
+    if (threadIdx.x == 0) sx_stamp(a, item, 0);
+    long long wcyc = 0;
     // ---- setup: centre c, scales, B operand (u_j, v_a), per-query eta ----
+    // the tile's queries staged in shared memory (coalesced 16-byte loads; aliases the A ring,
+    // which the producers only fill after the setup's last barrier)
+    float* Qf = reinterpret_cast<float*>(Aop);
+    {
+        const int nv = ds >> 2;
+        for (int i = threadIdx.x; i < nqt * nv; i += kSxThreads) {
+            const int n = i / nv, v = i - n * nv;
+            reinterpret_cast<float4*>(Qf)[i] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + n] * ds) + v);
+        }
+    }
+    __syncthreads();
     for (int j = threadIdx.x; j < dr; j += kSxThreads) {
         float s = 0.f;
         if (j < ds)
-            for (int n = 0; n < nqt; ++n) s += __ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j);
+            for (int n = 0; n < nqt; ++n) s += Qf[(size_t)n * ds + j];
         S.cen[j] = j < ds ? s / (float)nqt : 0.f;
     }
     __syncthreads();
@@ -133,7 +184,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         float mq = 0.f, mv = 0.f;
         for (int j = threadIdx.x; j < ds; j += kSxThreads) {
             const float c = S.cen[j];
-            for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(__ldg(a.Q + (size_t)a.qorder[q0 + n] * ds + j) - c));
+            for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(Qf[(size_t)n * ds + j] - c));
             for (int la = 0; la < na; ++la)
                 mv = fmaxf(mv, fabsf(c - __ldg(a.anc + (size_t)a.slot_anchor[slot0 + la] * dr + j)));
         }
@@ -146,7 +197,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         __syncthreads();
         if (threadIdx.x == 0) {
             float m = 0.f;
-            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
+            for (int w = 0; w < kSxThreads / 32; ++w) m = fmaxf(m, S.red[w]);
             int e = 0;
             if (m > 0.f) { frexpf(m, &e); e -= 15; }
             S.S = ldexpf(1.0f, max(-120, min(120, e)));
@@ -156,7 +207,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         __syncthreads();
         if (threadIdx.x == 0) {
             float m = 0.f;
-            for (int w = 0; w < 9; ++w) m = fmaxf(m, S.red[w]);
+            for (int w = 0; w < kSxThreads / 32; ++w) m = fmaxf(m, S.red[w]);
             int e = 0;
             if (m > 0.f) { frexpf(m, &e); e -= 15; }
             S.Sv = ldexpf(1.0f, max(-120, min(120, e)));
@@ -169,7 +220,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         const int n = i % kSxN, cc = i / kSxN;      // row n of B, 16-byte chunk cc (8 columns)
         __align__(16) __half h[8];
         const float* src = nullptr;
-        if (n < nqt) src = a.Q + (size_t)a.qorder[q0 + n] * ds;
+        if (n < nqt) src = Qf + (size_t)n * ds;
         else if (n >= 32 && n - 32 < na) src = a.anc + (size_t)a.slot_anchor[slot0 + (n - 32)] * dr;
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
@@ -177,7 +228,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             float v = 0.f;
             if (j < ds && src) {
                 const float c = S.cen[j];
-                v = n < 32 ? (__ldg(src + j) - c) * iSq : (c - __ldg(src + j)) * iSv;
+                v = n < 32 ? (src[j] - c) * iSq : (c - __ldg(src + j)) * iSv;
             }
             h[e] = __float2half_rn(v);
         }
@@ -201,54 +252,14 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             const float cn = sqrtf(sv) * (1.0f + 0x1p-18f);
             S.ca[la] = ((kSxEpsAcc + 0x1p-11f + 0x1p-23f) * (1.0f + 0x1p-9f) * cn + sqrtf((float)ds) * 0x1p-25f * Sv) *
                        (1.0f + 0x1p-10f);
-            S.cdist[la] = la < na ? cn : __int_as_float(0x7F800000);
         }
     }
-    // Stream order: the item's rows grouped by anchor (contiguous), anchors nearest to c first,
-    // so the rows closest to the tile come early and the running bounds U_j tighten before most
-    // of the union has been screened (fewer buffered pairs).  Results do not depend on it.
-    __syncthreads();                                           // S.cdist from every warp
-    if (warp == 0) {
-        for (int la = lane; la <= kSxAnc; la += 32) {         // first item row of anchor column la
-            int v = (int)(r1 - r0);
-            if (la < na) {
-                int64_t lo = r0, hi = r1;
-                while (lo < hi) {
-                    const int64_t m = (lo + hi) >> 1;
-                    if (RI[m].z < slot0 + (uint32_t)la) lo = m + 1;
-                    else hi = m;
-                }
-                v = (int)(lo - r0);
-            }
-            S.arow[la] = v;
-        }
-        __syncwarp();
-        for (int la = lane; la < kSxAnc; la += 32) {          // rank by (|c - a|, column)
-            int rk = 0;
-            const float me = S.cdist[la];
-            for (int o = 0; o < na; ++o) {
-                const float x = S.cdist[o];
-                rk += (x < me || (x == me && o < la)) ? 1 : 0;
-            }
-            if (la < na) S.aord[rk] = la;
-        }
-        __syncwarp();
-        if (lane == 0) {
-            int c = 0;
-            for (int kk = 0; kk < na; ++kk) {
-                S.cum[kk] = c;
-                c += S.arow[S.aord[kk] + 1] - S.arow[S.aord[kk]];
-            }
-            S.cum[na] = c;
-        }
-    }
-    // per query: qn = |q_j - c|, un = S |u_j| (of the fp16 values), eta_j
     for (int n = warp; n < QT; n += kSxThreads / 32) {
         float sq = 0.f, su = 0.f;
         if (n < nqt) {
-            const float* qq = a.Q + (size_t)a.qorder[q0 + n] * ds;
+            const float* qq = Qf + (size_t)n * ds;
             for (int j = lane; j < ds; j += 32) {
-                const float e = __ldg(qq + j) - S.cen[j];
+                const float e = qq[j] - S.cen[j];
                 sq = fmaf(e, e, sq);
                 const float u = __half2float(__float2half_rn(e * iSq));
                 su = fmaf(u, u, su);
@@ -269,12 +280,17 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
     if (threadIdx.x == 0) {
         for (int s = 0; s < nst; ++s) {
-            mbar_init(&S.afull[s], kSxProd);
+            mbar_init(&S.afull[s], 1);
             mbar_init(&S.aempty[s], 1);
         }
         for (int s = 0; s < 4; ++s) {
             mbar_init(&S.tfull[s], 1);
-            mbar_init(&S.tempty[s], 4);
+            mbar_init(&S.tempty[s], kSxEpiN);
+        }
+        for (int s = 0; s < kSxNM; ++s) {
+            mbar_init(&S.mfull[s], 1);
+            mbar_init(&S.cfull[s], 1);
+            mbar_init(&S.mempty[s], kSxEpiN);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -288,125 +304,134 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     tc_fence_after();
     const uint32_t tbase = S.tmem_base;
     const int nstage = nblk * np;
-    // stream position -> item-relative union row (anchors in |c - a| order)
-    auto srow = [&](int p) -> int64_t {
-        int lo = 0, hi = na;                                   // largest k with cum[k] <= p
-        while (hi - lo > 1) {
-            const int m = (lo + hi) >> 1;
-            if (S.cum[m] <= p) lo = m;
-            else hi = m;
-        }
-        return r0 + S.arow[S.aord[lo]] + (p - S.cum[lo]);
-    };
+    if (threadIdx.x == 0) sx_stamp(a, item, 1);
     const int nrow = (int)(r1 - r0);
 
-    if (warp < kSxProd) {
-        // ======================= producers =======================
-        // thread t: 16-byte chunk pc = t & 7 of rows rr + 16 i (i < 8), rr = t >> 3; a warp
-        // instruction copies 4 whole 128-byte row segments (coalesced) into 4 swizzled
-        // shared-memory lines (conflict-free).  Rows with an empty query mask are zero-filled.
-        const int t = threadIdx.x, pc = t & 7, rr = t >> 3;
-        constexpr int ahead = kSxAhead;
-        uint32_t pos[8];
-        bool ok[8];
-        auto issue = [&](int g) {
-            if (g < nstage) {
-                const int b = g / np, p = g - b * np;
-                if (p == 0) {
-                    // thread pc of each 8-thread group loads the entry of row rr + 16 pc; shuffles
-                    // hand every thread of the group the entries of its 8 rows
-                    const int sp = b * 128 + rr + 16 * pc;
-                    uint4 f = make_uint4(0u, 0u, 0u, 0u);
-                    if (sp < nrow) f = RI[srow(sp)];
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        const int src = (lane & ~7) | i;
-                        pos[i] = __shfl_sync(BLSH_FULL, f.x, src);
-                        ok[i] = __shfl_sync(BLSH_FULL, f.y, src) != 0u;
-                    }
-                }
-                const int slot = g % nst;
-                if (g >= nst) mbar_wait(&S.aempty[slot], (uint32_t)((g / nst - 1) & 1));
-                const uint32_t sb = smem_u32(Aop + (size_t)slot * kSxStage);
-#pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const int r = rr + 16 * i;
-                    const __half* src = a.Rh + (size_t)(ok[i] ? pos[i] : 0u) * dr + p * 64 + pc * 8;
-                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(sb + sw128_off(r, pc)),
-                                 "l"(src), "r"(ok[i] ? 16u : 0u)
-                                 : "memory");
-                }
+    if (warp == 0) {
+        // ======================= producer (bulk copies) =======================
+        // The item's rows are whole 8-row atoms (k_expand_atoms) and the fp16 table stores each
+        // 64-column panel's atoms as consecutive swizzled KBs (resid.cu), so a 128-row stage is
+        // one bulk copy per run of consecutive atoms among the block's 16 (lane i: run i; a
+        // bucket is one run), completing by transaction bytes on afull.  Block metadata (the
+        // block's 128 row entries, one contiguous 2 KB) is fetched kSxMA blocks ahead (mfull);
+        // the rows' bound constants follow per run with the block's first stage (cfull).  No
+        // thread waits on a dependent global load and nothing goes through the generic proxy.
+        long long wa = 0, wme = 0, wmf = 0;
+        const char* Rb = reinterpret_cast<const char*>(a.Rh);
+        const size_t pstride = (size_t)a.natom * 1024;          // bytes per panel of the table
+        auto fetch_meta = [&](int b) {                          // lane 0: block b's entries -> mrow
+            if (b >= nblk) return;
+            const int mb = b % kSxNM;
+            if (b >= kSxNM) {
+                const long long t0 = a.tstamp ? clock64() : 0;
+                mbar_wait1(&S.mempty[mb], (uint32_t)(((b / kSxNM) - 1) & 1));
+                if (a.tstamp) wme += clock64() - t0;
             }
-            asm volatile("cp.async.commit_group;" ::: "memory");   // (possibly empty: uniform group count)
+            const int nr = min(128, nrow - b * 128);
+            mbar_expect_tx(&S.mfull[mb], (uint32_t)nr * 16u);
+            bulk_g2s(&S.mrow[mb][0], RI + r0 + (int64_t)b * 128, (uint32_t)nr * 16u, &S.mfull[mb]);
         };
-        for (int g = 0; g < ahead; ++g) issue(g);
+        if (lane == 0)
+            for (int b = 0; b < kSxMA; ++b) fetch_meta(b);
+        __syncwarp();
+        uint32_t ra = 0;                                        // the run this lane starts: first atom, length
+        int rlen = 0, nat = 0;
+        int b = 0, p = 0, slot = 0, sph = 0;                    // block, panel, ring slot, slot phase
         for (int g = 0; g < nstage; ++g) {
-            issue(g + ahead);
-            asm volatile("cp.async.wait_group %0;" ::"n"(kSxAhead) : "memory");
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            const int mb = b % kSxNM;
+            if (p == 0) {
+                if (lane == 0) fetch_meta(b + kSxMA);
+                sx_wait(a, &S.mfull[mb], (uint32_t)((b / kSxNM) & 1), wmf);
+                nat = min(128, nrow - b * 128) >> 3;
+                // runs of consecutive atoms: lane i < nat holds atom i (block rows 8i..8i+7); a run
+                // starts where the atom does not follow its predecessor, and its first lane copies it
+                const uint32_t at = lane < nat ? (S.mrow[mb][8 * lane].x >> 3) : 0u;
+                const uint32_t prev = __shfl_up_sync(BLSH_FULL, at, 1);
+                const bool start = lane < nat && (lane == 0 || prev + 1u != at);
+                const unsigned sm = __ballot_sync(BLSH_FULL, start);
+                const unsigned after = sm & ~((2u << lane) - 1u);      // run starts after this lane
+                ra = at;
+                rlen = start ? (after ? __ffs(after) - 1 : nat) - lane : 0;
+                if (lane == 0) mbar_expect_tx(&S.cfull[mb], (uint32_t)nat * 128u);
+                __syncwarp();
+                if (rlen) bulk_g2s(&S.mcon[mb][8 * lane], a.rconst + (size_t)ra * 8, (uint32_t)rlen * 128u, &S.cfull[mb]);
+            }
+            if (g >= nst) sx_wait(a, &S.aempty[slot], (uint32_t)(sph ^ 1), wa);
+            if (lane == 0) mbar_expect_tx(&S.afull[slot], (uint32_t)nat * 1024u);
             __syncwarp();
-            if (lane == 0) mbar_arrive(&S.afull[g % nst]);
+            if (rlen) {
+                if (!(a.dbgmode & 2))
+                    bulk_g2s(Aop + (size_t)slot * kSxStage + lane * 1024, Rb + p * pstride + (size_t)ra * 1024,
+                             (uint32_t)rlen * 1024u, &S.afull[slot]);
+                else
+                    mbar_complete_tx(&S.afull[slot], (uint32_t)rlen * 1024u);   // ablation: no row loads
+            }
+            if (++p == np) { p = 0; ++b; }
+            if (++slot == nst) { slot = 0; sph ^= 1; }
+        }
+        if (lane == 0 && a.tstamp) {
+            sx_stamp(a, item, 2);
+            a.tstamp[item * 16 + 6] = wa;
+            a.tstamp[item * 16 + 10] = wmf;
+            a.tstamp[item * 16 + 11] = wme;
         }
     } else if (warp == kSxMma) {
         // ======================= MMA issuer =======================
+        long long wt = 0;
         for (int b = 0; b < nblk; ++b) {
             const int ts = b & 3;
-            if (b >= 4) mbar_wait(&S.tempty[ts], (uint32_t)(((b >> 2) - 1) & 1));
+            if (b >= 4) sx_wait(a, &S.tempty[ts], (uint32_t)(((b >> 2) - 1) & 1), wt);
             tc_fence_after();
             const uint32_t dt = tbase + (uint32_t)ts * 128u;
             for (int p = 0; p < np; ++p) {
                 const int g = b * np + p;
                 const int slot = g % nst;
-                mbar_wait(&S.afull[slot], (uint32_t)((g / nst) & 1));
+                sx_wait(a, &S.afull[slot], (uint32_t)((g / nst) & 1), wcyc);
                 tc_fence_after();
                 if (lane == 0) {
                     const uint32_t as = smem_u32(Aop + (size_t)slot * kSxStage);
                     const uint32_t bs = smem_u32(Bop + (size_t)p * kSxPanelB);
 #pragma unroll
                     for (int kk = 0; kk < 4; ++kk)
-                        sx_mma(dt, sw128_desc(as + 32u * kk), sw128_desc(bs + 32u * kk), (p > 0 || kk > 0) ? 1u : 0u);
+                        if (!(a.dbgmode & 4))
+                            sx_mma(dt, sw128_desc(as + 32u * kk), sw128_desc(bs + 32u * kk), (p > 0 || kk > 0) ? 1u : 0u);
                     tc_commit(&S.aempty[slot]);
                     if (p == np - 1) tc_commit(&S.tfull[ts]);
                 }
                 __syncwarp();
             }
         }
-    } else {
+        if (lane == 0 && a.tstamp) { sx_stamp(a, item, 3); a.tstamp[item * 16 + 7] = wcyc; a.tstamp[item * 16 + 8] = wt; }
+    } else if (warp >= kSxEpi0) {
         // ======================= epilogue =======================
-        const int ew = warp - kSxEpi0;          // 0..3
+        const int ew = warp - kSxEpi0;          // 0..7
         const int quad = warp & 3;              // TMEM lane quadrant of this warp
+        const int half = ew >> 2;               // rows 16 half .. 16 half + 15 of the quadrant
+        const bool mine_row = (lane >> 4) == half;
         const int j = lane;                     // query of this lane (screen phase)
         const float eta = S.eta[j];
         float ulr[KT];
 #pragma unroll
         for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
-        int my_cnt = 0;
+        int my_cnt = 0, n_ins = 0, n_cmp = 0;
+        long long wec = 0;
         bool my_fail = false;
-        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * 4 + ew) * kTcScap;
+        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * kSxEpiN + ew) * kTcScap;
         float* Tt = S.tr[ew];
-        // this lane's row of block b (row phase)
-        auto row_meta = [&](int b, uint4& ri, float4& rc, float& sb) {
-            const int sp = b * 128 + quad * 32 + lane;
-            ri = sp < nrow ? RI[srow(sp)] : make_uint4(0u, 0u, 0u, 0u);
-            rc = make_float4(0.f, 0.f, 0.f, 0.f);
-            sb = 0.f;
-            if (ri.y != 0u) {
-                rc = __ldg(a.rconst + ri.x);
-                sb = rc.y;                      // the group's scale s_g
-            }
-        };
-        uint4 ri_n;
-        float4 rc_n;
-        float sb_n;
-        if (nblk > 0) row_meta(0, ri_n, rc_n, sb_n);
         for (int b = 0; b < nblk; ++b) {
-            const uint4 ri = ri_n;
-            const float4 rc = rc_n;
-            const float sbv = sb_n;
-            if (b + 1 < nblk) row_meta(b + 1, ri_n, rc_n, sb_n);
+            const int mb = b % kSxNM;
             const int ts = b & 3;
-            mbar_wait(&S.tfull[ts], (uint32_t)((b >> 2) & 1));
+            sx_wait(a, &S.tfull[ts], (uint32_t)((b >> 2) & 1), wcyc);
             tc_fence_after();
+            // this lane's row (row phase): entry and bound constants from the metadata ring
+            sx_wait(a, &S.mfull[mb], (uint32_t)((b / kSxNM) & 1), wec);
+            sx_wait(a, &S.cfull[mb], (uint32_t)((b / kSxNM) & 1), wec);
+            const int rrow = quad * 32 + lane;
+            const uint4 ri = b * 128 + rrow < nrow ? S.mrow[mb][rrow] : make_uint4(0u, 0u, 0u, 0u);
+            const float4 rc = S.mcon[mb][rrow];
+            const float sbv = rc.y;             // the group's scale s_g
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&S.mempty[mb]);
             float dot[32];
             const uint32_t ta = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)ts * 128u;
             tmem_ld32(ta, dot);
@@ -451,20 +476,24 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                     a.dbg[4096 + 1059] = (float)nqt;
                 }
             }
-            // transpose: row lane writes its 32 dots, column j -> Tt[j][lane]
+            // transpose this warp's 16 rows: row lane writes its 32 dots, column j -> Tt[j][row]
+            if (mine_row) {
+                const int r16 = lane & 15;
 #pragma unroll
-            for (int jj = 0; jj < 32; ++jj) Tt[jj * 33 + lane] = dot[jj];
-            S.rf[ew][lane] = make_float4(beta, m, E, rc.z);
-            S.ru[ew][lane] = make_uint4(ri.y, ri.x, ri.z, 0u);
+                for (int jj = 0; jj < 32; ++jj) Tt[jj * 17 + r16] = dot[jj];
+                S.rf[ew][r16] = make_float4(beta, m, E, rc.z);
+                S.ru[ew][r16] = make_uint4(ri.y, ri.x, ri.z, 0u);
+            }
             __syncwarp();
+            if (a.dbgmode & 1) continue;                           // ablation: no screen loop
             const float kth0 = ulr[KT - 1];
             float U = fminf(kth0, __uint_as_float(S.umin[j]));    // any warp's bound is valid
 #pragma unroll 8
-            for (int i = 0; i < 32; ++i) {
+            for (int i = 0; i < 16; ++i) {
                 const uint4 ru = S.ru[ew][i];                      // broadcast
                 const float4 rf = S.rf[ew][i];
                 const float Kv = __ldg(a.ktab + (size_t)ru.z * QT + j);
-                const float d2 = Kv + fmaf(rf.y, Tt[j * 33 + i], rf.x);
+                const float d2 = Kv + fmaf(rf.y, Tt[j * 17 + i], rf.x);
                 const float err = fmaf(eta, rf.w, rf.z);
                 const float lo = fmaf(d2, 1.0f - kSxDelta, -err);
                 if (((ru.x >> j) & 1u) && lo <= U && !my_fail) {   // rare: keep the pair
@@ -473,10 +502,15 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
 #pragma unroll
                         for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
                         ulr[0] = fminf(ulr[0], up);
-                        U = fminf(U, ulr[KT - 1]);
+                        if (ulr[KT - 1] < U) {                     // share the tighter bound at once
+                            U = ulr[KT - 1];
+                            atomicMin(&S.umin[j], __float_as_uint(U));
+                        }
                     }
                     const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
+                    ++n_ins;
                     if (my_cnt == kTcScap) {                       // full: drop what the tighter U excludes
+                        ++n_cmp;
                         int c2 = 0;
                         const ulonglong2* B2 = reinterpret_cast<const ulonglong2*>(SBj);
                         for (int t0 = 0; t0 < kTcScap / 2; t0 += 8) {   // 8 independent 16-byte loads per batch
@@ -495,11 +529,19 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                     if (!my_fail) SBj[my_cnt++] = e;
                 }
             }
-            if (ulr[KT - 1] < kth0) atomicMin(&S.umin[j], __float_as_uint(ulr[KT - 1]));
+            (void)kth0;
             __syncwarp();                                          // Tt / rf / ru reused by the next block
         }
         S.scnt[ew][j] = my_fail ? -1 : my_cnt;
+        if (warp == kSxEpi0 && lane == 0 && a.tstamp) {
+            sx_stamp(a, item, 4);
+            a.tstamp[item * 16 + 9] = wcyc;
+            a.tstamp[item * 16 + 12] = wec;
+        }
         if (a.counters && my_cnt) atomicAdd(a.counters, (unsigned long long)my_cnt);   // kept pairs
+        if (a.counters && n_ins) atomicAdd(a.counters + 2, (unsigned long long)n_ins);   // buffer insertions
+        if (a.counters && n_cmp) atomicAdd(a.counters + 3, (unsigned long long)n_cmp);   // compactions
+        if (a.counters && my_fail) atomicAdd(a.counters + 4, 1ull);                       // overflowed lists
     }
     tc_fence_before();
     __syncthreads();
@@ -507,13 +549,14 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         tc_fence_after();
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
     }
+    if (threadIdx.x == 0) sx_stamp(a, item, 5);
     // ---- hand-off to k_tc_rescore: final bound U_j, buffered pair counts ----
     if (threadIdx.x < QT) {
         const int j = threadIdx.x;
         a.ufin[(size_t)item * QT + j] = j < nqt ? S.umin[j] : 0u;
 #pragma unroll
-        for (int w = 0; w < 4; ++w)
-            a.scnt[((size_t)item * QT + j) * 4 + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
+        for (int w = 0; w < kSxEpiN; ++w)
+            a.scnt[((size_t)item * QT + j) * kSxEpiN + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
     }
 }
 

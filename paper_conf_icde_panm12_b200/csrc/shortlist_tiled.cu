@@ -36,7 +36,8 @@ constexpr int kTW = 8;            // warps per CTA (each owns 4 tile queries)
 
 struct Seg {
     uint32_t start, len, mask, off;   // table rows [start, start+len), query mask, rows before it in the union
-    uint32_t abase;                   // tile-local index of the anchor block of row `start` (screen K table)
+    uint32_t abase;                   // tile-local index of the anchor group of row `start` (screen K table)
+    uint32_t atbase;                  // tile-local index of the 8-row atom of row `start` (fp16 screen rows)
 };
 
 // ---------------------------------------------------------------------------
@@ -49,7 +50,8 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
                                                             int32_t* __restrict__ nseg,
                                                             int64_t* __restrict__ rows,
                                                             int64_t* __restrict__ nanch,
-                                                            const uint32_t* __restrict__ rgrp) {
+                                                            const uint32_t* __restrict__ rgrp,
+                                                            int64_t* __restrict__ natom) {
     extern __shared__ uint32_t sm[];
     const int cap = 2 * QT * (T + 1);
     int npow = 1;
@@ -78,7 +80,7 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
     __syncthreads();
     const int cnt = s_cnt;
     if (cnt == 0) {
-        if (tid == 0) { nseg[t] = 0; rows[t] = 0; nanch[t] = 0; }
+        if (tid == 0) { nseg[t] = 0; rows[t] = 0; nanch[t] = 0; if (natom) natom[t] = 0; }
         return;
     }
     int np2 = 32;                                   // >= one warp of (padding) keys; npow >= 2 * QT
@@ -189,37 +191,46 @@ __global__ void __launch_bounds__(kPrepThreads) k_tile_prep(const uint2* __restr
                 const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
                 if (tid >= o) inc += y;
             }
-            if (v) S[out + __popc(bm & lanemask_lt())] = Seg{bnd[i], len, tog[i], off + inc - len, 0u};
+            if (v) S[out + __popc(bm & lanemask_lt())] = Seg{bnd[i], len, tog[i], off + inc - len, 0u, 0u};
             off += __shfl_sync(BLSH_FULL, inc, 31);
             out += __popc(bm);
         }
         __syncwarp();
-        // anchor groups (resid.cu: runs of table rows) of the union, numbered in row order:
-        // segment i covers groups [a0, a1]; it shares a0 with segment i-1 when that one ends in it
-        uint32_t na = 0, prev_last = 0xFFFFFFFFu;
-        for (int base = 0; base < out; base += 32) {
-            const int i = base + tid;
-            uint32_t a0 = 0, a1 = 0, pl = 0xFFFFFFFFu;
-            if (i < out) {
-                const Seg sg = S[i];
-                a0 = rgrp ? rgrp[sg.start] : 0u;
-                a1 = rgrp ? rgrp[sg.start + sg.len - 1] : 0u;
-            }
-            const uint32_t up = __shfl_up_sync(BLSH_FULL, a1, 1);
-            pl = tid == 0 ? prev_last : up;
-            const uint32_t shared = (i < out && pl == a0) ? 1u : 0u;
-            const uint32_t c = i < out ? a1 - a0 + 1u - shared : 0u;
-            uint32_t inc = c;
+        // Runs of table rows the union touches, numbered in row order: anchor groups
+        // (resid.cu) and 8-row atoms.  Segment i covers runs [a0, a1]; it shares a0 with
+        // segment i-1 when that one ends in it.  Returns the number of distinct runs.
+        auto number_runs = [&](auto run_of, bool anchors) {
+            uint32_t na = 0, prev_last = 0xFFFFFFFFu;
+            for (int base = 0; base < out; base += 32) {
+                const int i = base + tid;
+                uint32_t a0 = 0, a1 = 0;
+                if (i < out) {
+                    const Seg sg = S[i];
+                    a0 = run_of(sg.start);
+                    a1 = run_of(sg.start + sg.len - 1);
+                }
+                const uint32_t up = __shfl_up_sync(BLSH_FULL, a1, 1);
+                const uint32_t pl = tid == 0 ? prev_last : up;
+                const uint32_t shared = (i < out && pl == a0) ? 1u : 0u;
+                const uint32_t c = i < out ? a1 - a0 + 1u - shared : 0u;
+                uint32_t inc = c;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
-                if (tid >= o) inc += y;
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(BLSH_FULL, inc, o);
+                    if (tid >= o) inc += y;
+                }
+                if (i < out) {
+                    if (anchors) S[i].abase = na + inc - c - shared;
+                    else S[i].atbase = na + inc - c - shared;
+                }
+                na += __shfl_sync(BLSH_FULL, inc, 31);
+                prev_last = __shfl_sync(BLSH_FULL, a1, min(31, out - 1 - base));
             }
-            if (i < out) S[i].abase = na + inc - c - shared;
-            na += __shfl_sync(BLSH_FULL, inc, 31);
-            prev_last = __shfl_sync(BLSH_FULL, a1, min(31, out - 1 - base));
-        }
-        if (tid == 0) { nseg[t] = out; rows[t] = off; nanch[t] = na; }
+            return na;
+        };
+        const uint32_t na = number_runs([&](uint32_t r) { return rgrp ? rgrp[r] : 0u; }, true);
+        const uint32_t nat = number_runs([](uint32_t r) { return r >> 3; }, false);
+        if (tid == 0) { nseg[t] = out; rows[t] = off; nanch[t] = na; if (natom) natom[t] = 8 * (int64_t)nat; }
     }
 }
 
@@ -258,6 +269,65 @@ __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ seg
 // MMA, k_screen_f16).  One thread per tile walks its rows; the anchor slot (rowinfo.z) is
 // non-decreasing along a tile's rows.  Pass 1 (item_r0 == NULL) counts, pass 2 writes
 // every item's first row (item_r0[item_off[t] + i], tile-relative).
+// fp16 screen: the tile's union at 8-row-atom granularity, one entry per atom row
+// (atom-row index = 8 x the atom's tile-local index + (row & 7)): union rows carry (table row,
+// query mask, K slot); the other rows of a touched atom carry mask 0 and the K slot of the
+// atom's previous union row (or its first), so the slot stays non-decreasing along the
+// tile's rows (k_tile_items splits items on it).  One CTA per tile, three phases.
+__global__ void __launch_bounds__(256) k_expand_atoms(const Seg* __restrict__ segs, const int32_t* __restrict__ nseg,
+                                                      int segcap, const int64_t* __restrict__ arows_off,
+                                                      const int64_t* __restrict__ aoff, const uint32_t* __restrict__ rgrp,
+                                                      uint4* __restrict__ rowinfo, uint32_t* __restrict__ slot_anchor) {
+    const int64_t t = blockIdx.x;
+    const Seg* S = segs + (size_t)t * segcap;
+    uint4* out = rowinfo + arows_off[t];
+    const int64_t ab = aoff[t];
+    const int ns = nseg[t];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    // phase 1: the atoms each segment introduces (all but a first atom shared with its predecessor)
+    for (int sI = warp; sI < ns; sI += 8) {
+        const Seg sg = S[sI];
+        const uint32_t a0 = sg.start >> 3, a1 = (sg.start + sg.len - 1) >> 3;
+        const bool shared = sI > 0 && ((S[sI - 1].start + S[sI - 1].len - 1) >> 3) == a0;
+        for (uint32_t k = (shared ? 1u : 0u) * 8u + lane; k < (a1 - a0 + 1u) * 8u; k += 32) {
+            const uint32_t row = a0 * 8u + k;
+            out[(size_t)(sg.atbase + (k >> 3)) * 8 + (k & 7)] = make_uint4(row, 0u, 0u, 0u);
+        }
+    }
+    __syncthreads();
+    // phase 2: the union rows
+    for (int sI = warp; sI < ns; sI += 8) {
+        const Seg sg = S[sI];
+        const uint32_t a0 = sg.start >> 3;
+        const uint32_t g0 = rgrp[sg.start];
+        for (uint32_t i = lane; i < sg.len; i += 32) {
+            const uint32_t row = sg.start + i;
+            const uint32_t grp = rgrp[row];
+            const int64_t slot = ab + sg.abase + (grp - g0);
+            out[(size_t)(sg.atbase + ((row >> 3) - a0)) * 8 + (row & 7)] = make_uint4(row, sg.mask, (uint32_t)slot, 0u);
+            if (i == 0 || rgrp[row - 1] != grp) slot_anchor[slot] = grp;
+        }
+    }
+    __syncthreads();
+    // phase 3: K slots of the atoms' non-union rows (monotone)
+    const int64_t nat = (arows_off[t + 1] - arows_off[t]) >> 3;
+    for (int64_t at = threadIdx.x; at < nat; at += 256) {
+        uint4 e[8];
+#pragma unroll
+        for (int r = 0; r < 8; ++r) e[r] = out[at * 8 + r];
+        uint32_t cur = 0;
+        bool found = false;
+#pragma unroll
+        for (int r = 0; r < 8; ++r)
+            if (!found && e[r].y != 0u) { cur = e[r].z; found = true; }
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            if (e[r].y != 0u) cur = e[r].z;
+            else out[at * 8 + r].z = cur;
+        }
+    }
+}
+
 __global__ void k_tile_items(const int64_t* __restrict__ rows, const int64_t* __restrict__ rows_off,
                              const uint4* __restrict__ rowinfo, int64_t ntiles, int chr, int amax,
                              int64_t* __restrict__ items, const int64_t* __restrict__ item_off,
@@ -278,7 +348,8 @@ __global__ void k_tile_items(const int64_t* __restrict__ rows, const int64_t* __
                     if (RI[m].z >= lim) hi = m;
                     else lo = m + 1;
                 }
-                e = lo;
+                e = lo & ~(int64_t)7;              // whole atoms (an atom spans <= 8 groups)
+                if (e <= r) e = r + 8;
             }
         }
         if (item_r0) item_r0[item_off[t] + it] = r;
@@ -301,7 +372,19 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
 // Warp-wide wait (every caller is a whole warp).  Lanes may leave the try_wait
 // loop on different iterations; the __syncwarp reconverges them so that the
 // warp collectives that follow take the converged fast path.
+#ifndef BLSH_SPIN_WAIT
+#define BLSH_SPIN_WAIT 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#if BLSH_SPIN_WAIT
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+#else
     asm volatile(
         "{\n\t.reg .pred p;\n"
         "WAIT_%=:\n\t"
@@ -309,6 +392,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
         "r"(parity)
         : "memory");
+#endif
     __syncwarp();
 }
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -337,12 +421,14 @@ struct TiledArgs {
     float* dbg;                     // optional (BLSH_TC_DEBUG): item 0, block 0 dots / |x'|^2 / rows
     unsigned long long* sbuf;       // TC: [n_items][QT][scap] buffered (lower bound, row) pairs
     int scap;
+    int nlist;                      // TC screens: buffered-pair lists per (item, query): epilogue warps
     int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA, 32 phase timers
     unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
     const int64_t* rows_off;        // [ntiles + 1] union rows before each tile
     const uint4* rowinfo;           // TC: [total rows] (table row, query mask, K slot, 0) per union row
     int dr;                         // screen: fp16 columns of the compact rows
-    const __half* Rh;               // screen: [n][dr] fp16 residual rows (resid.cu)
+    const __half* Rh;               // screen: fp16 rows, panel-major swizzled 8-row atoms (resid.cu)
+    int64_t natom;                  // screen: atoms of the table (Rh panel stride = natom KB)
     const float4* rconst;           // screen: [n] per-row bound constants
     const float* ktab;              // screen: [K slots][QT] K_aj = |q_j - a|^2
     const float* anc;               // screen: [anchor groups][dr] fp32 anchors
@@ -578,10 +664,10 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
     const int64_t nq = a.nq;
     // tile arrays are sized for the worst case (one query per tile)
     const size_t slot = (((size_t)(nq + 1) * 8) + 255) & ~size_t(255);
-    tilebuf.ensure(slot * 15 + 256);
+    tilebuf.ensure(slot * 16 + 256);
     char* tb = tilebuf.as<char>();
     unsigned long long* counters = reinterpret_cast<unsigned long long*>(tb + 5 * slot);
-    BLSH_CUDA(cudaMemsetAsync(counters, 0, 16, s));
+    BLSH_CUDA(cudaMemsetAsync(counters, 0, 64, s));
     int64_t* tile_off = reinterpret_cast<int64_t*>(tb + 6 * slot);
     int32_t* tile_of = reinterpret_cast<int32_t*>(tb + 7 * slot);
     int64_t* d2bits = reinterpret_cast<int64_t*>(tb + 8 * slot);
@@ -644,22 +730,26 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     int npow = 1;
     while (npow < segcap) npow <<= 1;
     const size_t prep_smem = (size_t)3 * npow * 4;
-    int64_t* nanch = reinterpret_cast<int64_t*>(tb + 13 * slot);   // anchor blocks per tile (screen K table)
+    int64_t* nanch = reinterpret_cast<int64_t*>(tb + 13 * slot);   // anchor groups per tile (screen K table)
     int64_t* aoff = reinterpret_cast<int64_t*>(tb + 14 * slot);
-    BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
-    k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, tile_off, segcap,
-                                                                  segbuf.as<Seg>(), nseg, rows, nanch, a.rgrp);
-    BLSH_LAUNCH_CHECK();
-    ++*launches;
-    scan_exclusive_i64(rows, rows_off, ntiles, scan, s);
-    *launches += 3;
+    int64_t* arows = reinterpret_cast<int64_t*>(tb + 15 * slot);   // fp16 screen: atom rows per tile
     const bool use_tc = kind == 2;   // chosen by shortlist_kind()
     const bool use_f16 = use_tc && screen_variant() == 0;
+    BLSH_CUDA(cudaFuncSetAttribute(k_tile_prep, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)prep_smem));
+    k_tile_prep<<<(unsigned)ntiles, kPrepThreads, prep_smem, s>>>(a.ivl, T, qorder, tile_off, segcap,
+                                                                  segbuf.as<Seg>(), nseg, rows, nanch, a.rgrp,
+                                                                  use_f16 ? arows : nullptr);
+    BLSH_LAUNCH_CHECK();
+    ++*launches;
+    // the rows the short-list kernels walk: union rows, or (fp16 screen) the rows of the union's atoms
+    int64_t* wrows = use_f16 ? arows : rows;
+    scan_exclusive_i64(wrows, rows_off, ntiles, scan, s);
+    *launches += 3;
     if (use_f16) {
         scan_exclusive_i64(nanch, aoff, ntiles, scan, s);
         *launches += 3;
     }
-    int64_t tot2[2] = {0, 0};   // union rows, K slots
+    int64_t tot2[2] = {0, 0};   // walked rows, K slots
     BLSH_CUDA(cudaMemcpyAsync(&tot2[0], rows_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     if (use_f16) BLSH_CUDA(cudaMemcpyAsync(&tot2[1], aoff + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
@@ -670,7 +760,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     const size_t slot_bytes = ((size_t)std::max<int64_t>(total_slots, 1) * 4 + 255) & ~size_t(255);
     const int64_t target = 148 * 4;
     int64_t chr = (total_rows + target - 1) / target;
-    chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 31) / 32 * 32));
+    chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 127) / 128 * 128));   // whole 128-row blocks
     // items <= rows / chr + (anchor splits: at most one per kSxAnc anchor slots) + one per tile
     const int64_t items_max = (total_rows + chr - 1) / chr + total_slots / kSxAnc + ntiles + 1;
     const size_t ir0_bytes = ((size_t)items_max * 8 + 255) & ~size_t(255);
@@ -679,39 +769,46 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     float* ktab = reinterpret_cast<float*>(rowbuf.as<char>() + rinfo_bytes);
     uint32_t* slot_anchor = reinterpret_cast<uint32_t*>(rowbuf.as<char>() + rinfo_bytes + ktab_bytes);
     int64_t* item_r0 = reinterpret_cast<int64_t*>(rowbuf.as<char>() + rinfo_bytes + ktab_bytes + slot_bytes);
-    if (use_tc && ntiles > 0) {
-        if (!use_f16) BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
-        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(segbuf.as<Seg>(), nseg, segcap, rows_off, aoff, ri,
-                                                       use_f16 ? slot_anchor : nullptr, use_f16 ? a.rgrp : nullptr);
+    if (use_f16 && ntiles > 0) {
+        k_expand_atoms<<<(unsigned)ntiles, 256, 0, s>>>(segbuf.as<Seg>(), nseg, segcap, rows_off, aoff, a.rgrp, ri,
+                                                        slot_anchor);
+        BLSH_LAUNCH_CHECK();
+        ++*launches;
+    } else if (use_tc && ntiles > 0) {
+        BLSH_CUDA(cudaMemsetAsync(aoff, 0, (size_t)(ntiles + 1) * 8, s));
+        k_expand_rows<<<(unsigned)ntiles, 256, 0, s>>>(segbuf.as<Seg>(), nseg, segcap, rows_off, aoff, ri, nullptr,
+                                                       nullptr);
         BLSH_LAUNCH_CHECK();
         ++*launches;
     }
     const unsigned gt = (unsigned)((ntiles + 255) / 256);
     const uint4* ri_split = use_f16 ? ri : nullptr;
-    k_tile_items<<<gt, 256, 0, s>>>(rows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, nullptr, nullptr);
+    k_tile_items<<<gt, 256, 0, s>>>(wrows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, nullptr, nullptr);
     BLSH_LAUNCH_CHECK();
     scan_exclusive_i64(items, item_off, ntiles, scan, s);
-    k_tile_items<<<gt, 256, 0, s>>>(rows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, item_off, item_r0);
+    k_tile_items<<<gt, 256, 0, s>>>(wrows, rows_off, ri_split, ntiles, (int)chr, kSxAnc, items, item_off, item_r0);
     BLSH_LAUNCH_CHECK();
     *launches += 5;
     int64_t n_items = 0;
     BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
-    constexpr int kScap = 4 * kTcScap;   // buffered (row, query) pairs per item and query (4 epilogue warps)
+    const int nlist = use_f16 ? kSxEpiN : 4;   // buffered-pair lists per (item, query): the screen's epilogue warps
+    const int kScap = nlist * kTcScap;
     const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
     const size_t ufin_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 4 + 255) & ~size_t(255);
-    const size_t scnt_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 16 + 255) & ~size_t(255);
+    const size_t scnt_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * nlist * 4 + 255) & ~size_t(255);
     partials.ensure(part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
-    ta.nseg = nseg; ta.rows = rows; ta.item_off = item_off; ta.partials = partials.as<unsigned long long>();
+    ta.nseg = nseg; ta.rows = wrows; ta.item_off = item_off; ta.partials = partials.as<unsigned long long>();
     ta.counters = counters;
     ta.tile_off = tile_off;
     ta.tile_of = tile_of;
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
+    ta.nlist = nlist;
     ta.rows_off = rows_off;
     ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes);
     ta.scnt = reinterpret_cast<int32_t*>(partials.as<char>() + part_bytes + sbuf_bytes + ufin_bytes);
@@ -720,6 +817,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.anc = a.anc;
     ta.dr = a.dr;
     ta.Rh = reinterpret_cast<const __half*>(a.Rh);
+    ta.natom = a.natom;
     ta.rconst = a.rconst;
     ta.ktab = ktab;
     ta.slot_anchor = slot_anchor;
@@ -788,8 +886,8 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     *n_items_out = n_items;
     *chr_out = (int)chr;
     *rows_out = total_rows;
-    unsigned long long ev[2] = {0, 0};
-    BLSH_CUDA(cudaMemcpyAsync(ev, counters, 16, cudaMemcpyDeviceToHost, s));
+    unsigned long long ev[5] = {0, 0, 0, 0, 0};
+    BLSH_CUDA(cudaMemcpyAsync(ev, counters, 40, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     *pairs_out = (int64_t)(use_tc ? ev[1] : ev[0]);   // TC: exact rescorings after the screen
     *kept_out = use_tc ? (int64_t)ev[0] : 0;
@@ -798,23 +896,23 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     // every work item loads its tile's queries: sum over tiles of |tile| x items(tile) ~ n_items x nq / ntiles
     *qload_rows_out = ntiles > 0 ? (double)n_items * (double)nq / (double)ntiles : 0.0;
     if (use_tc && std::getenv("BLSH_TC_MODE"))
-        std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld\n", (long long)n_items, ev[0], ev[1],
-                     (long long)total_rows);
+        std::fprintf(stderr, "[tc] items %lld kept %llu rescored %llu rows %lld insertions %llu compactions %llu "
+                     "overflowed %llu\n", (long long)n_items, ev[0], ev[1], (long long)total_rows, ev[2], ev[3], ev[4]);
     if (ta.tstamp) {   // mean phase durations over items (us)
         std::vector<unsigned long long> h((size_t)n_items * 16);
         BLSH_CUDA(cudaMemcpy(h.data(), ta.tstamp, h.size() * 8, cudaMemcpyDeviceToHost));
-        double acc[9] = {0};
-        unsigned long long pmax = 0, psum = 0;
+        double acc[16] = {0};
         for (int64_t i = 0; i < n_items; ++i) {
-            for (int p = 1; p < 9; ++p)
+            for (int p = 1; p < 6; ++p)
                 if (h[i * 16 + p]) acc[p] += (double)(h[i * 16 + p] - h[i * 16]) * 1e-3;
-            pmax = std::max(pmax, h[i * 16 + 9]);
-            psum += h[i * 16 + 9];
+            for (int p = 6; p < 13; ++p) acc[p] += (double)h[i * 16 + p] / 1965.0;   // cycles -> us at 1965 MHz
         }
-        std::fprintf(stderr, "[tc] phase us after start: setup %.1f conv %.1f mma %.1f epi %.1f sync %.1f compact %.1f "
-                     "rescore %.1f end %.1f; rescored pairs per item mean %.0f max %llu\n",
+        std::fprintf(stderr, "[tc] per item, us after start: setup %.1f producers %.1f mma %.1f epilogue %.1f end %.1f; "
+                     "waits (us): producers on aempty %.1f, mfull %.1f, mempty %.1f; mma on afull %.1f, tempty %.1f; "
+                     "epilogue on tfull %.1f, meta %.1f\n",
                      acc[1] / n_items, acc[2] / n_items, acc[3] / n_items, acc[4] / n_items, acc[5] / n_items,
-                     acc[6] / n_items, acc[8] / n_items, acc[7] / n_items, (double)psum / n_items, pmax);
+                     acc[6] / n_items, acc[10] / n_items, acc[11] / n_items, acc[7] / n_items, acc[8] / n_items,
+                     acc[9] / n_items, acc[12] / n_items);
     }
     if (ta.dbg) {
         std::vector<float> h(kDbgN);

@@ -563,7 +563,7 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
             }
     };
     bool failed = false;
-    for (int w = 0; w < 4; ++w) failed |= a.scnt[unit * 4 + w] < 0;
+    for (int w = 0; w < a.nlist; ++w) failed |= a.scnt[unit * a.nlist + w] < 0;
     if (failed) {
         // The screen could not separate this query's candidates (a buffer overflowed):
         // exact distance to every row of the item whose query mask has bit j.
@@ -576,9 +576,9 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
             score_rows(nm, e.x);
         }
     } else {
-        for (int w = 0; w < 4; ++w) {
-            const int cnt = a.scnt[unit * 4 + w];
-            const unsigned long long* Bf = a.sbuf + ((size_t)unit * 4 + w) * kTcScap;
+        for (int w = 0; w < a.nlist; ++w) {
+            const int cnt = a.scnt[unit * a.nlist + w];
+            const unsigned long long* Bf = a.sbuf + ((size_t)unit * a.nlist + w) * kTcScap;
             for (int base = 0; base < cnt; base += 32) {
                 const int i = base + lane;
                 const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
