@@ -3,9 +3,9 @@
 //
 // Work item = (query tile of <= QT = 32 queries, range of the tile's candidate union).
 // For a 128-row block of the union, one tcgen05.mma chain (kind::f16, M = 128,
-// N = 80, K = dr in steps of 16, fp32 accumulators in TMEM) computes, per row i,
+// N = 48, K = dr in steps of 16, fp32 accumulators in TMEM) computes, per row i,
 //   D_ij = r_i . u_j   (j < 32)    u_j = fp16((q_j - c) / S): the tile's centred queries
-//   D_ia = r_i . v_a   (a < 48)    v_a = fp16((c - a) / S_v): the item's anchors seen from c
+//   D_ia = r_i . v_a   (a < 16)    v_a = fp16((c - a) / S_v): the item's anchors seen from c
 // straight from the fp16 residual rows r_i in shared memory (no conversion pass: the
 // rows are copied by cp.async into the 128-byte-swizzled K-major layout the tensor core
 // reads).  Every operand is a small difference vector (queries and anchors near c, rows
@@ -14,7 +14,7 @@
 //   |q_j - x~|^2 = K_aj - 2 (q_j - c).(s r) - 2 (c - a).(s r) + |s r|^2
 //               ~ K_aj + beta_i + m_i D_ij,
 //   beta_i = nu_i - 2 S_v s D_i,a(i),   m_i = -2 S s.
-// An item spans <= 48 anchor groups (k_tile_items), so every row's anchor has a column.
+// An item spans <= 16 anchor groups (k_tile_items), so every row's anchor has a column.
 // Every rounding in that chain is bounded (DESIGN.md §7 "Screen bound"):
 //   |d2(q_j, x_i) - d~2| <= delta d~2 + E_i + eta_j n_i,
 // so lo = d~2 (1 - delta) - (E_i + eta_j n_i) <= d2 <= d~2 (1 + delta) + (E_i + eta_j n_i) = up.
@@ -31,19 +31,19 @@ constexpr int kSxMma = 1;                   // MMA warp index
 constexpr int kSxEpi0 = 4;                  // first epilogue warp
 constexpr int kSxEpiN = 8;                  // epilogue warps: 2 per TMEM lane quadrant (16 rows each)
 constexpr int kSxThreads = (kSxEpi0 + kSxEpiN) * 32;
-constexpr int kSxAnc = 48;                  // anchor columns per item
+constexpr int kSxAnc = 16;                  // anchor columns per item (items split at 16 anchor groups)
 constexpr int kSxN = 32 + kSxAnc;           // MMA N: 32 queries + the item's anchors
 constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
-constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 80 rows x 64 fp16 columns (10 KB)
+constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 48 rows x 64 fp16 columns (6 KB)
 constexpr int kSxMaxDr = 512;            // (the setup stages the tile's queries in the A ring)
 // A ring: NST stages of 16 KB (template: 8, or 6 / 4 when the B operand is large)
-// instruction descriptor: D f32, A/B f16, K-major both, N = 80, M = 128
+// instruction descriptor: D f32, A/B f16, K-major both, N = 48, M = 128
 constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u >> 4) << 24);
 // error model (DESIGN.md §7 "Screen bound")
 constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, relative to sum |a_k b_k|
 constexpr float kSxDelta = 0x1p-11f;        // relative slack on d~2 (AM-GM split 2^-12, K table 2^-13, fp32 ops)
 
-constexpr int kSxNM = 8;                    // block metadata ring (row entries + bound constants)
+constexpr int kSxNM = 6;                    // block metadata ring (row entries + bound constants)
 constexpr int kSxMA = 4;                    // metadata fetched this many blocks ahead of the producers
 
 struct SxSmem {
@@ -54,8 +54,9 @@ struct SxSmem {
     alignas(16) float4 mcon[kSxNM][128];   // per block: the rows' bound constants (resid.cu)
     uint32_t tmem_base;
     float S, Sv;
-    float red[16];
+    float red[16], red2[16];
     float ca[kSxAnc];               // per anchor column: error constant of the D_ia term
+    float kt[kSxAnc][QT];           // the item's K table rows: K_aj = |q_j - a|^2 (k_anchor_k)
     alignas(16) float eta[QT];
     uint32_t umin[QT];
     int scnt[kSxEpiN][QT];
@@ -159,58 +160,61 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     if (threadIdx.x == 0) sx_stamp(a, item, 0);
     long long wcyc = 0;
     // ---- setup: centre c, scales, B operand (u_j, v_a), per-query eta ----
-    // the tile's queries staged in shared memory (coalesced 16-byte loads; aliases the A ring,
-    // which the producers only fill after the setup's last barrier)
+    // The tile's queries (rows 0..nqt-1) and the item's anchors (rows 32..) staged in shared
+    // memory with a row pitch of dr floats (coalesced 16-byte loads; aliases the A ring, which
+    // the producer only fills after the setup's last barrier).  Anchors beyond the ring's room
+    // are read from global memory.
     float* Qf = reinterpret_cast<float*>(Aop);
+    // the item's anchor slots: RI[r].z is non-decreasing; slot0 = its first, na <= kSxAnc
+    const uint32_t slot0 = r1 > r0 ? RI[r0].z : 0u;
+    const int na = r1 > r0 ? (int)(RI[r1 - 1].z - slot0) + 1 : 0;
+    const int na_st = min(na, (int)((size_t)NST * kSxStage / ((size_t)dr * 4)) - 32);
+    auto arow = [&](int la) -> const float* {
+        return la < na_st ? Qf + (size_t)(32 + la) * dr : a.anc + (size_t)a.slot_anchor[slot0 + la] * dr;
+    };
     {
-        const int nv = ds >> 2;
+        const int nv = ds >> 2, nvr = dr >> 2;
         for (int i = threadIdx.x; i < nqt * nv; i += kSxThreads) {
             const int n = i / nv, v = i - n * nv;
-            reinterpret_cast<float4*>(Qf)[i] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + n] * ds) + v);
+            reinterpret_cast<float4*>(Qf)[(size_t)n * nvr + v] =
+                __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)a.qorder[q0 + n] * ds) + v);
+        }
+        for (int i = threadIdx.x; i < na_st * nvr; i += kSxThreads) {
+            const int la = i / nvr, v = i - la * nvr;
+            reinterpret_cast<float4*>(Qf)[(size_t)(32 + la) * nvr + v] =
+                __ldg(reinterpret_cast<const float4*>(a.anc + (size_t)a.slot_anchor[slot0 + la] * dr) + v);
         }
     }
     __syncthreads();
     for (int j = threadIdx.x; j < dr; j += kSxThreads) {
         float s = 0.f;
         if (j < ds)
-            for (int n = 0; n < nqt; ++n) s += Qf[(size_t)n * ds + j];
+            for (int n = 0; n < nqt; ++n) s += Qf[(size_t)n * dr + j];
         S.cen[j] = j < ds ? s / (float)nqt : 0.f;
     }
     __syncthreads();
-    // the item's anchor slots: RI[r].z is non-decreasing; slot0 = its first, na <= kSxAnc
-    const uint32_t slot0 = r1 > r0 ? RI[r0].z : 0u;
-    const int na = r1 > r0 ? (int)(RI[r1 - 1].z - slot0) + 1 : 0;
     {   // S: max |q_jk - c_k|, S_v: max |c_k - a_k| over the item's anchors
         float mq = 0.f, mv = 0.f;
         for (int j = threadIdx.x; j < ds; j += kSxThreads) {
             const float c = S.cen[j];
-            for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(Qf[(size_t)n * ds + j] - c));
-            for (int la = 0; la < na; ++la)
-                mv = fmaxf(mv, fabsf(c - __ldg(a.anc + (size_t)a.slot_anchor[slot0 + la] * dr + j)));
+            for (int n = 0; n < nqt; ++n) mq = fmaxf(mq, fabsf(Qf[(size_t)n * dr + j] - c));
+            for (int la = 0; la < na; ++la) mv = fmaxf(mv, fabsf(c - arow(la)[j]));
         }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             mq = fmaxf(mq, __shfl_xor_sync(BLSH_FULL, mq, o));
             mv = fmaxf(mv, __shfl_xor_sync(BLSH_FULL, mv, o));
         }
-        if (lane == 0) S.red[warp] = mq;
+        if (lane == 0) { S.red[warp] = mq; S.red2[warp] = mv; }
         __syncthreads();
-        if (threadIdx.x == 0) {
+        if (threadIdx.x < 2) {
             float m = 0.f;
-            for (int w = 0; w < kSxThreads / 32; ++w) m = fmaxf(m, S.red[w]);
+            for (int w = 0; w < kSxThreads / 32; ++w) m = fmaxf(m, threadIdx.x ? S.red2[w] : S.red[w]);
             int e = 0;
             if (m > 0.f) { frexpf(m, &e); e -= 15; }
-            S.S = ldexpf(1.0f, max(-120, min(120, e)));
-        }
-        __syncthreads();
-        if (lane == 0) S.red[warp] = mv;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            float m = 0.f;
-            for (int w = 0; w < kSxThreads / 32; ++w) m = fmaxf(m, S.red[w]);
-            int e = 0;
-            if (m > 0.f) { frexpf(m, &e); e -= 15; }
-            S.Sv = ldexpf(1.0f, max(-120, min(120, e)));
+            const float sc = ldexpf(1.0f, max(-120, min(120, e)));
+            if (threadIdx.x == 0) S.S = sc;
+            else S.Sv = sc;
         }
         __syncthreads();
     }
@@ -220,15 +224,21 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         const int n = i % kSxN, cc = i / kSxN;      // row n of B, 16-byte chunk cc (8 columns)
         __align__(16) __half h[8];
         const float* src = nullptr;
-        if (n < nqt) src = Qf + (size_t)n * ds;
-        else if (n >= 32 && n - 32 < na) src = a.anc + (size_t)a.slot_anchor[slot0 + (n - 32)] * dr;
+        if (n < nqt) src = Qf + (size_t)n * dr;
+        else if (n >= 32 && n - 32 < na) src = arow(n - 32);
+        float vv[8];
+        if (src) {
+            const float4 x0 = reinterpret_cast<const float4*>(src)[2 * cc];
+            const float4 x1 = reinterpret_cast<const float4*>(src)[2 * cc + 1];
+            vv[0] = x0.x; vv[1] = x0.y; vv[2] = x0.z; vv[3] = x0.w; vv[4] = x1.x; vv[5] = x1.y; vv[6] = x1.z; vv[7] = x1.w;
+        }
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
             const int j = cc * 8 + e;
             float v = 0.f;
             if (j < ds && src) {
                 const float c = S.cen[j];
-                v = n < 32 ? (src[j] - c) * iSq : (c - __ldg(src + j)) * iSv;
+                v = n < 32 ? (vv[e] - c) * iSq : (c - vv[e]) * iSv;
             }
             h[e] = __float2half_rn(v);
         }
@@ -240,9 +250,9 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
     for (int la = warp; la < kSxAnc; la += kSxThreads / 32) {
         float sv = 0.f;
         if (la < na) {
-            const float* ar = a.anc + (size_t)a.slot_anchor[slot0 + la] * dr;
+            const float* ar = arow(la);
             for (int j = lane; j < ds; j += 32) {
-                const float e = S.cen[j] - __ldg(ar + j);
+                const float e = S.cen[j] - ar[j];
                 sv = fmaf(e, e, sv);
             }
         }
@@ -254,10 +264,11 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                        (1.0f + 0x1p-10f);
         }
     }
+    for (int i = threadIdx.x; i < na * QT; i += kSxThreads) S.kt[i / QT][i % QT] = __ldg(a.ktab + (size_t)slot0 * QT + i);
     for (int n = warp; n < QT; n += kSxThreads / 32) {
         float sq = 0.f, su = 0.f;
         if (n < nqt) {
-            const float* qq = Qf + (size_t)n * ds;
+            const float* qq = Qf + (size_t)n * dr;
             for (int j = lane; j < ds; j += 32) {
                 const float e = qq[j] - S.cen[j];
                 sq = fmaf(e, e, sq);
@@ -377,7 +388,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         }
     } else if (warp == kSxMma) {
         // ======================= MMA issuer =======================
-        long long wt = 0;
+        long long wt = 0, wis = 0;
         for (int b = 0; b < nblk; ++b) {
             const int ts = b & 3;
             if (b >= 4) sx_wait(a, &S.tempty[ts], (uint32_t)(((b >> 2) - 1) & 1), wt);
@@ -389,6 +400,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                 sx_wait(a, &S.afull[slot], (uint32_t)((g / nst) & 1), wcyc);
                 tc_fence_after();
                 if (lane == 0) {
+                    const long long ti0 = a.tstamp ? clock64() : 0;
                     const uint32_t as = smem_u32(Aop + (size_t)slot * kSxStage);
                     const uint32_t bs = smem_u32(Bop + (size_t)p * kSxPanelB);
 #pragma unroll
@@ -397,11 +409,17 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                             sx_mma(dt, sw128_desc(as + 32u * kk), sw128_desc(bs + 32u * kk), (p > 0 || kk > 0) ? 1u : 0u);
                     tc_commit(&S.aempty[slot]);
                     if (p == np - 1) tc_commit(&S.tfull[ts]);
+                    if (a.tstamp) wis += clock64() - ti0;
                 }
                 __syncwarp();
             }
         }
-        if (lane == 0 && a.tstamp) { sx_stamp(a, item, 3); a.tstamp[item * 16 + 7] = wcyc; a.tstamp[item * 16 + 8] = wt; }
+        if (lane == 0 && a.tstamp) {
+            sx_stamp(a, item, 3);
+            a.tstamp[item * 16 + 7] = wcyc;
+            a.tstamp[item * 16 + 8] = wt;
+            a.tstamp[item * 16 + 13] = wis;
+        }
     } else if (warp >= kSxEpi0) {
         // ======================= epilogue =======================
         const int ew = warp - kSxEpi0;          // 0..7
@@ -482,54 +500,67 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
 #pragma unroll
                 for (int jj = 0; jj < 32; ++jj) Tt[jj * 17 + r16] = dot[jj];
                 S.rf[ew][r16] = make_float4(beta, m, E, rc.z);
-                S.ru[ew][r16] = make_uint4(ri.y, ri.x, ri.z, 0u);
+                S.ru[ew][r16] = make_uint4(ri.y, ri.x, live ? (uint32_t)myla : 0u, 0u);   // K row: the item's anchor column
             }
             __syncwarp();
             if (a.dbgmode & 1) continue;                           // ablation: no screen loop
-            const float kth0 = ulr[KT - 1];
-            float U = fminf(kth0, __uint_as_float(S.umin[j]));    // any warp's bound is valid
-#pragma unroll 8
-            for (int i = 0; i < 16; ++i) {
+            float U = fminf(ulr[KT - 1], __uint_as_float(S.umin[j]));   // any warp's bound is valid
+            // pass 1 (branch-free): rows of this query whose lower bound clears the bound at the
+            // block start; pass 2 takes them in row order against the tightening bound, so the
+            // pairs kept are exactly those of a row-by-row loop
+            auto row_bounds = [&](int i, float& lo, float& up) {
                 const uint4 ru = S.ru[ew][i];                      // broadcast
                 const float4 rf = S.rf[ew][i];
-                const float Kv = __ldg(a.ktab + (size_t)ru.z * QT + j);
-                const float d2 = Kv + fmaf(rf.y, Tt[j * 17 + i], rf.x);
+                const float d2 = S.kt[ru.z][j] + fmaf(rf.y, Tt[j * 17 + i], rf.x);
                 const float err = fmaf(eta, rf.w, rf.z);
-                const float lo = fmaf(d2, 1.0f - kSxDelta, -err);
-                if (((ru.x >> j) & 1u) && lo <= U && !my_fail) {   // rare: keep the pair
-                    const float up = fmaf(d2, 1.0f + kSxDelta, err);
-                    if (up < U) {                                  // sorted insert; only bounds below U matter
+                lo = fmaf(d2, 1.0f - kSxDelta, -err);
+                up = fmaf(d2, 1.0f + kSxDelta, err);
+                return ru;
+            };
+            uint32_t pm = 0;
 #pragma unroll
-                        for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
-                        ulr[0] = fminf(ulr[0], up);
-                        if (ulr[KT - 1] < U) {                     // share the tighter bound at once
-                            U = ulr[KT - 1];
-                            atomicMin(&S.umin[j], __float_as_uint(U));
-                        }
-                    }
-                    const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
-                    ++n_ins;
-                    if (my_cnt == kTcScap) {                       // full: drop what the tighter U excludes
-                        ++n_cmp;
-                        int c2 = 0;
-                        const ulonglong2* B2 = reinterpret_cast<const ulonglong2*>(SBj);
-                        for (int t0 = 0; t0 < kTcScap / 2; t0 += 8) {   // 8 independent 16-byte loads per batch
-                            ulonglong2 f[8];
-#pragma unroll
-                            for (int u = 0; u < 8; ++u) f[u] = B2[t0 + u];
-#pragma unroll
-                            for (int u = 0; u < 8; ++u) {
-                                if (__uint_as_float((uint32_t)(f[u].x >> 32)) <= U) SBj[c2++] = f[u].x;
-                                if (__uint_as_float((uint32_t)(f[u].y >> 32)) <= U) SBj[c2++] = f[u].y;
-                            }
-                        }
-                        my_cnt = c2;
-                        if (my_cnt > 3 * kTcScap / 4) my_fail = true;   // exact scan of j's rows later
-                    }
-                    if (!my_fail) SBj[my_cnt++] = e;
-                }
+            for (int i = 0; i < 16; ++i) {
+                float lo, up;
+                const uint4 ru = row_bounds(i, lo, up);
+                pm |= ((((ru.x >> j) & 1u) != 0u) && lo <= U) ? (1u << i) : 0u;
             }
-            (void)kth0;
+            if (my_fail) pm = 0;
+            while (pm) {
+                const int i = __ffs(pm) - 1;
+                pm &= pm - 1;
+                float lo, up;
+                const uint4 ru = row_bounds(i, lo, up);
+                if (lo > U) continue;                              // the bound tightened since pass 1
+                if (up < U) {                                      // sorted insert; only bounds below U matter
+#pragma unroll
+                    for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
+                    ulr[0] = fminf(ulr[0], up);
+                    if (ulr[KT - 1] < U) {                         // share the tighter bound at once
+                        U = ulr[KT - 1];
+                        atomicMin(&S.umin[j], __float_as_uint(U));
+                    }
+                }
+                const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
+                ++n_ins;
+                if (my_cnt == kTcScap) {                           // full: drop what the tighter U excludes
+                    ++n_cmp;
+                    int c2 = 0;
+                    const ulonglong2* B2 = reinterpret_cast<const ulonglong2*>(SBj);
+                    for (int t0 = 0; t0 < kTcScap / 2; t0 += 8) {  // 8 independent 16-byte loads per batch
+                        ulonglong2 f[8];
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) f[u] = B2[t0 + u];
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) {
+                            if (__uint_as_float((uint32_t)(f[u].x >> 32)) <= U) SBj[c2++] = f[u].x;
+                            if (__uint_as_float((uint32_t)(f[u].y >> 32)) <= U) SBj[c2++] = f[u].y;
+                        }
+                    }
+                    my_cnt = c2;
+                    if (my_cnt > 3 * kTcScap / 4) { my_fail = true; break; }   // exact scan of j's rows later
+                }
+                SBj[my_cnt++] = e;
+            }
             __syncwarp();                                          // Tt / rf / ru reused by the next block
         }
         S.scnt[ew][j] = my_fail ? -1 : my_cnt;

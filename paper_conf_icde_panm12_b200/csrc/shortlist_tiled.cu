@@ -761,8 +761,10 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     const int64_t target = 148 * 4;
     int64_t chr = (total_rows + target - 1) / target;
     chr = std::min<int64_t>(16384, std::max<int64_t>(1024, (chr + 127) / 128 * 128));   // whole 128-row blocks
-    // items <= rows / chr + (anchor splits: at most one per kSxAnc anchor slots) + one per tile
-    const int64_t items_max = (total_rows + chr - 1) / chr + total_slots / kSxAnc + ntiles + 1;
+    // items <= rows / chr + anchor splits + one per tile; an item cut at the anchor limit spans
+    // >= kSxAnc - 7 anchor slots (it is cut at a whole atom, and an atom spans <= 8 slots)
+    static_assert(kSxAnc >= 8, "items must span whole atoms");
+    const int64_t items_max = (total_rows + chr - 1) / chr + total_slots / (kSxAnc - 7) + ntiles + 1;
     const size_t ir0_bytes = ((size_t)items_max * 8 + 255) & ~size_t(255);
     rowbuf.ensure(rinfo_bytes + ktab_bytes + slot_bytes + ir0_bytes);
     uint4* ri = use_tc ? reinterpret_cast<uint4*>(rowbuf.as<char>()) : nullptr;
@@ -905,14 +907,14 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         for (int64_t i = 0; i < n_items; ++i) {
             for (int p = 1; p < 6; ++p)
                 if (h[i * 16 + p]) acc[p] += (double)(h[i * 16 + p] - h[i * 16]) * 1e-3;
-            for (int p = 6; p < 13; ++p) acc[p] += (double)h[i * 16 + p] / 1965.0;   // cycles -> us at 1965 MHz
+            for (int p = 6; p < 14; ++p) acc[p] += (double)h[i * 16 + p] / 1965.0;   // cycles -> us at 1965 MHz
         }
         std::fprintf(stderr, "[tc] per item, us after start: setup %.1f producers %.1f mma %.1f epilogue %.1f end %.1f; "
                      "waits (us): producers on aempty %.1f, mfull %.1f, mempty %.1f; mma on afull %.1f, tempty %.1f; "
-                     "epilogue on tfull %.1f, meta %.1f\n",
+                     "epilogue on tfull %.1f, meta %.1f; mma issue+commit %.1f\n",
                      acc[1] / n_items, acc[2] / n_items, acc[3] / n_items, acc[4] / n_items, acc[5] / n_items,
                      acc[6] / n_items, acc[10] / n_items, acc[11] / n_items, acc[7] / n_items, acc[8] / n_items,
-                     acc[9] / n_items, acc[12] / n_items);
+                     acc[9] / n_items, acc[12] / n_items, acc[13] / n_items);
     }
     if (ta.dbg) {
         std::vector<float> h(kDbgN);

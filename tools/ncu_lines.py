@@ -56,6 +56,8 @@ def main():
     lm = line_map(ksub)
     agg = collections.Counter()
     ex = collections.Counter()
+    stalls = [(i, h) for i, h in enumerate(hdr) if h.startswith("stall_") and "Not Issued" not in h]
+    why = collections.defaultdict(collections.Counter)
     tot = 0
     for r in body:
         off = int(r[ia], 16) - base
@@ -63,10 +65,16 @@ def main():
         s = int(r[isamp] or 0)
         agg[loc] += s
         ex[loc] += int(r[iex] or 0)
+        for i, h in stalls:
+            try:
+                why[loc][h[6:]] += int(r[i] or 0)
+            except ValueError:
+                pass
         tot += s
     print(f"total samples {tot}")
     for loc, s in agg.most_common(top):
-        print(f"{100.0 * s / max(tot, 1):6.2f}%  {s:9d}  inst {ex[loc]:12d}  {loc}")
+        w = ", ".join(f"{k} {v * 100 // max(s, 1)}%" for k, v in why[loc].most_common(2) if v)
+        print(f"{100.0 * s / max(tot, 1):6.2f}%  {s:9d}  inst {ex[loc]:12d}  {loc}  [{w}]")
 
 
 if __name__ == "__main__":
