@@ -234,6 +234,44 @@ def l2_copy_gbs() -> float:
     return 2 * a.numel() * 4 / (best * 1e-3) / 1e9
 
 
+def leaf_ceiling(cfg, ix, X, Q):
+    """SURVEY D6 leaf ceiling: the fraction of the ground-truth 10-NN (committed oracle sample) that
+    lie in the query's own RP-tree leaf -- the recall@10 no probing of that leaf can exceed.
+    Point leaves from the table directory (PERM, UOFF, LEAF_U), query leaves from the last
+    keep_stages query (Q_LEAF).  None without a matching ground-truth file."""
+    g = _gt_file(cfg, X, Q)
+    if g is None:
+        return None
+    perm = ix.export("PERM").astype(np.int64)
+    uoff = ix.export("UOFF").astype(np.int64)
+    leaf_u = ix.export("LEAF_U").astype(np.int64)
+    row_start = uoff[leaf_u]                               # first table row of every leaf (+ end)
+    pos_leaf = np.searchsorted(row_start, np.arange(perm.shape[0]), side="right") - 1
+    pt_leaf = np.full(X.shape[0], -1, np.int64)
+    pt_leaf[perm] = pos_leaf
+    qleaf = ix.export("Q_LEAF").astype(np.int64)[g["qidx"]]
+    gi = g["ids"][:, :10]
+    return float((pt_leaf[gi] == qleaf[:, None]).mean())
+
+
+def _gt_file(cfg, X, Q):
+    """The committed ground-truth sample of this workload if its size and fingerprints match."""
+    path = os.path.join(ROOT, "bench_data", f"{cfg.name}_gt.npz")
+    if not os.path.exists(path):
+        return None
+    g = np.load(path)
+    if int(g["n"]) != X.shape[0] or int(g["nq"]) != Q.shape[0]:
+        return None
+    import torch
+    qidx = torch.as_tensor(g["qidx"], device=Q.device)
+    fpx = float(X[:: max(1, X.shape[0] // 997)].double().sum())
+    fpq = float(Q[qidx].double().sum())
+    if abs(fpx - float(g["fp_x"])) > 1e-6 * max(1.0, abs(float(g["fp_x"]))) or \
+       abs(fpq - float(g["fp_q"])) > 1e-6 * max(1.0, abs(float(g["fp_q"]))):
+        return None
+    return g
+
+
 def error_ratio(gt_d2, our_d2):
     """Eq. 4: kappa = (1/k) sum_i |v - N(v)_i| / |v - I(v)_i| over the sample
     (0/0 = 1; a padded answer contributes 0), from fp64 ground-truth and reported d^2."""
@@ -449,9 +487,12 @@ def run_ours(a):
         # kernel reads it (fp16 screen: 2 dr + 16 B; fp32 kernels: 4 d_stride (+ metadata)); plus
         # the query batch once.  Bytes served again from L2 (tiles sharing rows) are NOT counted.
         distinct = None
-        if cfg.L == 1 and world == 1:
+        ceiling = None
+        if world == 1:
             ix.query(Q, k, keep_stages=True, **kw)
-            distinct = distinct_candidate_rows(ix, cfg.T, info.n_owned)
+            if cfg.L == 1:
+                distinct = distinct_candidate_rows(ix, cfg.T, info.n_owned)
+            ceiling = leaf_ceiling(cfg, ix, X, Q)
         if distinct is None:
             distinct = min(total_cand, info.n_owned)
         per_row = (row_bytes - 16) if (kind == 2 and skind == 1) else row_bytes   # rowinfo is per union row, not per table row
@@ -489,6 +530,7 @@ def run_ours(a):
                        "l2": "no flush: table (%.1f GB) and query batch (%.0f MB) exceed the 126 MB L2"
                              % (cfg.n * info.d_stride * 4 / 1e9, nq * cfg.d * 4 / 1e6)},
             "recall@10": recall, "recall_note": recall_note, "error_ratio@10": kappa,
+            "leaf_ceiling@10": ceiling,
             "selectivity": total_cand / nq / cfg.n, "mean_candidates": total_cand / nq,
             "build_s": build_s, "datagen_s": gen_s,
             "roofline": roof,

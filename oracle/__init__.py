@@ -82,6 +82,8 @@ def lib():
         L.orc_e8_second_ring.argtypes = [P]
         L.orc_e8_parent.restype = None
         L.orc_e8_parent.argtypes = [P, P]
+        L.orc_query_ex.restype = i32
+        L.orc_query_ex.argtypes = [P, P, i64, i32, i32, i32, i32, i32, i64, i32, i32, P, P, P]
         L.orc_query_union.restype = i32
         L.orc_query_union.argtypes = [P, i32, P, i64, i32, i32, i32, P, P, P]
         L.orc_gen_table_params.restype = None
@@ -350,15 +352,15 @@ class OracleIndex:
         return out
 
     def query(self, Q, k: int, probe: int = 0, T: int = 1, hierarchy: int = 0,
-              hier_step_bits: int = 0, min_cand: int = 0):
+              hier_step_bits: int = 0, min_cand: int = 0, curve_perturb: int = 0, msb_min: int = 0):
         Q = _f32(Q)
         nq = Q.shape[0]
         ids = np.empty((nq, k), np.int64)
         d2 = np.empty((nq, k), np.float32)
         nc = np.empty(nq, np.int64)
         if self.L == 1:
-            rc = lib().orc_query(self._h, _p(Q), nq, k, probe, T, hierarchy, hier_step_bits,
-                                 min_cand, _p(ids), _p(d2), _p(nc))
+            rc = lib().orc_query_ex(self._h, _p(Q), nq, k, probe, T, hierarchy, hier_step_bits,
+                                    min_cand, curve_perturb, msb_min, _p(ids), _p(d2), _p(nc))
         elif hierarchy:
             raise OracleError("the Morton hierarchy is defined for L = 1 only (R24)")
         else:

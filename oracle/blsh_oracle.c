@@ -942,12 +942,27 @@ static void orc_shortlist(const float *X, int d, const float *q, const int64_t *
  * hierarchy (Z^M only): Morton-prefix widening (Eq. 7-8)
  * with threshold tau = min_cand, or the lower median of the base counts of
  * this batch when min_cand == 0 (R18).  Returns 0, or 1 on invalid args. */
+/* Number of leading bits two B*M-bit Morton keys share ("the number of most
+ * significant bits shared"), B*M when equal. */
+static int orc_shared_msb(u128 a, u128 b, int BM)
+{
+    u128 x = a ^ b;
+    int len = 0;
+    while (x) { len++; x >>= 1; }
+    return BM - len;
+}
+
+/* hierarchy = 2 (R32): P:132's shared-MSB climb.  curve_perturb (R31): P:132's
+ * bit-perturbed repeats of the Morton-curve search (probe = 3). */
 static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
-                          int hier_step, int64_t min_cand, int64_t *out_ids, float *out_d2, int64_t *out_ncand,
-                          int do_shortlist)
+                          int hier_step, int64_t min_cand, int curve_perturb, int msb_min,
+                          int64_t *out_ids, float *out_d2, int64_t *out_ncand, int do_shortlist)
 {
     const int M = ix->M, d = ix->d, B = ix->B;
     if (k < 1 || T < 1) return 1;
+    if (curve_perturb < 0 || curve_perturb > M || (curve_perturb > 0 && probe != 3)) return 1;
+    if (hierarchy < 0 || hierarchy > 2 || (hierarchy == 2 && ix->quantizer != 0)) return 1;
+    if (msb_min < 0 || msb_min > B * M) return 1;
     if (probe == 0 && T != 1) return 1;
     if (probe == 1 && (ix->quantizer != 0 || M > 10 || T > orc_pow3(M))) return 1;
     if (probe == 2 && (ix->quantizer != 1 || T > 256 || (M == 16 && T > 481))) return 1;
@@ -1014,14 +1029,48 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
         if (probe == 3) {
             /* P:132 Morton-curve neighbours (R25): insertion position of the
              * (clamped) home key among the leaf's sorted bucket keys, then the
-             * buckets after / before it alternately: offsets 0, -1, +1, -2, ... */
-            int64_t p0 = ix->leaf_u[g];
-            for (int64_t u = ix->leaf_u[g]; u < ix->leaf_u[g + 1]; u++)
-                if (ix->ukey[u] < hkey[q]) p0 = u + 1;
+             * buckets after / before it alternately: offsets 0, -1, +1, -2, ...
+             * With curve_perturb = P > 0 (R31, "perturb some bits of the query
+             * Morton code and repeat this process several times"): keys
+             * kappa_0 = home key, kappa_r = home key with bit 0 of coordinate c_r
+             * flipped (one cell towards +1 if that bit is 0, else towards -1),
+             * c_1, c_2, ... = coordinates by ascending (distance to that cell
+             * boundary x_i(delta_i) of R11, i); probe j searches around the
+             * insertion position of kappa_(j mod (P+1)) with offset number
+             * j div (P+1); a bucket already probed is an empty probe. */
+            const int R = curve_perturb + 1;
+            u128 keys[17];
+            keys[0] = hkey[q];
+            if (R > 1 && !nonfin) {
+                int ord[16];
+                float xd[16];
+                for (int i = 0; i < M; i++) {
+                    const float xm = t[i] - floorf(t[i]);                    /* x_i(-1) */
+                    const int up = (((clamped[i] + (1 << (B - 1))) & 1) == 0); /* bit 0 of u_i is 0: +1 */
+                    xd[i] = up ? 1.0f - xm : xm;
+                    ord[i] = i;
+                }
+                for (int i = 1; i < M; i++) {          /* insertion sort: ties keep index order */
+                    int c = ord[i], j = i - 1;
+                    while (j >= 0 && xd[ord[j]] > xd[c]) { ord[j + 1] = ord[j]; j--; }
+                    ord[j + 1] = c;
+                }
+                for (int r = 1; r < R; r++) keys[r] = hkey[q] ^ ((u128)1 << (M - 1 - ord[r - 1]));
+            }
+            int64_t pr[17];
+            for (int r = 0; r < R; r++) {
+                pr[r] = ix->leaf_u[g];
+                for (int64_t u = ix->leaf_u[g]; u < ix->leaf_u[g + 1]; u++)
+                    if (ix->ukey[u] < keys[r]) pr[r] = u + 1;
+            }
+            int64_t *pb = (int64_t *)malloc(sizeof(int64_t) * (size_t)T);
             for (int p = 0; p < T; p++) {
-                int64_t off = (p % 2 == 1) ? -(int64_t)((p + 1) / 2) : (int64_t)(p / 2);
-                int64_t b = p0 + off;
+                const int r = p % R, mo = p / R;
+                int64_t off = (mo % 2 == 1) ? -(int64_t)((mo + 1) / 2) : (int64_t)(mo / 2);
+                int64_t b = pr[r] + off;
                 int valid = !nonfin && b >= ix->leaf_u[g] && b < ix->leaf_u[g + 1];
+                for (int pp = 0; pp < p && valid; pp++) if (pb[pp] == b) valid = 0;
+                pb[p] = valid ? b : -1;
                 u128 pk = valid ? ix->ukey[b] : 0;
                 ix->lq_pkey[((size_t)q * T + p) * 2] = (uint64_t)(pk >> 64);
                 ix->lq_pkey[((size_t)q * T + p) * 2 + 1] = (uint64_t)pk;
@@ -1030,6 +1079,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
                 be[(size_t)q * T + p] = valid ? ix->uoff[b + 1] : 0;
                 base += be[(size_t)q * T + p] - bs[(size_t)q * T + p];
             }
+            free(pb);
         }
         for (int p = 0; p < T && probe != 3; p++) {
             int32_t pc[16];
@@ -1072,14 +1122,14 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
 
     /* threshold tau (median of the short-list sizes of the query set) */
     int64_t tau = min_cand;
-    if (hierarchy && min_cand == 0 && nq > 0) {
+    if (hierarchy == 1 && min_cand == 0 && nq > 0) {
         int64_t *c = (int64_t *)malloc(sizeof(int64_t) * nqs);
         memcpy(c, ix->lq_base, sizeof(int64_t) * nqs);
         qsort(c, (size_t)nq, sizeof(int64_t), orc_cmp_i64);
         tau = c[(nq - 1) / 2];
         free(c);
     }
-    ix->lq_tau = hierarchy ? tau : 0;
+    ix->lq_tau = hierarchy == 1 ? tau : 0;
 
     /* E8 hierarchy (R27): a node at level j = the leaf's buckets whose
      * level-j code equals the query's; matches are closed upwards (the level-j+1
@@ -1088,7 +1138,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
      * code, <= ORC_E8_LEVELS) to the deepest node matching the query,
      * and P:249 widens from there until the node holds >= tau points: the first
      * level j <= m_g with a match and |node| >= tau; otherwise the whole leaf. */
-    if (hierarchy && ix->quantizer == 1) {
+    if (hierarchy == 1 && ix->quantizer == 1) {
         #pragma omp parallel for schedule(dynamic, 4)
         for (int64_t q = 0; q < nq; q++) {
             if (ix->lq_base[q] >= tau || (ix->lq_oor[q] & 4)) continue;
@@ -1138,7 +1188,7 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     }
 
     /* hierarchy: widen along Morton prefixes until |R| >= tau (Eq. 8) */
-    if (hierarchy && ix->quantizer == 0) {
+    if (hierarchy == 1 && ix->quantizer == 0) {
         const int BM = B * M;
         #pragma omp parallel for schedule(dynamic, 16)
         for (int64_t q = 0; q < nq; q++) {
@@ -1161,6 +1211,42 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
                     break;
                 }
             }
+        }
+    }
+
+    /* P:132 shared-MSB climb (R32, hierarchy = 2): s* = the larger number of
+     * most significant bits the (clamped) home key shares with the keys just
+     * before and after its insertion position in the leaf's sorted keys; when
+     * s* is small (< msb_min, default B*M: the home bucket is empty) the query
+     * goes up to the level of s* shared bits and uses that larger bucket, the
+     * leaf's buckets whose keys share those s* bits with it: A = A0 u R. */
+    if (hierarchy == 2) {
+        const int BM = B * M;
+        const int sig = msb_min > 0 ? msb_min : BM;
+        #pragma omp parallel for schedule(dynamic, 16)
+        for (int64_t q = 0; q < nq; q++) {
+            if (ix->lq_oor[q] & 4) continue;
+            int g = ix->lq_leaf[q];
+            int64_t ul = ix->leaf_u[g], uh = ix->leaf_u[g + 1];
+            if (uh <= ul) continue;
+            int64_t p0 = ul;
+            for (int64_t u = ul; u < uh; u++) if (ix->ukey[u] < hkey[q]) p0 = u + 1;
+            int sstar = 0;
+            if (p0 > ul) { int c = orc_shared_msb(hkey[q], ix->ukey[p0 - 1], BM); if (c > sstar) sstar = c; }
+            if (p0 < uh) { int c = orc_shared_msb(hkey[q], ix->ukey[p0], BM); if (c > sstar) sstar = c; }
+            if (sstar >= sig) continue;
+            int cb = BM - sstar;
+            u128 mask = cb >= 128 ? ~(u128)0 : (((u128)1 << cb) - 1);
+            u128 lo = hkey[q] & ~mask, hi = lo | mask;
+            int64_t s = -1, e = -1;
+            for (int64_t u = ul; u < uh; u++) {
+                if (ix->ukey[u] >= lo && ix->ukey[u] <= hi) {
+                    if (s < 0) s = ix->uoff[u];
+                    e = ix->uoff[u + 1];
+                }
+            }
+            if (s < 0) { s = 0; e = 0; }
+            hs[q] = s; he[q] = e; ix->lq_level[q] = cb;
         }
     }
 
@@ -1206,8 +1292,18 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
 int orc_query(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
               int hier_step, int64_t min_cand, int64_t *out_ids, float *out_d2, int64_t *out_ncand)
 {
-    return orc_query_impl(ix, Q, nq, k, probe, T, hierarchy, hier_step, min_cand, out_ids, out_d2,
+    return orc_query_impl(ix, Q, nq, k, probe, T, hierarchy, hier_step, min_cand, 0, 0, out_ids, out_d2,
                           out_ncand, 1);
+}
+
+/* orc_query with P:132's remaining options: curve_perturb (R31) and the shared-MSB
+ * climb threshold msb_min (R32, hierarchy = 2; 0 = B*M). */
+int orc_query_ex(orc_index *ix, const float *Q, int64_t nq, int k, int probe, int T, int hierarchy,
+                 int hier_step, int64_t min_cand, int curve_perturb, int msb_min, int64_t *out_ids,
+                 float *out_d2, int64_t *out_ncand)
+{
+    return orc_query_impl(ix, Q, nq, k, probe, T, hierarchy, hier_step, min_cand, curve_perturb, msb_min,
+                          out_ids, out_d2, out_ncand, 1);
 }
 
 /* L > 1 tables: "each of them is constructed independently with
@@ -1222,7 +1318,7 @@ int orc_query_union(orc_index **tabs, int L, const float *Q, int64_t nq, int k, 
 {
     if (L < 1) return 1;
     for (int l = 0; l < L; l++)
-        if (orc_query_impl(tabs[l], Q, nq, k, probe, T, 0, 0, 0, out_ids, out_d2, NULL, 0)) return 1;
+        if (orc_query_impl(tabs[l], Q, nq, k, probe, T, 0, 0, 0, 0, 0, out_ids, out_d2, NULL, 0)) return 1;
     const int d = tabs[0]->d;
     #pragma omp parallel for schedule(dynamic, 16)
     for (int64_t q = 0; q < nq; q++) {

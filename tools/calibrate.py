@@ -58,8 +58,12 @@ def main():
     ap.add_argument("--lattice", action="store_true")
     ap.add_argument("--hier", action="store_true", help="Morton hierarchy with tau = batch median")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--G", type=int, default=None, help="override the config's leaf count")
     a = ap.parse_args()
     cfg = synth.CONFIGS[a.config]
+    if a.G:
+        from dataclasses import replace
+        cfg = replace(cfg, G=a.G)
     t0 = time.time()
     X, Q = synth.make_dataset(cfg, backend="torch", device="cuda:0")
     torch.cuda.synchronize()

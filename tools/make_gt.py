@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--config", default="c4")
     ap.add_argument("--sample", type=int, default=200)
     ap.add_argument("--k", type=int, default=50)
+    ap.add_argument("--out-dir", default=os.path.join(ROOT, "bench_data"))
     a = ap.parse_args()
     import torch
     cfg = synth.CONFIGS[a.config]
@@ -44,8 +45,8 @@ def main():
     t0 = time.time()
     ids, d2 = oracle.bruteforce(Xh, Qs, a.k)
     print(f"brute force {len(qidx)} x {Xh.shape[0]} in {time.time() - t0:.1f}s on {oracle.num_threads()} threads")
-    os.makedirs(os.path.join(ROOT, "bench_data"), exist_ok=True)
-    out = os.path.join(ROOT, "bench_data", f"{cfg.name}_gt.npz")
+    os.makedirs(a.out_dir, exist_ok=True)
+    out = os.path.join(a.out_dir, f"{cfg.name}_gt.npz")
     np.savez_compressed(out, n=Xh.shape[0], nq=cfg.nq, qidx=qidx, ids=ids, d2=d2, fp_x=fp_x, fp_q=fp_q)
     print("wrote", out)
 

@@ -11,6 +11,9 @@ KEYS = ['gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__bytes_write.sum
         'smsp__issue_active.avg.pct_of_peak_sustained_active', 'launch__grid_size', 'launch__block_size',
         'sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active',
         'l1tex__data_pipe_lsu_wavefronts_mem_shared.sum']
+# prefixes printed for every matching counter (tensor pipe, L2 throughput)
+PREFIXES = ['sm__pipe_tensor', 'sm__pipe_tc', 'sm__inst_executed_pipe_tc', 'lts__t_bytes.sum',
+            'lts__throughput.avg.pct', 'l1tex__throughput.avg.pct', 'sm__pipe_shared_cycles_active']
 
 
 def main(path, top=12):
@@ -20,6 +23,9 @@ def main(path, top=12):
         for i, h in enumerate(hdr):
             if h == w:
                 print(f"{w:70s} {vals[i]:>20s} {units[i]}")
+    for i, h in enumerate(hdr):
+        if any(h.startswith(p) for p in PREFIXES):
+            print(f"{h:70s} {vals[i]:>20s} {units[i]}")
     st = []
     for i, h in enumerate(hdr):
         if h.startswith('smsp__pcsamp_warps_issue_stalled') and not h.endswith('not_issued'):
