@@ -93,7 +93,11 @@ typedef struct {
     int32_t n_probes;       /* T >= 1 including the home bucket; <= 3^M (M <= 10), <= 256 (Morton curve) or
                                <= 256 (E8: home, the 240 roots, then probes 242..256 from the second ring of
                                recursive probing, R26)                                                */
-    int32_t hierarchy;      /* 1 = Morton-prefix widening (Eq. 7-8, R17); Z^M index only               */
+    int32_t hierarchy;      /* 1 = Morton-prefix widening until |R| >= tau (Eq. 7-8, R17) on a Z^M index,
+                               the E8 code hierarchy (R27) on an E8 index; 2 = P:132's shared-MSB
+                               climb (R32, Z^M): a query whose home key shares fewer than msb_min leading
+                               bits with the keys before/after its insertion position also takes the leaf's
+                               buckets that share those bits with it                                         */
     int32_t hier_step_bits; /* key bits cleared per widening step: 0 = M (one Eq. 8 level), or 1..M           */
     int64_t min_cand;       /* tau (R18); 0 = lower median of the base counts of this batch           */
     void*   stream;         /* cudaStream_t                                                                   */
@@ -105,6 +109,12 @@ typedef struct {
                                over a set of queries" taken over the whole sharded batch, so a sharded index
                                widens exactly like one GPU).  NULL = this call's own counts; must be non-NULL
                                for that case when world > 1.  Read on `stream`; owned by the caller.          */
+    int32_t curve_perturb;  /* probe = 3 only, 0..M: P:132's bit-perturbed repeats of the curve search (R31):
+                               keys = the home key and the home key with bit 0 of its curve_perturb nearest
+                               coordinates flipped; probe j searches around key j mod (curve_perturb + 1);
+                               an already probed bucket is an empty probe                                     */
+    int32_t msb_min;        /* hierarchy = 2: climb when the shared-MSB count s* < msb_min; 0 = B*M (every
+                               query whose home bucket is empty)                                              */
 } blsh_query_params;
 
 void blsh_build_params_default(blsh_build_params* p);

@@ -38,7 +38,8 @@ class BuildParams(C.Structure):
 class QueryParams(C.Structure):
     _fields_ = [("probe", C.c_int32), ("n_probes", C.c_int32), ("hierarchy", C.c_int32),
                 ("hier_step_bits", C.c_int32), ("min_cand", C.c_int64), ("stream", C.c_void_p),
-                ("keep_stages", C.c_int32), ("timing", C.c_int32), ("global_base", C.c_void_p)]
+                ("keep_stages", C.c_int32), ("timing", C.c_int32), ("global_base", C.c_void_p),
+                ("curve_perturb", C.c_int32), ("msb_min", C.c_int32)]
 
 
 class Info(C.Structure):
@@ -187,9 +188,11 @@ def blsh_build(X, n_leaves: int = 1, M: int = 8, W: float = 4.0, seed: int = 42,
     return Index(h, n, d, M)
 
 
-def _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, stream, global_base=None):
+def _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, stream, global_base=None,
+             curve_perturb=0, msb_min=0):
     p = QueryParams()
     lib().blsh_query_params_default(C.byref(p))
+    p.curve_perturb, p.msb_min = curve_perturb, msb_min
     p.probe, p.n_probes, p.hierarchy, p.hier_step_bits = probe, n_probes, int(hierarchy), hier_step_bits
     p.min_cand, p.keep_stages, p.timing, p.stream = min_cand, int(bool(keep_stages)), int(bool(timing)), stream
     if global_base is not None:
@@ -208,7 +211,7 @@ def _alloc_like(Q, shape, kind):
 
 def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
                hier_step_bits: int = 0, min_cand: int = 0, keep_stages: bool = False, timing: bool = False,
-               out=None, global_base=None):
+               out=None, global_base=None, curve_perturb: int = 0, msb_min: int = 0):
     """-> (ids [nq,k] int64, dist2 [nq,k] fp32, ncand [nq] int64), on Q's device."""
     Q = _f32(Q)
     nq = int(Q.shape[0])
@@ -216,7 +219,7 @@ def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hie
         out = (_alloc_like(Q, (nq, k), "i64"), _alloc_like(Q, (nq, k), "f32"), _alloc_like(Q, (nq,), "i64"))
     ids, d2, nc = out
     p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, keep_stages, timing, _stream_for(Q, ids),
-                 global_base)
+                 global_base, curve_perturb, msb_min)
     qp, kq, _ = _ptr(Q)
     ip, ki, _ = _ptr(ids)
     dp, kd, _ = _ptr(d2)
@@ -227,7 +230,7 @@ def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hie
 
 def blsh_query_packed(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
                       hier_step_bits: int = 0, min_cand: int = 0, timing: bool = False, out=None,
-                      global_base=None):
+                      global_base=None, curve_perturb: int = 0, msb_min: int = 0):
     """-> (packed [nq,k] (uint64 bits; int64 for torch), ncand [nq])."""
     Q = _f32(Q)
     nq = int(Q.shape[0])
@@ -235,7 +238,7 @@ def blsh_query_packed(index: "Index", Q, k: int, probe: int = 0, n_probes: int =
         out = (_alloc_like(Q, (nq, k), "u64"), _alloc_like(Q, (nq,), "i64"))
     pk, nc = out
     p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, False, timing, _stream_for(Q, pk),
-                 global_base)
+                 global_base, curve_perturb, msb_min)
     qp, kq, _ = _ptr(Q)
     pp, kp, _ = _ptr(pk)
     np_, kn, _ = _ptr(nc)
@@ -244,13 +247,13 @@ def blsh_query_packed(index: "Index", Q, k: int, probe: int = 0, n_probes: int =
 
 
 def blsh_query_base_counts(index: "Index", Q, probe: int = 0, n_probes: int = 1, timing: bool = False,
-                           out=None, **_ignored):
+                           out=None, curve_perturb: int = 0, **_ignored):
     """a1-a4 only: |A0(q)| [nq] int64 (0 for queries another shard owns), on Q's device."""
     Q = _f32(Q)
     nq = int(Q.shape[0])
     if out is None:
         out = _alloc_like(Q, (nq,), "i64")
-    p = _qparams(probe, n_probes, 0, 0, 0, False, timing, _stream_for(Q, out))
+    p = _qparams(probe, n_probes, 0, 0, 0, False, timing, _stream_for(Q, out), None, curve_perturb)
     qp, kq, _ = _ptr(Q)
     op, ko, _ = _ptr(out)
     _check(lib().blsh_query_base_counts(index.handle, qp, nq, C.byref(p), op))

@@ -356,7 +356,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         add((size_t)nq * (T + 1), 8); add(nq, 8); add(nq, 8);
         if (keep) { add((size_t)nq * T, 16); add((size_t)nq * T, 4); }
     }
-    const bool e8h = p.hierarchy && ix.quantizer == 1;   // E8 code hierarchy
+    const bool e8h = p.hierarchy == 1 && ix.quantizer == 1;   // E8 code hierarchy
     const bool list_path = L > 1 || e8h;                   // candidates as deduplicated position lists
     if (list_path) { add(nq + 1, 8); add(nq, 8); add(L, 8); add(L, 8); }
     if (e8h) { add(nq, 8); add(nq, 8); add(nq, 8); }
@@ -444,6 +444,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     a.nq = nq; a.d = ix.d; a.ds = ds; a.G = ix.G; a.M = M; a.B = ix.B; a.depth = ix.depth;
     a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi;
     a.probe = p.probe; a.T = T; a.hstep = p.hier_step_bits > 0 ? p.hier_step_bits : M;
+    a.cperturb = p.probe == 3 ? p.curve_perturb : 0; a.msb_min = p.msb_min;
     {
         const char* rh = std::getenv("BLSH_RH_STAGE");   // ablation: 1 = stage query rows in shared memory
         a.rh_direct = (rh && rh[0] == '1') ? 0 : 1;
@@ -509,7 +510,9 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
         ix.has_stages = keep;
         return;
     }
-    if (p.hierarchy) {
+    if (p.hierarchy == 2) {   // P:132 shared-MSB climb (R32): no threshold statistic
+        launch_msb_climb(a, s); ++launches;
+    } else if (p.hierarchy) {
         if (p.min_cand == 0) {
             launch_median(p.global_base ? p.global_base : w.base, nq, w.tau, s);
             ++launches;
@@ -638,7 +641,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
                             : stt.shortlist_bytes;
     stt.pairs_scored = pairs;
     stt.shortlist_flops = 3.0 * ix.d * (double)total;
-    if (p.hierarchy) {
+    if (p.hierarchy == 1) {
         int64_t tau = p.min_cand;
         if (p.min_cand == 0) BLSH_CUDA(cudaMemcpy(&tau, w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost));
         stt.tau = tau;
@@ -686,7 +689,15 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
         return fail(BLSH_ERR_INVALID, "probe must be 0, 1, 2 or 3");
     }
     if (p->n_probes > 256) return fail(BLSH_ERR_UNSUPPORTED, "n_probes > 256");
-    if (p->hierarchy) {
+    if (p->curve_perturb < 0 || p->curve_perturb > idx->M)
+        return fail(BLSH_ERR_INVALID, "curve_perturb must be in [0, M]");
+    if (p->curve_perturb > 0 && p->probe != 3) return fail(BLSH_ERR_INVALID, "curve_perturb needs probe = 3");
+    if (p->hierarchy < 0 || p->hierarchy > 2) return fail(BLSH_ERR_INVALID, "hierarchy must be 0, 1 or 2");
+    if (p->hierarchy == 2 && idx->quantizer != 0) return fail(BLSH_ERR_INVALID, "the shared-MSB climb needs a Z^M index");
+    if (p->msb_min < 0 || p->msb_min > idx->B * idx->M) return fail(BLSH_ERR_INVALID, "msb_min must be in [0, B*M]");
+    if (p->hierarchy == 2) {
+        if (idx->L > 1) return fail(BLSH_ERR_UNSUPPORTED, "the Morton hierarchy is defined for one table (R24)");
+    } else if (p->hierarchy) {
         if (idx->L > 1) return fail(BLSH_ERR_UNSUPPORTED, "the Morton hierarchy is defined for one table (R24)");
         if (p->hier_step_bits < 0 || p->hier_step_bits > idx->M) return fail(BLSH_ERR_INVALID, "hier_step_bits must be in [0, M]");
         if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");

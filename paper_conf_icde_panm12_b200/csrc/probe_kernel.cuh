@@ -281,21 +281,93 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
 // bucket p is its home bucket); offsets outside the leaf are empty probes that
 // count toward T.  Every probe is one whole bucket, so the intervals are
 // disjoint (and the hierarchy's containment rule applies unchanged).
-__device__ int64_t probe_curve(const QueryArgs& a, int64_t q, int lane, int64_t ulo, int64_t uhi, uint2* ivl) {
-    const int T = a.T;
-    const Key128 k = a.qkey[q];
-    int64_t lo = ulo, hi = uhi;
-    while (lo < hi) {   // every lane runs the same search (keys L1/L2-resident)
+//
+// R31 ("perturb some bits of the query Morton code and repeat this process
+// several times [23]"): with P = a.cperturb > 0 the search is repeated for the keys
+// kappa_r = home key with bit 0 of coordinate c_r flipped (key bit M-1-c_r: one cell
+// towards +1 when that bit is 0, else towards -1), c_1, c_2, .. = the coordinates by
+// ascending (x_i(delta_i), i) (R11's boundary distances, fp32); probe j searches around
+// key j mod (P+1) with offset number j div (P+1); a bucket already probed by an earlier
+// probe is an empty probe (the intervals stay disjoint).
+__device__ __forceinline__ int64_t curve_lower(const QueryArgs& a, int64_t lo, int64_t hi, const Key128& k) {
+    while (lo < hi) {   // every lane that calls it runs the same search (keys L1/L2-resident)
         const int64_t mid = (lo + hi) >> 1;
         if (key_lt(a.ukey[mid], k)) lo = mid + 1;
         else hi = mid;
     }
-    const int64_t p0 = lo;
+    return lo;
+}
+
+__device__ int64_t probe_curve(const QueryArgs& a, int64_t q, int lane, int64_t ulo, int64_t uhi, uint2* ivl) {
+    const int T = a.T, M = a.M;
+    const int R = a.cperturb + 1;
+    const Key128 k = a.qkey[q];
+    const int64_t p0 = curve_lower(a, ulo, uhi, k);
+    // perturbed keys: lane i < M owns coordinate i; its rank among the coordinates decides
+    // which key (r = rank + 1) it holds, and it searches that key's insertion position
+    int64_t pmine = p0;
+    int rank = 32;
+    if (R > 1) {
+        float xd = 0.f;
+        if (lane < M) {
+            const float t = a.qt[(size_t)q * M + lane];
+            const float xm = __fsub_rn(t, floorf(t));                      // x_i(-1)
+            const bool up = ((k.lo >> (M - 1 - lane)) & 1ull) == 0ull;       // bit 0 of u_i
+            xd = up ? __fsub_rn(1.0f, xm) : xm;
+        }
+        rank = 0;
+        for (int j = 0; j < M; ++j) {
+            const float xj = __shfl_sync(BLSH_FULL, xd, j);
+            rank += (xj < xd || (xj == xd && j < lane)) ? 1 : 0;
+        }
+        if (lane < M && rank < R - 1) {
+            const Key128 kp{k.hi, k.lo ^ (1ull << (M - 1 - lane))};
+            pmine = curve_lower(a, ulo, uhi, kp);
+        }
+    }
+    constexpr int kMaxRounds = 8;                  // T <= 256 probes, 32 per round
+    const int nround = (T + 31) >> 5;
+    int64_t bj[kMaxRounds];
+#pragma unroll
+    for (int t = 0; t < kMaxRounds; ++t) {
+        bj[t] = -1;
+        const int j = lane + 32 * t;
+        if (t >= nround) continue;
+        const int r = j % R, m = j / R;
+        int64_t pr = p0;
+        for (int rr = 1; rr < R; ++rr) {           // the lane holding key rr: rank rr - 1
+            const unsigned hold = __ballot_sync(BLSH_FULL, lane < M && rank == rr - 1);
+            const int64_t v = __shfl_sync(BLSH_FULL, pmine, __ffs(hold) - 1);
+            if (r == rr) pr = v;
+        }
+        const int64_t off = (m & 1) ? -(int64_t)((m + 1) >> 1) : (int64_t)(m >> 1);
+        const int64_t b = pr + off;
+        if (j < T && b >= ulo && b < uhi) bj[t] = b;
+    }
+    // a bucket probed before is an empty probe: compare with every earlier in-range probe
+    bool dup[kMaxRounds];
+#pragma unroll
+    for (int t = 0; t < kMaxRounds; ++t) dup[t] = false;
+    if (R > 1) {
+#pragma unroll
+        for (int tt = 0; tt < kMaxRounds; ++tt) {
+            if (tt >= nround) break;
+            for (int sl = 0; sl < 32; ++sl) {
+                const int64_t v = __shfl_sync(BLSH_FULL, bj[tt], sl);
+                const int jj = sl + 32 * tt;
+#pragma unroll
+                for (int t = 0; t < kMaxRounds; ++t)
+                    if (v >= 0 && v == bj[t] && jj < lane + 32 * t) dup[t] = true;
+            }
+        }
+    }
     int64_t mysum = 0;
-    for (int p = lane; p < T; p += 32) {
-        const int64_t off = (p & 1) ? -(int64_t)((p + 1) >> 1) : (int64_t)(p >> 1);
-        const int64_t b = p0 + off;
-        const bool valid = b >= ulo && b < uhi;
+#pragma unroll
+    for (int t = 0; t < kMaxRounds; ++t) {
+        const int p = lane + 32 * t;
+        if (t >= nround || p >= T) continue;
+        const int64_t b = bj[t];
+        const bool valid = b >= 0 && !dup[t];
         uint2 iv = make_uint2(0, 0);
         Key128 kb{0, 0};
         if (valid) {

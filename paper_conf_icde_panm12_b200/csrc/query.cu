@@ -558,7 +558,68 @@ __global__ void k_widen(QueryArgs a, const int64_t* __restrict__ tau_p, int64_t 
     if (a.level) a.level[q] = cb;
 }
 
+// P:132's shared-MSB climb (R32, hierarchy = 2), one thread per query: s* = the larger
+// number of leading bits the clamped home key shares with the leaf's keys just before and
+// after its insertion position; when s* < msb_min (default B*M: the home bucket is empty)
+// the query also takes the leaf's buckets whose keys share those s* bits with it (one
+// contiguous bucket range, containing the neighbour), with k_widen's containment rule.
+__device__ __forceinline__ int shared_msb(const Key128& x, const Key128& y, int BM) {
+    const unsigned long long h = x.hi ^ y.hi, l = x.lo ^ y.lo;
+    const int len = h ? 128 - __clzll((long long)h) : (l ? 64 - __clzll((long long)l) : 0);
+    return BM - len;
+}
+
+__global__ void k_msb_climb(QueryArgs a) {
+    const int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (q >= a.nq) return;
+    if (a.qoor[q] & 6) return;
+    const int g = a.qleaf[q];
+    const int64_t ulo = a.leaf_u[g], uhi = a.leaf_u[g + 1];
+    if (uhi <= ulo) return;
+    const int BM = a.B * a.M;
+    const Key128 k0 = a.qkey[q];
+    const int64_t p0 = lower_key(a.ukey, ulo, uhi, k0);
+    int sstar = 0;
+    if (p0 > ulo) sstar = max(sstar, shared_msb(k0, a.ukey[p0 - 1], BM));
+    if (p0 < uhi) sstar = max(sstar, shared_msb(k0, a.ukey[p0], BM));
+    const int sig = a.msb_min > 0 ? a.msb_min : BM;
+    if (sstar >= sig) return;
+    const int cb = BM - sstar;
+    Key128 lo = k0, hi = k0;
+    if (cb >= 128) { lo = Key128{0, 0}; hi = Key128{~0ull, ~0ull}; }
+    else if (cb >= 64) {
+        const unsigned long long mh = cb == 64 ? 0ull : ((1ull << (cb - 64)) - 1ull);
+        lo = Key128{k0.hi & ~mh, 0ull};
+        hi = Key128{lo.hi | mh, ~0ull};
+    } else {
+        const unsigned long long ml = (1ull << cb) - 1ull;
+        lo = Key128{k0.hi, k0.lo & ~ml};
+        hi = Key128{k0.hi, lo.lo | ml};
+    }
+    const int64_t ua = lower_key(a.ukey, ulo, uhi, lo);
+    const int64_t ub = upper_key(a.ukey, ua, uhi, hi);
+    const int64_t s = ua < ub ? (int64_t)a.uoff[ua] : 0;
+    const int64_t e = ua < ub ? (int64_t)a.uoff[ub] : 0;
+    uint2* ivl = a.ivl + (size_t)q * (a.T + 1);
+    int64_t c = a.base[q];
+    for (int p = 0; p < a.T; ++p) {
+        const uint2 iv = ivl[p];
+        if (iv.y > iv.x && (int64_t)iv.x >= s && (int64_t)iv.y <= e) {
+            c -= (int64_t)(iv.y - iv.x);
+            ivl[p] = make_uint2(0, 0);
+        }
+    }
+    ivl[a.T] = make_uint2((uint32_t)s, (uint32_t)e);
+    a.cnt[q] = c + (e - s);
+    if (a.level) a.level[q] = cb;
+}
+
 }  // namespace
+
+void launch_msb_climb(const QueryArgs& a, cudaStream_t s) {
+    k_msb_climb<<<(unsigned)((a.nq + 127) / 128), 128, 0, s>>>(a);
+    BLSH_LAUNCH_CHECK();
+}
 
 void upload_e8_roots() {
     // __constant__ / __device__ tables are per device: track the upload per device, under a lock

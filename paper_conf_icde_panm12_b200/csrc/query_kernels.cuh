@@ -11,6 +11,8 @@ struct QueryArgs {
     int64_t nq;
     int d, ds, G, M, B, depth, quantizer, leaf_lo, leaf_hi;
     int probe, T, hstep;
+    int cperturb;            // probe = 3: bit-perturbed curve keys (R31)
+    int msb_min;             // hierarchy = 2: climb threshold on the shared-MSB count (R32; B*M when 0)
     int rh_direct;           // a1/a2 read query rows through L1 instead of staging them in shared memory
     // queries
     const float* Q;          // [nq][ds]
@@ -52,6 +54,7 @@ struct QueryArgs {
 void upload_e8_roots();
 int launch_route_hash(const QueryArgs& a, cudaStream_t s);   // returns kernels launched
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s);
+void launch_msb_climb(const QueryArgs& a, cudaStream_t s);
 // a2 only (queries already routed and grouped by leaf in a.lperm): hash with a.A / a.bvec
 void launch_hash(const QueryArgs& a, cudaStream_t s);
 // a2 of several hash tables in one launch (tables 1..L-1 of an L-table index)

@@ -35,6 +35,7 @@ constexpr int kSxAnc = 16;                  // anchor columns per item (items sp
 constexpr int kSxN = 32 + kSxAnc;           // MMA N: 32 queries + the item's anchors
 constexpr uint32_t kSxStage = 128 * 128;    // one A stage: 128 rows x 64 fp16 columns (16 KB)
 constexpr uint32_t kSxPanelB = kSxN * 128;  // one B panel: 48 rows x 64 fp16 columns (6 KB)
+constexpr int kSxMaxK = 64;                 // k supported (per-lane bound lists of KT <= 64; the rescoring's warp top-k holds 64)
 constexpr int kSxMaxDr = 512;            // (the setup stages the tile's queries in the A ring)
 // A ring: NST stages of 16 KB (template: 8, or 6 / 4 when the B operand is large)
 // instruction descriptor: D f32, A/B f16, K-major both, N = 48, M = 128

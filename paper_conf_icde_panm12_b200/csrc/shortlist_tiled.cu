@@ -629,7 +629,7 @@ int shortlist_kind(int ds, int dr, int T, int k) {
     const bool simt_ok = tiled_smem_bytes(ds) <= 227 * 1024;
     const bool tc_ok = screen_variant() == 1
                            ? (k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024)
-                           : (k <= kTcMaxK && dr >= 64 && dr <= kSxMaxDr && screen_stages(dr) > 0);
+                           : (k <= kSxMaxK && dr >= 64 && dr <= kSxMaxDr && screen_stages(dr) > 0);
     if (mode && std::strcmp(mode, "simt") == 0) return simt_ok ? 1 : 0;
     if (tc_ok) return 2;
     return simt_ok ? 1 : 0;
@@ -851,10 +851,15 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_f16) {
-            auto pick = [&](auto k8, auto k12, auto k16, auto k32) { return k <= 8 ? k8 : (k <= 12 ? k12 : (k <= 16 ? k16 : k32)); };
-            auto kern = nst == 8 ? pick(k_screen_f16<8, 8>, k_screen_f16<12, 8>, k_screen_f16<16, 8>, k_screen_f16<32, 8>)
-                      : nst == 6 ? pick(k_screen_f16<8, 6>, k_screen_f16<12, 6>, k_screen_f16<16, 6>, k_screen_f16<32, 6>)
-                                 : pick(k_screen_f16<8, 4>, k_screen_f16<12, 4>, k_screen_f16<16, 4>, k_screen_f16<32, 4>);
+            auto pick = [&](auto k8, auto k12, auto k16, auto k32, auto k64) {
+                return k <= 8 ? k8 : (k <= 12 ? k12 : (k <= 16 ? k16 : (k <= 32 ? k32 : k64)));
+            };
+            auto kern = nst == 8 ? pick(k_screen_f16<8, 8>, k_screen_f16<12, 8>, k_screen_f16<16, 8>, k_screen_f16<32, 8>,
+                                        k_screen_f16<64, 8>)
+                      : nst == 6 ? pick(k_screen_f16<8, 6>, k_screen_f16<12, 6>, k_screen_f16<16, 6>, k_screen_f16<32, 6>,
+                                        k_screen_f16<64, 6>)
+                                 : pick(k_screen_f16<8, 4>, k_screen_f16<12, 4>, k_screen_f16<16, 4>, k_screen_f16<32, 4>,
+                                        k_screen_f16<64, 4>);
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kSxThreads, tc_smem, s>>>(ta);
         } else if (use_tc) {

@@ -96,12 +96,14 @@ class ShardedIndex:
         ix = blsh.blsh_build(X, rank=dist.get_rank(group), world=dist.get_world_size(group), **build_kw)
         return cls(ix, group)
 
-    def global_base_counts(self, Q, probe: int = 0, n_probes: int = 1):
+    def global_base_counts(self, Q, probe: int = 0, n_probes: int = 1, curve_perturb: int = 0):
         """|A0(q)| of every query of the batch over all shards (SUM all-reduce of the per-rank counts)."""
         import torch
         kw = {}
         if not (isinstance(Q, torch.Tensor) and Q.is_cuda) and torch.cuda.is_available():
             kw["out"] = torch.empty((int(Q.shape[0]),), dtype=torch.int64, device="cuda")   # all-reduce on device
+        if curve_perturb:
+            kw["curve_perturb"] = curve_perturb
         base = self.index.base_counts(Q, probe=probe, n_probes=n_probes, **kw)
         if self.world > 1:
             self.dist.all_reduce(base, op=self.dist.ReduceOp.SUM, group=self.group)
@@ -146,8 +148,9 @@ class ShardedIndex:
         rank's list; required when Q is a host array (the all-gather runs on device memory)."""
         import torch
         nq = int(Q.shape[0])
-        if kw.get("hierarchy") and not kw.get("min_cand") and kw.get("global_base") is None:
-            kw["global_base"] = self.global_base_counts(Q, kw.get("probe", 0), kw.get("n_probes", 1))
+        if kw.get("hierarchy") == 1 and not kw.get("min_cand") and kw.get("global_base") is None:
+            kw["global_base"] = self.global_base_counts(Q, kw.get("probe", 0), kw.get("n_probes", 1),
+                                                        kw.get("curve_perturb", 0))
         if packed_out is not None:
             kw["out"] = packed_out
         pk, nc = self.index.query_packed(Q, k, timing=timing, **kw)

@@ -80,3 +80,53 @@ def test_curve_rejected_on_e8(blsh, c1):
     ix = blsh.blsh_build(torch.from_numpy(X).cuda(), n_leaves=4, quantizer=1)
     with pytest.raises(blsh.BlshError):
         ix.query(torch.from_numpy(Q).cuda(), 10, probe=3, n_probes=4)
+
+
+# P:132's remaining parts: bit-perturbed repeats of the curve search (R31) and the
+# shared-MSB climb (R32), bit-exact against the oracle (probe keys, validity, levels,
+# candidate sets), distances within 1e-5.
+
+@pytest.mark.parametrize("P,T", [(1, 4), (3, 8), (8, 18), (8, 256), (2, 33)])
+@pytest.mark.parametrize("k", [10, 50])
+def test_curve_perturbed(c1_pair_w1, c1, P, T, k):
+    X, Q = c1
+    run_query_pair(*c1_pair_w1, X, Q, k, probe=3, T=T, curve_perturb=P)
+
+
+@pytest.mark.parametrize("W,msb_min,probe,T", [(1.0, 0, 0, 1), (1.0, 0, 1, 4), (1.0, 112, 3, 3), (1.0, 124, 3, 5)])
+def test_msb_climb(blsh, orc, c1, W, msb_min, probe, T):
+    X, Q = c1
+    ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=W, seed=42)
+    run_query_pair(ix, ox, X, Q, 10, probe=probe, T=T, hierarchy=2, msb_min=msb_min)
+
+
+def test_msb_climb_with_perturbed_curve(c1_pair_w1, c1):
+    X, Q = c1
+    run_query_pair(*c1_pair_w1, X, Q, 10, probe=3, T=6, hierarchy=2, curve_perturb=2)
+
+
+def test_msb_climb_low_density_queries(blsh, orc):
+    """C3-shaped data with between-cluster queries (P:129 low-density regions): the climb
+    triggers for many queries; M = 6 keys (B*M = 96 < 128 bits)."""
+    cfg = synth.CONFIGS["c3"]
+    from dataclasses import replace
+    cfg = replace(cfg, n=20000, nq=300, backend="numpy")
+    X, Q = synth.make_dataset(cfg)
+    ix, ox = build_pair(blsh, orc, X, G=8, M=6, W=0.6, seed=7)
+    _, _, nc = run_query_pair(ix, ox, X, Q, 20, probe=3, T=2, hierarchy=2, curve_perturb=3)
+    assert (ix.export("Q_LEVEL") > 0).sum() > 10
+
+
+def test_perturb_and_climb_rejected(blsh, c1):
+    X, Q = c1
+    Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
+    ix = blsh.blsh_build(Xd, n_leaves=4, M=8, W=1.0)
+    with pytest.raises(blsh.BlshError):
+        ix.query(Qd, 10, probe=1, n_probes=4, curve_perturb=1)
+    with pytest.raises(blsh.BlshError):
+        ix.query(Qd, 10, probe=3, n_probes=4, curve_perturb=9)
+    with pytest.raises(blsh.BlshError):
+        ix.query(Qd, 10, hierarchy=2, msb_min=129)
+    e8 = blsh.blsh_build(Xd, n_leaves=4, quantizer=1)
+    with pytest.raises(blsh.BlshError):
+        e8.query(Qd, 10, hierarchy=2)

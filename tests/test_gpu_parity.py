@@ -51,15 +51,16 @@ def compare_build(ix, ox, owned_all=True):
 
 
 def run_query_pair(ix, ox, X, Q, k, probe=0, T=1, hierarchy=0, hier_step_bits=0, min_cand=0, device=True,
-                   check_stages=True):
+                   check_stages=True, **extra):
+    """extra: curve_perturb / msb_min (R31/R32), passed to both sides."""
     Qin = torch.from_numpy(Q).cuda() if device else Q
     ids, d2, nc = ix.query(Qin, k, probe=probe, n_probes=T, hierarchy=hierarchy, hier_step_bits=hier_step_bits,
-                           min_cand=min_cand, keep_stages=True)
+                           min_cand=min_cand, keep_stages=True, **extra)
     if device:
         torch.cuda.synchronize()
         ids, d2, nc = ids.cpu().numpy(), d2.cpu().numpy(), nc.cpu().numpy()
     oi, od, onc = ox.query(Q, k, probe=probe, T=T, hierarchy=hierarchy, hier_step_bits=hier_step_bits,
-                           min_cand=min_cand)
+                           min_cand=min_cand, **extra)
     if check_stages:
         assert np.array_equal(ix.export("Q_LEAF"), ox.get("q_leaf")), "query leaf differs"
         assert np.array_equal(ix.export("Q_T").view(np.uint32), ox.get("q_t").ravel().view(np.uint32)), "t differs"
@@ -331,7 +332,7 @@ def test_tiled_shortlist_variants(blsh, orc, c1, monkeypatch, mode):
     else:
         monkeypatch.setenv("BLSH_SHORTLIST", "tc")
     ix, ox = build_pair(blsh, orc, X, G=4, M=8, W=4.0, seed=21)
-    for k, T in [(1, 1), (10, 16), (16, 64)] + ([(32, 16)] if mode == "tc" else []):
+    for k, T in [(1, 1), (10, 16), (16, 64), (50, 16), (64, 8)] + ([(32, 16)] if mode == "tc" else []):
         run_query_pair(ix, ox, X, Q, k, probe=1 if T > 1 else 0, T=T)
         assert ix.stats().tiled == (1 if mode == "simt" else 2)
 
@@ -371,7 +372,7 @@ def test_tc_screen_equals_warp(blsh, orc, monkeypatch, shape):
         Q = synth.sample_points(mix, 100, 53)
         G, W, T = 2, 3.0, 4
     ix, ox = build_pair(blsh, orc, X, G=G, M=8, W=W, seed=5)
-    for k in (1, 10, 16, 17, 24, 32):
+    for k in (1, 10, 16, 17, 24, 32, 33, 50, 64):
         a = _query_mode(ix, Q, k, "warp", monkeypatch, probe=1, n_probes=T)
         b = _query_mode(ix, Q, k, "tc", monkeypatch, probe=1, n_probes=T)
         assert a[3] == 0 and b[3] == 2
