@@ -325,9 +325,117 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
 
 namespace blsh {
 
+static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
+                           const blsh_query_params& p, int64_t* out_ids, float* out_d2,
+                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base);
+
+// A shard answers only the queries of its own leaves.  It routes the whole
+// batch (a1; every rank must, to learn the owners), then runs a2-a5 on the compacted batch
+// of its own queries -- leaf-grouped by the routing pass, so they are one contiguous run of
+// lperm -- and scatters the answers back among padding rows.  The Morton hierarchy's batch
+// median tau (R18) stays a statistic of the whole batch: it is taken over global_base
+// before the compaction and passed on as an explicit threshold.  With keep_stages (per-query
+// exports of the full batch) or for base counts, the unsharded path runs instead.
 void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k, const blsh_query_params& p,
                int64_t* out_ids, float* out_d2, unsigned long long* out_packed, int64_t* out_ncand, bool out_host,
                int64_t* out_base) {
+    const bool shard = ix.leaf_lo > 0 || ix.leaf_hi < ix.G;
+    if (!shard || p.keep_stages || out_base || nq == 0) {
+        run_query_core(ix, Q, q_host, nq, k, p, out_ids, out_d2, out_packed, out_ncand, out_host, out_base);
+        return;
+    }
+    cudaStream_t s = (cudaStream_t)p.stream;
+    QueryWork& w = ix.qw;
+    const int ds = ix.ds, G = ix.G;
+    int launches = 0;
+    const bool q_direct = !q_host && ds == ix.d && (reinterpret_cast<uintptr_t>(Q) & 15u) == 0;
+    const float* Qdev = Q;
+    if (!q_direct) {
+        w.sh_qfull.ensure((size_t)nq * ds * sizeof(float));
+        if (ds != ix.d) BLSH_CUDA(cudaMemsetAsync(w.sh_qfull.p, 0, (size_t)nq * ds * sizeof(float), s));
+        BLSH_CUDA(cudaMemcpy2DAsync(w.sh_qfull.p, ds * sizeof(float), Q, ix.d * sizeof(float), ix.d * sizeof(float), nq,
+                                    q_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice, s));
+        Qdev = w.sh_qfull.as<float>();
+    }
+    // carve: leaf [nq], lperm [nq], leaf counts + cursors [2G], tau, compact rows and outputs
+    size_t need = 0;
+    auto add = [&](size_t cnt, size_t el) { need += Arena::need(cnt, el); };
+    add(nq, 4); add(nq, 4); add((size_t)2 * G, 4); add(4, 8);
+    add((size_t)nq * ds, 4); add((size_t)nq * k, 8); add((size_t)nq * k, 4); add((size_t)nq * k, 8); add(nq, 8);
+    add((size_t)nq * k, 8); add((size_t)nq * k, 4); add((size_t)nq * k, 8); add(nq, 8);
+    w.sh_buf.ensure(need);
+    Arena ar{w.sh_buf.as<char>(), 0, w.sh_buf.bytes};
+    int32_t* qleaf = ar.take<int32_t>(nq);
+    uint32_t* lperm = ar.take<uint32_t>(nq);
+    int32_t* lcnt = ar.take<int32_t>((size_t)2 * G);
+    int64_t* tau_d = ar.take<int64_t>(4);
+    float* Qc = ar.take<float>((size_t)nq * ds);
+    int64_t* ids_c = ar.take<int64_t>((size_t)nq * k);
+    float* d2_c = ar.take<float>((size_t)nq * k);
+    unsigned long long* pk_c = ar.take<unsigned long long>((size_t)nq * k);
+    int64_t* nc_c = ar.take<int64_t>(nq);
+    QueryArgs a{};
+    a.nq = nq; a.d = ix.d; a.ds = ds; a.G = G; a.M = ix.M; a.B = ix.B; a.depth = ix.depth;
+    a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi; a.rh_direct = 1;
+    a.Q = Qdev; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
+    a.ntype = ix.ntype.as<int32_t>(); a.qleaf = qleaf; a.lperm = lperm; a.lcnt = lcnt;
+    launches += launch_route_group(a, s);
+    std::vector<int32_t> cnt_h((size_t)G);
+    BLSH_CUDA(cudaMemcpyAsync(cnt_h.data(), lcnt, (size_t)G * 4, cudaMemcpyDeviceToHost, s));
+    blsh_query_params p2 = p;
+    p2.global_base = nullptr;
+    int64_t tau = 0;
+    const bool med = p.hierarchy == 1 && p.min_cand == 0;
+    if (med) {   // R18 over the whole batch (check_query guarantees global_base on a shard)
+        launch_median(p.global_base, nq, tau_d, s);
+        ++launches;
+        BLSH_CUDA(cudaMemcpyAsync(&tau, tau_d, 8, cudaMemcpyDeviceToHost, s));
+    }
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    if (med) {
+        if (tau > 0) p2.min_cand = tau;
+        else p2.hierarchy = 0;   // tau = 0: no query is below it, nothing widens
+    }
+    int64_t off = 0, nown = 0;
+    for (int g = 0; g < G; ++g) {
+        if (g < ix.leaf_lo) off += cnt_h[g];
+        else if (g < ix.leaf_hi) nown += cnt_h[g];
+    }
+    const uint32_t* own = lperm + off;   // the owned queries, grouped by leaf
+    launch_gather_rows(Qdev, ds, own, nown, Qc, s);
+    ++launches;
+    int64_t* d_ids = out_ids;
+    float* d_d2 = out_d2;
+    unsigned long long* d_pk = out_packed;
+    int64_t* d_nc = out_ncand;
+    if (out_host) {
+        d_ids = out_ids ? ar.take<int64_t>((size_t)nq * k) : nullptr;
+        d_d2 = out_d2 ? ar.take<float>((size_t)nq * k) : nullptr;
+        d_pk = out_packed ? ar.take<unsigned long long>((size_t)nq * k) : nullptr;
+        d_nc = out_ncand ? ar.take<int64_t>(nq) : nullptr;
+    }
+    if (nown > 0)
+        run_query_core(ix, Qc, false, nown, k, p2, out_ids ? ids_c : nullptr, out_d2 ? d2_c : nullptr,
+                       out_packed ? pk_c : nullptr, nc_c, false, nullptr);
+    else
+        ix.stats = blsh_stats{};
+    launch_shard_outputs(own, nq, nown, k, ids_c, d2_c, pk_c, nc_c, d_ids, d_d2, d_pk, d_nc, s);
+    launches += nown > 0 ? 2 : 1;
+    if (out_host) {
+        if (out_ids) BLSH_CUDA(cudaMemcpyAsync(out_ids, d_ids, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
+        if (out_d2) BLSH_CUDA(cudaMemcpyAsync(out_d2, d_d2, (size_t)nq * k * 4, cudaMemcpyDeviceToHost, s));
+        if (out_ncand) BLSH_CUDA(cudaMemcpyAsync(out_ncand, d_nc, (size_t)nq * 8, cudaMemcpyDeviceToHost, s));
+        if (out_packed) BLSH_CUDA(cudaMemcpyAsync(out_packed, d_pk, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
+    }
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    ix.stats.nq = nq;
+    ix.stats.launches += launches;
+    if (med) ix.stats.tau = tau;
+}
+
+static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
+                           const blsh_query_params& p, int64_t* out_ids, float* out_d2,
+                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base) {
     cudaStream_t s = (cudaStream_t)p.stream;
     QueryWork& w = ix.qw;
     const int T = p.n_probes, M = ix.M, ds = ix.ds;
@@ -483,7 +591,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[2], s));
     // query-tiled short-list ahead: fork the query sort + tile formation (a1/a2 outputs only)
-    const int kind_pre = (list_path || out_base) ? 0 : shortlist_kind(ds, ix.dr, T, k);
+    const int kind_pre = (list_path || out_base) ? 0 : shortlist_kind(nq, ds, ix.dr, T, k);
     if (kind_pre > 0) {
         if (!w.side) {
             BLSH_CUDA(cudaStreamCreateWithFlags(&w.side, cudaStreamNonBlocking));

@@ -122,6 +122,7 @@ struct QueryWork {
     };
     std::vector<TableQuery> tq;
     DevBuf listbuf;               // deduplicated candidate positions (u32), at raw_off[q]
+    DevBuf sh_qfull, sh_buf;      // sharded index: the whole batch on the device; routing + compact batch
     int64_t* raw_off = nullptr;   // [nq+1] scan of the per-query sums of the table counts
     bool list_valid = false;      // the last query built candidate lists (listbuf / raw_off / cnt)
     // side stream: the query sort and tile formation run while a3/a4 run on the caller's stream

@@ -707,6 +707,80 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     return 4;
 }
 
+// a1 alone over a batch, queries grouped by leaf (lperm), leaf counts in a.lcnt[0..G):
+// the sharded path's first pass (run_query: a rank routes the whole batch, then works
+// on the queries of its own leaves only).
+int launch_route_group(const QueryArgs& a, cudaStream_t s) {
+    if (a.nq == 0) return 0;
+    const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
+    const size_t smem_r = a.rh_direct ? 16 : (size_t)kRHQ * (a.ds + 4) * sizeof(float);
+    BLSH_CUDA(cudaMemsetAsync(a.lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
+    BLSH_CUDA(cudaFuncSetAttribute(k_route, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_r));
+    k_route<<<grid, kRHQ, smem_r, s>>>(a, a.lcnt);
+    BLSH_LAUNCH_CHECK();
+    k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, a.G, a.lcnt + a.G);
+    BLSH_LAUNCH_CHECK();
+    k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, a.lcnt + a.G, a.lperm);
+    BLSH_LAUNCH_CHECK();
+    return 3;
+}
+
+namespace {
+// compact batch: row i = query idx[i] of the full batch (ds floats per row, 16-byte vectors)
+__global__ void k_gather_rows(const float* __restrict__ Q, int ds, const uint32_t* __restrict__ idx, int64_t n,
+                              float* __restrict__ out) {
+    const int nv = ds >> 2;
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t >= n * nv) return;
+    const int64_t i = t / nv;
+    const int v = (int)(t - i * nv);
+    reinterpret_cast<float4*>(out)[t] = __ldg(reinterpret_cast<const float4*>(Q + (size_t)idx[i] * ds) + v);
+}
+// full outputs: padding everywhere, then the compact rows at their queries
+__global__ void k_shard_pad(int64_t nq, int k, int64_t* ids, float* d2, unsigned long long* pk, int64_t* nc) {
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t < nq * k) {
+        if (ids) ids[t] = -1;
+        if (d2) d2[t] = __int_as_float(0x7F800000);
+        if (pk) pk[t] = 0x7F800000FFFFFFFFull;
+    }
+    if (nc && t < nq) nc[t] = 0;
+}
+__global__ void k_shard_scatter(const uint32_t* __restrict__ idx, int64_t n, int k, const int64_t* ids_c,
+                                const float* d2_c, const unsigned long long* pk_c, const int64_t* nc_c, int64_t* ids,
+                                float* d2, unsigned long long* pk, int64_t* nc) {
+    const int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (t >= n * k) return;
+    const int64_t i = t / k;
+    const int j = (int)(t - i * k);
+    const int64_t o = (int64_t)idx[i] * k + j;
+    if (ids) ids[o] = ids_c[t];
+    if (d2) d2[o] = d2_c[t];
+    if (pk) pk[o] = pk_c[t];
+    if (nc && j == 0) nc[idx[i]] = nc_c[i];
+}
+}  // namespace
+
+void launch_gather_rows(const float* Q, int ds, const uint32_t* idx, int64_t n, float* out, cudaStream_t s) {
+    if (n == 0) return;
+    const int64_t tot = n * (ds >> 2);
+    k_gather_rows<<<(unsigned)((tot + 255) / 256), 256, 0, s>>>(Q, ds, idx, n, out);
+    BLSH_LAUNCH_CHECK();
+}
+
+void launch_shard_outputs(const uint32_t* idx, int64_t nq, int64_t n, int k, const int64_t* ids_c, const float* d2_c,
+                          const unsigned long long* pk_c, const int64_t* nc_c, int64_t* ids, float* d2,
+                          unsigned long long* pk, int64_t* nc, cudaStream_t s) {
+    const int64_t tp = std::max<int64_t>(nq * k, nq);
+    k_shard_pad<<<(unsigned)((tp + 255) / 256), 256, 0, s>>>(nq, k, ids, d2, pk, nc);
+    BLSH_LAUNCH_CHECK();
+    if (n > 0) {
+        k_shard_scatter<<<(unsigned)((n * k + 255) / 256), 256, 0, s>>>(idx, n, k, ids_c, d2_c, pk_c, nc_c, ids, d2,
+                                                                      pk, nc);
+        BLSH_LAUNCH_CHECK();
+    }
+}
+
 void launch_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);

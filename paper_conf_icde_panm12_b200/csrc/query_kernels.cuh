@@ -55,6 +55,11 @@ void upload_e8_roots();
 int launch_route_hash(const QueryArgs& a, cudaStream_t s);   // returns kernels launched
 void launch_probe_lookup(const QueryArgs& a, cudaStream_t s);
 void launch_msb_climb(const QueryArgs& a, cudaStream_t s);
+int launch_route_group(const QueryArgs& a, cudaStream_t s);
+void launch_gather_rows(const float* Q, int ds, const uint32_t* idx, int64_t n, float* out, cudaStream_t s);
+void launch_shard_outputs(const uint32_t* idx, int64_t nq, int64_t n, int k, const int64_t* ids_c, const float* d2_c,
+                          const unsigned long long* pk_c, const int64_t* nc_c, int64_t* ids, float* d2,
+                          unsigned long long* pk, int64_t* nc, cudaStream_t s);
 // a2 only (queries already routed and grouped by leaf in a.lperm): hash with a.A / a.bvec
 void launch_hash(const QueryArgs& a, cudaStream_t s);
 // a2 of several hash tables in one launch (tables 1..L-1 of an L-table index)
@@ -140,7 +145,7 @@ struct ShortlistArgs {
 // 0: warp short-list, 1: SIMT query-tiled, 2: tensor-core screened query-tiled.  The TC
 // kernel is the default where it applies (k <= 32, d_stride a multiple of 64 and <= 512);
 // BLSH_SHORTLIST=warp|simt forces the others.
-int shortlist_kind(int ds, int dr, int T, int k);
+int shortlist_kind(int64_t nq, int ds, int dr, int T, int k);
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
 int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, ScanTemp& scan, cudaStream_t s,
                    int* launches);

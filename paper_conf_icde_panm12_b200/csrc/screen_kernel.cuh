@@ -60,6 +60,7 @@ struct SxSmem {
     float kt[kSxAnc][QT];           // the item's K table rows: K_aj = |q_j - a|^2 (k_anchor_k)
     alignas(16) float eta[QT];
     uint32_t umin[QT];
+    float ksub[kSxEpiN][QT];        // per epilogue warp and query: the ceil(k/8)-th smallest upper bound it has seen
     int scnt[kSxEpiN][QT];
     float tr[kSxEpiN][32 * 17];     // per epilogue warp: transposed dots [query][row of its 16]
     float4 rf[kSxEpiN][16];         // per epilogue warp and row: beta, m, E, n
@@ -290,6 +291,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         }
     }
     if (threadIdx.x < QT) S.umin[threadIdx.x] = 0x7F800000u;
+    for (int i = threadIdx.x; i < kSxEpiN * QT; i += kSxThreads) (&S.ksub[0][0])[i] = __int_as_float(0x7F800000);
     if (threadIdx.x == 0) {
         for (int s = 0; s < nst; ++s) {
             mbar_init(&S.afull[s], 1);
@@ -429,6 +431,14 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         const bool mine_row = (lane >> 4) == half;
         const int j = lane;                     // query of this lane (screen phase)
         const float eta = S.eta[j];
+        // Two valid bounds on query j's k-th smallest distance among the item's rows: the k-th
+        // smallest upper bound one warp has seen (ulr[KT - 1]; any warp's), and -- since the 8
+        // warps see disjoint rows -- the largest over the warps of each one's kk-th smallest,
+        // kk = ceil(k / 8): every warp holds >= kk bounds below it, >= k in all.  The second is
+        // near the true k-th (each warp sees 1/8 of the rows); the first is what a warp alone knows.
+        const int kk = (k + kSxEpiN - 1) / kSxEpiN;
+        const int isub = KT - k + kk - 1;       // position of the kk-th smallest in the sorted list
+        volatile float* ksub_all = &S.ksub[0][0];
         float ulr[KT];
 #pragma unroll
         for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
@@ -506,6 +516,15 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             __syncwarp();
             if (a.dbgmode & 1) continue;                           // ablation: no screen loop
             float U = fminf(ulr[KT - 1], __uint_as_float(S.umin[j]));   // any warp's bound is valid
+            {
+                float us = ksub_all[j];
+#pragma unroll
+                for (int w = 1; w < kSxEpiN; ++w) us = fmaxf(us, ksub_all[w * QT + j]);
+                if (us < U) {
+                    U = us;
+                    atomicMin(&S.umin[j], __float_as_uint(us));
+                }
+            }
             // pass 1 (branch-free): rows of this query whose lower bound clears the bound at the
             // block start; pass 2 takes them in row order against the tightening bound, so the
             // pairs kept are exactly those of a row-by-row loop
@@ -536,6 +555,10 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
 #pragma unroll
                     for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
                     ulr[0] = fminf(ulr[0], up);
+                    float sub = ulr[0];
+#pragma unroll
+                    for (int p = 1; p < KT; ++p) sub = p == isub ? ulr[p] : sub;
+                    ksub_all[ew * QT + j] = sub;                   // only decreases: stale reads stay valid
                     if (ulr[KT - 1] < U) {                         // share the tighter bound at once
                         U = ulr[KT - 1];
                         atomicMin(&S.umin[j], __float_as_uint(U));

@@ -30,6 +30,7 @@ namespace blsh {
 namespace {
 
 constexpr int QT = 32;            // queries per tile
+constexpr int64_t kSmallBatch = 128;   // batches up to this size take the warp short-list
 constexpr int kPrepThreads = 256;
 constexpr int kRows = 32;         // rows per stage (one per lane)
 constexpr int kTW = 8;            // warps per CTA (each owns 4 tile queries)
@@ -619,9 +620,12 @@ static int screen_variant() {
     return v;
 }
 
-int shortlist_kind(int ds, int dr, int T, int k) {
+int shortlist_kind(int64_t nq, int ds, int dr, int T, int k) {
     const char* mode = std::getenv("BLSH_SHORTLIST");
     if (mode && std::strcmp(mode, "warp") == 0) return 0;
+    // small batches (<= 4 tiles): the tiled path's planning launches and host round trips
+    // (~0.6 ms) exceed the warp short-list's whole run (profiles/r02/c5_sweep.jsonl, B <= 100)
+    if (!mode && nq <= kSmallBatch) return 0;
     if (k > 64) return 0;   // large k: warp short-list emitting every key + k_select
     int cap = 2 * QT * (T + 1), npow = 1;
     while (npow < cap) npow <<= 1;

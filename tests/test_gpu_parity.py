@@ -4,6 +4,8 @@ Bit-exact: parameters, tree, per-point leaf/code/key, table, per-query
 leaf/t/code/key/probe keys/candidate sets.  Distances within 1e-5 relative,
 ids equal except ties (parity_utils.check_topk).
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -79,6 +81,18 @@ def run_query_pair(ix, ox, X, Q, k, probe=0, T=1, hierarchy=0, hier_step_bits=0,
         assert np.array_equal(gc[q], oc[q]), f"candidate set of query {q} differs"
     assert np.array_equal(nc, onc)
     check_topk(ids, d2, oi, od, X, Q, cands=oc)
+    if len(Q) <= 128 and k <= 64 and device and "BLSH_SHORTLIST" not in os.environ:
+        # small batches default to the warp short-list: the tiled tensor-core path must
+        # return the same bits on them (the large-batch product path)
+        os.environ["BLSH_SHORTLIST"] = "tc"
+        try:
+            i2, d22, n2 = ix.query(Qin, k, probe=probe, n_probes=T, hierarchy=hierarchy,
+                                   hier_step_bits=hier_step_bits, min_cand=min_cand, **extra)
+            torch.cuda.synchronize()
+        finally:
+            del os.environ["BLSH_SHORTLIST"]
+        assert np.array_equal(i2.cpu().numpy(), ids) and np.array_equal(d22.cpu().numpy().view(np.uint32), d2.view(np.uint32))
+        assert np.array_equal(n2.cpu().numpy(), nc)
     return ids, d2, nc
 
 
@@ -310,6 +324,9 @@ def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
     assert ix.stats().tiled == 0
     monkeypatch.delenv("BLSH_SHORTLIST")
     run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
+    assert ix.stats().tiled == 0, "batches of <= 128 queries take the warp short-list by default"
+    Q2 = np.concatenate([Q, Q, Q])                  # 300 queries: the tiled path
+    run_query_pair(ix, ox, X, Q2, 10, probe=1, T=16)
     assert ix.stats().tiled >= 1
 
 
