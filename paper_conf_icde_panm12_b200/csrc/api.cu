@@ -687,7 +687,8 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     if (tiled) {
         // a5, query-tiled: sort queries by bi-level code, stream each tile's candidate union once
         int chr = 0;
-        run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.rowbuf, w.partials, w.scan, d_ids, d_d2, d_pk, d_nc,
+        run_tiled_shortlist(a, qorder, k, w.segbuf, w.tilebuf, w.rowbuf, w.partials, w.keybuf, w.scan, d_ids, d_d2,
+                            d_pk, d_nc,
                             ix.Xp.as<float>(), ix.perm.as<uint32_t>(), s, &launches, &n_items, &chr, &union_rows,
                             tm ? ix.ev[4] : nullptr, tm ? ix.ev[8] : nullptr, tm ? ix.ev[5] : nullptr, &pairs,
                             &kept, &qload_rows, kind, ntiles_pre, &kslots, &screen_kind);

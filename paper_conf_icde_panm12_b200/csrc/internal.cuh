@@ -93,6 +93,7 @@ struct QueryWork {
     DevBuf partials;   // per-item partial top-k lists
     DevBuf host_stage; // device staging for host outputs
     DevBuf segbuf, tilebuf;   // tiled short-list: per-tile segments, tile arrays
+    DevBuf keybuf;            // tiled short-list, large k: per-query segments of exact (d^2, id) keys
     DevBuf rowbuf;            // tiled short-list: per-union-row entries, K table, item rows
     SortBufs qsort;           // query sort by (leaf, key)
     ScanTemp scan;

@@ -436,16 +436,23 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         // warps see disjoint rows -- the largest over the warps of each one's kk-th smallest,
         // kk = ceil(k / 8): every warp holds >= kk bounds below it, >= k in all.  The second is
         // near the true k-th (each warp sees 1/8 of the rows); the first is what a warp alone knows.
+        // For k > KT (large k, KT = 64) a warp keeps only its kk smallest and only the second
+        // bound is used.
+        // (Used from KT = 32 on: at k <= 16 it buys few rescorings and costs screen time.)
+        constexpr bool kSub = KT >= 32;
         const int kk = (k + kSxEpiN - 1) / kSxEpiN;
-        const int isub = KT - k + kk - 1;       // position of the kk-th smallest in the sorted list
+        const bool own_valid = k <= KT;
+        const int klist = own_valid ? k : kk;   // real entries of the list
+        const int isub = KT - klist + kk - 1;   // position of the kk-th smallest in the sorted list
         volatile float* ksub_all = &S.ksub[0][0];
         float ulr[KT];
 #pragma unroll
-        for (int p = 0; p < KT; ++p) ulr[p] = p < KT - k ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
+        for (int p = 0; p < KT; ++p) ulr[p] = p < KT - klist ? __int_as_float(0xFF800000) : __int_as_float(0x7F800000);
         int my_cnt = 0, n_ins = 0, n_cmp = 0;
         long long wec = 0;
         bool my_fail = false;
-        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * kSxEpiN + ew) * kTcScap;
+        const int scapw = a.scapw;              // buffered pairs per (item, query, epilogue warp)
+        unsigned long long* SBj = a.sbuf + (((size_t)item * QT + j) * kSxEpiN + ew) * scapw;
         float* Tt = S.tr[ew];
         for (int b = 0; b < nblk; ++b) {
             const int mb = b % kSxNM;
@@ -515,8 +522,8 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
             }
             __syncwarp();
             if (a.dbgmode & 1) continue;                           // ablation: no screen loop
-            float U = fminf(ulr[KT - 1], __uint_as_float(S.umin[j]));   // any warp's bound is valid
-            {
+            float U = own_valid ? fminf(ulr[KT - 1], __uint_as_float(S.umin[j])) : __uint_as_float(S.umin[j]);
+            if (kSub) {
                 float us = ksub_all[j];
 #pragma unroll
                 for (int w = 1; w < kSxEpiN; ++w) us = fmaxf(us, ksub_all[w * QT + j]);
@@ -555,22 +562,24 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
 #pragma unroll
                     for (int p = KT - 1; p > 0; --p) ulr[p] = fmaxf(ulr[p - 1], fminf(ulr[p], up));
                     ulr[0] = fminf(ulr[0], up);
-                    float sub = ulr[0];
+                    if (kSub) {
+                        float sub = ulr[0];
 #pragma unroll
-                    for (int p = 1; p < KT; ++p) sub = p == isub ? ulr[p] : sub;
-                    ksub_all[ew * QT + j] = sub;                   // only decreases: stale reads stay valid
-                    if (ulr[KT - 1] < U) {                         // share the tighter bound at once
+                        for (int p = 1; p < KT; ++p) sub = p == isub ? ulr[p] : sub;
+                        ksub_all[ew * QT + j] = sub;               // only decreases: stale reads stay valid
+                    }
+                    if (own_valid && ulr[KT - 1] < U) {            // share the tighter bound at once
                         U = ulr[KT - 1];
                         atomicMin(&S.umin[j], __float_as_uint(U));
                     }
                 }
                 const unsigned long long e = ((unsigned long long)__float_as_uint(fmaxf(lo, 0.f)) << 32) | ru.y;
                 ++n_ins;
-                if (my_cnt == kTcScap) {                           // full: drop what the tighter U excludes
+                if (my_cnt == scapw) {                             // full: drop what the tighter U excludes
                     ++n_cmp;
                     int c2 = 0;
                     const ulonglong2* B2 = reinterpret_cast<const ulonglong2*>(SBj);
-                    for (int t0 = 0; t0 < kTcScap / 2; t0 += 8) {  // 8 independent 16-byte loads per batch
+                    for (int t0 = 0; t0 < scapw / 2; t0 += 8) {    // 8 independent 16-byte loads per batch
                         ulonglong2 f[8];
 #pragma unroll
                         for (int u = 0; u < 8; ++u) f[u] = B2[t0 + u];
@@ -581,7 +590,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
                         }
                     }
                     my_cnt = c2;
-                    if (my_cnt > 3 * kTcScap / 4) { my_fail = true; break; }   // exact scan of j's rows later
+                    if (my_cnt > 3 * scapw / 4) { my_fail = true; break; }     // exact scan of j's rows later
                 }
                 SBj[my_cnt++] = e;
             }
@@ -611,7 +620,7 @@ __global__ void __launch_bounds__(kSxThreads, 1) k_screen_f16(TiledArgs a) {
         a.ufin[(size_t)item * QT + j] = j < nqt ? S.umin[j] : 0u;
 #pragma unroll
         for (int w = 0; w < kSxEpiN; ++w)
-            a.scnt[((size_t)item * QT + j) * kSxEpiN + w] = j < nqt ? min(S.scnt[w][j], kTcScap) : 0;
+            a.scnt[((size_t)item * QT + j) * kSxEpiN + w] = j < nqt ? min(S.scnt[w][j], a.scapw) : 0;
     }
 }
 
@@ -648,4 +657,174 @@ __global__ void __launch_bounds__(256) k_anchor_k(const float* __restrict__ Q, i
         }
         ktab[(size_t)sl * QT + lane] = lane < nqt ? (s0 + s1) + (s2 + s3) : 0.f;
     }
+}
+
+// ---------------------------------------------------------------------------
+// Large k (64 < k <= kSxMaxKLarge, the paper's k = 500 of P:217) after the fp16 screen:
+// every surviving (row, query) pair of a work item gets its exact fp32 distance (the warp
+// short-list's form, R22) and its packed (d^2, id) key goes to the query's key segment;
+// launch_select then keeps the k smallest per query (as the warp large-k path does).
+//   k_unit_counts    keys per (item, query) unit: its buffered pairs, or (a buffer
+//                    overflowed) every row of the item whose query mask has bit j
+//   k_query_counts   per query: total over its tile's items, each unit's offset in it
+//   k_tc_emit        one warp per unit: exact distances, keys at the unit's offset;
+//                    buffered pairs the final bound excludes become padding keys
+// ---------------------------------------------------------------------------
+constexpr int kSxMaxKLarge = 512;   // kk = ceil(k / 8) <= 64: the KT = 64 lists hold it
+
+__global__ void __launch_bounds__(256) k_unit_counts(TiledArgs a, int64_t* __restrict__ ucnt) {
+    const int lane = threadIdx.x & 31;
+    const int64_t unit = blockIdx.x * (int64_t)8 + (threadIdx.x >> 5);
+    if (unit >= a.n_items * QT) return;
+    const int64_t item = unit / QT;
+    const int j = (int)(unit % QT);
+    int64_t r0, r1;
+    const int64_t t = item_tile_rows(a, item, &r0, &r1);
+    if (j >= (int)(a.tile_off[t + 1] - a.tile_off[t])) {
+        if (lane == 0) ucnt[unit] = 0;
+        return;
+    }
+    bool failed = false;
+    int64_t c = 0;
+    for (int w = 0; w < a.nlist; ++w) {
+        const int v = a.scnt[unit * a.nlist + w];
+        failed |= v < 0;
+        c += v > 0 ? v : 0;
+    }
+    if (failed) {
+        const uint4* RI = a.rowinfo + a.rows_off[t];
+        c = 0;
+        for (int64_t base = r0; base < r1; base += 32) {
+            const int64_t i = base + lane;
+            const uint4 e = i < r1 ? RI[i] : make_uint4(0u, 0u, 0u, 0u);
+            c += __popc(__ballot_sync(BLSH_FULL, (e.y >> j) & 1u));
+        }
+    }
+    if (lane == 0) ucnt[unit] = c;
+}
+
+__global__ void __launch_bounds__(256) k_query_counts(TiledArgs a, const int64_t* __restrict__ ucnt,
+                                                      int64_t* __restrict__ uloc, int64_t* __restrict__ qcnt) {
+    const int64_t pos = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (pos >= a.nq) return;
+    const int64_t t = a.tile_of[pos];
+    const int j = (int)(pos - a.tile_off[t]);
+    int64_t c = 0;
+    for (int64_t it = a.item_off[t]; it < a.item_off[t + 1]; ++it) {
+        uloc[it * QT + j] = c;
+        c += ucnt[it * QT + j];
+    }
+    qcnt[a.qorder[pos]] = c;
+}
+
+template <int NV>
+__global__ void __launch_bounds__(256) k_tc_emit(TiledArgs a, const int64_t* __restrict__ uloc,
+                                                 const int64_t* __restrict__ cand_off,
+                                                 unsigned long long* __restrict__ keys) {
+    const int lane = threadIdx.x & 31;
+    const int64_t unit = blockIdx.x * (int64_t)8 + (threadIdx.x >> 5);
+    if (unit >= a.n_items * QT) return;
+    const int64_t item = unit / QT;
+    const int j = (int)(unit % QT);
+    int64_t r0, r1;
+    const int64_t t = item_tile_rows(a, item, &r0, &r1);
+    const int64_t q0 = a.tile_off[t];
+    if (j >= (int)(a.tile_off[t + 1] - q0)) return;
+    const int nv = a.ds >> 2;
+    const uint32_t qid = a.qorder[q0 + j];
+    unsigned long long* seg = keys + cand_off[qid] + uloc[unit];
+    const float U = __uint_as_float(a.ufin[unit]);
+    const float4* qrow = reinterpret_cast<const float4*>(a.Q + (size_t)qid * a.ds);
+    float4 qv[NV];
+#pragma unroll
+    for (int u = 0; u < NV; ++u) {
+        const int v = lane + 32 * u;
+        qv[u] = v < nv ? __ldg(qrow + v) : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    int rescored = 0;
+    // rows of the set bits of nm (lane i holds row position rpos); row r of a group goes to
+    // slot sbase + (compact ? its rank among the set bits : its source lane)
+    auto score_rows = [&](unsigned nm, uint32_t rpos, int64_t sbase, bool compact) {
+        int done = 0;
+        while (nm) {
+            uint32_t row[4];
+            int src[4];
+            int nr = 0;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                row[r] = 0u;
+                src[r] = 0;
+                if (nm) {
+                    src[r] = __ffs(nm) - 1;
+                    nm &= nm - 1;
+                    row[r] = (uint32_t)__shfl_sync(BLSH_FULL, rpos, src[r]);
+                    nr = r + 1;
+                }
+            }
+            float part[4];
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                part[r] = 0.0f;
+                if (r < nr) {
+                    const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)row[r] * a.ds);
+#pragma unroll
+                    for (int u = 0; u < NV; ++u) {
+                        const int v = lane + 32 * u;
+                        if (v < nv) {
+                            const float4 x = __ldg(xr + v);
+                            const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                            part[r] = fmaf(dx, dx, part[r]);
+                            part[r] = fmaf(dy, dy, part[r]);
+                            part[r] = fmaf(dz, dz, part[r]);
+                            part[r] = fmaf(dw, dw, part[r]);
+                        }
+                    }
+                }
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+                for (int r = 0; r < 4; ++r) part[r] += __shfl_xor_sync(BLSH_FULL, part[r], o);
+            }
+            const uint32_t rl = (lane & 3) == 0 ? row[0] : (lane & 3) == 1 ? row[1] : (lane & 3) == 2 ? row[2] : row[3];
+            const uint32_t idl = lane < nr ? __ldg(a.perm + rl) : 0u;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const uint32_t id = __shfl_sync(BLSH_FULL, idl, r);
+                if (r < nr && lane == r) seg[sbase + (compact ? done + r : src[r])] = pack_entry(part[r], id);
+            }
+            done += nr;
+        }
+    };
+    bool failed = false;
+    for (int w = 0; w < a.nlist; ++w) failed |= a.scnt[unit * a.nlist + w] < 0;
+    if (failed) {
+        const uint4* RI = a.rowinfo + a.rows_off[t];
+        int64_t at = 0;
+        for (int64_t base = r0; base < r1; base += 32) {
+            const int64_t i = base + lane;
+            const uint4 e = i < r1 ? RI[i] : make_uint4(0u, 0u, 0u, 0u);
+            const unsigned nm = __ballot_sync(BLSH_FULL, (e.y >> j) & 1u);
+            rescored += __popc(nm);
+            score_rows(nm, e.x, at, true);
+            at += __popc(nm);
+        }
+    } else {
+        int64_t at = 0;
+        for (int w = 0; w < a.nlist; ++w) {
+            const int cnt = a.scnt[unit * a.nlist + w];
+            const unsigned long long* Bf = a.sbuf + ((size_t)unit * a.nlist + w) * a.scapw;
+            for (int base = 0; base < cnt; base += 32) {
+                const int i = base + lane;
+                const unsigned long long e = i < cnt ? Bf[i] : ~0ull;
+                const bool need = i < cnt && __uint_as_float((uint32_t)(e >> 32)) <= U;
+                if (i < cnt && !need) seg[at + lane] = kEmpty;     // excluded by the final bound: padding
+                const unsigned nm = __ballot_sync(BLSH_FULL, need);
+                rescored += __popc(nm);
+                score_rows(nm, (uint32_t)(e & 0xFFFFFFFFull), at, false);
+                at += min(32, cnt - base);
+            }
+        }
+    }
+    if (lane == 0 && a.counters && rescored) atomicAdd(a.counters + 1, (unsigned long long)rescored);
 }

@@ -422,6 +422,7 @@ struct TiledArgs {
     float* dbg;                     // optional (BLSH_TC_DEBUG): item 0, block 0 dots / |x'|^2 / rows
     unsigned long long* sbuf;       // TC: [n_items][QT][scap] buffered (lower bound, row) pairs
     int scap;
+    int scapw;                      // per list (scap = nlist x scapw)
     int nlist;                      // TC screens: buffered-pair lists per (item, query): epilogue warps
     int dbgmode;                    // ablation (BLSH_TC_MODE): 1 skip screen, 2 skip row loads, 4 skip MMA, 32 phase timers
     unsigned long long* tstamp;     // BLSH_TC_MODE & 32: [n_items][8] globaltimer stamps per phase
@@ -626,14 +627,16 @@ int shortlist_kind(int64_t nq, int ds, int dr, int T, int k) {
     // small batches (<= 4 tiles): the tiled path's planning launches and host round trips
     // (~0.6 ms) exceed the warp short-list's whole run (profiles/r02/c5_sweep.jsonl, B <= 100)
     if (!mode && nq <= kSmallBatch) return 0;
-    if (k > 64) return 0;   // large k: warp short-list emitting every key + k_select
+    // large k (64 < k <= 512): the fp16 screen (kk lists) + exact keys per query + k_select;
+    // beyond, or without the fp16 screen: the warp short-list emitting every key + k_select
+    if (k > 64 && (k > kSxMaxKLarge || screen_variant() != 0 || (mode && std::strcmp(mode, "simt") == 0))) return 0;
     int cap = 2 * QT * (T + 1), npow = 1;
     while (npow < cap) npow <<= 1;
     if ((size_t)3 * npow * 4 > 227 * 1024) return 0;   // tile prep does not fit
-    const bool simt_ok = tiled_smem_bytes(ds) <= 227 * 1024;
+    const bool simt_ok = k <= 64 && tiled_smem_bytes(ds) <= 227 * 1024;
     const bool tc_ok = screen_variant() == 1
                            ? (k <= kTcMaxK && ds % kTcChunk == 0 && ds <= 512 && tc_smem_bytes(ds) <= 227 * 1024)
-                           : (k <= kSxMaxK && dr >= 64 && dr <= kSxMaxDr && screen_stages(dr) > 0);
+                           : ((k <= kSxMaxK || k <= kSxMaxKLarge) && dr >= 64 && dr <= kSxMaxDr && screen_stages(dr) > 0);
     if (mode && std::strcmp(mode, "simt") == 0) return simt_ok ? 1 : 0;
     if (tc_ok) return 2;
     return simt_ok ? 1 : 0;
@@ -711,7 +714,7 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
 
 void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevBuf& segbuf, DevBuf& tilebuf,
                          DevBuf& rowbuf,
-                         DevBuf& partials, ScanTemp& scan, int64_t* out_ids, float* out_d2,
+                         DevBuf& partials, DevBuf& keybuf, ScanTemp& scan, int64_t* out_ids, float* out_d2,
                          unsigned long long* out_packed, int64_t* out_ncand, const float* Xp, const uint32_t* perm,
                          cudaStream_t s, int* launches, int64_t* n_items_out, int* chr_out, int64_t* rows_out,
                          cudaEvent_t ev_sl0, cudaEvent_t ev_mid, cudaEvent_t ev_sl1, int64_t* pairs_out,
@@ -799,12 +802,18 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     BLSH_CUDA(cudaMemcpyAsync(&n_items, item_off + ntiles, 8, cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
     const int nlist = use_f16 ? kSxEpiN : 4;   // buffered-pair lists per (item, query): the screen's epilogue warps
-    const int kScap = nlist * kTcScap;
-    const size_t part_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
+    const bool large_k = k > 64;               // fp16 screen + exact keys per query + launch_select
+    // large k: each warp's list holds ~kk = ceil(k/8) survivors (+ the bound's slack)
+    const int scapw = large_k ? ((2 * ((k + kSxEpiN - 1) / kSxEpiN) + 64 + 15) / 16) * 16 : kTcScap;
+    const int kScap = nlist * scapw;
+    const size_t part_bytes = large_k ? 0 : ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
     const size_t ufin_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * 4 + 255) & ~size_t(255);
     const size_t scnt_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * nlist * 4 + 255) & ~size_t(255);
-    partials.ensure(part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes);
+    // large k: unit counts, unit offsets in their query's segment, query counts, segment offsets
+    const size_t unit_bytes = large_k ? (((size_t)std::max<int64_t>(n_items, 1) * QT * 8 + 255) & ~size_t(255)) : 0;
+    const size_t q_bytes = large_k ? (((size_t)(nq + 1) * 8 + 255) & ~size_t(255)) : 0;
+    partials.ensure(part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes + 2 * unit_bytes + 2 * q_bytes);
     TiledArgs ta{};
     ta.nq = nq; ta.ntiles = ntiles; ta.n_items = n_items; ta.d = a.d; ta.ds = a.ds; ta.k = k; ta.chr = (int)chr;
     ta.segcap = segcap; ta.Q = a.Q; ta.Xp = Xp; ta.perm = perm; ta.qorder = qorder; ta.segs = segbuf.as<Seg>();
@@ -814,6 +823,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     ta.tile_of = tile_of;
     ta.sbuf = reinterpret_cast<unsigned long long*>(partials.as<char>() + part_bytes);
     ta.scap = kScap;
+    ta.scapw = scapw;
     ta.nlist = nlist;
     ta.rows_off = rows_off;
     ta.ufin = reinterpret_cast<uint32_t*>(partials.as<char>() + part_bytes + sbuf_bytes);
@@ -855,7 +865,7 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     if (ev_sl0) BLSH_CUDA(cudaEventRecord(ev_sl0, s));
     if (n_items > 0) {
         if (use_f16) {
-            auto pick = [&](auto k8, auto k12, auto k16, auto k32, auto k64) {
+            auto pick = [&](auto k8, auto k12, auto k16, auto k32, auto k64) {   // k > 64: KT = 64 (kk lists)
                 return k <= 8 ? k8 : (k <= 12 ? k12 : (k <= 16 ? k16 : (k <= 32 ? k32 : k64)));
             };
             auto kern = nst == 8 ? pick(k_screen_f16<8, 8>, k_screen_f16<12, 8>, k_screen_f16<16, 8>, k_screen_f16<32, 8>,
@@ -872,7 +882,39 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
             BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem));
             kern<<<(unsigned)n_items, kTcThreads, tc_smem, s>>>(ta);
         }
-        if (use_tc) {
+        if (use_tc && large_k) {
+            BLSH_LAUNCH_CHECK();
+            ++*launches;
+            if (ev_mid) BLSH_CUDA(cudaEventRecord(ev_mid, s));
+            char* pb = partials.as<char>() + part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes;
+            int64_t* ucnt = reinterpret_cast<int64_t*>(pb);
+            int64_t* uloc = reinterpret_cast<int64_t*>(pb + unit_bytes);
+            int64_t* qcnt = reinterpret_cast<int64_t*>(pb + 2 * unit_bytes);
+            int64_t* coff = reinterpret_cast<int64_t*>(pb + 2 * unit_bytes + q_bytes);
+            const unsigned rg = (unsigned)((n_items * QT + 7) / 8);
+            BLSH_CUDA(cudaMemsetAsync(qcnt, 0, (size_t)nq * 8, s));
+            k_unit_counts<<<rg, 256, 0, s>>>(ta, ucnt);
+            BLSH_LAUNCH_CHECK();
+            k_query_counts<<<(unsigned)((nq + 255) / 256), 256, 0, s>>>(ta, ucnt, uloc, qcnt);
+            BLSH_LAUNCH_CHECK();
+            scan_exclusive_i64(qcnt, coff, nq, scan, s);
+            *launches += 5;
+            int64_t nkeys = 0;
+            BLSH_CUDA(cudaMemcpyAsync(&nkeys, coff + nq, 8, cudaMemcpyDeviceToHost, s));
+            BLSH_CUDA(cudaStreamSynchronize(s));
+            keybuf.ensure((size_t)std::max<int64_t>(nkeys, 1) * 8);
+            unsigned long long* keys = keybuf.as<unsigned long long>();
+            const int nvq = (a.ds / 4 + 31) / 32;
+            if (nvq <= 1) k_tc_emit<1><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else if (nvq == 2) k_tc_emit<2><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else if (nvq == 3) k_tc_emit<3><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else k_tc_emit<4><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            BLSH_LAUNCH_CHECK();
+            ++*launches;
+            if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
+            launch_select(keys, coff, nq, k, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand, s);
+            *launches += 2;
+        } else if (use_tc) {
             BLSH_LAUNCH_CHECK();
             ++*launches;
             if (ev_mid) BLSH_CUDA(cudaEventRecord(ev_mid, s));
@@ -890,10 +932,22 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
         ++*launches;
     }
     if (ev_mid && !use_tc) BLSH_CUDA(cudaEventRecord(ev_mid, s));
-    if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
-    k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed, out_ncand);
-    BLSH_LAUNCH_CHECK();
-    ++*launches;
+    if (!(large_k && n_items > 0)) {
+        if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
+        if (large_k) {   // no work item: padding only
+            char* pb = partials.as<char>() + part_bytes + sbuf_bytes + ufin_bytes + scnt_bytes;
+            int64_t* coff = reinterpret_cast<int64_t*>(pb + 2 * unit_bytes + q_bytes);
+            BLSH_CUDA(cudaMemsetAsync(coff, 0, (size_t)(nq + 1) * 8, s));
+            launch_select(keybuf.as<unsigned long long>(), coff, nq, k, a.qoor, a.cnt, out_ids, out_d2, out_packed,
+                          out_ncand, s);
+            *launches += 2;
+        } else {
+            k_merge_tiled<<<(unsigned)((nq + 7) / 8), 256, 0, s>>>(ta, a.qoor, a.cnt, out_ids, out_d2, out_packed,
+                                                                   out_ncand);
+            BLSH_LAUNCH_CHECK();
+            ++*launches;
+        }
+    }
     *n_items_out = n_items;
     *chr_out = (int)chr;
     *rows_out = total_rows;

@@ -578,7 +578,7 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     } else {
         for (int w = 0; w < a.nlist; ++w) {
             const int cnt = a.scnt[unit * a.nlist + w];
-            const unsigned long long* Bf = a.sbuf + ((size_t)unit * a.nlist + w) * kTcScap;
+            const unsigned long long* Bf = a.sbuf + ((size_t)unit * a.nlist + w) * a.scapw;
             for (int base = 0; base < cnt; base += 32) {
                 const int i = base + lane;
                 const unsigned long long e = i < cnt ? Bf[i] : ~0ull;

@@ -148,3 +148,63 @@ def test_large_k_sharded_merge_matches_single(blsh, orc, c1):
     mi, md = blsh.blsh_merge_topk(torch.cat(parts).contiguous(), 2, len(Q), 256)
     torch.cuda.synchronize()
     assert torch.equal(mi, i1) and torch.equal(md.view(torch.int32), d1.view(torch.int32))
+
+
+# Large k on the tensor-core path (64 < k <= 512): the fp16 screen keeps ceil(k/8) bounds per
+# epilogue warp, every survivor gets the exact fp32 distance, k_select keeps the k smallest.
+@pytest.mark.parametrize("k,T", [(65, 8), (100, 16), (500, 64), (512, 4)])
+def test_large_k_tc_vs_oracle(c1_pair, c1, monkeypatch, k, T):
+    X, Q = c1
+    monkeypatch.setenv("BLSH_SHORTLIST", "tc")
+    run_query_pair(*c1_pair, X, Q, k, probe=1, T=T)
+    assert c1_pair[0].stats().tiled == 2
+
+
+def test_large_k_tc_hierarchy_and_default_batch(c1_pair, c1):
+    X, Q = c1
+    Q3 = np.concatenate([Q, Q[::-1], Q[::2]])      # 250 queries: the tiled path by default
+    run_query_pair(*c1_pair, X, Q3, 300, probe=1, T=8, hierarchy=1)
+    assert c1_pair[0].stats().tiled == 2
+
+
+def _mode(ix, Q, k, mode, monkeypatch, **kw):
+    monkeypatch.setenv("BLSH_SHORTLIST", mode)
+    ids, d2, nc = ix.query(torch.from_numpy(Q).cuda(), k, **kw)
+    torch.cuda.synchronize()
+    t = ix.stats().tiled
+    monkeypatch.delenv("BLSH_SHORTLIST")
+    return ids.cpu().numpy(), d2.cpu().numpy(), nc.cpu().numpy(), t
+
+
+@pytest.mark.parametrize("shape", ["lowrank384", "dup_overflow"])
+def test_large_k_tc_equals_warp(blsh, orc, monkeypatch, shape):
+    """Bit identity of the large-k TC path with the warp large-k path (ids, d^2 bits, counts);
+    dup_overflow: 10 points repeated 1000x, so the per-warp pair buffers overflow and the
+    items' rows are scored exhaustively."""
+    if shape == "lowrank384":
+        mix = synth.mixture(384, 64, 16, 0.02, 31)
+        X = synth.sample_points(mix, 20000, 32)
+        Q = synth.sample_points(mix, 400, 33)
+        G, W, T = 4, 1.2, 16
+    else:
+        mix = synth.mixture(128, 8, 8, 0.05, 51)
+        X = np.repeat(synth.sample_points(mix, 10, 52), 1000, axis=0)
+        Q = synth.sample_points(mix, 100, 53)
+        G, W, T = 2, 3.0, 4
+    ix, ox = build_pair(blsh, orc, X, G=G, M=8, W=W, seed=5)
+    for k in (65, 128, 500, 512):
+        a = _mode(ix, Q, k, "warp", monkeypatch, probe=1, n_probes=T)
+        b = _mode(ix, Q, k, "tc", monkeypatch, probe=1, n_probes=T)
+        assert a[3] == 0 and b[3] == 2
+        np.testing.assert_array_equal(a[2], b[2])
+        np.testing.assert_array_equal(a[0], b[0])
+        np.testing.assert_array_equal(a[1].view(np.uint32), b[1].view(np.uint32))
+    monkeypatch.setenv("BLSH_SHORTLIST", "tc")
+    run_query_pair(ix, ox, X, Q[:60], 200, probe=1, T=T)
+
+
+def test_k_above_512_stays_on_warp_path(c1_pair, c1):
+    X, Q = c1
+    Q3 = np.concatenate([Q, Q, Q])
+    run_query_pair(*c1_pair, X, Q3, 600, probe=1, T=4)
+    assert c1_pair[0].stats().tiled == 0

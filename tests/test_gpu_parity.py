@@ -324,6 +324,7 @@ def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
     assert ix.stats().tiled == 0
     monkeypatch.delenv("BLSH_SHORTLIST")
     run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
+    ix.query(torch.from_numpy(Q).cuda(), 10, probe=1, n_probes=16)
     assert ix.stats().tiled == 0, "batches of <= 128 queries take the warp short-list by default"
     Q2 = np.concatenate([Q, Q, Q])                  # 300 queries: the tiled path
     run_query_pair(ix, ox, X, Q2, 10, probe=1, T=16)

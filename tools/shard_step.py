@@ -46,7 +46,7 @@ def main():
     X, Q = synth.make_dataset(cfg, backend="torch", device="cuda:0")
     kw = dict(probe=cfg.probe, n_probes=cfg.T)
     full = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
-    ms_full = timed(lambda: full.query(Q, cfg.k, **kw))
+    ms_full = timed(lambda: full.query(Q, cfg.k, timing=True, **kw))
     st_full = full.stats()
     ids_f, d2_f, _ = full.query(Q, cfg.k, **kw)
     del full
@@ -56,8 +56,13 @@ def main():
     parts = []
     for r in range(a.world):
         sh = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index, rank=r, world=a.world)
-        ms = timed(lambda: sh.query_packed(Q, cfg.k, **kw), reps=3)
+        ms = timed(lambda: sh.query_packed(Q, cfg.k, timing=True, **kw), reps=3)
         out["ms_shard"][r] = ms
+        st = sh.stats()
+        out.setdefault("stage_shard", {})[r] = dict(nq_owned=st.n_active, route_hash=st.ms_route_hash,
+                                                    probe=st.ms_probe, plan=st.ms_plan, screen=st.ms_screen,
+                                                    rescore=st.ms_rescore, merge=st.ms_merge, total=st.ms_total,
+                                                    items=st.n_items, launches=st.launches)
         parts.append(sh.query_packed(Q, cfg.k, **kw)[0].clone())
         del sh
         torch.cuda.empty_cache()
