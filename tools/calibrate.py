@@ -59,11 +59,14 @@ def main():
     ap.add_argument("--hier", action="store_true", help="Morton hierarchy with tau = batch median")
     ap.add_argument("--out", default=None)
     ap.add_argument("--G", type=int, default=None, help="override the config's leaf count")
+    ap.add_argument("--L", type=int, default=1, help="hash tables per leaf (P:43)")
+    ap.add_argument("--k", type=int, default=None, help="k of the timed full batch (default: the config's)")
     a = ap.parse_args()
     cfg = synth.CONFIGS[a.config]
     if a.G:
         from dataclasses import replace
         cfg = replace(cfg, G=a.G)
+    kq = a.k or cfg.k
     t0 = time.time()
     X, Q = synth.make_dataset(cfg, backend="torch", device="cuda:0")
     torch.cuda.synchronize()
@@ -79,7 +82,7 @@ def main():
         W = wm * r10
         t1 = time.time()
         ix = blsh.blsh_build(X, n_leaves=cfg.G, M=cfg.M, W=W, seed=cfg.seed_index, keep_stages=True,
-                             quantizer=1 if a.lattice else 0)
+                             quantizer=1 if a.lattice else 0, n_tables=a.L)
         torch.cuda.synchronize()
         bt = time.time() - t1
         pleaf = torch.as_tensor(ix.export("POINT_LEAF"), device="cuda").long()
@@ -93,14 +96,14 @@ def main():
             sel = float(nc.double().mean() / X.shape[0])
             # full batch timing
             for _ in range(2):
-                ix.query(Q, cfg.k, probe=probe, n_probes=T, **hk)
+                ix.query(Q, kq, probe=probe, n_probes=T, **hk)
             torch.cuda.synchronize()
             t2 = time.time()
-            ix.query(Q, cfg.k, probe=probe, n_probes=T, timing=True, **hk)
+            ix.query(Q, kq, probe=probe, n_probes=T, timing=True, **hk)
             torch.cuda.synchronize()
             dt = time.time() - t2
             st = ix.stats()
-            row = dict(W_mult=wm, W=W, T=T, recall10=float(hit), selectivity=sel, ceiling=ceiling,
+            row = dict(L=a.L, k=kq, W_mult=wm, W=W, T=T, recall10=float(hit), selectivity=sel, ceiling=ceiling,
                        qps=Q.shape[0] / dt, ms=dt * 1e3, sl_ms=st.ms_shortlist, probe_ms=st.ms_probe,
                        mean_cand=float(st.total_cand) / Q.shape[0], build_s=bt,
                        sl_gbs=st.shortlist_bytes / (st.ms_shortlist * 1e-3) / 1e9 if st.ms_shortlist > 0 else 0)
