@@ -996,6 +996,13 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
     int32_t roots[240 * 8];
     orc_e8_roots(roots);
     int32_t *ring2 = NULL;           /* recursive E8 probing (R26) */
+    /* R33 ("If the number of candidates computed is not enough, we
+     * recursively probe the adjacent buckets of the 240 probed buckets"): with
+     * min_cand = tau > 0 and no hierarchy, the second-ring probes 241..T-1 of
+     * the lattice sequence are taken one by one, in sequence order, only while
+     * the candidates of the probes before them number fewer than tau; a probe
+     * not taken is invalid (key 0, no bucket). */
+    const int e8_rec = probe == 2 && hierarchy == 0 && min_cand > 0 && M == 8 && T > 241;
     if (probe == 2 && T > 241 && M == 8) {
         ring2 = (int32_t *)malloc(sizeof(int32_t) * 8 * ORC_E8_S2);
         orc_e8_second_ring(ring2);
@@ -1093,6 +1100,8 @@ static int orc_query_impl(orc_index *ix, const float *Q, int64_t nq, int k, int 
                     if (!(f >= lo && f <= hi)) valid = 0;
                     else pc[i] = (int32_t)f;
                 }
+            } else if (e8_rec && p > 240 && base >= min_cand) {
+                valid = 0;      /* R33: enough candidates, the recursion stops */
             } else {
                 /* E8: home c, then c + r for the selected roots */
                 valid = ok;
