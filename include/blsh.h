@@ -99,7 +99,12 @@ typedef struct {
                                bits with the keys before/after its insertion position also takes the leaf's
                                buckets that share those bits with it                                         */
     int32_t hier_step_bits; /* key bits cleared per widening step: 0 = M (one Eq. 8 level), or 1..M           */
-    int64_t min_cand;       /* tau (R18); 0 = lower median of the base counts of this batch           */
+    int64_t min_cand;       /* tau (R18); 0 = lower median of the base counts of this batch.         
+                               probe = 2 (E8, M = 8) with hierarchy = 0 and min_cand > 0: recursive lattice
+                               probing ("if the number of candidates computed is not enough, we
+                               recursively probe the adjacent buckets of the 240 probed buckets", R33): the
+                               second-ring probes 241..n_probes-1 are taken in order only while the probes
+                               before them hold < min_cand candidates (not taken: Q_PVALID 0); needs L = 1  */
     void*   stream;         /* cudaStream_t                                                                   */
     int32_t keep_stages;    /* 1 = keep per-query stages of this call for blsh_export                         */
     int32_t timing;         /* 1 = record per-stage CUDA-event times into blsh_last_stats                     */
@@ -141,6 +146,24 @@ blsh_status blsh_build(const float* X, int64_t n, int32_t d, const blsh_build_pa
 blsh_status blsh_query(const blsh_index* idx, const float* Q, int64_t nq, int32_t k,
                        const blsh_query_params* p, int64_t* out_ids, float* out_dist2,
                        int64_t* out_ncand);
+
+/* a1-a5 over a stream of n_batches independent HOST batches (serving form of
+ * blsh_query; the same problem statement, per batch): batch b is
+ * Q[b] [nq x d] fp32 in host memory, its answers go to out_ids[b] [nq x k],
+ * out_dist2[b] [nq x k] and out_ncand[b] [nq] (may be NULL) in host memory.
+ * Results equal n_batches separate blsh_query calls (every batch-level
+ * statistic, e.g. the hierarchy's median tau R18, is taken per batch).  The
+ * library uploads batch b+1 and downloads batch b-1 on its own copy stream
+ * while batch b is searched on p->stream (two device staging buffers for the
+ * queries and for the answers), so with page-locked host buffers the copies
+ * overlap the search.  Pointers in the arrays may repeat (e.g. one host batch
+ * searched n_batches times); an output buffer is overwritten in batch order.
+ * Host buffers only (BLSH_ERR_INVALID for device pointers); returns after
+ * every copy has completed. */
+blsh_status blsh_query_pipelined(const blsh_index* idx, int32_t n_batches, const float* const* Q,
+                                 int64_t nq, int32_t k, const blsh_query_params* p,
+                                 int64_t* const* out_ids, float* const* out_dist2,
+                                 int64_t* const* out_ncand);
 
 /* Multi-GPU form of blsh_query: each row is k packed u64 entries
  * (float_bits(d^2) << 32) | id32, ascending; padding = 0x7F800000FFFFFFFF.

@@ -89,6 +89,8 @@ def lib():
         L.blsh_build.restype = i32
         L.blsh_query.argtypes = [P, P, i64, i32, C.POINTER(QueryParams), P, P, P]
         L.blsh_query.restype = i32
+        L.blsh_query_pipelined.argtypes = [P, i32, P, i64, i32, C.POINTER(QueryParams), P, P, P]
+        L.blsh_query_pipelined.restype = i32
         L.blsh_query_packed.argtypes = [P, P, i64, i32, C.POINTER(QueryParams), P, P]
         L.blsh_query_packed.restype = i32
         L.blsh_query_base_counts.argtypes = [P, P, i64, C.POINTER(QueryParams), P]
@@ -110,6 +112,7 @@ def lib():
 
 
 EXPORTED_SYMBOLS = ("blsh_build_params_default", "blsh_query_params_default", "blsh_build", "blsh_query",
+                    "blsh_query_pipelined",
                     "blsh_query_packed", "blsh_query_base_counts", "blsh_merge_topk", "blsh_export", "blsh_index_info",
                     "blsh_last_stats", "blsh_free", "blsh_last_error")
 
@@ -228,6 +231,41 @@ def blsh_query(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hie
     return ids, d2, nc
 
 
+def blsh_query_pipelined(index: "Index", Qs, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
+                         hier_step_bits: int = 0, min_cand: int = 0, timing: bool = False, outs=None,
+                         global_base=None, curve_perturb: int = 0, msb_min: int = 0):
+    """Qs: a list of HOST batches [nq, d] (equal nq; entries may repeat).  -> list of
+    (ids, dist2, ncand) host arrays, one per batch (``outs`` supplies them; entries may repeat)."""
+    Qs = [_f32(Q) for Q in Qs]
+    nb = len(Qs)
+    if nb == 0:
+        return []
+    nq = int(Qs[0].shape[0])
+    if any(int(Q.shape[0]) != nq for Q in Qs):
+        raise ValueError("every batch must have the same number of queries")
+    if outs is None:
+        outs = [(_alloc_like(Q, (nq, k), "i64"), _alloc_like(Q, (nq, k), "f32"), _alloc_like(Q, (nq,), "i64"))
+                for Q in Qs]
+    p = _qparams(probe, n_probes, hierarchy, hier_step_bits, min_cand, False, timing, C.c_void_p(0),
+                 global_base, curve_perturb, msb_min)
+    keep = []
+
+    def arr(items):
+        ptrs = []
+        for a in items:
+            ptr, ka, _ = _ptr(a)
+            keep.append(ka)
+            ptrs.append(ptr.value if ptr is not None else None)
+        return (C.c_void_p * nb)(*ptrs)
+
+    qa = arr(Qs)
+    ia = arr([o[0] for o in outs])
+    da = arr([o[1] for o in outs])
+    na = arr([o[2] for o in outs])
+    _check(lib().blsh_query_pipelined(index.handle, nb, qa, nq, k, C.byref(p), ia, da, na))
+    return outs
+
+
 def blsh_query_packed(index: "Index", Q, k: int, probe: int = 0, n_probes: int = 1, hierarchy: int = 0,
                       hier_step_bits: int = 0, min_cand: int = 0, timing: bool = False, out=None,
                       global_base=None, curve_perturb: int = 0, msb_min: int = 0):
@@ -322,6 +360,9 @@ class Index:
 
     def query(self, Q, k, **kw):
         return blsh_query(self, Q, k, **kw)
+
+    def query_pipelined(self, Qs, k, **kw):
+        return blsh_query_pipelined(self, Qs, k, **kw)
 
     def query_packed(self, Q, k, **kw):
         return blsh_query_packed(self, Q, k, **kw)

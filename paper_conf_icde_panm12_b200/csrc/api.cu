@@ -433,6 +433,70 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     if (med) ix.stats.tau = tau;
 }
 
+// Serving form (include/blsh.h blsh_query_pipelined): batch b is searched on p.stream from device
+// staging buffer b % 2 while the copy stream uploads batch b + 1 into the other buffer and then
+// downloads batch b - 1's answers.  Every batch is one run_query call on device memory, so the
+// answers are those of separate blsh_query calls.  Ordering (events):
+//   up[i]   on copy, after the upload of a batch into pl_q[i]    -> the search of that batch waits
+//   free[i] on s,    after the search of a batch in slot i        -> the download of its answers waits
+//   dl[i]   on copy, after the download of slot i's answers       -> the search two batches later waits
+// The upload of batch b + 2 into slot i is queued on the copy stream after the download of batch b
+// (slot i), which itself waits for free[i]: the buffer is never overwritten while in use.
+void run_query_pipelined(const blsh_index& ix, int nb, const float* const* Q, int64_t nq, int k,
+                         const blsh_query_params& p, int64_t* const* out_ids, float* const* out_d2,
+                         int64_t* const* out_ncand) {
+    cudaStream_t s = (cudaStream_t)p.stream;
+    QueryWork& w = ix.qw;
+    if (!w.copy) {
+        BLSH_CUDA(cudaStreamCreateWithFlags(&w.copy, cudaStreamNonBlocking));
+        for (int i = 0; i < 2; ++i) {
+            BLSH_CUDA(cudaEventCreateWithFlags(&w.pl_up[i], cudaEventDisableTiming));
+            BLSH_CUDA(cudaEventCreateWithFlags(&w.pl_free[i], cudaEventDisableTiming));
+            BLSH_CUDA(cudaEventCreateWithFlags(&w.pl_dl[i], cudaEventDisableTiming));
+        }
+    }
+    cudaStream_t cs = w.copy;
+    const size_t qb = (size_t)nq * ix.d * sizeof(float);
+    const size_t ib = ((size_t)nq * k * 8 + 255) & ~size_t(255);
+    const size_t db = ((size_t)nq * k * 4 + 255) & ~size_t(255);
+    const size_t cb = (size_t)nq * 8;
+    for (int i = 0; i < 2; ++i) {
+        w.pl_q[i].ensure(qb);
+        w.pl_out[i].ensure(ib + db + cb);
+    }
+    // the copy stream starts after everything already queued on s (earlier users of the buffers)
+    BLSH_CUDA(cudaEventRecord(w.pl_free[0], s));
+    BLSH_CUDA(cudaStreamWaitEvent(cs, w.pl_free[0], 0));
+    auto upload = [&](int b) {
+        const int i = b & 1;
+        BLSH_CUDA(cudaMemcpyAsync(w.pl_q[i].p, Q[b], qb, cudaMemcpyHostToDevice, cs));
+        BLSH_CUDA(cudaEventRecord(w.pl_up[i], cs));
+    };
+    upload(0);
+    int launches = 0;
+    for (int b = 0; b < nb; ++b) {
+        const int i = b & 1;
+        if (b + 1 < nb) upload(b + 1);
+        BLSH_CUDA(cudaStreamWaitEvent(s, w.pl_up[i], 0));
+        if (b >= 2) BLSH_CUDA(cudaStreamWaitEvent(s, w.pl_dl[i], 0));
+        char* ob = w.pl_out[i].as<char>();
+        int64_t* di = reinterpret_cast<int64_t*>(ob);
+        float* dd = reinterpret_cast<float*>(ob + ib);
+        int64_t* dn = reinterpret_cast<int64_t*>(ob + ib + db);
+        run_query(ix, w.pl_q[i].as<float>(), false, nq, k, p, di, dd, nullptr, dn, false, nullptr);
+        launches += ix.stats.launches;
+        BLSH_CUDA(cudaEventRecord(w.pl_free[i], s));
+        BLSH_CUDA(cudaStreamWaitEvent(cs, w.pl_free[i], 0));
+        BLSH_CUDA(cudaMemcpyAsync(out_ids[b], di, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, cs));
+        BLSH_CUDA(cudaMemcpyAsync(out_d2[b], dd, (size_t)nq * k * 4, cudaMemcpyDeviceToHost, cs));
+        if (out_ncand && out_ncand[b]) BLSH_CUDA(cudaMemcpyAsync(out_ncand[b], dn, cb, cudaMemcpyDeviceToHost, cs));
+        BLSH_CUDA(cudaEventRecord(w.pl_dl[i], cs));
+    }
+    BLSH_CUDA(cudaStreamSynchronize(cs));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    ix.stats.launches = launches;   // all batches' kernel launches (the other stats: the last batch)
+}
+
 static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
                            const blsh_query_params& p, int64_t* out_ids, float* out_d2,
                            unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base) {
@@ -553,6 +617,7 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi;
     a.probe = p.probe; a.T = T; a.hstep = p.hier_step_bits > 0 ? p.hier_step_bits : M;
     a.cperturb = p.probe == 3 ? p.curve_perturb : 0; a.msb_min = p.msb_min;
+    a.rec_tau = (p.probe == 2 && p.hierarchy == 0 && p.min_cand > 0) ? p.min_cand : 0;   // R33
     {
         const char* rh = std::getenv("BLSH_RH_STAGE");   // ablation: 1 = stage query rows in shared memory
         a.rh_direct = (rh && rh[0] == '1') ? 0 : 1;
@@ -814,6 +879,9 @@ blsh_status check_query(const blsh_index* idx, const float* Q, int64_t nq, int32
             return fail(BLSH_ERR_INVALID, "batch-median tau on a sharded index needs p->global_base "
                                           "(blsh_query_base_counts summed over ranks) or an explicit min_cand");
     }
+    if (p->min_cand < 0) return fail(BLSH_ERR_INVALID, "min_cand must be >= 0");
+    if (p->probe == 2 && p->hierarchy == 0 && p->min_cand > 0 && idx->L > 1)
+        return fail(BLSH_ERR_UNSUPPORTED, "recursive lattice probing (min_cand without hierarchy, R33) needs L = 1");
     if (p->global_base && !is_device_ptr(p->global_base)) return fail(BLSH_ERR_INVALID, "global_base must be device memory");
     return BLSH_OK;
 }
@@ -833,6 +901,25 @@ blsh_status blsh_query(const blsh_index* idx, const float* Q, int64_t nq, int32_
     if (o_host != !is_device_ptr(out_dist2) || (out_ncand && o_host != !is_device_ptr(out_ncand)))
         return fail(BLSH_ERR_INVALID, "outputs must all be host or all be device memory");
     return guarded([&] { blsh::run_query(*idx, Q, q_host, nq, k, *p, out_ids, out_dist2, nullptr, out_ncand, o_host, nullptr); });
+}
+
+blsh_status blsh_query_pipelined(const blsh_index* idx, int32_t n_batches, const float* const* Q, int64_t nq, int32_t k,
+                                 const blsh_query_params* p, int64_t* const* out_ids, float* const* out_dist2,
+                                 int64_t* const* out_ncand) {
+    if (n_batches < 0) return fail(BLSH_ERR_INVALID, "n_batches must be >= 0");
+    if (n_batches == 0) return BLSH_OK;
+    if (!Q || !out_ids || !out_dist2) return fail(BLSH_ERR_INVALID, "pointer arrays are NULL");
+    for (int32_t b = 0; b < n_batches; ++b) {
+        blsh_status c = check_query(idx, Q[b], nq, k, p);
+        if (c != BLSH_OK) return c;
+        if (nq == 0) continue;
+        if (!out_ids[b] || !out_dist2[b]) return fail(BLSH_ERR_INVALID, "outputs are NULL");
+        if (is_device_ptr(Q[b]) || is_device_ptr(out_ids[b]) || is_device_ptr(out_dist2[b]) ||
+            (out_ncand && out_ncand[b] && is_device_ptr(out_ncand[b])))
+            return fail(BLSH_ERR_INVALID, "blsh_query_pipelined takes host buffers only");
+    }
+    if (nq == 0) return BLSH_OK;
+    return guarded([&] { blsh::run_query_pipelined(*idx, n_batches, Q, nq, k, *p, out_ids, out_dist2, out_ncand); });
 }
 
 blsh_status blsh_query_packed(const blsh_index* idx, const float* Q, int64_t nq, int32_t k, const blsh_query_params* p,

@@ -130,6 +130,10 @@ struct QueryWork {
     ScanTemp scan2;
     cudaStream_t side = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    // blsh_query_pipelined: double-buffered query uploads / answer downloads on a copy stream
+    DevBuf pl_q[2], pl_out[2];
+    cudaStream_t copy = nullptr;
+    cudaEvent_t pl_up[2] = {nullptr, nullptr}, pl_free[2] = {nullptr, nullptr}, pl_dl[2] = {nullptr, nullptr};
     QueryWork() = default;
     QueryWork(const QueryWork&) = delete;
     QueryWork& operator=(const QueryWork&) = delete;
@@ -137,6 +141,12 @@ struct QueryWork {
         if (ev_fork) cudaEventDestroy(ev_fork);
         if (ev_join) cudaEventDestroy(ev_join);
         if (side) cudaStreamDestroy(side);
+        for (int i = 0; i < 2; ++i) {
+            if (pl_up[i]) cudaEventDestroy(pl_up[i]);
+            if (pl_free[i]) cudaEventDestroy(pl_free[i]);
+            if (pl_dl[i]) cudaEventDestroy(pl_dl[i]);
+        }
+        if (copy) cudaStreamDestroy(copy);
     }
 };
 
@@ -266,6 +276,10 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
                const blsh_query_params& p, int64_t* out_ids, float* out_d2,
                unsigned long long* out_packed, int64_t* out_ncand, bool out_host,
                int64_t* out_base);   // non-NULL: stop after a4 and write |A0(q)| (blsh_query_base_counts)
+// blsh_query_pipelined: n_batches host batches, uploads/downloads overlapped with the search
+void run_query_pipelined(const blsh_index& ix, int nb, const float* const* Q, int64_t nq, int k,
+                         const blsh_query_params& p, int64_t* const* out_ids, float* const* out_d2,
+                         int64_t* const* out_ncand);
 
 void merge_lists(const unsigned long long* packed, int n_lists, int64_t nq, int k,
                  int64_t* out_ids, float* out_d2, cudaStream_t s);

@@ -228,6 +228,14 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
         else warp_select(sm, 480u, 0xFFFFFFFFu, T - 1, [&](uint32_t x) { return lat2_score(t, code, x); });
     }
     int64_t mysum = 0;
+    // R33 ("if the number of candidates computed is not enough, we recursively probe the
+    // adjacent buckets of the 240 probed buckets"): with rec_tau > 0 the second-ring probes
+    // p = 241..T-1 (T <= 256: the last lane-strided round, lane = p - 224) are looked up first and
+    // decided after the loop: probe p is taken iff the probes before it hold < rec_tau candidates.
+    const bool rec = a.rec_tau > 0 && M == 8 && T > 241;
+    Key128 rk{0, 0};
+    uint2 riv = make_uint2(0, 0);
+    bool rvalid = false, rpend = false;
     for (int p = lane; p < T; p += 32) {
         int32_t pc[16];
         bool valid = !(oor & 1);
@@ -261,11 +269,38 @@ __device__ int64_t probe_e8(const QueryArgs& a, ProbeSmem& sm, int64_t q, int la
             const int64_t u = find_bucket(a.ukey, ulo, uhi, k);
             if (u >= 0) iv = make_uint2(a.uoff[u], a.uoff[u + 1]);
         }
+        if (rec && p > 240) {   // decided below
+            rk = k; riv = iv; rvalid = valid; rpend = true;
+            continue;
+        }
         ivl[p] = iv;
         mysum += (int64_t)(iv.y - iv.x);
         if (a.pkey) {
             a.pkey[(size_t)q * T + p] = k;
             a.pvalid[(size_t)q * T + p] = valid ? 1 : 0;
+        }
+    }
+    if (rec) {
+        int64_t before = mysum;                       // probes 0..240: every lane's sum
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) before += __shfl_xor_sync(BLSH_FULL, before, o);
+        const int64_t sz = rpend ? (int64_t)(riv.y - riv.x) : 0;
+        int64_t inc = sz;                             // inclusive scan over lanes = ring probes in order
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int64_t v = __shfl_up_sync(BLSH_FULL, inc, o);
+            if (lane >= o) inc += v;
+        }
+        if (rpend) {
+            const int p = lane + 224;
+            const bool take = before + (inc - sz) < a.rec_tau;
+            const uint2 iv = take ? riv : make_uint2(0, 0);
+            ivl[p] = iv;
+            mysum += (int64_t)(iv.y - iv.x);
+            if (a.pkey) {
+                a.pkey[(size_t)q * T + p] = take && rvalid ? rk : Key128{0, 0};
+                a.pvalid[(size_t)q * T + p] = take && rvalid ? 1 : 0;
+            }
         }
     }
     return mysum;

@@ -804,7 +804,11 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     const int nlist = use_f16 ? kSxEpiN : 4;   // buffered-pair lists per (item, query): the screen's epilogue warps
     const bool large_k = k > 64;               // fp16 screen + exact keys per query + launch_select
     // large k: each warp's list holds ~kk = ceil(k/8) survivors (+ the bound's slack)
-    const int scapw = large_k ? ((2 * ((k + kSxEpiN - 1) / kSxEpiN) + 64 + 15) / 16) * 16 : kTcScap;
+    static const int scap_small = [] {   // BLSH_SCAPW (experiments): buffered pairs per list for k <= 64
+        const char* e = std::getenv("BLSH_SCAPW");
+        return e ? std::max(32, std::atoi(e) / 16 * 16) : kTcScap;
+    }();
+    const int scapw = large_k ? ((2 * ((k + kSxEpiN - 1) / kSxEpiN) + 64 + 15) / 16) * 16 : (use_f16 ? scap_small : kTcScap);
     const int kScap = nlist * scapw;
     const size_t part_bytes = large_k ? 0 : ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);

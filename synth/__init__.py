@@ -72,27 +72,31 @@ CONFIGS = {
                  G=4, M=8, W=4.0, seed_data=1001, seed_query=2001,
                  notes="BASELINE configs[0]: CPU-oracle-in-seconds case"),
     "c2": Config("c2", n=22_000, d=512, n_clusters=64, spread=0.02, rank=16, nq=1_000, k=50,
-                 G=16, M=8, W=1.6, seed_data=1002, seed_query=2002,
-                 notes="BASELINE configs[1]: LabelMe-shaped, standard LSH per subgroup"),
+                 G=4, M=8, W=7.03, L=4, seed_data=1002, seed_query=2002,
+                 notes="BASELINE configs[1]: LabelMe-shaped, standard LSH per subgroup (L = 4 tables); "
+                       "G = 4, W = 16 r10 (calibrated r02ai: recall@10 0.953, leaf ceiling 0.963)"),
     "c3": Config("c3", n=1_000_000, d=384, n_clusters=256, spread=0.02, rank=16, nq=10_000,
-                 k=50, G=16, M=8, W=1.2, probe=1, T=16, hierarchy=1, min_cand=0, zipf=0.8,
+                 k=50, G=8, M=8, W=2.41, probe=1, T=16, hierarchy=1, min_cand=0, zipf=0.8,
                  between=0.05, backend="torch", seed_data=1003, seed_query=2003,
-                 notes="BASELINE configs[2]: Tiny-Images-shaped, multiprobe + Morton hierarchy"),
+                 notes="BASELINE configs[2]: Tiny-Images-shaped, multiprobe + Morton hierarchy; "
+                       "G = 8, W = 8 r10 (calibrated r02ah: recall@10 0.922, leaf ceiling 0.935)"),
     "c4": Config("c4", n=10_000_000, d=384, n_clusters=1024, spread=0.02, rank=16,
-                 nq=100_000, k=10, G=64, M=8, W=1.65, probe=1, T=32, backend="torch",
+                 nq=100_000, k=10, G=64, M=8, W=2.33, probe=1, T=16, backend="torch",
                  seed_data=1004, seed_query=2004,
-                 notes="BASELINE configs[3]: 10M x 384 sharded by subgroup, NCCL top-k merge"),
+                 notes="BASELINE configs[3]: 10M x 384 sharded by subgroup, NCCL top-k merge; "
+                       "W = 8 r10, T = 16 (recalibrated r02ai under the fp16 screen: recall@10 0.930)"),
     "c5": Config("c5", n=1_000_000, d=384, n_clusters=256, spread=0.02, rank=16, nq=100_000,
-                 k=10, G=16, M=8, W=1.2, probe=1, T=16, backend="torch",
+                 k=10, G=16, M=8, W=2.51, probe=1, T=16, backend="torch",
                  seed_data=1005, seed_query=2005,
                  notes="BASELINE configs[4]: sweep base (probes 1-64, lattice vs multiprobe, batch)"),
     # The paper's own evaluation setting: 100,000 items hashed, another
     # 100,000 items of the same distribution as queries, L = 10 tables, M = 8,
     # k = 500 (Tiny-Images-shaped 384-d data).
     "p217": Config("p217", n=100_000, d=384, n_clusters=64, spread=0.02, rank=16, nq=100_000,
-                   k=500, G=16, M=8, W=1.2, probe=0, T=1, L=10, backend="torch",
+                   k=500, G=16, M=8, W=1.90, probe=0, T=1, L=10, backend="torch",
                    seed_data=1006, seed_query=2006,
-                   notes="P:217 evaluation setting: L = 10, M = 8, k = 500, 100k items / 100k queries"),
+                   notes="P:217 evaluation setting: L = 10, M = 8, k = 500, 100k items / 100k queries; "
+                         "W = 5.66 r10 (calibrated r02aj: recall@10 0.911, leaf ceiling 0.937)"),
 }
 
 

@@ -308,9 +308,14 @@ def test_c2_full(blsh, orc):
     """BASELINE configs[1] at full size: LabelMe-shaped 22k x 512, 1000 queries, k = 50."""
     cfg = synth.CONFIGS["c2"]
     X, Q = synth.make_dataset(cfg)
-    ix, ox = build_pair(blsh, orc, X, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
-    compare_build(ix, ox)
-    run_query_pair(ix, ox, X, Q, cfg.k)
+    if cfg.L == 1:
+        ix, ox = build_pair(blsh, orc, X, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
+        compare_build(ix, ox)
+        run_query_pair(ix, ox, X, Q, cfg.k)
+    else:   # standard LSH with L tables per subgroup (P:43, R24): the L-table parity helpers
+        import test_gpu_tables as tt
+        ix, ox = tt.build_pair(blsh, orc, X, cfg.L, G=cfg.G, M=cfg.M, W=cfg.W, seed=cfg.seed_index)
+        tt.run_pair(ix, ox, X, Q, cfg.k, cfg.L, probe=cfg.probe, T=cfg.T)
 
 
 def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
