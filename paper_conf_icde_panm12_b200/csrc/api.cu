@@ -376,7 +376,7 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
     int64_t* nc_c = ar.take<int64_t>(nq);
     QueryArgs a{};
     a.nq = nq; a.d = ix.d; a.ds = ds; a.G = G; a.M = ix.M; a.B = ix.B; a.depth = ix.depth;
-    a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi; a.rh_direct = 1;
+    a.quantizer = ix.quantizer; a.leaf_lo = ix.leaf_lo; a.leaf_hi = ix.leaf_hi;
     a.Q = Qdev; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
     a.ntype = ix.ntype.as<int32_t>(); a.qleaf = qleaf; a.lperm = lperm; a.lcnt = lcnt;
     launches += launch_route_group(a, s);
@@ -618,10 +618,6 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     a.probe = p.probe; a.T = T; a.hstep = p.hier_step_bits > 0 ? p.hier_step_bits : M;
     a.cperturb = p.probe == 3 ? p.curve_perturb : 0; a.msb_min = p.msb_min;
     a.rec_tau = (p.probe == 2 && p.hierarchy == 0 && p.min_cand > 0) ? p.min_cand : 0;   // R33
-    {
-        const char* rh = std::getenv("BLSH_RH_STAGE");   // ablation: 1 = stage query rows in shared memory
-        a.rh_direct = (rh && rh[0] == '1') ? 0 : 1;
-    }
     a.Q = Qdev; a.dirs = ix.dirs.as<float>(); a.mu = ix.mu.as<float>(); a.theta = ix.theta.as<float>();
     a.ntype = ix.ntype.as<int32_t>(); a.A = ix.A.as<float>(); a.bvec = ix.b.as<float>(); a.Wl = ix.W.as<float>();
     a.ukey = ix.ukey.as<Key128>(); a.uoff = ix.uoff.as<uint32_t>(); a.leaf_u = ix.leaf_u.as<int64_t>();

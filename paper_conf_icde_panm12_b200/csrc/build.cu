@@ -12,7 +12,6 @@ namespace blsh {
 namespace {
 
 constexpr int kTR = 256;
-constexpr int kDC = 32;
 
 struct HTile {
     int32_t leaf;
@@ -20,8 +19,10 @@ struct HTile {
     int64_t start;   // position in `order`
 };
 
-// One thread per row: M canonical fp32 chains against the leaf's a_i (R1),
-// then t_i = (dot + b_i) / W, quantise, Morton key.
+// One lane per row, 32 rows per warp, a tile of <= 256 rows of one leaf per block: the
+// leaf's a_i in shared memory (pitch ds, broadcast 16-byte reads), the rows streamed as
+// 32-column chunks staged by coalesced 16-byte loads (ChunkStager); M canonical fp32
+// chains per lane (R1), then t_i = (dot + b_i) / W, quantise, Morton key.
 template <int MM>
 __global__ void __launch_bounds__(kTR) k_hash_rows(const float* __restrict__ Xs, int ds, int d,
                                                    const uint32_t* __restrict__ order,
@@ -32,38 +33,57 @@ __global__ void __launch_bounds__(kTR) k_hash_rows(const float* __restrict__ Xs,
                                                    unsigned long long* __restrict__ key_lo,
                                                    uint32_t* __restrict__ leaf_o, uint32_t* __restrict__ id_o,
                                                    int32_t* __restrict__ code_out, int* __restrict__ bad) {
-    __shared__ float xs[kTR][kDC + 1];
-    __shared__ float as_[MM][kDC];
-    __shared__ uint32_t rid[kTR];
+    extern __shared__ __align__(16) float hsm[];
+    float* as_ = hsm;                                               // [MM][ds]
+    float* tile = hsm + (size_t)MM * ds + (size_t)(threadIdx.x >> 5) * 32 * kRowPitch;
     const HTile t = tiles[blockIdx.x];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int r = threadIdx.x;
-    if (r < t.len) rid[r] = order[t.start + r];
     const float* Ag = A + (size_t)t.leaf * MM * d;
+    for (int i = threadIdx.x; i < MM * d; i += kTR) {
+        const int ii = i / d, jj = i - ii * d;
+        as_[(size_t)ii * ds + jj] = __ldg(Ag + i);
+    }
     __syncthreads();
+    const int r0 = warp * 32;
+    if (r0 >= t.len) return;
+    const int nrow = min(32, t.len - r0);
+    const uint32_t* rid = order + t.start + r0;
+    auto qid = [&](int r) { return (int64_t)rid[r]; };
     float s[MM];
 #pragma unroll
     for (int i = 0; i < MM; ++i) s[i] = 0.0f;
-    for (int dc = 0; dc < d; dc += kDC) {
-        const int w = min(kDC, d - dc);
-#pragma unroll 4
-        for (int rr = warp; rr < t.len; rr += kTR / 32)
-            if (lane < w) xs[rr][lane] = Xs[(size_t)rid[rr] * ds + dc + lane];
-        for (int i = threadIdx.x; i < MM * kDC; i += kTR) {
-            const int ii = i / kDC, jj = i % kDC;
-            if (jj < w) as_[ii][jj] = Ag[(size_t)ii * d + dc + jj];
-        }
-        __syncthreads();
-        if (r < t.len) {
-            for (int jj = 0; jj < w; ++jj) {
-                const float x = xs[r][jj];
+    ChunkStager cst;
+    cst.load(Xs, ds, qid, nrow, 0, lane);
+    for (int j0 = 0; j0 < d; j0 += 32) {
+        cst.store(tile, lane);
+        __syncwarp();
+        if (j0 + 32 < d) cst.load(Xs, ds, qid, nrow, j0 + 32, lane);   // in flight during this chunk
+        const int jn = min(32, d - j0);
+        const float* xr = tile + lane * kRowPitch;
+        if (jn == 32) {
+#pragma unroll 2
+            for (int jj = 0; jj < 32; jj += 4) {
+                const float4 x = *reinterpret_cast<const float4*>(xr + jj);
 #pragma unroll
-                for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(as_[i][jj], x, s[i]);
+                for (int i = 0; i < MM; ++i) {
+                    const float4 w = *reinterpret_cast<const float4*>(as_ + (size_t)i * ds + j0 + jj);
+                    s[i] = __fmaf_rn(w.x, x.x, s[i]);
+                    s[i] = __fmaf_rn(w.y, x.y, s[i]);
+                    s[i] = __fmaf_rn(w.z, x.z, s[i]);
+                    s[i] = __fmaf_rn(w.w, x.w, s[i]);
+                }
+            }
+        } else {
+            for (int jj = 0; jj < jn; ++jj) {
+                const float x = xr[jj];
+#pragma unroll
+                for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(as_[(size_t)i * ds + j0 + jj], x, s[i]);
             }
         }
-        __syncthreads();
+        __syncwarp();
     }
-    if (r >= t.len) return;
+    if (lane >= nrow) return;
+    const int r = r0 + lane;
     const float W = Wl[t.leaf];
     float tv[MM];
 #pragma unroll
@@ -73,7 +93,7 @@ __global__ void __launch_bounds__(kTR) k_hash_rows(const float* __restrict__ Xs,
     if (!ok) atomicOr(bad, 1);
     const Key128 k = morton_key(code, MM, B);
     const int64_t o = t.start + r - pos_lo;
-    const uint32_t id = rid[r];
+    const uint32_t id = rid[lane];
     key_hi[o] = k.hi;
     key_lo[o] = k.lo;
     leaf_o[o] = (uint32_t)t.leaf;
@@ -206,9 +226,11 @@ bool hash_points(const blsh_index& ix, const float* Xs, const uint32_t* order, c
     bad_d.alloc(sizeof(int));
     BLSH_CUDA(cudaMemsetAsync(bad_d.p, 0, sizeof(int), s));
     const unsigned nt = (unsigned)tiles.size();
+    const size_t hsmem = ((size_t)ix.M * ix.ds + (size_t)(kTR / 32) * 32 * kRowPitch) * sizeof(float);
 #define BLSH_HASH_CASE(MMV)                                                                                    \
     case MMV:                                                                                                  \
-        k_hash_rows<MMV><<<nt, kTR, 0, s>>>(Xs, ix.ds, ix.d, order, tiles_d.as<HTile>(), pos_lo,              \
+        BLSH_CUDA(cudaFuncSetAttribute(k_hash_rows<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem)); \
+        k_hash_rows<MMV><<<nt, kTR, hsmem, s>>>(Xs, ix.ds, ix.d, order, tiles_d.as<HTile>(), pos_lo,              \
                                             A, b, ix.W.as<float>(), ix.B,                                     \
                                             ix.quantizer, key_hi, key_lo, leaf, id, code_out, bad_d.as<int>()); \
         break;

@@ -92,4 +92,31 @@ __device__ __forceinline__ bool quantise(const float* t, int M, int B, int quant
     return ok;
 }
 
+// A warp's [32 rows x 32 columns] chunks of fp32 rows (row pitch ds floats, ds % 4 == 0),
+// staged through registers into shared memory tile[r * kRowPitch + c]: coalesced 16-byte
+// loads (8 lanes per row's 128-byte chunk, 4 rows per instruction), rows qid(0..nrow-1),
+// zeros beyond.  load(j0) issues the 8 loads of chunk j0 into registers (the next chunk's
+// loads are in flight while the current one is consumed), store() writes them to the tile.
+// Read back by lane = row, the 16-byte reads of 8 lanes fall in distinct bank groups (pitch 36).
+constexpr int kRowPitch = 36;
+struct ChunkStager {
+    float4 v[8];
+    template <class QID>
+    __device__ __forceinline__ void load(const float* __restrict__ Q, int ds, QID qid, int nrow, int j0, int lane) {
+        const int c4 = lane & 7, rr = lane >> 3;
+        const int col = j0 + 4 * c4;
+#pragma unroll
+        for (int r4 = 0; r4 < 8; ++r4) {
+            const int r = 4 * r4 + rr;
+            v[r4] = (r < nrow && col < ds) ? __ldg(reinterpret_cast<const float4*>(Q + (size_t)qid(r) * ds + col))
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+    }
+    __device__ __forceinline__ void store(float* tile, int lane) const {
+        const int c4 = lane & 7, rr = lane >> 3;
+#pragma unroll
+        for (int r4 = 0; r4 < 8; ++r4) *reinterpret_cast<float4*>(tile + (4 * r4 + rr) * kRowPitch + 4 * c4) = v[r4];
+    }
+};
+
 }  // namespace blsh

@@ -26,80 +26,112 @@ namespace {
 // ---------------------------------------------------------------------------
 // a1 + a2
 // ---------------------------------------------------------------------------
-// a1 and a2 run as two passes so that the projection reads its leaf's M x d
-// matrix from shared memory:
-//   k_route       one warp per block, one query per lane: the 32 query rows are
-//                 staged into shared memory with coalesced 16-byte loads (row
-//                 pitch ds + 4 floats, so the lanes' 16-byte reads at the same
-//                 column fall into distinct bank groups); each lane descends the
-//                 tree with its query's canonical chains (R1: strictly ascending
-//                 j, explicit fmaf), node vectors through L1; leaf histogram.
+// Both passes read the query rows as 32-column chunks of 32 rows per warp, staged in
+// shared memory with coalesced 16-byte loads (each row's 128-byte chunk is one line) and
+// read back by lane = query (row pitch 36 floats: the 16-byte reads of 8 lanes fall in
+// distinct bank groups).  A lane's chains stay canonical (R1: one fmaf per column, j
+// strictly ascending from 0.0f); the chunking only changes where x_j comes from.
+//   k_route       ceil(depth / 3) passes; a pass evaluates the <= 7 nodes of the
+//                 3-level subtree below the lane's current node (independent chains:
+//                 the FMA latency is hidden, the rows are read ceil(depth / 3) times
+//                 instead of depth times), then descends 3 levels; leaf histogram.
 //   k_leaf_scan / k_leaf_scatter   group the queries by leaf (lperm).
-//   k_hash        32 leaf-grouped queries per block; the block's leaf matrix A_g
-//                 is staged in shared memory (broadcast reads), the rows again;
-//                 each lane runs its M projection chains, Eq. 2 / E8, Morton key.
-constexpr int kRHQ = 32;
-
-__device__ __forceinline__ void stage_rows(const QueryArgs& a, float4* rows4, const uint32_t* qids, int64_t q0,
-                                           int nrow, int lane) {
-    const int nv4 = a.ds >> 2, pitch4 = nv4 + 1;
-    for (int r = 0; r < nrow; ++r) {
-        const int64_t q = qids ? (int64_t)qids[q0 + r] : q0 + r;
-        for (int v = lane; v < nv4; v += 32)
-            rows4[r * pitch4 + v] = __ldg(reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds) + v);
-    }
-}
+//   k_hash        128 leaf-grouped queries per block; the leaf matrix A_g of the
+//                 block's first query is staged in shared memory (pitch ds, broadcast
+//                 reads); each lane runs its M projection chains, Eq. 2 / E8, Morton key.
+constexpr int kRHW = 4;              // warps per block (32 queries each)
+constexpr int kRHQ = 32 * kRHW;      // queries per block
+constexpr int kRHP = kRowPitch;      // staged chunk row pitch (floats, hashcore.cuh)
 
 __global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict__ lcnt) {
-    extern __shared__ __align__(16) float rh_rows[];
-    const int lane = threadIdx.x;
-    const int64_t q0 = blockIdx.x * (int64_t)kRHQ;
-    const int nrow = (int)min((int64_t)kRHQ, a.nq - q0);
-    float4* rows4 = reinterpret_cast<float4*>(rh_rows);
-    if (!a.rh_direct) stage_rows(a, rows4, nullptr, q0, nrow, lane);
-    __syncwarp();
-    if (lane >= nrow) return;
-    const int64_t q = q0 + lane;
-    // rh_direct: each lane reads its own row through L1 (no staging: more blocks per SM)
-    const float4* x4 = a.rh_direct ? reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds)
-                                   : rows4 + lane * ((a.ds >> 2) + 1);
-    const int d = a.d;
-    const int nfull = d >> 2, rem = d & 3;
+    __shared__ __align__(16) float tiles[kRHW][32 * kRHP];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t q0 = blockIdx.x * (int64_t)kRHQ + warp * 32;
+    if (q0 >= a.nq) return;
+    const int nrow = (int)min((int64_t)32, a.nq - q0);
+    float* tile = tiles[warp];
+    const bool act = lane < nrow;
+    const int d = a.d, ds = a.ds;
+    auto qid = [&](int r) { return q0 + r; };
     int v = 0;
-    for (int l = 0; l < a.depth; ++l) {
-        float s = 0.0f;
-        if (a.ntype[v] == 0) {
-            const float4* dir4 = reinterpret_cast<const float4*>(a.dirs + (size_t)v * a.ds);
-#pragma unroll 4
-            for (int j4 = 0; j4 < nfull; ++j4) {
-                const float4 xv = x4[j4], dv = __ldg(dir4 + j4);
-                s = __fmaf_rn(dv.x, xv.x, s);
-                s = __fmaf_rn(dv.y, xv.y, s);
-                s = __fmaf_rn(dv.z, xv.z, s);
-                s = __fmaf_rn(dv.w, xv.w, s);
-            }
-            if (rem) {
-                const float4 xv = x4[nfull], dv = __ldg(dir4 + nfull);
-                s = __fmaf_rn(dv.x, xv.x, s);
-                if (rem > 1) s = __fmaf_rn(dv.y, xv.y, s);
-                if (rem > 2) s = __fmaf_rn(dv.z, xv.z, s);
-            }
-        } else {
-            const float4* mu4 = reinterpret_cast<const float4*>(a.mu + (size_t)v * a.ds);
-            for (int j4 = 0; j4 < (d + 3) >> 2; ++j4) {
-                const float4 xv = x4[j4], mv = __ldg(mu4 + j4);
-                const float xs[4] = {xv.x, xv.y, xv.z, xv.w}, ms[4] = {mv.x, mv.y, mv.z, mv.w};
+    for (int l0 = 0; l0 < a.depth; l0 += 3) {
+        const int nl = min(3, a.depth - l0);
+        const int nn = (1 << nl) - 1;
+        const float* vec[7];
+        bool mean[7];
+        bool anymean = false;
 #pragma unroll
-                for (int c = 0; c < 4; ++c) {
-                    if (4 * j4 + c < d) {
-                        const float e = __fsub_rn(xs[c], ms[c]);
-                        s = __fmaf_rn(e, e, s);
+        for (int i = 0; i < 7; ++i) {
+            const int ll = i == 0 ? 0 : (i < 3 ? 1 : 2);
+            const int nid = ((v + 1) << ll) - 1 + (i - ((1 << ll) - 1));   // heap order below v
+            const bool use = i < nn;
+            mean[i] = use && a.ntype[nid] != 0;
+            vec[i] = use ? (mean[i] ? a.mu : a.dirs) + (size_t)nid * ds : a.dirs;
+            anymean |= act && mean[i];
+        }
+        const bool generic = __any_sync(BLSH_FULL, anymean);
+        float s[7];
+#pragma unroll
+        for (int i = 0; i < 7; ++i) s[i] = 0.0f;
+        ChunkStager cst;
+        cst.load(a.Q, ds, qid, nrow, 0, lane);
+        for (int j0 = 0; j0 < d; j0 += 32) {
+            cst.store(tile, lane);
+            __syncwarp();
+            if (j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);   // in flight during this chunk
+            const int jn = min(32, d - j0);
+            const float* xr = tile + lane * kRHP;
+            if (!generic) {   // hyperplane nodes only: s_i = fmaf(dir_ij, x_j, s_i)
+                if (jn == 32) {
+#pragma unroll 2
+                    for (int jj = 0; jj < 32; jj += 4) {
+                        const float4 x = *reinterpret_cast<const float4*>(xr + jj);
+#pragma unroll
+                        for (int i = 0; i < 7; ++i) {
+                            if (i < nn) {
+                                const float4 w = __ldg(reinterpret_cast<const float4*>(vec[i] + j0 + jj));
+                                s[i] = __fmaf_rn(w.x, x.x, s[i]);
+                                s[i] = __fmaf_rn(w.y, x.y, s[i]);
+                                s[i] = __fmaf_rn(w.z, x.z, s[i]);
+                                s[i] = __fmaf_rn(w.w, x.w, s[i]);
+                            }
+                        }
+                    }
+                } else {
+                    for (int jj = 0; jj < jn; ++jj) {
+                        const float x = xr[jj];
+#pragma unroll
+                        for (int i = 0; i < 7; ++i)
+                            if (i < nn) s[i] = __fmaf_rn(__ldg(vec[i] + j0 + jj), x, s[i]);
+                    }
+                }
+            } else {          // some mean-rule node: s_i += (x_j - mu_ij)^2 there (R4), same j order
+                for (int jj = 0; jj < jn; ++jj) {
+                    const float x = xr[jj];
+#pragma unroll
+                    for (int i = 0; i < 7; ++i) {
+                        if (i < nn) {
+                            const float w = __ldg(vec[i] + j0 + jj);
+                            const float e = __fsub_rn(x, w);
+                            s[i] = mean[i] ? __fmaf_rn(e, e, s[i]) : __fmaf_rn(w, x, s[i]);
+                        }
                     }
                 }
             }
+            __syncwarp();
         }
-        v = 2 * v + 1 + (s > a.theta[v] ? 1 : 0);
+        int li = 0;
+        for (int ll = 0; ll < nl; ++ll) {
+            const int nid = ((v + 1) << ll) - 1 + (li - ((1 << ll) - 1));
+            float sl = s[0];
+#pragma unroll
+            for (int i = 1; i < 7; ++i) sl = i == li ? s[i] : sl;
+            li = 2 * li + 1 + (sl > a.theta[nid] ? 1 : 0);
+        }
+        v = ((v + 1) << nl) - 1 + (li - ((1 << nl) - 1));
     }
+    if (!act) return;
+    const int64_t q = q0 + lane;
     const int g = v - (a.G - 1);
     a.qleaf[q] = g;
     atomicAdd(&lcnt[g], 1);
@@ -145,40 +177,65 @@ __global__ void k_leaf_scatter(const int32_t* __restrict__ qleaf, int64_t nq, in
 }
 
 template <int MM>
-__device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __restrict__ lperm, float* rh_rows) {
-    const int lane = threadIdx.x;
-    const int64_t p0 = blockIdx.x * (int64_t)kRHQ;
-    const int nrow = (int)min((int64_t)kRHQ, a.nq - p0);
-    const int d = a.d;
-    float4* rows4 = reinterpret_cast<float4*>(rh_rows);
-    float* As = rh_rows + (a.rh_direct ? (size_t)0 : (size_t)kRHQ * (a.ds + 4));   // [MM][d] of the block's first leaf
-    const int g0 = a.qleaf[lperm[p0]];
+__device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __restrict__ lperm, float* smem) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t pb = blockIdx.x * (int64_t)kRHQ;
+    const int d = a.d, ds = a.ds;
+    float* As = smem;                                   // [MM][ds] of the block's first query's leaf
+    float* tile = smem + (size_t)MM * ds + (size_t)warp * 32 * kRHP;
+    const int g0 = a.qleaf[lperm[pb]];
     const float* Ag0 = a.A + (size_t)g0 * MM * d;
-    for (int i = lane; i < MM * d; i += 32) As[i] = __ldg(Ag0 + i);
-    if (!a.rh_direct) stage_rows(a, rows4, lperm, p0, nrow, lane);
-    __syncwarp();
-    if (lane >= nrow) return;
-    const int64_t q = lperm[p0 + lane];
-    const float4* x4 = a.rh_direct ? reinterpret_cast<const float4*>(a.Q + (size_t)q * a.ds)
-                                   : rows4 + lane * ((a.ds >> 2) + 1);
-    const int g = a.qleaf[q];
-    const bool active = g >= a.leaf_lo && g < a.leaf_hi;
-    const float* Ag = g == g0 ? As : a.A + (size_t)g * MM * d;   // generic: shared (broadcast) or global
+    for (int i = threadIdx.x; i < MM * d; i += kRHQ) {
+        const int r = i / d, c = i - r * d;
+        As[(size_t)r * ds + c] = __ldg(Ag0 + i);
+    }
+    __syncthreads();
+    const int64_t p0 = pb + warp * 32;
+    if (p0 >= a.nq) return;
+    const int nrow = (int)min((int64_t)32, a.nq - p0);
+    const bool act = lane < nrow;
+    const int64_t q = act ? lperm[p0 + lane] : 0;
+    const int g = act ? a.qleaf[q] : g0;
+    const bool shared_a = __all_sync(BLSH_FULL, g == g0);
+    const float* Ag = a.A + (size_t)g * MM * d;        // generic path: this lane's leaf, row pitch d
+    auto qid = [&](int r) { return (int64_t)lperm[p0 + r]; };
     float s[MM];
 #pragma unroll
     for (int i = 0; i < MM; ++i) s[i] = 0.0f;
-    for (int j4 = 0; j4 < (d + 3) >> 2; ++j4) {
-        const float4 xv = x4[j4];
-        const float xs[4] = {xv.x, xv.y, xv.z, xv.w};
+    ChunkStager cst;
+    cst.load(a.Q, ds, qid, nrow, 0, lane);
+    for (int j0 = 0; j0 < d; j0 += 32) {
+        cst.store(tile, lane);
+        __syncwarp();
+        if (j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);   // in flight during this chunk
+        const int jn = min(32, d - j0);
+        const float* xr = tile + lane * kRHP;
+        if (shared_a && jn == 32) {   // the block's leaf: broadcast 16-byte reads of A_g
+#pragma unroll 1
+            for (int jj = 0; jj < 32; jj += 4) {
+                const float4 x = *reinterpret_cast<const float4*>(xr + jj);
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            const int j = 4 * j4 + c;
-            if (j < d) {
+                for (int i = 0; i < MM; ++i) {
+                    const float4 w = *reinterpret_cast<const float4*>(As + (size_t)i * ds + j0 + jj);
+                    s[i] = __fmaf_rn(w.x, x.x, s[i]);
+                    s[i] = __fmaf_rn(w.y, x.y, s[i]);
+                    s[i] = __fmaf_rn(w.z, x.z, s[i]);
+                    s[i] = __fmaf_rn(w.w, x.w, s[i]);
+                }
+            }
+        } else {
+            for (int jj = 0; jj < jn; ++jj) {
+                const float x = xr[jj];
+                const int j = j0 + jj;
 #pragma unroll
-                for (int i = 0; i < MM; ++i) s[i] = __fmaf_rn(Ag[(size_t)i * d + j], xs[c], s[i]);
+                for (int i = 0; i < MM; ++i)
+                    s[i] = __fmaf_rn(g == g0 ? As[(size_t)i * ds + j] : __ldg(Ag + (size_t)i * d + j), x, s[i]);
             }
         }
+        __syncwarp();
     }
+    if (!act) return;
+    const bool active = g >= a.leaf_lo && g < a.leaf_hi;
     const float W = a.Wl[g];
     float t[MM];
 #pragma unroll
@@ -200,19 +257,19 @@ __device__ __forceinline__ void hash_body(const QueryArgs& a, const uint32_t* __
 
 template <int MM>
 __global__ void __launch_bounds__(kRHQ) k_hash(QueryArgs a, const uint32_t* __restrict__ lperm) {
-    extern __shared__ __align__(16) float rh_rows[];
-    hash_body<MM>(a, lperm, rh_rows);
+    extern __shared__ __align__(16) float rh_smem[];
+    hash_body<MM>(a, lperm, rh_smem);
 }
 
 // a2 of hash tables 1..L-1 in one launch (blockIdx.y = table - 1): the tables'
 // blocks run together instead of one latency-bound launch per table.
 template <int MM>
 __global__ void __launch_bounds__(kRHQ) k_hash_tables(QueryArgs a, const __grid_constant__ HashTables ht) {
-    extern __shared__ __align__(16) float rh_rows[];
+    extern __shared__ __align__(16) float rh_smem[];
     const int t = blockIdx.y;
     QueryArgs b = a;
     b.A = ht.A[t]; b.bvec = ht.b[t]; b.qt = ht.qt[t]; b.qcode = ht.qcode[t]; b.qoor = ht.qoor[t]; b.qkey = ht.qkey[t];
-    hash_body<MM>(b, a.lperm, rh_rows);
+    hash_body<MM>(b, a.lperm, rh_smem);
 }
 
 // ---------------------------------------------------------------------------
@@ -675,16 +732,19 @@ void upload_e8_roots() {
     done_dev[dev] = true;
 }
 
+// k_hash: A_g [M][ds] + one staged chunk per warp
+static size_t hash_smem(const QueryArgs& a) {
+    return ((size_t)a.M * a.ds + (size_t)kRHW * 32 * kRHP) * sizeof(float);
+}
+
 int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    const size_t smem_r = a.rh_direct ? 16 : (size_t)kRHQ * (a.ds + 4) * sizeof(float);
-    const size_t smem_h = (a.rh_direct ? 0 : smem_r) + (size_t)a.M * a.d * sizeof(float);
+    const size_t smem_h = hash_smem(a);
     int32_t* lcnt = a.lcnt;
     int32_t* lcur = a.lcnt + a.G;
     BLSH_CUDA(cudaMemsetAsync(lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    BLSH_CUDA(cudaFuncSetAttribute(k_route, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_r));
-    k_route<<<grid, kRHQ, smem_r, s>>>(a, lcnt);
+    k_route<<<grid, kRHQ, 0, s>>>(a, lcnt);
     BLSH_LAUNCH_CHECK();
     k_leaf_scan<<<1, 1024, 0, s>>>(lcnt, a.G, lcur);
     BLSH_LAUNCH_CHECK();
@@ -713,10 +773,8 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
 int launch_route_group(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    const size_t smem_r = a.rh_direct ? 16 : (size_t)kRHQ * (a.ds + 4) * sizeof(float);
     BLSH_CUDA(cudaMemsetAsync(a.lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    BLSH_CUDA(cudaFuncSetAttribute(k_route, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_r));
-    k_route<<<grid, kRHQ, smem_r, s>>>(a, a.lcnt);
+    k_route<<<grid, kRHQ, 0, s>>>(a, a.lcnt);
     BLSH_LAUNCH_CHECK();
     k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, a.G, a.lcnt + a.G);
     BLSH_LAUNCH_CHECK();
@@ -784,7 +842,7 @@ void launch_shard_outputs(const uint32_t* idx, int64_t nq, int64_t n, int k, con
 void launch_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    const size_t smem_h = (a.rh_direct ? 0 : (size_t)kRHQ * (a.ds + 4) * sizeof(float)) + (size_t)a.M * a.d * sizeof(float);
+    const size_t smem_h = hash_smem(a);
 #define BLSH_H_CASE(MMV)                                                                                    \
     case MMV:                                                                                              \
         BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
@@ -804,7 +862,7 @@ void launch_hash(const QueryArgs& a, cudaStream_t s) {
 void launch_hash_tables(const QueryArgs& a, const HashTables& ht, cudaStream_t s) {
     if (a.nq == 0 || ht.n == 0) return;
     const dim3 grid((unsigned)((a.nq + kRHQ - 1) / kRHQ), (unsigned)ht.n);
-    const size_t smem_h = (a.rh_direct ? 0 : (size_t)kRHQ * (a.ds + 4) * sizeof(float)) + (size_t)a.M * a.d * sizeof(float);
+    const size_t smem_h = hash_smem(a);
 #define BLSH_HT_CASE(MMV)                                                                                     \
     case MMV:                                                                                                \
         BLSH_CUDA(cudaFuncSetAttribute(k_hash_tables<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \

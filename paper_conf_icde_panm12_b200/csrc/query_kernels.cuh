@@ -13,7 +13,6 @@ struct QueryArgs {
     int probe, T, hstep;
     int cperturb;            // probe = 3: bit-perturbed curve keys (R31)
     int msb_min;             // hierarchy = 2: climb threshold on the shared-MSB count (R32; B*M when 0)
-    int rh_direct;           // a1/a2 read query rows through L1 instead of staging them in shared memory
     int64_t rec_tau;         // probe = 2, T > 241: second-ring probes only while |A| < rec_tau (R33; 0 = all)
     // queries
     const float* Q;          // [nq][ds]

@@ -274,58 +274,77 @@ __global__ void __launch_bounds__(256) k_expand_rows(const Seg* __restrict__ seg
 // (atom-row index = 8 x the atom's tile-local index + (row & 7)): union rows carry (table row,
 // query mask, K slot); the other rows of a touched atom carry mask 0 and the K slot of the
 // atom's previous union row (or its first), so the slot stays non-decreasing along the
-// tile's rows (k_tile_items splits items on it).  One CTA per tile, three phases.
+// tile's rows (k_tile_items splits items on it).  One CTA per tile, one thread per atom: the
+// thread finds the first segment touching its atom (binary search over the segments' last
+// atoms, which are non-decreasing), walks the atom's 8 rows through that segment and the
+// later ones starting inside the atom, fills the non-union rows' K slots in registers; the
+// CTA's 256 atoms (32 KB) leave through shared memory (XOR-swizzled 16-byte slots) as
+// coalesced stores.  Every entry is written once.
 __global__ void __launch_bounds__(256) k_expand_atoms(const Seg* __restrict__ segs, const int32_t* __restrict__ nseg,
                                                       int segcap, const int64_t* __restrict__ arows_off,
                                                       const int64_t* __restrict__ aoff, const uint32_t* __restrict__ rgrp,
                                                       uint4* __restrict__ rowinfo, uint32_t* __restrict__ slot_anchor) {
+    __shared__ uint4 stage[256 * 8];
     const int64_t t = blockIdx.x;
     const Seg* S = segs + (size_t)t * segcap;
     uint4* out = rowinfo + arows_off[t];
     const int64_t ab = aoff[t];
     const int ns = nseg[t];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    // phase 1: the atoms each segment introduces (all but a first atom shared with its predecessor)
-    for (int sI = warp; sI < ns; sI += 8) {
-        const Seg sg = S[sI];
-        const uint32_t a0 = sg.start >> 3, a1 = (sg.start + sg.len - 1) >> 3;
-        const bool shared = sI > 0 && ((S[sI - 1].start + S[sI - 1].len - 1) >> 3) == a0;
-        for (uint32_t k = (shared ? 1u : 0u) * 8u + lane; k < (a1 - a0 + 1u) * 8u; k += 32) {
-            const uint32_t row = a0 * 8u + k;
-            out[(size_t)(sg.atbase + (k >> 3)) * 8 + (k & 7)] = make_uint4(row, 0u, 0u, 0u);
-        }
-    }
-    __syncthreads();
-    // phase 2: the union rows
-    for (int sI = warp; sI < ns; sI += 8) {
-        const Seg sg = S[sI];
-        const uint32_t a0 = sg.start >> 3;
-        const uint32_t g0 = rgrp[sg.start];
-        for (uint32_t i = lane; i < sg.len; i += 32) {
-            const uint32_t row = sg.start + i;
-            const uint32_t grp = rgrp[row];
-            const int64_t slot = ab + sg.abase + (grp - g0);
-            out[(size_t)(sg.atbase + ((row >> 3) - a0)) * 8 + (row & 7)] = make_uint4(row, sg.mask, (uint32_t)slot, 0u);
-            if (i == 0 || rgrp[row - 1] != grp) slot_anchor[slot] = grp;
-        }
-    }
-    __syncthreads();
-    // phase 3: K slots of the atoms' non-union rows (monotone)
     const int64_t nat = (arows_off[t + 1] - arows_off[t]) >> 3;
-    for (int64_t at = threadIdx.x; at < nat; at += 256) {
-        uint4 e[8];
+    const int tid = threadIdx.x;
+    auto last_atom = [&](const Seg& g) { return (int64_t)g.atbase + ((g.start + g.len - 1) >> 3) - (g.start >> 3); };
+    int lo = 0;
+    for (int64_t base = 0; base < nat; base += 256) {
+        const int64_t A = base + tid;
+        if (A < nat) {
+            int l = lo, h = ns - 1;
+            while (l < h) {
+                const int m = (l + h) >> 1;
+                if (last_atom(S[m]) >= A) h = m;
+                else l = m + 1;
+            }
+            lo = l;
+            int sj = l;
+            Seg cs = S[sj];
+            const uint32_t at = (cs.start >> 3) + (uint32_t)(A - cs.atbase);
+            uint32_t cg0 = rgrp[cs.start];
+            uint4 e[8];
 #pragma unroll
-        for (int r = 0; r < 8; ++r) e[r] = out[at * 8 + r];
-        uint32_t cur = 0;
-        bool found = false;
+            for (int r = 0; r < 8; ++r) {
+                const uint32_t row = at * 8u + (uint32_t)r;
+                while (row >= cs.start + cs.len && sj + 1 < ns && S[sj + 1].start <= row) {
+                    cs = S[++sj];
+                    cg0 = rgrp[cs.start];
+                }
+                if (row >= cs.start && row < cs.start + cs.len) {
+                    const uint32_t grp = rgrp[row];
+                    const int64_t slot = ab + cs.abase + (grp - cg0);
+                    e[r] = make_uint4(row, cs.mask, (uint32_t)slot, 0u);
+                    if (row == cs.start || rgrp[row - 1] != grp) slot_anchor[slot] = grp;
+                } else {
+                    e[r] = make_uint4(row, 0u, 0u, 0u);
+                }
+            }
+            uint32_t cur = 0;
+            bool found = false;
 #pragma unroll
-        for (int r = 0; r < 8; ++r)
-            if (!found && e[r].y != 0u) { cur = e[r].z; found = true; }
+            for (int r = 0; r < 8; ++r)
+                if (!found && e[r].y != 0u) { cur = e[r].z; found = true; }
 #pragma unroll
-        for (int r = 0; r < 8; ++r) {
-            if (e[r].y != 0u) cur = e[r].z;
-            else out[at * 8 + r].z = cur;
+            for (int r = 0; r < 8; ++r) {
+                if (e[r].y != 0u) cur = e[r].z;
+                else e[r].z = cur;
+                stage[tid * 8 + (r ^ (tid & 7))] = e[r];
+            }
         }
+        __syncthreads();
+        const int cnt = (int)min((int64_t)256, nat - base) * 8;
+        uint4* o = out + base * 8;
+        for (int i = tid; i < cnt; i += 256) {
+            const int a8 = i >> 3, r = i & 7;
+            o[i] = stage[a8 * 8 + (r ^ (a8 & 7))];
+        }
+        __syncthreads();
     }
 }
 
@@ -804,10 +823,15 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     const int nlist = use_f16 ? kSxEpiN : 4;   // buffered-pair lists per (item, query): the screen's epilogue warps
     const bool large_k = k > 64;               // fp16 screen + exact keys per query + launch_select
     // large k: each warp's list holds ~kk = ceil(k/8) survivors (+ the bound's slack)
-    static const int scap_small = [] {   // BLSH_SCAPW (experiments): buffered pairs per list for k <= 64
+    // fp16 screen, k <= 64: buffered pairs per (item, query, epilogue warp).  k <= 16 (KT <= 16): 96;
+    // 16 < k <= 64: 384 -- with k = 50 on c3 (58k candidates per query, 6 queries per union row)
+    // 96 overflowed 87k lists (every row of those rescored: 207M exact pairs, 40 ms), 192 6.4k,
+    // 384 none (8M pairs, 1.8 ms; profiles/r02/r02ak).  BLSH_SCAPW overrides (experiments).
+    static const int scap_env = [] {
         const char* e = std::getenv("BLSH_SCAPW");
-        return e ? std::max(32, std::atoi(e) / 16 * 16) : kTcScap;
+        return e ? std::max(32, std::atoi(e) / 16 * 16) : 0;
     }();
+    const int scap_small = scap_env ? scap_env : (k <= 16 ? kTcScap : 384);
     const int scapw = large_k ? ((2 * ((k + kSxEpiN - 1) / kSxEpiN) + 64 + 15) / 16) * 16 : (use_f16 ? scap_small : kTcScap);
     const int kScap = nlist * scapw;
     const size_t part_bytes = large_k ? 0 : ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);

@@ -507,13 +507,16 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
         qv[u] = v < nv ? __ldg(qrow + v) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
     int rescored = 0;
-    // rows of the set bits of nm: lane i of the warp holds row position rpos (from its entry)
+    // rows of the set bits of nm: lane i of the warp holds row position rpos (from its entry);
+    // kRB rows per round: their 16-byte loads are all in flight together (the kernel waits on
+    // DRAM: random fp32 rows, long_scoreboard 63% of stalls with 4 rows per round, r02ak)
+    constexpr int kRB = 8;
     auto score_rows = [&](unsigned nm, uint32_t rpos) {
             while (nm) {
-                uint32_t row[4];
+                uint32_t row[kRB];
                 int nr = 0;
 #pragma unroll
-                for (int r = 0; r < 4; ++r) {
+                for (int r = 0; r < kRB; ++r) {
                     row[r] = 0u;
                     if (nm) {
                         const int src = __ffs(nm) - 1;
@@ -522,9 +525,9 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
                         nr = r + 1;
                     }
                 }
-                float part[4];
+                float part[kRB];
 #pragma unroll
-                for (int r = 0; r < 4; ++r) {
+                for (int r = 0; r < kRB; ++r) {
                     part[r] = 0.0f;
                     if (r < nr) {
                         const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)row[r] * a.ds);
@@ -545,12 +548,14 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
 #pragma unroll
                 for (int o = 16; o > 0; o >>= 1) {
 #pragma unroll
-                    for (int r = 0; r < 4; ++r) part[r] += __shfl_xor_sync(BLSH_FULL, part[r], o);
+                    for (int r = 0; r < kRB; ++r) part[r] += __shfl_xor_sync(BLSH_FULL, part[r], o);
                 }
-                const uint32_t rl = (lane & 3) == 0 ? row[0] : (lane & 3) == 1 ? row[1] : (lane & 3) == 2 ? row[2] : row[3];
+                uint32_t rl = row[0];
+#pragma unroll
+                for (int r = 1; r < kRB; ++r) rl = (lane & (kRB - 1)) == r ? row[r] : rl;
                 const uint32_t idl = lane < nr ? __ldg(a.perm + rl) : 0u;
 #pragma unroll
-                for (int r = 0; r < 4; ++r) {
+                for (int r = 0; r < kRB; ++r) {
                     const uint32_t id = __shfl_sync(BLSH_FULL, idl, r);
                     if (r < nr) {
                         const unsigned long long key = pack_entry(part[r], id);

@@ -9,4 +9,5 @@ BLSH_RH_STAGE=1 timeout 600 python bench.py --no-cpu-baseline --no-e2e > gpurun_
 for kre in k_route k_hash k_expand_atoms k_probe_lookup k_tc_rescore k_tile_prep; do
   timeout 600 bash tools/prof.sh full r02ak_$kre "$kre"
   python tools/ncu_summary.py gpurun_out/raw_r02ak_$kre.csv > gpurun_out/r02ak_ncu_$kre.txt 2>&1
+  ncu -i gpurun_out/prof_r02ak_$kre.ncu-rep --page source --csv > gpurun_out/src_r02ak_$kre.csv 2>/dev/null; rm -f gpurun_out/prof_r02ak_$kre.ncu-rep
 done
