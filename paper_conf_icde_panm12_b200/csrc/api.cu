@@ -736,8 +736,14 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     // plan: chunking of the candidate lists
     scan_exclusive_i64(w.cnt, cand_off, nq, w.scan, s); launches += 3;
     int64_t total = 0;
-    BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    BLSH_CUDA(cudaStreamSynchronize(s));
+    // small batches on the warp short-list plan without host round trips: chunks of 256, item
+    // count and candidate total stay on the device, buffers sized by |A(q)| <= the leaf's rows
+    // (R21: candidates come from the query's own leaf); one synchronisation per call
+    const bool nosync = kind_pre == 0 && !list_path && nq <= small_batch_limit();
+    if (!nosync) {
+        BLSH_CUDA(cudaMemcpyAsync(&total, cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+    }
     const int kind = kind_pre;   // lists: warp short-list over the positions
     const bool tiled = kind > 0;
     int64_t n_items = 0, union_rows = 0, pairs = total, kept = 0, kslots = 0;
@@ -757,14 +763,26 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[6], s));
     } else {
         const int64_t target = 148 * 8 * 4;
-        ch = (total + target - 1) / std::max<int64_t>(target, 1);
-        ch = std::min<int64_t>(4096, std::max<int64_t>(256, (ch + 31) / 32 * 32));
+        int64_t total_cap = total;
+        if (nosync) {
+            // a few queries: short chunks, so that their candidates spread over many warps
+            // (one warp streams its chunk with 4 rows in flight: latency-bound)
+            ch = nq <= 4 ? 32 : (nq <= 32 ? 64 : 256);
+            total_cap = nq * std::max<int64_t>(ix.max_leaf_rows, 1);
+        } else {
+            ch = (total + target - 1) / std::max<int64_t>(target, 1);
+            ch = std::min<int64_t>(4096, std::max<int64_t>(256, (ch + 31) / 32 * 32));
+        }
         launch_items(w.cnt, nq, (int)ch, items, s); ++launches;
         scan_exclusive_i64(items, w.item_off, nq, w.scan, s); launches += 3;
-        BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        BLSH_CUDA(cudaStreamSynchronize(s));
+        if (nosync) {
+            n_items = nq + (total_cap + ch - 1) / ch;   // >= sum of ceil(|A(q)| / ch): the grid's bound
+        } else {
+            BLSH_CUDA(cudaMemcpyAsync(&n_items, w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+            BLSH_CUDA(cudaStreamSynchronize(s));
+        }
         const bool large_k = k > 64;
-        if (large_k) w.partials.ensure((size_t)std::max<int64_t>(total, 1) * sizeof(unsigned long long));
+        if (large_k) w.partials.ensure((size_t)std::max<int64_t>(total_cap, 1) * sizeof(unsigned long long));
         else w.partials.ensure((size_t)std::max<int64_t>(n_items, 1) * k * sizeof(unsigned long long));
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[4], s));
         // a5, one warp per (query, chunk)
@@ -776,6 +794,7 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
         sa.list = list_path ? w.listbuf.as<uint32_t>() : nullptr;
         sa.list_off = list_path ? w.raw_off : nullptr;
         sa.cand_keys = large_k ? w.partials.as<unsigned long long>() : nullptr;
+        sa.n_items_dev = nosync ? w.item_off + nq : nullptr;
         launch_shortlist(sa, s); if (n_items) ++launches;
         if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[5], s));
         if (large_k) launch_select(sa.cand_keys, cand_off, nq, k, w.qoor, w.cnt, d_ids, d_d2, d_pk, d_nc, s);
@@ -791,7 +810,19 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
         if (out_packed) BLSH_CUDA(cudaMemcpyAsync(out_packed, d_pk, (size_t)nq * k * 8, cudaMemcpyDeviceToHost, s));
     }
     if (tm) BLSH_CUDA(cudaEventRecord(ix.ev[7], s));
+    if (nosync) {   // the statistics of the device-side plan
+        BLSH_CUDA(cudaMemcpyAsync(&w.host_scalars[0], cand_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        BLSH_CUDA(cudaMemcpyAsync(&w.host_scalars[1], w.item_off + nq, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    }
+    const bool tau_dev = p.hierarchy == 1 && p.min_cand == 0;
+    if (tau_dev) BLSH_CUDA(cudaMemcpyAsync(&w.host_scalars[2], w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     BLSH_CUDA(cudaStreamSynchronize(s));
+    if (nosync) {
+        total = w.host_scalars[0];
+        n_items = w.host_scalars[1];
+        union_rows = total;
+        pairs = total;
+    }
     stt.total_cand = total;
     stt.n_items = n_items;
     stt.chunk = (int32_t)ch;
@@ -813,7 +844,7 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     stt.shortlist_flops = 3.0 * ix.d * (double)total;
     if (p.hierarchy == 1) {
         int64_t tau = p.min_cand;
-        if (p.min_cand == 0) BLSH_CUDA(cudaMemcpy(&tau, w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        if (tau_dev) tau = w.host_scalars[2];
         stt.tau = tau;
     }
     if (tm) {

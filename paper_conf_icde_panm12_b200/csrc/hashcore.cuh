@@ -108,7 +108,9 @@ struct ChunkStager {
 #pragma unroll
         for (int r4 = 0; r4 < 8; ++r4) {
             const int r = 4 * r4 + rr;
-            v[r4] = (r < nrow && col < ds) ? __ldg(reinterpret_cast<const float4*>(Q + (size_t)qid(r) * ds + col))
+            // streaming loads (evict-first): a row chunk is read once per pass, L1 keeps the
+            // parameters (tree nodes, A_g) the chains read again and again
+            v[r4] = (r < nrow && col < ds) ? __ldcs(reinterpret_cast<const float4*>(Q + (size_t)qid(r) * ds + col))
                                            : make_float4(0.f, 0.f, 0.f, 0.f);
         }
     }

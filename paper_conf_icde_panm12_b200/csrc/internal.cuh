@@ -130,6 +130,7 @@ struct QueryWork {
     ScanTemp scan2;
     cudaStream_t side = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    int64_t host_scalars[3] = {0, 0, 0};   // plan statistics and tau, read back with the answers
     // blsh_query_pipelined: double-buffered query uploads / answer downloads on a copy stream
     DevBuf pl_q[2], pl_out[2];
     cudaStream_t copy = nullptr;

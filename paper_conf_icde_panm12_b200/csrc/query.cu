@@ -43,6 +43,10 @@ constexpr int kRHW = 4;              // warps per block (32 queries each)
 constexpr int kRHQ = 32 * kRHW;      // queries per block
 constexpr int kRHP = kRowPitch;      // staged chunk row pitch (floats, hashcore.cuh)
 
+// PREFETCH: the next chunk's loads are in flight while a chunk is consumed (latency: small
+// batches); without, 64 instead of 117 registers and more warps per SM (throughput: 309 vs
+// 458 us at c4, r02am)
+template <bool PREFETCH>
 __global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict__ lcnt) {
     __shared__ __align__(16) float tiles[kRHW][32 * kRHP];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -74,11 +78,12 @@ __global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict
 #pragma unroll
         for (int i = 0; i < 7; ++i) s[i] = 0.0f;
         ChunkStager cst;
-        cst.load(a.Q, ds, qid, nrow, 0, lane);
+        if (PREFETCH) cst.load(a.Q, ds, qid, nrow, 0, lane);
         for (int j0 = 0; j0 < d; j0 += 32) {
+            if (!PREFETCH) cst.load(a.Q, ds, qid, nrow, j0, lane);
             cst.store(tile, lane);
             __syncwarp();
-            if (j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);   // in flight during this chunk
+            if (PREFETCH && j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);
             const int jn = min(32, d - j0);
             const float* xr = tile + lane * kRHP;
             if (!generic) {   // hyperplane nodes only: s_i = fmaf(dir_ij, x_j, s_i)
@@ -732,6 +737,7 @@ void upload_e8_roots() {
     done_dev[dev] = true;
 }
 
+constexpr int64_t kRoutePrefetchBelow = 16384;   // batches smaller than this fill < 1 wave of k_route
 // k_hash: A_g [M][ds] + one staged chunk per warp
 static size_t hash_smem(const QueryArgs& a) {
     return ((size_t)a.M * a.ds + (size_t)kRHW * 32 * kRHP) * sizeof(float);
@@ -744,7 +750,8 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     int32_t* lcnt = a.lcnt;
     int32_t* lcur = a.lcnt + a.G;
     BLSH_CUDA(cudaMemsetAsync(lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    k_route<<<grid, kRHQ, 0, s>>>(a, lcnt);
+    if (a.nq < kRoutePrefetchBelow) k_route<true><<<grid, kRHQ, 0, s>>>(a, lcnt);
+    else k_route<false><<<grid, kRHQ, 0, s>>>(a, lcnt);
     BLSH_LAUNCH_CHECK();
     k_leaf_scan<<<1, 1024, 0, s>>>(lcnt, a.G, lcur);
     BLSH_LAUNCH_CHECK();
@@ -774,7 +781,8 @@ int launch_route_group(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
     BLSH_CUDA(cudaMemsetAsync(a.lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    k_route<<<grid, kRHQ, 0, s>>>(a, a.lcnt);
+    if (a.nq < kRoutePrefetchBelow) k_route<true><<<grid, kRHQ, 0, s>>>(a, a.lcnt);
+    else k_route<false><<<grid, kRHQ, 0, s>>>(a, a.lcnt);
     BLSH_LAUNCH_CHECK();
     k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, a.G, a.lcnt + a.G);
     BLSH_LAUNCH_CHECK();

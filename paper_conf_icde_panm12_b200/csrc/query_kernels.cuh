@@ -139,6 +139,8 @@ struct ShortlistArgs {
     unsigned long long* cand_keys;  // [total] non-NULL: emit every candidate key (large k)
     const uint32_t* list;           // non-NULL (L > 1): deduplicated candidate positions per query
     const int64_t* list_off;        // [nq+1] start of each query's list
+    const int64_t* n_items_dev;     // non-NULL: the item count lives on the device (n_items is then an upper
+                                    // bound for the grid; small batches plan without a host round trip)
 };
 
 // query-tiled short-list (shortlist_tiled.cu)
@@ -146,6 +148,7 @@ struct ShortlistArgs {
 // kernel is the default where it applies (k <= 32, d_stride a multiple of 64 and <= 512);
 // BLSH_SHORTLIST=warp|simt forces the others.
 int shortlist_kind(int64_t nq, int ds, int dr, int T, int k);
+int64_t small_batch_limit();   // batches up to this size take the warp short-list
 void sort_queries(const QueryArgs& a, SortBufs& sb, uint32_t* qorder, cudaStream_t s, int* launches);
 int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, ScanTemp& scan, cudaStream_t s,
                    int* launches);

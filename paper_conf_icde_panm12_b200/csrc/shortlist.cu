@@ -60,8 +60,10 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     // items differ in length, and a block would otherwise hold its slot until its slowest warp ends)
     // (list mode; the interval mode keeps one item per warp: neighbouring items, which share
     // rows in L2, then run together)
-    for (int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5); item < a.n_items;
-         item += LIST ? (int64_t)gridDim.x * kSLWarps : a.n_items) {
+    // (with the item count on the device -- small batches -- the grid is bounded and strides too)
+    const int64_t n_items = a.n_items_dev ? *a.n_items_dev : a.n_items;
+    for (int64_t item = blockIdx.x * (int64_t)kSLWarps + (threadIdx.x >> 5); item < n_items;
+         item += (LIST || a.n_items_dev) ? (int64_t)gridDim.x * kSLWarps : n_items) {
     // query of this item: last q with item_off[q] <= item
     int64_t lo = 0, hi = a.nq;
     while (hi - lo > 1) {
@@ -487,7 +489,7 @@ void launch_items(const int64_t* cnt, int64_t nq, int chunk, int64_t* items, cud
 void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     if (a.n_items == 0) return;
     const int64_t blocks = (a.n_items + kSLWarps - 1) / kSLWarps;
-    const unsigned grid = (unsigned)(a.list ? std::min<int64_t>(blocks, 148 * 8) : blocks);
+    const unsigned grid = (unsigned)((a.list || a.n_items_dev) ? std::min<int64_t>(blocks, 148 * 8) : blocks);
     const int nvl = ((a.ds >> 2) + 31) / 32;
 
 #define BLSH_SL_CASE(V)                                                                             \

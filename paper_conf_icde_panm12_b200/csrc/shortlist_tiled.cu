@@ -640,6 +640,8 @@ static int screen_variant() {
     return v;
 }
 
+int64_t small_batch_limit() { return kSmallBatch; }
+
 int shortlist_kind(int64_t nq, int ds, int dr, int T, int k) {
     const char* mode = std::getenv("BLSH_SHORTLIST");
     if (mode && std::strcmp(mode, "warp") == 0) return 0;

@@ -508,9 +508,9 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     }
     int rescored = 0;
     // rows of the set bits of nm: lane i of the warp holds row position rpos (from its entry);
-    // kRB rows per round: their 16-byte loads are all in flight together (the kernel waits on
-    // DRAM: random fp32 rows, long_scoreboard 63% of stalls with 4 rows per round, r02ak)
-    constexpr int kRB = 8;
+    // kRB rows per round, their 16-byte loads in flight together (8 rows: 80 registers and a
+    // stack frame, fewer warps, 0.95 -> 1.28 ms at c4, r02am; 4 kept)
+    constexpr int kRB = 4;
     auto score_rows = [&](unsigned nm, uint32_t rpos) {
             while (nm) {
                 uint32_t row[kRB];

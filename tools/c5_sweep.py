@@ -76,6 +76,8 @@ def main():
     ap.add_argument("--wmult", default="2.83,4,5.66,8")
     ap.add_argument("--families", default="multiprobe,e8_lattice,morton_curve")
     ap.add_argument("--batches", default="1,10,100,1000,10000,100000")
+    ap.add_argument("--points", default=None,
+                    help="skip the probe sweep: batch sweep at family:W_mult:T[,...] (e.g. multiprobe:8:16)")
     a = ap.parse_args()
     cfg = synth.CONFIGS[a.config]
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
@@ -96,7 +98,11 @@ def main():
               r10=r10, gt="bench_data/%s_gt.npz (%d queries, oracle fp64 brute force)" % (cfg.name, len(g["qidx"]))))
     k = cfg.k
     best = {}
-    for fam in a.families.split(","):
+    if a.points:
+        for pt in a.points.split(","):
+            fam, wm, T = pt.split(":")
+            best[fam] = (None, dict(W=float(wm) * r10, T=int(T), recall10=None))
+    for fam in ([] if a.points else a.families.split(",")):
         fk = FAMILIES[fam]
         for wm in [float(w) for w in a.wmult.split(",")]:
             W = wm * r10
