@@ -825,16 +825,18 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
     const int nlist = use_f16 ? kSxEpiN : 4;   // buffered-pair lists per (item, query): the screen's epilogue warps
     const bool large_k = k > 64;               // fp16 screen + exact keys per query + launch_select
     // large k: each warp's list holds ~kk = ceil(k/8) survivors (+ the bound's slack)
-    // fp16 screen, k <= 64: buffered pairs per (item, query, epilogue warp).  k <= 16 (KT <= 16): 96;
-    // 16 < k <= 64: 384 -- with k = 50 on c3 (58k candidates per query, 6 queries per union row)
-    // 96 overflowed 87k lists (every row of those rescored: 207M exact pairs, 40 ms), 192 6.4k,
-    // 384 none (8M pairs, 1.8 ms; profiles/r02/r02ak).  BLSH_SCAPW overrides (experiments).
+    // fp16 screen: buffered pairs per (item, query, epilogue warp): 384.  A list that overflows
+    // sends every row of its unit to exact rescoring, by one warp: with 96 (k <= 64) c3 at k = 50
+    // (58k candidates per query) overflowed 87k lists (207M exact pairs, 40 ms; 384: none, 8M,
+    // 1.8 ms), c5 with Morton-curve probing T = 64 spent 8.6 ms on a few overflowed units, and the
+    // large-k lists (2 kk + 64) overflowed on c3 at k = 500 (428M exact pairs, 76 ms) (r02ak,
+    // r02ao).  The buffers are plain HBM (n_items x 32 x 8 x 384 x 8 B: 3.1 GB at c4); the TF32
+    // screen keeps its 96.  BLSH_SCAPW overrides (experiments).
     static const int scap_env = [] {
         const char* e = std::getenv("BLSH_SCAPW");
         return e ? std::max(32, std::atoi(e) / 16 * 16) : 0;
     }();
-    const int scap_small = scap_env ? scap_env : (k <= 16 ? kTcScap : 384);
-    const int scapw = large_k ? ((2 * ((k + kSxEpiN - 1) / kSxEpiN) + 64 + 15) / 16) * 16 : (use_f16 ? scap_small : kTcScap);
+    const int scapw = use_f16 ? (scap_env ? scap_env : 384) : kTcScap;
     const int kScap = nlist * scapw;
     const size_t part_bytes = large_k ? 0 : ((size_t)std::max<int64_t>(n_items, 1) * QT * k * 8 + 255) & ~size_t(255);
     const size_t sbuf_bytes = ((size_t)std::max<int64_t>(n_items, 1) * QT * kScap * 8 + 255) & ~size_t(255);
