@@ -403,3 +403,26 @@ def test_tc_screen_equals_warp(blsh, orc, monkeypatch, shape):
         np.testing.assert_array_equal(a[0], b[0])
         np.testing.assert_array_equal(a[1].view(np.uint32), b[1].view(np.uint32))
     run_query_pair(ix, ox, X, Q[:60], 10, probe=1, T=T)
+
+
+def test_sharded_merge_against_oracle(blsh, orc):
+    """SURVEY §8(e) against the oracle directly: world = 4 leaf shards (each answers its
+    compacted ~150 owned queries on the tiled tcgen05 screen), packed lists merged with
+    blsh_merge_topk; counts equal the oracle's |A(q)| and the merged top-k passes check_topk
+    against the oracle's single-index answer."""
+    X, Q = synth.make_dataset(synth.CONFIGS["c1"], n=10000, nq=600)
+    Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
+    ox = orc.OracleIndex(X, G=8, M=8, W=4.0, seed=5)
+    oi, od, onc = ox.query(Q, 10, probe=1, T=16)
+    lists, counts = [], []
+    for r in range(4):
+        sh = blsh.blsh_build(Xd, n_leaves=8, M=8, W=4.0, seed=5, rank=r, world=4)
+        pk, nc = sh.query_packed(Qd, 10, probe=1, n_probes=16)
+        lists.append(pk)
+        counts.append(nc)
+        sh.close()
+    packed = torch.stack(lists).contiguous()
+    mi, md = blsh.blsh_merge_topk(packed, 4, len(Q), 10)
+    torch.cuda.synchronize()
+    assert np.array_equal(torch.stack(counts).sum(0).cpu().numpy(), onc)
+    check_topk(mi.cpu().numpy(), md.cpu().numpy(), oi, od, X, Q, cands=ox.candidates())

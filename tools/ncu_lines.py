@@ -1,6 +1,6 @@
 """Aggregate ncu per-instruction stall samples by CUDA source line.
 
-    python tools/ncu_lines.py <rep.ncu-rep> <kernel-substring> [top]
+    python tools/ncu_lines.py <rep.ncu-rep | source-page.csv> <kernel-substring> [top]
 
 Reads the SASS source page of the capture (`ncu -i … --page source --csv`), maps
 each instruction offset to its source line with `nvdisasm -g` of the kernel's
@@ -47,7 +47,10 @@ def line_map(kernel_sub):
 def main():
     rep, ksub = sys.argv[1], sys.argv[2]
     top = int(sys.argv[3]) if len(sys.argv) > 3 else 30
-    txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv"], capture_output=True, text=True).stdout
+    if rep.endswith(".csv"):   # an exported source page (ncu -i rep --page source --csv > file.csv)
+        txt = open(rep).read()
+    else:
+        txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(txt)))
     hdr = rows[1]
     ia, isamp, iex = hdr.index("Address"), hdr.index("Warp Stall Sampling (All Samples)"), hdr.index("Instructions Executed")
