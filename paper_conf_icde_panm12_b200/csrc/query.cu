@@ -31,10 +31,12 @@ namespace {
 // read back by lane = query (row pitch 36 floats: the 16-byte reads of 8 lanes fall in
 // distinct bank groups).  A lane's chains stay canonical (R1: one fmaf per column, j
 // strictly ascending from 0.0f); the chunking only changes where x_j comes from.
-//   k_route       ceil(depth / 3) passes; a pass evaluates the <= 7 nodes of the
-//                 3-level subtree below the lane's current node (independent chains:
+//   k_route_pass  ceil(depth / 3) passes; a pass evaluates the <= 7 nodes of the
+//                 3-level subtree below the query's current node (independent chains:
 //                 the FMA latency is hidden, the rows are read ceil(depth / 3) times
-//                 instead of depth times), then descends 3 levels; leaf histogram.
+//                 instead of depth times), then descends 3 levels; between passes the
+//                 queries are regrouped by the node reached, so a block's queries share
+//                 their subtree and read its node vectors from shared memory.
 //   k_leaf_scan / k_leaf_scatter   group the queries by leaf (lperm).
 //   k_hash        128 leaf-grouped queries per block; the leaf matrix A_g of the
 //                 block's first query is staged in shared memory (pitch ds, broadcast
@@ -43,103 +45,114 @@ constexpr int kRHW = 4;              // warps per block (32 queries each)
 constexpr int kRHQ = 32 * kRHW;      // queries per block
 constexpr int kRHP = kRowPitch;      // staged chunk row pitch (floats, hashcore.cuh)
 
-// PREFETCH: the next chunk's loads are in flight while a chunk is consumed (latency: small
-// batches); without, 64 instead of 117 registers and more warps per SM (throughput: 309 vs
-// 458 us at c4, r02am)
+// One pass of a1 over levels [l0, l0 + 3): queries in `order` (NULL: batch order), grouped by
+// the node they reached (qleaf holds its index within level l0; 0 at l0 = 0).  The block stages
+// the 3-level subtree (<= 7 node vectors, dir or mu by the node's rule) below its first query's
+// node in shared memory; a warp whose 32 queries all sit at that node reads it as broadcast
+// 16-byte loads, other warps read their lanes' nodes through L1.  Every lane runs <= 7
+// independent canonical chains (R1) over the row chunks, descends, and writes its node's index
+// within level l0 + nl into qleaf, counted in cnt (the next grouping / the leaf histogram).
+// PREFETCH: the next chunk's loads are in flight while a chunk is consumed (small batches).
 template <bool PREFETCH>
-__global__ void __launch_bounds__(kRHQ) k_route(QueryArgs a, int32_t* __restrict__ lcnt) {
-    __shared__ __align__(16) float tiles[kRHW][32 * kRHP];
+__global__ void __launch_bounds__(kRHQ) k_route_pass(QueryArgs a, int l0, const uint32_t* __restrict__ order,
+                                                     int32_t* __restrict__ cnt) {
+    extern __shared__ __align__(16) float rt_smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int64_t q0 = blockIdx.x * (int64_t)kRHQ + warp * 32;
-    if (q0 >= a.nq) return;
-    const int nrow = (int)min((int64_t)32, a.nq - q0);
-    float* tile = tiles[warp];
-    const bool act = lane < nrow;
     const int d = a.d, ds = a.ds;
-    auto qid = [&](int r) { return q0 + r; };
-    int v = 0;
-    for (int l0 = 0; l0 < a.depth; l0 += 3) {
-        const int nl = min(3, a.depth - l0);
-        const int nn = (1 << nl) - 1;
-        const float* vec[7];
-        bool mean[7];
-        bool anymean = false;
+    const int nl = min(3, a.depth - l0);
+    const int nn = (1 << nl) - 1;
+    float* nvec = rt_smem;                                  // [7][ds]: the leader's subtree
+    float* tile = rt_smem + (size_t)7 * ds + (size_t)warp * 32 * kRHP;
+    const int64_t pb = blockIdx.x * (int64_t)kRHQ;
+    const int vbase = (1 << l0) - 1;                        // first node of level l0
+    const int v_lead = vbase + (l0 ? a.qleaf[order ? order[pb] : pb] : 0);
+    auto node_of = [&](int v, int i) {                      // heap index of subtree entry i below v
+        const int ll = i == 0 ? 0 : (i < 3 ? 1 : 2);
+        return ((v + 1) << ll) - 1 + (i - ((1 << ll) - 1));
+    };
+    for (int e = threadIdx.x; e < nn * (ds >> 2); e += kRHQ) {
+        const int i = e / (ds >> 2), c4 = e - i * (ds >> 2);
+        const int nid = node_of(v_lead, i);
+        const float* src = (a.ntype[nid] != 0 ? a.mu : a.dirs) + (size_t)nid * ds;
+        reinterpret_cast<float4*>(nvec + (size_t)i * ds)[c4] = __ldg(reinterpret_cast<const float4*>(src) + c4);
+    }
+    __syncthreads();
+    const int64_t p0 = pb + warp * 32;
+    if (p0 >= a.nq) return;
+    const int nrow = (int)min((int64_t)32, a.nq - p0);
+    const bool act = lane < nrow;
+    const int64_t q = act ? (order ? (int64_t)order[p0 + lane] : p0 + lane) : 0;
+    const int v = act ? vbase + (l0 ? a.qleaf[q] : 0) : v_lead;
+    const bool lead = __all_sync(BLSH_FULL, v == v_lead);
+    const float* vec[7];
+    bool mean[7];
+    bool anymean = false;
 #pragma unroll
-        for (int i = 0; i < 7; ++i) {
-            const int ll = i == 0 ? 0 : (i < 3 ? 1 : 2);
-            const int nid = ((v + 1) << ll) - 1 + (i - ((1 << ll) - 1));   // heap order below v
-            const bool use = i < nn;
-            mean[i] = use && a.ntype[nid] != 0;
-            vec[i] = use ? (mean[i] ? a.mu : a.dirs) + (size_t)nid * ds : a.dirs;
-            anymean |= act && mean[i];
-        }
-        const bool generic = __any_sync(BLSH_FULL, anymean);
-        float s[7];
+    for (int i = 0; i < 7; ++i) {
+        const bool use = i < nn;
+        const int nid = use ? node_of(v, i) : 0;
+        mean[i] = use && a.ntype[nid] != 0;
+        vec[i] = lead ? nvec + (size_t)i * ds : ((mean[i] ? a.mu : a.dirs) + (size_t)nid * ds);
+        anymean |= act && mean[i];
+    }
+    const bool generic = __any_sync(BLSH_FULL, anymean);
+    auto qid = [&](int r) { return order ? (int64_t)order[p0 + r] : p0 + r; };
+    float s[7];
 #pragma unroll
-        for (int i = 0; i < 7; ++i) s[i] = 0.0f;
-        ChunkStager cst;
-        if (PREFETCH) cst.load(a.Q, ds, qid, nrow, 0, lane);
-        for (int j0 = 0; j0 < d; j0 += 32) {
-            if (!PREFETCH) cst.load(a.Q, ds, qid, nrow, j0, lane);
-            cst.store(tile, lane);
-            __syncwarp();
-            if (PREFETCH && j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);
-            const int jn = min(32, d - j0);
-            const float* xr = tile + lane * kRHP;
-            if (!generic) {   // hyperplane nodes only: s_i = fmaf(dir_ij, x_j, s_i)
-                if (jn == 32) {
+    for (int i = 0; i < 7; ++i) s[i] = 0.0f;
+    ChunkStager cst;
+    if (PREFETCH) cst.load(a.Q, ds, qid, nrow, 0, lane);
+    for (int j0 = 0; j0 < d; j0 += 32) {
+        if (!PREFETCH) cst.load(a.Q, ds, qid, nrow, j0, lane);
+        cst.store(tile, lane);
+        __syncwarp();
+        if (PREFETCH && j0 + 32 < d) cst.load(a.Q, ds, qid, nrow, j0 + 32, lane);
+        const int jn = min(32, d - j0);
+        const float* xr = tile + lane * kRHP;
+        if (!generic && jn == 32) {   // hyperplane nodes only: s_i = fmaf(dir_ij, x_j, s_i)
 #pragma unroll 2
-                    for (int jj = 0; jj < 32; jj += 4) {
-                        const float4 x = *reinterpret_cast<const float4*>(xr + jj);
+            for (int jj = 0; jj < 32; jj += 4) {
+                const float4 x = *reinterpret_cast<const float4*>(xr + jj);
 #pragma unroll
-                        for (int i = 0; i < 7; ++i) {
-                            if (i < nn) {
-                                const float4 w = __ldg(reinterpret_cast<const float4*>(vec[i] + j0 + jj));
-                                s[i] = __fmaf_rn(w.x, x.x, s[i]);
-                                s[i] = __fmaf_rn(w.y, x.y, s[i]);
-                                s[i] = __fmaf_rn(w.z, x.z, s[i]);
-                                s[i] = __fmaf_rn(w.w, x.w, s[i]);
-                            }
-                        }
-                    }
-                } else {
-                    for (int jj = 0; jj < jn; ++jj) {
-                        const float x = xr[jj];
-#pragma unroll
-                        for (int i = 0; i < 7; ++i)
-                            if (i < nn) s[i] = __fmaf_rn(__ldg(vec[i] + j0 + jj), x, s[i]);
-                    }
-                }
-            } else {          // some mean-rule node: s_i += (x_j - mu_ij)^2 there (R4), same j order
-                for (int jj = 0; jj < jn; ++jj) {
-                    const float x = xr[jj];
-#pragma unroll
-                    for (int i = 0; i < 7; ++i) {
-                        if (i < nn) {
-                            const float w = __ldg(vec[i] + j0 + jj);
-                            const float e = __fsub_rn(x, w);
-                            s[i] = mean[i] ? __fmaf_rn(e, e, s[i]) : __fmaf_rn(w, x, s[i]);
-                        }
+                for (int i = 0; i < 7; ++i) {
+                    if (i < nn) {
+                        const float4 w = lead ? *reinterpret_cast<const float4*>(vec[i] + j0 + jj)
+                                              : __ldg(reinterpret_cast<const float4*>(vec[i] + j0 + jj));
+                        s[i] = __fmaf_rn(w.x, x.x, s[i]);
+                        s[i] = __fmaf_rn(w.y, x.y, s[i]);
+                        s[i] = __fmaf_rn(w.z, x.z, s[i]);
+                        s[i] = __fmaf_rn(w.w, x.w, s[i]);
                     }
                 }
             }
-            __syncwarp();
-        }
-        int li = 0;
-        for (int ll = 0; ll < nl; ++ll) {
-            const int nid = ((v + 1) << ll) - 1 + (li - ((1 << ll) - 1));
-            float sl = s[0];
+        } else {          // a mean-rule node somewhere (R4: s_i += (x_j - mu_ij)^2), or a ragged chunk
+            for (int jj = 0; jj < jn; ++jj) {
+                const float x = xr[jj];
 #pragma unroll
-            for (int i = 1; i < 7; ++i) sl = i == li ? s[i] : sl;
-            li = 2 * li + 1 + (sl > a.theta[nid] ? 1 : 0);
+                for (int i = 0; i < 7; ++i) {
+                    if (i < nn) {
+                        const float w = vec[i][j0 + jj];
+                        const float e = __fsub_rn(x, w);
+                        s[i] = mean[i] ? __fmaf_rn(e, e, s[i]) : __fmaf_rn(w, x, s[i]);
+                    }
+                }
+            }
         }
-        v = ((v + 1) << nl) - 1 + (li - ((1 << nl) - 1));
+        __syncwarp();
     }
     if (!act) return;
-    const int64_t q = q0 + lane;
-    const int g = v - (a.G - 1);
-    a.qleaf[q] = g;
-    atomicAdd(&lcnt[g], 1);
+    int li = 0;
+    for (int ll = 0; ll < nl; ++ll) {
+        const int nid = node_of(v, li);
+        float sl = s[0];
+#pragma unroll
+        for (int i = 1; i < 7; ++i) sl = i == li ? s[i] : sl;
+        li = 2 * li + 1 + (sl > a.theta[nid] ? 1 : 0);
+    }
+    const int vn = ((v + 1) << nl) - 1 + (li - ((1 << nl) - 1));   // node reached (level l0 + nl)
+    const int rel = vn - ((1 << (l0 + nl)) - 1);
+    a.qleaf[q] = rel;
+    atomicAdd(&cnt[rel], 1);
 }
 
 // exclusive scan of the G leaf counts into the scatter cursors (one block)
@@ -743,16 +756,44 @@ static size_t hash_smem(const QueryArgs& a) {
     return ((size_t)a.M * a.ds + (size_t)kRHW * 32 * kRHP) * sizeof(float);
 }
 
+// a1: ceil(depth / 3) passes of k_route_pass, the queries regrouped by the node they reached
+// between passes (k_leaf_scan / k_leaf_scatter over that level's nodes, into a.lperm); leaves in
+// a.qleaf and the leaf histogram in a.lcnt[0, G) on return.  Returns the kernels launched.
+static int launch_route(const QueryArgs& a, cudaStream_t s) {
+    const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
+    const size_t smem = ((size_t)7 * a.ds + (size_t)kRHW * 32 * kRHP) * sizeof(float);
+    if (smem > 48 * 1024) {
+        BLSH_CUDA(cudaFuncSetAttribute(k_route_pass<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        BLSH_CUDA(cudaFuncSetAttribute(k_route_pass<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    }
+    int launches = 0;
+    const uint32_t* order = nullptr;
+    for (int l0 = 0;; l0 += 3) {
+        const int nl = std::max(0, std::min(3, a.depth - l0));
+        const int nbins = 1 << (l0 + nl);
+        BLSH_CUDA(cudaMemsetAsync(a.lcnt, 0, (size_t)nbins * sizeof(int32_t), s));
+        if (a.nq < kRoutePrefetchBelow) k_route_pass<true><<<grid, kRHQ, smem, s>>>(a, l0, order, a.lcnt);
+        else k_route_pass<false><<<grid, kRHQ, smem, s>>>(a, l0, order, a.lcnt);
+        BLSH_LAUNCH_CHECK();
+        ++launches;
+        if (l0 + 3 >= a.depth) break;
+        k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, nbins, a.lcnt + a.G);
+        BLSH_LAUNCH_CHECK();
+        k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, a.lcnt + a.G, a.lperm);
+        BLSH_LAUNCH_CHECK();
+        launches += 2;
+        order = a.lperm;
+    }
+    return launches;
+}
+
 int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
     const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
     const size_t smem_h = hash_smem(a);
     int32_t* lcnt = a.lcnt;
     int32_t* lcur = a.lcnt + a.G;
-    BLSH_CUDA(cudaMemsetAsync(lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    if (a.nq < kRoutePrefetchBelow) k_route<true><<<grid, kRHQ, 0, s>>>(a, lcnt);
-    else k_route<false><<<grid, kRHQ, 0, s>>>(a, lcnt);
-    BLSH_LAUNCH_CHECK();
+    int launches = launch_route(a, s);
     k_leaf_scan<<<1, 1024, 0, s>>>(lcnt, a.G, lcur);
     BLSH_LAUNCH_CHECK();
     k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, lcur, a.lperm);
@@ -771,7 +812,7 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     }
 #undef BLSH_RH_CASE
     BLSH_LAUNCH_CHECK();
-    return 4;
+    return launches + 3;
 }
 
 // a1 alone over a batch, queries grouped by leaf (lperm), leaf counts in a.lcnt[0..G):
@@ -779,16 +820,12 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
 // on the queries of its own leaves only).
 int launch_route_group(const QueryArgs& a, cudaStream_t s) {
     if (a.nq == 0) return 0;
-    const unsigned grid = (unsigned)((a.nq + kRHQ - 1) / kRHQ);
-    BLSH_CUDA(cudaMemsetAsync(a.lcnt, 0, (size_t)a.G * sizeof(int32_t), s));
-    if (a.nq < kRoutePrefetchBelow) k_route<true><<<grid, kRHQ, 0, s>>>(a, a.lcnt);
-    else k_route<false><<<grid, kRHQ, 0, s>>>(a, a.lcnt);
-    BLSH_LAUNCH_CHECK();
+    int launches = launch_route(a, s);
     k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, a.G, a.lcnt + a.G);
     BLSH_LAUNCH_CHECK();
     k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, a.lcnt + a.G, a.lperm);
     BLSH_LAUNCH_CHECK();
-    return 3;
+    return launches + 2;
 }
 
 namespace {

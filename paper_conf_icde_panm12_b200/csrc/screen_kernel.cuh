@@ -44,8 +44,17 @@ constexpr uint32_t kSxIdesc = (1u << 4) | ((uint32_t)(kSxN >> 3) << 17) | ((128u
 constexpr float kSxEpsAcc = 0x1p-14f;       // tensor-core fp32 accumulation, relative to sum |a_k b_k|
 constexpr float kSxDelta = 0x1p-11f;        // relative slack on d~2 (AM-GM split 2^-12, K table 2^-13, fp32 ops)
 
-constexpr int kSxNM = 6;                    // block metadata ring (row entries + bound constants)
-constexpr int kSxMA = 4;                    // metadata fetched this many blocks ahead of the producers
+// metadata ring depth: 8 (screen 5.09 -> 4.93 ms at c4: the producers' waits for the epilogue
+// to release ring slots fell from 22 to 10 us per item; 6 / 7 slots or fetching 5-6 blocks
+// ahead measured no better, r02ar); 8 fills the 227 KB of shared memory at d_r = 384, NST = 8
+#ifndef BLSH_SX_NM   // (experiments: variant builds with -DBLSH_SX_NM=.. -DBLSH_SX_MA=..)
+#define BLSH_SX_NM 8
+#endif
+#ifndef BLSH_SX_MA
+#define BLSH_SX_MA 4
+#endif
+constexpr int kSxNM = BLSH_SX_NM;           // block metadata ring (row entries + bound constants)
+constexpr int kSxMA = BLSH_SX_MA;           // metadata fetched this many blocks ahead of the producers
 
 struct SxSmem {
     uint64_t afull[8], aempty[8];
