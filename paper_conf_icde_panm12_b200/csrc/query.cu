@@ -751,6 +751,7 @@ void upload_e8_roots() {
 }
 
 constexpr int64_t kRoutePrefetchBelow = 16384;   // batches smaller than this fill < 1 wave of k_route
+constexpr int64_t kRouteGroupFrom = 4096;        // regroup the queries between route passes from this batch size
 // k_hash: A_g [M][ds] + one staged chunk per warp
 static size_t hash_smem(const QueryArgs& a) {
     return ((size_t)a.M * a.ds + (size_t)kRHW * 32 * kRHP) * sizeof(float);
@@ -777,6 +778,9 @@ static int launch_route(const QueryArgs& a, cudaStream_t s) {
         BLSH_LAUNCH_CHECK();
         ++launches;
         if (l0 + 3 >= a.depth) break;
+        // small batches: no regrouping (two launches of latency for a few warps); their lanes
+        // read their subtrees' vectors through L1
+        if (a.nq < kRouteGroupFrom) continue;
         k_leaf_scan<<<1, 1024, 0, s>>>(a.lcnt, nbins, a.lcnt + a.G);
         BLSH_LAUNCH_CHECK();
         k_leaf_scatter<<<(unsigned)((a.nq + 255) / 256), 256, 0, s>>>(a.qleaf, a.nq, a.lcnt + a.G, a.lperm);
@@ -800,7 +804,8 @@ int launch_route_hash(const QueryArgs& a, cudaStream_t s) {
     BLSH_LAUNCH_CHECK();
 #define BLSH_RH_CASE(MMV)                                                                                   \
     case MMV:                                                                                              \
-        BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        if (smem_h > 48 * 1024)                                                                            \
+            BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
         k_hash<MMV><<<grid, kRHQ, smem_h, s>>>(a, a.lperm);                                                 \
         break;
     switch (a.M) {
@@ -890,7 +895,8 @@ void launch_hash(const QueryArgs& a, cudaStream_t s) {
     const size_t smem_h = hash_smem(a);
 #define BLSH_H_CASE(MMV)                                                                                    \
     case MMV:                                                                                              \
-        BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        if (smem_h > 48 * 1024)                                                                            \
+            BLSH_CUDA(cudaFuncSetAttribute(k_hash<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
         k_hash<MMV><<<grid, kRHQ, smem_h, s>>>(a, a.lperm);                                                 \
         break;
     switch (a.M) {
@@ -910,7 +916,8 @@ void launch_hash_tables(const QueryArgs& a, const HashTables& ht, cudaStream_t s
     const size_t smem_h = hash_smem(a);
 #define BLSH_HT_CASE(MMV)                                                                                     \
     case MMV:                                                                                                \
-        BLSH_CUDA(cudaFuncSetAttribute(k_hash_tables<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
+        if (smem_h > 48 * 1024)                                                                              \
+            BLSH_CUDA(cudaFuncSetAttribute(k_hash_tables<MMV>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_h)); \
         k_hash_tables<MMV><<<grid, kRHQ, smem_h, s>>>(a, ht);                                                 \
         break;
     switch (a.M) {

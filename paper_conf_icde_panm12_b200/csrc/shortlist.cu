@@ -56,6 +56,8 @@ constexpr int kRG = 4;   // rows per distance group (loads in flight per lane: k
 template <int NV, bool EMIT, bool LIST>
 __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int lane = threadIdx.x & 31;
+    extern __shared__ float4 sl_stage[];   // [kSLWarps][kRG][NV][32]: row loads in flight
+    float4* stg = sl_stage + (size_t)(threadIdx.x >> 5) * kRG * NV * 32;
     // grid-stride over the work items (a warp takes the next item as soon as it is done:
     // items differ in length, and a block would otherwise hold its slot until its slowest warp ends)
     // (list mode; the interval mode keeps one item per warp: neighbouring items, which share
@@ -87,23 +89,39 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     unsigned long long thr = kEmpty;
     // Rows r[0..nr) (table positions) that are candidates c, c+1, .. of q.
     auto group = [&](const int64_t (&r)[kRG], int nr, int64_t c) {
-        float part[kRG];
+        // the group's kRG x NV 16-byte loads in flight together: cp.async into this warp's
+        // staging slots [j][u][lane], one wait, then the chains read the lane's own slots (with
+        // register loads the compiler consumed each row before issuing the next: 3 LDG.128 in
+        // flight per lane in the SASS)
 #pragma unroll
         for (int j = 0; j < kRG; ++j) {
-            part[j] = 0.0f;
             if (j < nr) {
                 const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
 #pragma unroll
                 for (int u = 0; u < NV; ++u) {
                     const int v = lane + 32 * u;
                     if (v < nv) {
-                        const float4 x = __ldg(xr + v);
-                        float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
-                        part[j] = fmaf(dx, dx, part[j]);
-                        part[j] = fmaf(dy, dy, part[j]);
-                        part[j] = fmaf(dz, dz, part[j]);
-                        part[j] = fmaf(dw, dw, part[j]);
+                        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(stg + (j * NV + u) * 32 + lane);
+                        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(xr + v) : "memory");
                     }
+                }
+            }
+        }
+        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+        float part[kRG];
+#pragma unroll
+        for (int j = 0; j < kRG; ++j) {
+            part[j] = 0.0f;
+#pragma unroll
+            for (int u = 0; u < NV; ++u) {
+                const int v = lane + 32 * u;
+                if (v < nv) {
+                    const float4 x = stg[(j * NV + u) * 32 + lane];
+                    float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                    part[j] = fmaf(dx, dx, part[j]);
+                    part[j] = fmaf(dy, dy, part[j]);
+                    part[j] = fmaf(dz, dz, part[j]);
+                    part[j] = fmaf(dw, dw, part[j]);
                 }
             }
         }
@@ -202,16 +220,25 @@ __global__ void __launch_bounds__(256) k_merge(ShortlistArgs a, const int32_t* _
     const int k = a.k;
     TopK tk{kEmpty, kEmpty};
     unsigned long long thr = kEmpty;
-    for (int64_t it = a.item_off[q]; it < a.item_off[q + 1]; ++it) {
+    const int64_t it0 = a.item_off[q], it1 = a.item_off[q + 1];
+    auto load = [&](int64_t it, unsigned long long& l0, unsigned long long& l1) {
         const unsigned long long* L = a.partials + (size_t)it * k;
-        const unsigned long long l0 = lane < k ? L[lane] : kEmpty;
-        const unsigned long long l1 = lane + 32 < k ? L[lane + 32] : kEmpty;
+        l0 = lane < k ? L[lane] : kEmpty;
+        l1 = lane + 32 < k ? L[lane + 32] : kEmpty;
+    };
+    unsigned long long c0 = kEmpty, c1 = kEmpty;
+    if (it0 < it1) load(it0, c0, c1);
+    for (int64_t it = it0; it < it1; ++it) {
+        unsigned long long n0 = kEmpty, n1 = kEmpty;
+        if (it + 1 < it1) load(it + 1, n0, n1);   // the next list is in flight during this one's inserts
         for (int j = 0; j < k; ++j) {
-            const unsigned long long v = __shfl_sync(BLSH_FULL, j < 32 ? l0 : l1, j & 31);
+            const unsigned long long v = __shfl_sync(BLSH_FULL, j < 32 ? c0 : c1, j & 31);
             if (v >= thr) break;
             topk_insert(tk, v, lane);
             thr = topk_thr(tk, k);
         }
+        c0 = n0;
+        c1 = n1;
     }
     write_out(tk, q, k, lane, out_ids, out_d2, out_packed);
     if (lane == 0 && out_ncand) out_ncand[q] = (qoor[q] & 2) ? 0 : a.cnt[q];
@@ -492,14 +519,19 @@ void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     const unsigned grid = (unsigned)((a.list || a.n_items_dev) ? std::min<int64_t>(blocks, 148 * 8) : blocks);
     const int nvl = ((a.ds >> 2) + 31) / 32;
 
+    const int smem = kSLWarps * kRG * nvl * 32 * 16;
+    auto go = [&](auto kern) {
+        if (smem > 48 * 1024) BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        kern<<<grid, kSLWarps * 32, smem, s>>>(a);
+    };
 #define BLSH_SL_CASE(V)                                                                             \
     case V:                                                                                         \
         if (a.list) {                                                                               \
-            if (a.cand_keys) k_shortlist<V, true, true><<<grid, kSLWarps * 32, 0, s>>>(a);          \
-            else k_shortlist<V, false, true><<<grid, kSLWarps * 32, 0, s>>>(a);                     \
+            if (a.cand_keys) go(k_shortlist<V, true, true>);                                        \
+            else go(k_shortlist<V, false, true>);                                                   \
         } else {                                                                                    \
-            if (a.cand_keys) k_shortlist<V, true, false><<<grid, kSLWarps * 32, 0, s>>>(a);         \
-            else k_shortlist<V, false, false><<<grid, kSLWarps * 32, 0, s>>>(a);                    \
+            if (a.cand_keys) go(k_shortlist<V, true, false>);                                       \
+            else go(k_shortlist<V, false, false>);                                                  \
         }                                                                                           \
         break;
     switch (nvl) {
