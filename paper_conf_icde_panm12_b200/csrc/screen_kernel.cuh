@@ -753,8 +753,6 @@ __global__ void __launch_bounds__(256) k_tc_emit(TiledArgs a, const int64_t* __r
         qv[u] = v < nv ? __ldg(qrow + v) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
     int rescored = 0;
-    extern __shared__ float4 em_stage[];   // [8 warps][4 rows][NV][32]
-    float4* stg = em_stage + (size_t)(threadIdx.x >> 5) * 4 * NV * 32;
     // rows of the set bits of nm (lane i holds row position rpos); row r of a group goes to
     // slot sbase + (compact ? its rank among the set bits : its source lane)
     auto score_rows = [&](unsigned nm, uint32_t rpos, int64_t sbase, bool compact) {
@@ -774,37 +772,23 @@ __global__ void __launch_bounds__(256) k_tc_emit(TiledArgs a, const int64_t* __r
                     nr = r + 1;
                 }
             }
-            // the rows' 16-byte loads in flight together (cp.async into this warp's staging slots,
-            // as in k_tc_rescore), then the chains
+            float part[4];
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
+                part[r] = 0.0f;
                 if (r < nr) {
                     const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)row[r] * a.ds);
 #pragma unroll
                     for (int u = 0; u < NV; ++u) {
                         const int v = lane + 32 * u;
                         if (v < nv) {
-                            const uint32_t dst = smem_u32(stg + (r * NV + u) * 32 + lane);
-                            asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(xr + v) : "memory");
+                            const float4 x = __ldg(xr + v);
+                            const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                            part[r] = fmaf(dx, dx, part[r]);
+                            part[r] = fmaf(dy, dy, part[r]);
+                            part[r] = fmaf(dz, dz, part[r]);
+                            part[r] = fmaf(dw, dw, part[r]);
                         }
-                    }
-                }
-            }
-            asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-            float part[4];
-#pragma unroll
-            for (int r = 0; r < 4; ++r) {
-                part[r] = 0.0f;
-#pragma unroll
-                for (int u = 0; u < NV; ++u) {
-                    const int v = lane + 32 * u;
-                    if (v < nv) {
-                        const float4 x = stg[(r * NV + u) * 32 + lane];
-                        const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
-                        part[r] = fmaf(dx, dx, part[r]);
-                        part[r] = fmaf(dy, dy, part[r]);
-                        part[r] = fmaf(dz, dz, part[r]);
-                        part[r] = fmaf(dw, dw, part[r]);
                     }
                 }
             }

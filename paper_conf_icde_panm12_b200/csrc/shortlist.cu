@@ -56,7 +56,7 @@ constexpr int kRG = 4;   // rows per distance group (loads in flight per lane: k
 template <int NV, bool EMIT, bool LIST>
 __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     const int lane = threadIdx.x & 31;
-    extern __shared__ float4 sl_stage[];   // [kSLWarps][kRG][NV][32]: row loads in flight
+    extern __shared__ float4 sl_stage[];   // interval mode: [kSLWarps][kRG][NV][32], row loads in flight
     float4* stg = sl_stage + (size_t)(threadIdx.x >> 5) * kRG * NV * 32;
     // grid-stride over the work items (a warp takes the next item as soon as it is done:
     // items differ in length, and a block would otherwise hold its slot until its slowest warp ends)
@@ -89,39 +89,65 @@ __global__ void __launch_bounds__(kSLWarps * 32) k_shortlist(ShortlistArgs a) {
     unsigned long long thr = kEmpty;
     // Rows r[0..nr) (table positions) that are candidates c, c+1, .. of q.
     auto group = [&](const int64_t (&r)[kRG], int nr, int64_t c) {
-        // the group's kRG x NV 16-byte loads in flight together: cp.async into this warp's
-        // staging slots [j][u][lane], one wait, then the chains read the lane's own slots (with
-        // register loads the compiler consumed each row before issuing the next: 3 LDG.128 in
-        // flight per lane in the SASS)
+        float part[kRG];
+        if constexpr (!LIST) {
+            // interval mode (rows streamed once, the no-reuse regime): the group's kRG x NV 16-byte
+            // loads in flight together, by cp.async into this warp's staging slots [j][u][lane],
+            // one wait, then the chains read the lane's own slots (register loads: the compiler
+            // consumed each row before issuing the next, 3 LDG.128 in flight per lane; c5 with
+            // tiles off 0.79 -> 0.98 of measured HBM, r02au)
 #pragma unroll
-        for (int j = 0; j < kRG; ++j) {
-            if (j < nr) {
-                const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
+            for (int j = 0; j < kRG; ++j) {
+                if (j < nr) {
+                    const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
+#pragma unroll
+                    for (int u = 0; u < NV; ++u) {
+                        const int v = lane + 32 * u;
+                        if (v < nv) {
+                            const uint32_t dst = (uint32_t)__cvta_generic_to_shared(stg + (j * NV + u) * 32 + lane);
+                            asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(xr + v) : "memory");
+                        }
+                    }
+                }
+            }
+            asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+#pragma unroll
+            for (int j = 0; j < kRG; ++j) {
+                part[j] = 0.0f;
 #pragma unroll
                 for (int u = 0; u < NV; ++u) {
                     const int v = lane + 32 * u;
                     if (v < nv) {
-                        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(stg + (j * NV + u) * 32 + lane);
-                        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(xr + v) : "memory");
+                        const float4 x = stg[(j * NV + u) * 32 + lane];
+                        float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                        part[j] = fmaf(dx, dx, part[j]);
+                        part[j] = fmaf(dy, dy, part[j]);
+                        part[j] = fmaf(dz, dz, part[j]);
+                        part[j] = fmaf(dw, dw, part[j]);
                     }
                 }
             }
-        }
-        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-        float part[kRG];
+        } else {
+            // list mode (L > 1 tables, the E8 node: rows gathered, many served from L2): register
+            // loads, which the compiler overlaps with the previous row's chain (the staging's
+            // issue-then-wait measured slower here: p217 13.0 -> 17.3 ms, r02au)
 #pragma unroll
-        for (int j = 0; j < kRG; ++j) {
-            part[j] = 0.0f;
+            for (int j = 0; j < kRG; ++j) {
+                part[j] = 0.0f;
+                if (j < nr) {
+                    const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)r[j] * a.ds);
 #pragma unroll
-            for (int u = 0; u < NV; ++u) {
-                const int v = lane + 32 * u;
-                if (v < nv) {
-                    const float4 x = stg[(j * NV + u) * 32 + lane];
-                    float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
-                    part[j] = fmaf(dx, dx, part[j]);
-                    part[j] = fmaf(dy, dy, part[j]);
-                    part[j] = fmaf(dz, dz, part[j]);
-                    part[j] = fmaf(dw, dw, part[j]);
+                    for (int u = 0; u < NV; ++u) {
+                        const int v = lane + 32 * u;
+                        if (v < nv) {
+                            const float4 x = __ldg(xr + v);
+                            float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                            part[j] = fmaf(dx, dx, part[j]);
+                            part[j] = fmaf(dy, dy, part[j]);
+                            part[j] = fmaf(dz, dz, part[j]);
+                            part[j] = fmaf(dw, dw, part[j]);
+                        }
+                    }
                 }
             }
         }
@@ -519,7 +545,7 @@ void launch_shortlist(const ShortlistArgs& a, cudaStream_t s) {
     const unsigned grid = (unsigned)((a.list || a.n_items_dev) ? std::min<int64_t>(blocks, 148 * 8) : blocks);
     const int nvl = ((a.ds >> 2) + 31) / 32;
 
-    const int smem = kSLWarps * kRG * nvl * 32 * 16;
+    const int smem = a.list ? 0 : kSLWarps * kRG * nvl * 32 * 16;   // interval mode stages its row loads
     auto go = [&](auto kern) {
         if (smem > 48 * 1024) BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         kern<<<grid, kSLWarps * 32, smem, s>>>(a);

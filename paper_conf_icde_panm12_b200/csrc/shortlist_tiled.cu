@@ -937,16 +937,10 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
             keybuf.ensure((size_t)std::max<int64_t>(nkeys, 1) * 8);
             unsigned long long* keys = keybuf.as<unsigned long long>();
             const int nvq = (a.ds / 4 + 31) / 32;
-            auto em_launch = [&](auto kern, int nvt) {   // cp.async staging: 8 warps x 4 rows x NV x 32 x 16 B
-                const int smem_em = 8 * 4 * nvt * 32 * 16;
-                if (smem_em > 48 * 1024)
-                    BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_em));
-                kern<<<rg, 256, smem_em, s>>>(ta, uloc, coff, keys);
-            };
-            if (nvq <= 1) em_launch(k_tc_emit<1>, 1);
-            else if (nvq == 2) em_launch(k_tc_emit<2>, 2);
-            else if (nvq == 3) em_launch(k_tc_emit<3>, 3);
-            else em_launch(k_tc_emit<4>, 4);
+            if (nvq <= 1) k_tc_emit<1><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else if (nvq == 2) k_tc_emit<2><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else if (nvq == 3) k_tc_emit<3><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
+            else k_tc_emit<4><<<rg, 256, 0, s>>>(ta, uloc, coff, keys);
             BLSH_LAUNCH_CHECK();
             ++*launches;
             if (ev_sl1) BLSH_CUDA(cudaEventRecord(ev_sl1, s));
@@ -958,17 +952,12 @@ void run_tiled_shortlist(const QueryArgs& a, const uint32_t* qorder, int k, DevB
             if (ev_mid) BLSH_CUDA(cudaEventRecord(ev_mid, s));
             const unsigned rg = (unsigned)((n_items * QT + 7) / 8);
             const int nvq = (a.ds / 4 + 31) / 32;
-            // k_tc_rescore's cp.async staging: 8 warps x 4 rows x NV x 32 lanes x 16 B
-            auto rs_launch = [&](auto kern, int nvt) {
-                const int smem_rs = 8 * 4 * nvt * 32 * 16;
-                if (smem_rs > 48 * 1024)
-                    BLSH_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_rs));
-                kern<<<rg, 256, smem_rs, s>>>(ta);
-            };
-            if (nvq <= 1) rs_launch(k_tc_rescore<1>, 1);
-            else if (nvq == 2) rs_launch(k_tc_rescore<2>, 2);
-            else if (nvq == 3) rs_launch(k_tc_rescore<3>, 3);
-            else rs_launch(k_tc_rescore<4>, 4);
+            // (cp.async staging of the rescored rows, as in k_shortlist's interval mode, measured
+            // slower here: 0.92 -> 1.09 ms at c4, the rows of a tile's queries overlap in L1/L2, r02au)
+            if (nvq <= 1) k_tc_rescore<1><<<rg, 256, 0, s>>>(ta);
+            else if (nvq == 2) k_tc_rescore<2><<<rg, 256, 0, s>>>(ta);
+            else if (nvq == 3) k_tc_rescore<3><<<rg, 256, 0, s>>>(ta);
+            else k_tc_rescore<4><<<rg, 256, 0, s>>>(ta);
         } else {
             BLSH_CUDA(cudaFuncSetAttribute(k_shortlist_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             k_shortlist_tiled<<<(unsigned)n_items, kTiledThreads, smem, s>>>(ta);

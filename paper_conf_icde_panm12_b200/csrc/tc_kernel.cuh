@@ -511,8 +511,6 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
     // kRB rows per round, their 16-byte loads in flight together (8 rows: 80 registers and a
     // stack frame, fewer warps, 0.95 -> 1.28 ms at c4, r02am; 4 kept)
     constexpr int kRB = 4;
-    extern __shared__ float4 rs_stage[];   // [8 warps][kRB][NV][32]
-    float4* stg = rs_stage + (size_t)(threadIdx.x >> 5) * kRB * NV * 32;
     auto score_rows = [&](unsigned nm, uint32_t rpos) {
             while (nm) {
                 uint32_t row[kRB];
@@ -527,44 +525,23 @@ __global__ void __launch_bounds__(256) k_tc_rescore(TiledArgs a) {
                         nr = r + 1;
                     }
                 }
-                // all kRB x NV 16-byte loads in flight together: cp.async into this warp's shared
-                // staging slots [r][u][lane], one wait, then the chains read the lane's own slots
-                // (with register loads the compiler consumed each row before issuing the next: SASS
-                // showed 3 LDG.128 in flight per lane, long_scoreboard 65% of stalls, r02at)
+                float part[kRB];
 #pragma unroll
                 for (int r = 0; r < kRB; ++r) {
+                    part[r] = 0.0f;
                     if (r < nr) {
                         const float4* xr = reinterpret_cast<const float4*>(a.Xp + (size_t)row[r] * a.ds);
 #pragma unroll
                         for (int u = 0; u < NV; ++u) {
                             const int v = lane + 32 * u;
                             if (v < nv) {
-                                const uint32_t dst = smem_u32(stg + (r * NV + u) * 32 + lane);
-                                asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(xr + v) : "memory");
+                                const float4 x = __ldg(xr + v);
+                                const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
+                                part[r] = fmaf(dx, dx, part[r]);
+                                part[r] = fmaf(dy, dy, part[r]);
+                                part[r] = fmaf(dz, dz, part[r]);
+                                part[r] = fmaf(dw, dw, part[r]);
                             }
-                        }
-                    }
-                }
-                asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-                float4 xv[kRB][NV];
-#pragma unroll
-                for (int r = 0; r < kRB; ++r)
-#pragma unroll
-                    for (int u = 0; u < NV; ++u) xv[r][u] = stg[(r * NV + u) * 32 + lane];
-                float part[kRB];
-#pragma unroll
-                for (int r = 0; r < kRB; ++r) {
-                    part[r] = 0.0f;
-#pragma unroll
-                    for (int u = 0; u < NV; ++u) {
-                        const int v = lane + 32 * u;
-                        if (v < nv) {
-                            const float4 x = xv[r][u];
-                            const float dx = qv[u].x - x.x, dy = qv[u].y - x.y, dz = qv[u].z - x.z, dw = qv[u].w - x.w;
-                            part[r] = fmaf(dx, dx, part[r]);
-                            part[r] = fmaf(dy, dy, part[r]);
-                            part[r] = fmaf(dz, dz, part[r]);
-                            part[r] = fmaf(dw, dw, part[r]);
                         }
                     }
                 }
