@@ -327,7 +327,114 @@ namespace blsh {
 
 static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
                            const blsh_query_params& p, int64_t* out_ids, float* out_d2,
-                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base);
+                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base,
+                           bool capture = false);
+static bool query_graph(const blsh_index& ix, const float* Q, int64_t nq, int k, const blsh_query_params& p,
+                        int64_t* out_ids, float* out_d2, int64_t* out_ncand);
+
+// Small batches (<= small_batch_limit() queries on the warp short-list, whose plan needs no host
+// round trip): the whole call -- route, hash, probes, plan, short-list, merge, ~17 launches whose
+// host-side issue dominated the latency (GPU span 0.21 ms for one query, r02at) -- is captured
+// once per (shape, parameters, workspace) into a CUDA graph on a private stream and replayed on the
+// caller's stream: copy the batch into the graph's input buffer, launch, copy the answers out.
+// The first call of a shape runs normally (allocating every workspace buffer), then captures.
+// Results are those of run_query_core (the same kernels on the same inputs).  BLSH_GRAPH=0
+// disables it (experiments).
+static bool query_graph(const blsh_index& ix, const float* Q, int64_t nq, int k, const blsh_query_params& p,
+                        int64_t* out_ids, float* out_d2, int64_t* out_ncand) {
+    static const bool enabled = [] {
+        const char* e = std::getenv("BLSH_GRAPH");
+        return !(e && e[0] == '0');
+    }();
+    if (!enabled || nq <= 0 || nq > small_batch_limit() || p.keep_stages || p.timing || p.global_base || ix.L > 1 ||
+        (p.hierarchy == 1 && ix.quantizer == 1) || shortlist_kind(nq, ix.ds, ix.dr, p.n_probes, k) != 0)
+        return false;
+    QueryWork& w = ix.qw;
+    cudaStream_t s = (cudaStream_t)p.stream;
+    const size_t qbytes = (size_t)nq * ix.d * sizeof(float);
+    const size_t ib = ((size_t)nq * k * 8 + 255) & ~size_t(255), db = ((size_t)nq * k * 4 + 255) & ~size_t(255);
+    w.g_q.ensure(qbytes);
+    w.g_out.ensure(ib + db + (size_t)nq * 8);
+    const float* gq = w.g_q.as<float>();
+    int64_t* gi = w.g_out.as<int64_t>();
+    float* gd = reinterpret_cast<float*>(w.g_out.as<char>() + ib);
+    int64_t* gn = reinterpret_cast<int64_t*>(w.g_out.as<char>() + ib + db);
+    BLSH_CUDA(cudaMemcpyAsync(w.g_q.p, Q, qbytes, cudaMemcpyDeviceToDevice, s));
+    auto key_of = [&](QueryWork::GraphEntry& e) {
+        e.nq = nq; e.min_cand = p.min_cand; e.k = k; e.T = p.n_probes; e.probe = p.probe; e.hierarchy = p.hierarchy;
+        e.hstep = p.hier_step_bits; e.cperturb = p.curve_perturb; e.msb_min = p.msb_min;
+        const DevBuf* b[6] = {&w.arena, &w.partials, &w.scan.blocks, &w.g_q, &w.g_out, &w.listbuf};
+        for (int i = 0; i < 6; ++i) { e.bufs[i] = b[i]->p; e.sizes[i] = b[i]->bytes; }
+    };
+    auto same = [](const QueryWork::GraphEntry& a, const QueryWork::GraphEntry& b) {
+        if (a.nq != b.nq || a.min_cand != b.min_cand || a.k != b.k || a.T != b.T || a.probe != b.probe ||
+            a.hierarchy != b.hierarchy || a.hstep != b.hstep || a.cperturb != b.cperturb || a.msb_min != b.msb_min)
+            return false;
+        for (int i = 0; i < 6; ++i)
+            if (a.bufs[i] != b.bufs[i] || a.sizes[i] != b.sizes[i]) return false;
+        return true;
+    };
+    QueryWork::GraphEntry key{};
+    key_of(key);
+    QueryWork::GraphEntry* hit = nullptr;
+    for (auto& e : w.graphs)
+        if (same(e, key)) { hit = &e; break; }
+    if (!hit) {
+        // run it once for real (allocates the workspace, gives this call's answers), then capture
+        run_query_core(ix, gq, false, nq, k, p, gi, gd, nullptr, gn, false, nullptr);
+        QueryWork::GraphEntry e{};
+        key_of(e);
+        e.stats = ix.stats;
+        if (!w.cap) BLSH_CUDA(cudaStreamCreateWithFlags(&w.cap, cudaStreamNonBlocking));
+        blsh_query_params pc = p;
+        pc.stream = w.cap;
+        cudaGraph_t g = nullptr;
+        BLSH_CUDA(cudaStreamBeginCapture(w.cap, cudaStreamCaptureModeRelaxed));
+        try {
+            run_query_core(ix, gq, false, nq, k, pc, gi, gd, nullptr, gn, false, nullptr, true);
+        } catch (...) {
+            cudaStreamEndCapture(w.cap, &g);
+            if (g) cudaGraphDestroy(g);
+            throw;
+        }
+        BLSH_CUDA(cudaStreamEndCapture(w.cap, &g));
+        cudaGraphExec_t ex = nullptr;
+        const cudaError_t ie = cudaGraphInstantiate(&ex, g, 0);
+        cudaGraphDestroy(g);
+        BLSH_CUDA(ie);
+        bool stale = true;   // the capture must not have grown a buffer (its key would then differ)
+        QueryWork::GraphEntry chk{};
+        key_of(chk);
+        stale = !same(chk, e);
+        if (stale) {
+            cudaGraphExecDestroy(ex);
+        } else {
+            e.exec = ex;
+            e.stats.launches = ix.stats.launches;
+            if (w.graphs.size() >= 16) {
+                cudaGraphExecDestroy(w.graphs.front().exec);
+                w.graphs.erase(w.graphs.begin());
+            }
+            w.graphs.push_back(e);
+        }
+        ix.stats = e.stats;
+    } else {
+        BLSH_CUDA(cudaGraphLaunch(hit->exec, s));
+        BLSH_CUDA(cudaStreamSynchronize(s));
+        blsh_stats st = hit->stats;   // shape statistics of the captured call, counts of this one
+        st.total_cand = w.host_scalars[0];
+        st.n_items = w.host_scalars[1];
+        st.union_rows = st.total_cand;
+        st.pairs_scored = st.total_cand;
+        if (p.hierarchy == 1 && p.min_cand == 0) st.tau = w.host_scalars[2];
+        ix.stats = st;
+    }
+    BLSH_CUDA(cudaMemcpyAsync(out_ids, gi, (size_t)nq * k * 8, cudaMemcpyDeviceToDevice, s));
+    BLSH_CUDA(cudaMemcpyAsync(out_d2, gd, (size_t)nq * k * 4, cudaMemcpyDeviceToDevice, s));
+    if (out_ncand) BLSH_CUDA(cudaMemcpyAsync(out_ncand, gn, (size_t)nq * 8, cudaMemcpyDeviceToDevice, s));
+    BLSH_CUDA(cudaStreamSynchronize(s));
+    return true;
+}
 
 // A shard answers only the queries of its own leaves.  It routes the whole
 // batch (a1; every rank must, to learn the owners), then runs a2-a5 on the compacted batch
@@ -340,6 +447,9 @@ void run_query(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, in
                int64_t* out_ids, float* out_d2, unsigned long long* out_packed, int64_t* out_ncand, bool out_host,
                int64_t* out_base) {
     const bool shard = ix.leaf_lo > 0 || ix.leaf_hi < ix.G;
+    if (!shard && !q_host && !out_host && !out_base && !out_packed && out_ids && out_d2 &&
+        query_graph(ix, Q, nq, k, p, out_ids, out_d2, out_ncand))
+        return;
     if (!shard || p.keep_stages || out_base || nq == 0) {
         run_query_core(ix, Q, q_host, nq, k, p, out_ids, out_d2, out_packed, out_ncand, out_host, out_base);
         return;
@@ -499,8 +609,10 @@ void run_query_pipelined(const blsh_index& ix, int nb, const float* const* Q, in
 
 static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, int64_t nq, int k,
                            const blsh_query_params& p, int64_t* out_ids, float* out_d2,
-                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base) {
+                           unsigned long long* out_packed, int64_t* out_ncand, bool out_host, int64_t* out_base,
+                           bool capture) {
     cudaStream_t s = (cudaStream_t)p.stream;
+    if (!ix.qw.host_scalars) BLSH_CUDA(cudaMallocHost(&ix.qw.host_scalars, 4 * sizeof(int64_t)));
     QueryWork& w = ix.qw;
     const int T = p.n_probes, M = ix.M, ds = ix.ds;
     const bool keep = p.keep_stages != 0;
@@ -816,6 +928,11 @@ static void run_query_core(const blsh_index& ix, const float* Q, bool q_host, in
     }
     const bool tau_dev = p.hierarchy == 1 && p.min_cand == 0;
     if (tau_dev) BLSH_CUDA(cudaMemcpyAsync(&w.host_scalars[2], w.tau, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    if (capture) {   // query_graph: the caller launches, synchronises and reads host_scalars
+        stt.launches = launches;
+        stt.chunk = (int32_t)ch;
+        return;
+    }
     BLSH_CUDA(cudaStreamSynchronize(s));
     if (nosync) {
         total = w.host_scalars[0];

@@ -130,7 +130,19 @@ struct QueryWork {
     ScanTemp scan2;
     cudaStream_t side = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
-    int64_t host_scalars[3] = {0, 0, 0};   // plan statistics and tau, read back with the answers
+    int64_t* host_scalars = nullptr;   // pinned [3]: plan statistics and tau, read back with the answers
+    // small batches: the whole call captured once per shape into a CUDA graph (api.cu, query_graph)
+    struct GraphEntry {
+        int64_t nq, min_cand;
+        int k, T, probe, hierarchy, hstep, cperturb, msb_min;
+        const void* bufs[6];
+        size_t sizes[6];
+        cudaGraphExec_t exec;
+        blsh_stats stats;
+    };
+    std::vector<GraphEntry> graphs;
+    DevBuf g_q, g_out;                 // the graphs' query batch and answers
+    cudaStream_t cap = nullptr;        // capture stream
     // blsh_query_pipelined: double-buffered query uploads / answer downloads on a copy stream
     DevBuf pl_q[2], pl_out[2];
     cudaStream_t copy = nullptr;
@@ -148,6 +160,10 @@ struct QueryWork {
             if (pl_dl[i]) cudaEventDestroy(pl_dl[i]);
         }
         if (copy) cudaStreamDestroy(copy);
+        for (auto& g : graphs)
+            if (g.exec) cudaGraphExecDestroy(g.exec);
+        if (cap) cudaStreamDestroy(cap);
+        if (host_scalars) cudaFreeHost(host_scalars);
     }
 };
 
