@@ -713,7 +713,11 @@ int64_t plan_tiles(const QueryArgs& a, const uint32_t* qorder, DevBuf& tilebuf, 
             launch_median(d2bits, nq - 1, med, s);
             *launches += 2;
         }
-        float jump = 16.0f;   // cut a tile where consecutive queries are > 16x the median squared step apart
+        // cut a tile where consecutive queries are > 2048x the median squared step apart: at 4-512x
+        // c3's tiles (Zipf clusters, 5% between-cluster queries) were fragmented -- 99 M union rows,
+        // screen 16.1 ms; 2048x: 47 M, 9.0 ms (512 k -> 819 k q/s) with c4 unchanged; at 8192x the
+        // tiles span clusters, the screen's bound loosens and c4 and c3 slow down (r02ax sweep)
+        float jump = 2048.0f;
         if (const char* e = std::getenv("BLSH_TILE_JUMP")) jump = (float)std::atof(e);   // (experiments)
         k_tile_flags<<<g256, 256, 0, s>>>(d2bits, med, a.qleaf, a.qoor, qorder, nq, brk, jump);
         BLSH_LAUNCH_CHECK();
