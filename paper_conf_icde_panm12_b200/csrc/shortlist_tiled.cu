@@ -647,7 +647,10 @@ int shortlist_kind(int64_t nq, int ds, int dr, int T, int k) {
     if (mode && std::strcmp(mode, "warp") == 0) return 0;
     // small batches (<= 4 tiles): the tiled path's planning launches and host round trips
     // (~0.6 ms) exceed the warp short-list's whole run (profiles/r02/c5_sweep.jsonl, B <= 100)
-    if (!mode && nq <= kSmallBatch) return 0;
+    // batches of up to 1 024 queries with few probes also stream faster without tiles: C5 at
+    // 1 000 queries, T = 16 multiprobe / T = 8 E8: warp 0.94 / 0.98 ms vs tiled 1.17 / 1.20 ms;
+    // with T = 64 Morton-curve probes the tiles win (1.38 vs 1.58 ms) (profiles/r02/c5_sweep_final)
+    if (!mode && (nq <= kSmallBatch || (nq <= 1024 && nq * (int64_t)T <= 16384))) return 0;
     // large k (64 < k <= 512): the fp16 screen (kk lists) + exact keys per query + k_select;
     // beyond, or without the fp16 screen: the warp short-list emitting every key + k_select
     if (k > 64 && (k > kSxMaxKLarge || screen_variant() != 0 || (mode && std::strcmp(mode, "simt") == 0))) return 0;

@@ -44,9 +44,9 @@ def test_curve_probes(c1_pair_w1, c1, T, k):
 @pytest.mark.parametrize("mode", ["warp", "simt", "tc"])
 def test_curve_shortlist_variants(c1_pair_w1, c1, monkeypatch, mode):
     X, Q = c1
-    if mode != "tc":
-        monkeypatch.setenv("BLSH_SHORTLIST", mode)
+    monkeypatch.setenv("BLSH_SHORTLIST", mode)   # (tc: forced; 100 queries would take the warp list)
     run_query_pair(*c1_pair_w1, X, Q, 10, probe=3, T=6)
+    assert c1_pair_w1[0].stats().tiled == {"warp": 0, "simt": 1, "tc": 2}[mode]
 
 
 def test_curve_with_hierarchy(c1_pair_w1, c1):

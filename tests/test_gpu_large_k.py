@@ -162,7 +162,7 @@ def test_large_k_tc_vs_oracle(c1_pair, c1, monkeypatch, k, T):
 
 def test_large_k_tc_hierarchy_and_default_batch(c1_pair, c1):
     X, Q = c1
-    Q3 = np.concatenate([Q, Q[::-1], Q[::2]])      # 250 queries: the tiled path by default
+    Q3 = np.concatenate([Q] * 11)                   # 1 100 queries (> 1 024): the tiled path by default
     run_query_pair(*c1_pair, X, Q3, 300, probe=1, T=8, hierarchy=1)
     assert c1_pair[0].stats().tiled == 2
 

@@ -331,7 +331,7 @@ def test_warp_shortlist_fallback(blsh, orc, c1, monkeypatch):
     run_query_pair(ix, ox, X, Q, 10, probe=1, T=16)
     ix.query(torch.from_numpy(Q).cuda(), 10, probe=1, n_probes=16)
     assert ix.stats().tiled == 0, "batches of <= 128 queries take the warp short-list by default"
-    Q2 = np.concatenate([Q, Q, Q])                  # 300 queries: the tiled path
+    Q2 = np.concatenate([Q] * 11)                   # 1 100 queries (> 1 024): the tiled path
     run_query_pair(ix, ox, X, Q2, 10, probe=1, T=16)
     assert ix.stats().tiled >= 1
 
@@ -407,10 +407,10 @@ def test_tc_screen_equals_warp(blsh, orc, monkeypatch, shape):
 
 def test_sharded_merge_against_oracle(blsh, orc):
     """SURVEY §8(e) against the oracle directly: world = 4 leaf shards (each answers its
-    compacted ~150 owned queries on the tiled tcgen05 screen), packed lists merged with
+    compacted ~1 250 owned queries on the tiled tcgen05 screen), packed lists merged with
     blsh_merge_topk; counts equal the oracle's |A(q)| and the merged top-k passes check_topk
     against the oracle's single-index answer."""
-    X, Q = synth.make_dataset(synth.CONFIGS["c1"], n=10000, nq=600)
+    X, Q = synth.make_dataset(synth.CONFIGS["c1"], n=10000, nq=5000)
     Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
     ox = orc.OracleIndex(X, G=8, M=8, W=4.0, seed=5)
     oi, od, onc = ox.query(Q, 10, probe=1, T=16)

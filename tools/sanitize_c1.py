@@ -24,8 +24,8 @@ from paper_conf_icde_panm12_b200 import blsh  # noqa: E402
 
 
 def main():
-    # 600 queries: batches above the small-batch limit (128) take the query-tiled paths
-    X, Q = synth.make_dataset(synth.CONFIGS["c1"], nq=600)
+    # 1 200 queries: batches above 1 024 take the query-tiled paths
+    X, Q = synth.make_dataset(synth.CONFIGS["c1"], nq=1200)
     Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
     cases = [
         (dict(), dict(probe=0, n_probes=1), 10),
